@@ -1,0 +1,253 @@
+/*
+ * nestgpu.h -- C ABI of the B200-native nested-method correlated-subquery
+ * engine (libnestgpu.so, sm_100a).
+ *
+ * The operation (Fig. 2, §II-D; Fig. 4, P:175-183,
+ * §III-B): for every outer tuple r of R that passes the outer local
+ * predicates, evaluate the subquery over S with r's correlated value bound in
+ * ("subquery(r.c1)"), store the scalar result in Res[i],
+ * then keep r iff the predicate on Res holds ("Selection(=, R.col1, Res)",
+ * P:183) and compact the survivors.  Template (north_star):
+ *
+ *   SELECT R.* FROM R
+ *   WHERE <outer_preds(R)>
+ *     AND lhs_mult*R.cmp <outer_op> rhs_mult*(SELECT AGG(S.agg) FROM S
+ *            WHERE <inner_preds(S)> AND R.key <corr_op> S.key)
+ *   -- or AND [NOT] EXISTS (SELECT * FROM S WHERE ...)
+ *
+ * The three entry points named by the north star are nestgpu_load_column
+ * (LoadToGPU), nestgpu_build_index (the sorted correlated-column
+ * index, §III-D "Indexing") and nestgpu_exec_correlated (the
+ * vectorised subquery loop, §III-D "Vectorization").  The rest manage
+ * the context, the memory pool (§III-C) and results.
+ *
+ * Conventions
+ *  - Every call returns nestgpu_status: 0 = OK, < 0 = error.  The message of
+ *    the last error is kept per context (nestgpu_last_error).  No exception,
+ *    abort() or CPU fallback ever crosses this boundary: if the device work
+ *    cannot be done, the call fails.
+ *  - Device memory and the CUDA stream are OWNED BY THE CALLER.  The library
+ *    carves every allocation out of the caller's arena (no cudaMalloc on any
+ *    path) and enqueues all work on the caller's stream.
+ *  - Host buffers passed in are borrowed for the duration of the call only.
+ *  - Column / index ids and result pointers belong to the context.  Result
+ *    device pointers stay valid until the next exec or release.
+ *  - A context is not thread-safe; use one per host thread / GPU.
+ *  - Semantics follow SQL-92 where the paper is silent (DESIGN.md readings
+ *    R1-R11): NULL compares UNKNOWN (not TRUE); an empty subquery gives
+ *    NULL for MIN/MAX/SUM/AVG, 0 for COUNT(*), false for EXISTS.
+ */
+#ifndef NESTGPU_H
+#define NESTGPU_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define NESTGPU_ABI_VERSION 1
+
+typedef int32_t nestgpu_status;
+enum {
+    NESTGPU_OK = 0,
+    NESTGPU_ERR_INVALID = -1,      /* bad argument / id / plan (nothing launched) */
+    NESTGPU_ERR_OOM = -2,          /* the caller's arena is exhausted */
+    NESTGPU_ERR_TYPE = -3,         /* dtype mismatch */
+    NESTGPU_ERR_UNSUPPORTED = -4,  /* valid SQL outside this engine's template */
+    NESTGPU_ERR_OVERFLOW = -5,     /* |S'| * max|payload| may exceed int64 (reading R5) */
+    NESTGPU_ERR_CUDA = -6,         /* a CUDA runtime call or launch failed */
+    NESTGPU_ERR_BUFFER = -7        /* caller's host buffer too small */
+};
+
+/* Column storage types (columnar store).  Decimals are scaled
+ * integers; dates are int32 days since 1970-01-01 (reading R11). */
+typedef enum {
+    NG_INT32 = 0,     /* int32 */
+    NG_INT64 = 1,     /* int64 */
+    NG_DECIMAL = 2,   /* int64, value * 10^scale */
+    NG_DATE = 3,      /* int32 days since 1970-01-01 */
+    NG_DECIMAL32 = 4  /* int32, value * 10^scale (fits when |value*10^scale| < 2^31) */
+} nestgpu_dtype;
+
+/* Comparison operators.  A correlated predicate always reads
+ * outer.key OP inner.key (reading R8). */
+typedef enum { NG_EQ = 0, NG_NE = 1, NG_LT = 2, NG_LE = 3, NG_GT = 4, NG_GE = 5 } nestgpu_cmp;
+
+/* Aggregates (type-JA subqueries; EXISTS as semi-join). */
+typedef enum {
+    NG_MIN = 0, NG_MAX = 1, NG_SUM = 2,
+    NG_COUNT = 3,       /* COUNT(*) over qualifying S rows */
+    NG_AVG = 4,         /* exact: compared as a*x*nn OP b*sum (reading R6) */
+    NG_EXISTS = 5, NG_NOT_EXISTS = 6
+} nestgpu_agg;
+
+typedef struct nestgpu_ctx nestgpu_ctx;   /* opaque */
+
+/* Local predicate on one table: col OP literal (rhs_col < 0) or col OP rhs_col.
+ * Columns are compared as int64 values (int32 storage is widened). */
+typedef struct {
+    int32_t col;
+    nestgpu_cmp op;
+    int64_t literal;
+    int32_t rhs_col;
+} nestgpu_pred;
+
+/* ---------------------------------------------------------------- context */
+
+/* Create a context on `device` over the caller's device buffer
+ * [d_arena, d_arena + arena_bytes) (>= 1 MiB, 256-B aligned) and the
+ * caller's cudaStream_t `cuda_stream` (NULL = legacy default stream).
+ * The library never frees d_arena.  Errors: INVALID, CUDA. */
+nestgpu_status nestgpu_create(int device, void *d_arena, size_t arena_bytes,
+                              void *cuda_stream, nestgpu_ctx **out);
+/* Destroy the context (waits for its stream).  NULL is a no-op. */
+nestgpu_status nestgpu_destroy(nestgpu_ctx *ctx);
+/* Message of the last failed call on ctx ("" if none).  Owned by ctx. */
+const char *nestgpu_last_error(const nestgpu_ctx *ctx);
+/* Number of kernels this context has launched since creation. */
+int64_t nestgpu_launch_count(const nestgpu_ctx *ctx);
+/* Switch the stream subsequent calls enqueue on. */
+nestgpu_status nestgpu_set_stream(nestgpu_ctx *ctx, void *cuda_stream);
+
+/* Memory pool (Fig. 7: "record where to free", then move the
+ * tail back).  nestgpu_mark returns the current tail of the persistent side of
+ * the arena; nestgpu_release drops every column, index and result created
+ * after that mark.  Errors: INVALID. */
+nestgpu_status nestgpu_mark(nestgpu_ctx *ctx, uint64_t *out_mark);
+nestgpu_status nestgpu_release(nestgpu_ctx *ctx, uint64_t mark);
+/* Bytes in use (persistent + scratch) and the high-water mark. */
+nestgpu_status nestgpu_arena_usage(const nestgpu_ctx *ctx, size_t *in_use, size_t *peak);
+
+/* ---------------------------------------------------------------- columns */
+
+/* LoadToGPU: copy n host values (and optional validity bytes,
+ * host_valid[i] == 0 means NULL; NULL pointer = NOT NULL column) into the
+ * arena, asynchronously on the context stream; the call returns after the
+ * copy has been enqueued AND completed (the host buffers are borrowed for the
+ * call only; pinned host memory makes the copy a DMA).  Values are stored in
+ * the dtype's width; `scale` is metadata for NG_DECIMAL / NG_DECIMAL32.
+ * n must be < 2^31.  Returns the new column id.  Errors: INVALID, OOM, CUDA. */
+nestgpu_status nestgpu_load_column(nestgpu_ctx *ctx, nestgpu_dtype dtype, int32_t scale,
+                                   const void *host_values, const uint8_t *host_valid,
+                                   int64_t n, int32_t *out_col);
+/* Reserve an uninitialised column (contents to be filled by the caller on
+ * the device, e.g. by an NCCL broadcast into nestgpu_column_info's pointers).
+ * with_valid != 0 reserves a validity byte array too. */
+nestgpu_status nestgpu_alloc_column(nestgpu_ctx *ctx, nestgpu_dtype dtype, int32_t scale,
+                                    int64_t n, int32_t with_valid, int32_t *out_col);
+typedef struct {
+    nestgpu_dtype dtype;
+    int32_t scale;
+    int64_t n;
+    void *d_values;      /* n * (4|8) bytes */
+    uint8_t *d_valid;    /* n bytes or NULL */
+} nestgpu_column_desc;
+nestgpu_status nestgpu_column_info(const nestgpu_ctx *ctx, int32_t col, nestgpu_column_desc *out);
+
+/* ---------------------------------------------------------------- index */
+
+/* Build the correlated-column index of P:315 over S' = rows of S whose
+ * inner_preds are all TRUE ("invariant component", executed once):
+ * a stable device radix sort of S' by the correlated key, carrying the
+ * aggregate payload.  key_cols: 1 column (int32/int64/date/decimal) or 2
+ * int32-storage columns (composite '=' key, packed; reading R9).
+ * payload_col: the column a MIN/MAX/SUM/AVG plan aggregates, or -1 (COUNT /
+ * EXISTS need none).  Rows with a NULL key component are dropped (they
+ * satisfy no correlated predicate); rows with a NULL payload are dropped too
+ * (MIN/MAX/SUM/AVG skip them), so an index with a nullable payload column
+ * cannot serve COUNT/EXISTS plans.  All columns must have S's row count.
+ * Synchronises the stream once (to size the sort).
+ * Errors: INVALID, TYPE, UNSUPPORTED, OOM, CUDA. */
+nestgpu_status nestgpu_build_index(nestgpu_ctx *ctx, const int32_t *key_cols, int32_t n_key_cols,
+                                   int32_t payload_col,
+                                   const nestgpu_pred *inner_preds, int32_t n_inner_preds,
+                                   int32_t *out_index);
+/* Drop an index (its arena bytes are reclaimed at the next release of a
+ * mark taken before it was built). */
+nestgpu_status nestgpu_drop_index(nestgpu_ctx *ctx, int32_t index);
+
+/* Device layout of an index, for the multi-GPU broadcast (sorted keys are
+ * order-preserving unsigned encodings: int32 k -> (uint32)k ^ 0x80000000,
+ * int64 k -> (uint64)k ^ 2^63, composite (k1,k2) -> enc32(k1) << 32 | enc32(k2)). */
+typedef struct {
+    int64_t n;              /* |S'| */
+    int32_t key_bytes;      /* 4 or 8 */
+    int32_t payload_bytes;  /* 0, 4 or 8 */
+    void *d_keys;           /* n * key_bytes, ascending */
+    void *d_payload;        /* n * payload_bytes, co-sorted, or NULL */
+} nestgpu_index_desc;
+nestgpu_status nestgpu_index_info(const nestgpu_ctx *ctx, int32_t index, nestgpu_index_desc *out);
+/* Receiving rank of a broadcast: create an index with the given shape whose
+ * contents the caller fills on the device (d_keys / d_payload of *out after
+ * the call).  key_cols / payload_col / inner_preds describe what it indexes
+ * (they are validated against plans exactly as for nestgpu_build_index). */
+nestgpu_status nestgpu_index_create_empty(nestgpu_ctx *ctx, int64_t n, int32_t key_bytes,
+                                          int32_t payload_bytes,
+                                          const int32_t *key_cols, int32_t n_key_cols,
+                                          int32_t payload_col,
+                                          const nestgpu_pred *inner_preds, int32_t n_inner_preds,
+                                          nestgpu_index_desc *out, int32_t *out_index);
+
+/* ---------------------------------------------------------------- exec */
+
+typedef struct {
+    const nestgpu_pred *outer_preds; int32_t n_outer_preds;   /* over R, conjunctive */
+    int32_t outer_key_cols[2];                                /* correlated outer column(s) */
+    int32_t inner_key_cols[2];                                /* correlated inner column(s) */
+    int32_t n_key_cols;                                       /* 1, or 2 (composite, '=' only) */
+    nestgpu_cmp corr_op;                                      /* outer.key OP inner.key */
+    const nestgpu_pred *inner_preds; int32_t n_inner_preds;   /* over S, conjunctive, invariant */
+    nestgpu_agg agg;
+    int32_t agg_col;                                          /* S column; ignored for COUNT/EXISTS */
+    int32_t outer_cmp_col;                                    /* R column x; ignored for EXISTS */
+    nestgpu_cmp outer_op;                                     /* lhs_mult*x OP rhs_mult*v */
+    int64_t lhs_mult, rhs_mult;                               /* 1 .. 2^31-1 (reading R7) */
+    int32_t index;                                            /* -1: tiled nested loop over S'; else index id */
+    int64_t row_id_base;                                      /* added to emitted row ids (R shard offset) */
+    int32_t emit_all;                                         /* 0: survivors only; 1: every R' tuple */
+} nestgpu_plan;
+
+typedef struct {
+    int64_t n_rows;               /* survivors, or |R'| if emit_all */
+    const int64_t *d_row_ids;     /* ascending R row ids (+ row_id_base) */
+    const int64_t *d_values;      /* Res[i]: MIN/MAX/SUM value, COUNT, AVG rounded at
+                                     scale+6 (reading R6), EXISTS 0/1 */
+    const uint8_t *d_valid;       /* 0: the subquery value is NULL */
+    const uint8_t *d_passed;      /* outer predicate TRUE (always 1 unless emit_all) */
+    const int64_t *d_avg_sum;     /* AVG only: exact sum of non-NULL payloads */
+    const int64_t *d_avg_cnt;     /* AVG only: number of non-NULL payloads (nn) */
+} nestgpu_result;
+
+/* Execute one correlated subquery plan.  R is the set of columns the outer_*
+ * fields name (all with one row count), S the columns the inner_* / agg
+ * fields name.  index >= 0: S' comes from that index (its key columns, payload
+ * and inner predicates must match the plan: INVALID otherwise); index == -1:
+ * S is filtered here and the tiled block-nested-loop kernel runs.  Work is
+ * enqueued on the context stream; the call synchronises once at the end to
+ * read the survivor count.  Errors: INVALID, TYPE, UNSUPPORTED, OVERFLOW,
+ * OOM, CUDA.  Nothing is launched when validation fails. */
+nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *ctx, const nestgpu_plan *plan,
+                                       nestgpu_result *out);
+
+/* Copy up to cap rows of a result to host buffers (each pointer may be NULL
+ * to skip that field).  BUFFER if cap < n_rows (nothing copied).  Synchronous. */
+nestgpu_status nestgpu_result_to_host(nestgpu_ctx *ctx, const nestgpu_result *res,
+                                      int64_t *row_ids, int64_t *values, uint8_t *valid,
+                                      uint8_t *passed, int64_t *avg_sum, int64_t *avg_cnt,
+                                      int64_t cap);
+
+/* Per-stage device times (ms, CUDA events on the context stream) of the last
+ * exec / build_index when profiling is on (nestgpu_set_profiling(ctx, 1)).
+ * Stage order: 0 outer filter, 1 inner filter, 2 sort, 3 subquery kernel
+ * (range-agg or nested loop), 4 finalize+compact, 5 total.  NaN if a stage
+ * did not run. */
+#define NESTGPU_N_STAGES 6
+nestgpu_status nestgpu_set_profiling(nestgpu_ctx *ctx, int32_t on);
+nestgpu_status nestgpu_last_profile(const nestgpu_ctx *ctx, float *ms, int32_t n);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* NESTGPU_H */

@@ -1,0 +1,793 @@
+// api.cpp -- the C ABI (include/nestgpu.h): context, memory pool, columnar
+// store, index build, plan validation and the exec pipeline.
+//
+// Pipeline of nestgpu_exec_correlated (one stream, no device allocation, one
+// host synchronisation at the end):
+//   a2  filter_kernel(R, outer preds)        -> R' ids + encoded keys
+//   a3  filter_kernel(S, inner preds)        -> S' (key, payload)   [BNL path]
+//       or the index built by nestgpu_build_index (a3 + a4, once)   [index path]
+//   a5+a6 range_short/long kernels            -> per-R' partials     [index path]
+//   a7  bnl_kernel                            -> per-R' partials     [BNL path]
+//   a8+a9 finalize_kernel                     -> compacted result
+//   D2H of the survivor count.
+#include <cuda_runtime.h>
+
+#include <climits>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/nestgpu.h"
+#include "internal.h"
+
+namespace {
+
+struct Column {
+    nestgpu_dtype dtype;
+    int32_t scale;
+    int64_t n;
+    void *d;
+    uint8_t *valid;
+    size_t off;
+    bool alive;
+    bool stats;         // host-side min/max known
+    long long mn, mx;
+};
+
+struct IndexRec {
+    bool alive;
+    size_t off;
+    int64_t n;
+    int kb, vb;
+    void *keys;
+    void *payload;
+    long long *d_n;     // device copy of n
+    int32_t key_cols[2];
+    int n_key;
+    int32_t payload_col;
+    std::vector<nestgpu_pred> inner;
+    bool payload_nullable;
+};
+
+constexpr int PIN_WORDS = 8 * 256 + 64;
+constexpr size_t ALIGN = 256;
+
+}  // namespace
+
+struct nestgpu_ctx {
+    int device;
+    char *base;
+    size_t size;
+    size_t lo;     // persistent tail (grows up)
+    size_t hi;     // scratch head (grows down from size)
+    size_t peak;
+    cudaStream_t stream;
+    std::string err;
+    long long launches;
+    int num_sms;
+    std::vector<Column> cols;
+    std::vector<IndexRec> idx;
+    unsigned *pinned;  // host pinned words for small D2H / H2D
+    bool profiling;
+    cudaEvent_t ev[NESTGPU_N_STAGES][2];
+    bool ran[NESTGPU_N_STAGES];
+};
+
+namespace {
+
+nestgpu_status fail(nestgpu_ctx *c, nestgpu_status code, const char *fmt, ...)
+{
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    if (c) c->err = buf;
+    return code;
+}
+
+#define CUDA_TRY(ctx, expr)                                                                         \
+    do {                                                                                            \
+        cudaError_t e_ = (expr);                                                                    \
+        if (e_ != cudaSuccess)                                                                      \
+            return fail(ctx, NESTGPU_ERR_CUDA, "%s: %s (%s:%d)", #expr, cudaGetErrorString(e_),     \
+                        __FILE__, __LINE__);                                                        \
+    } while (0)
+
+size_t align_up(size_t x) { return (x + ALIGN - 1) / ALIGN * ALIGN; }
+
+void *palloc(nestgpu_ctx *c, size_t bytes)
+{
+    size_t b = align_up(bytes + 16);  // +16: bulk copies / vector loads may read a ragged tail
+    if (c->lo + b > c->hi) return nullptr;
+    void *p = c->base + c->lo;
+    c->lo += b;
+    size_t used = c->lo + (c->size - c->hi);
+    if (used > c->peak) c->peak = used;
+    return p;
+}
+
+void *salloc(nestgpu_ctx *c, size_t bytes)
+{
+    size_t b = align_up(bytes + 16);
+    if (c->hi < c->lo + b) return nullptr;
+    c->hi -= b;
+    size_t used = c->lo + (c->size - c->hi);
+    if (used > c->peak) c->peak = used;
+    return c->base + c->hi;
+}
+
+int dtype_width(nestgpu_dtype t)
+{
+    switch (t) {
+    case NG_INT32: case NG_DATE: case NG_DECIMAL32: return 4;
+    case NG_INT64: case NG_DECIMAL: return 8;
+    }
+    return 0;
+}
+
+bool valid_op(int op) { return op >= NG_EQ && op <= NG_GE; }
+
+const Column *col_get(const nestgpu_ctx *c, int32_t id)
+{
+    if (id < 0 || id >= (int32_t)c->cols.size() || !c->cols[id].alive) return nullptr;
+    return &c->cols[id];
+}
+
+// Build the device predicate set for a conjunction over a relation of n rows.
+nestgpu_status make_preds(nestgpu_ctx *c, const nestgpu_pred *p, int32_t np, int64_t n, ng::PredSet &out,
+                          const char *what)
+{
+    if (np < 0 || np > ng::MAX_PREDS) return fail(c, NESTGPU_ERR_UNSUPPORTED, "%s: at most %d predicates", what, ng::MAX_PREDS);
+    if (np > 0 && !p) return fail(c, NESTGPU_ERR_INVALID, "%s: null predicate array", what);
+    memset(&out, 0, sizeof out);
+    out.n = np;
+    for (int k = 0; k < np; k++) {
+        const Column *a = col_get(c, p[k].col);
+        if (!a) return fail(c, NESTGPU_ERR_INVALID, "%s[%d]: unknown column %d", what, k, p[k].col);
+        if (a->n != n) return fail(c, NESTGPU_ERR_INVALID, "%s[%d]: column %d has %lld rows, relation has %lld", what, k, p[k].col, (long long)a->n, (long long)n);
+        if (!valid_op(p[k].op)) return fail(c, NESTGPU_ERR_INVALID, "%s[%d]: bad operator", what, k);
+        ng::DevPred &d = out.p[k];
+        d.col = a->d;
+        d.valid = a->valid;
+        d.w = dtype_width(a->dtype);
+        d.op = p[k].op;
+        d.lit = p[k].literal;
+        if (p[k].rhs_col >= 0) {
+            const Column *b = col_get(c, p[k].rhs_col);
+            if (!b) return fail(c, NESTGPU_ERR_INVALID, "%s[%d]: unknown rhs column %d", what, k, p[k].rhs_col);
+            if (b->n != n) return fail(c, NESTGPU_ERR_INVALID, "%s[%d]: rhs column row count differs", what, k);
+            d.rhs = b->d;
+            d.rhs_valid = b->valid;
+            d.rhs_w = dtype_width(b->dtype);
+        }
+    }
+    return NESTGPU_OK;
+}
+
+bool same_preds(const nestgpu_pred *a, int32_t na, const std::vector<nestgpu_pred> &b)
+{
+    if ((size_t)na != b.size()) return false;
+    for (int i = 0; i < na; i++)
+        if (a[i].col != b[i].col || a[i].op != b[i].op || a[i].rhs_col != b[i].rhs_col ||
+            (a[i].rhs_col < 0 && a[i].literal != b[i].literal))
+            return false;
+    return true;
+}
+
+// Key source: one column, or two int32-storage columns (composite '=').
+nestgpu_status make_key(nestgpu_ctx *c, const int32_t *cols, int32_t nk, int64_t &n, ng::KeySrc &ks, const char *what)
+{
+    if (nk != 1 && nk != 2) return fail(c, NESTGPU_ERR_INVALID, "%s: 1 or 2 key columns", what);
+    const Column *a = col_get(c, cols[0]);
+    if (!a) return fail(c, NESTGPU_ERR_INVALID, "%s: unknown key column %d", what, cols[0]);
+    memset(&ks, 0, sizeof ks);
+    ks.c0 = a->d;
+    ks.v0 = a->valid;
+    ks.w0 = dtype_width(a->dtype);
+    ks.n_key = nk;
+    n = a->n;
+    if (nk == 2) {
+        const Column *b = col_get(c, cols[1]);
+        if (!b) return fail(c, NESTGPU_ERR_INVALID, "%s: unknown key column %d", what, cols[1]);
+        if (b->n != n) return fail(c, NESTGPU_ERR_INVALID, "%s: key columns differ in row count", what);
+        if (dtype_width(a->dtype) != 4 || dtype_width(b->dtype) != 4)
+            return fail(c, NESTGPU_ERR_UNSUPPORTED, "%s: composite keys need int32-storage columns", what);
+        ks.c1 = b->d;
+        ks.v1 = b->valid;
+    }
+    return NESTGPU_OK;
+}
+
+int key_bytes(const nestgpu_ctx *c, const int32_t *cols, int32_t nk)
+{
+    return (nk == 1 && dtype_width(c->cols[cols[0]].dtype) == 4) ? 4 : 8;
+}
+
+void prof_begin(nestgpu_ctx *c, int s)
+{
+    if (c->profiling) {
+        cudaEventRecord(c->ev[s][0], c->stream);
+        c->ran[s] = true;
+    }
+}
+void prof_end(nestgpu_ctx *c, int s)
+{
+    if (c->profiling) cudaEventRecord(c->ev[s][1], c->stream);
+}
+
+// Host-side min/max of a column (lazily, one small D2H) for the SUM/AVG
+// overflow pre-check (reading R5).
+nestgpu_status column_stats(nestgpu_ctx *c, Column &col);
+
+}  // namespace
+
+namespace ng {
+cudaError_t launch_minmax(const void *col, int w, const uint8_t *valid, long long n, long long *out2, cudaStream_t st,
+                          long long *launches);
+}
+
+namespace {
+nestgpu_status column_stats(nestgpu_ctx *c, Column &col)
+{
+    if (col.stats) return NESTGPU_OK;
+    long long *d = (long long *)salloc(c, 16);
+    if (!d) return fail(c, NESTGPU_ERR_OOM, "arena exhausted (stats)");
+    CUDA_TRY(c, ng::launch_minmax(col.d, dtype_width(col.dtype), col.valid, col.n, d, c->stream, &c->launches));
+    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, d, 16, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    memcpy(&col.mn, c->pinned, 8);
+    memcpy(&col.mx, (char *)c->pinned + 8, 8);
+    col.stats = true;
+    return NESTGPU_OK;
+}
+}  // namespace
+
+extern "C" {
+
+nestgpu_status nestgpu_create(int device, void *d_arena, size_t arena_bytes, void *cuda_stream, nestgpu_ctx **out)
+{
+    if (!out) return NESTGPU_ERR_INVALID;
+    *out = nullptr;
+    if (!d_arena || arena_bytes < (1u << 20) || ((uintptr_t)d_arena % ALIGN) != 0) return NESTGPU_ERR_INVALID;
+    if (cudaSetDevice(device) != cudaSuccess) return NESTGPU_ERR_CUDA;
+    nestgpu_ctx *c = new nestgpu_ctx();
+    c->device = device;
+    c->base = (char *)d_arena;
+    c->size = arena_bytes / ALIGN * ALIGN;
+    c->lo = 0;
+    c->hi = c->size;
+    c->peak = 0;
+    c->stream = (cudaStream_t)cuda_stream;
+    c->launches = 0;
+    c->profiling = false;
+    if (cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess ||
+        cudaMallocHost((void **)&c->pinned, PIN_WORDS * sizeof(unsigned)) != cudaSuccess) {
+        delete c;
+        return NESTGPU_ERR_CUDA;
+    }
+    for (int s = 0; s < NESTGPU_N_STAGES; s++) {
+        cudaEventCreate(&c->ev[s][0]);
+        cudaEventCreate(&c->ev[s][1]);
+        c->ran[s] = false;
+    }
+    *out = c;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_destroy(nestgpu_ctx *c)
+{
+    if (!c) return NESTGPU_OK;
+    cudaSetDevice(c->device);
+    cudaStreamSynchronize(c->stream);
+    for (int s = 0; s < NESTGPU_N_STAGES; s++) {
+        cudaEventDestroy(c->ev[s][0]);
+        cudaEventDestroy(c->ev[s][1]);
+    }
+    cudaFreeHost(c->pinned);
+    delete c;
+    return NESTGPU_OK;
+}
+
+const char *nestgpu_last_error(const nestgpu_ctx *c) { return c ? c->err.c_str() : "null context"; }
+int64_t nestgpu_launch_count(const nestgpu_ctx *c) { return c ? c->launches : 0; }
+
+nestgpu_status nestgpu_set_stream(nestgpu_ctx *c, void *s)
+{
+    if (!c) return NESTGPU_ERR_INVALID;
+    c->stream = (cudaStream_t)s;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_mark(nestgpu_ctx *c, uint64_t *m)
+{
+    if (!c || !m) return NESTGPU_ERR_INVALID;
+    *m = c->lo;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_release(nestgpu_ctx *c, uint64_t m)
+{
+    if (!c) return NESTGPU_ERR_INVALID;
+    if (m > c->lo) return fail(c, NESTGPU_ERR_INVALID, "release: mark %llu beyond tail %zu", (unsigned long long)m, c->lo);
+    cudaSetDevice(c->device);
+    // Work already enqueued may still read the released bytes.
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    c->lo = m;
+    c->hi = c->size;
+    for (auto &col : c->cols)
+        if (col.alive && col.off >= m) col.alive = false;
+    for (auto &ix : c->idx)
+        if (ix.alive && ix.off >= m) ix.alive = false;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_arena_usage(const nestgpu_ctx *c, size_t *in_use, size_t *peak)
+{
+    if (!c) return NESTGPU_ERR_INVALID;
+    if (in_use) *in_use = c->lo + (c->size - c->hi);
+    if (peak) *peak = c->peak;
+    return NESTGPU_OK;
+}
+
+static nestgpu_status new_column(nestgpu_ctx *c, nestgpu_dtype dtype, int32_t scale, int64_t n, bool with_valid,
+                                 int32_t *out)
+{
+    const int w = dtype_width(dtype);
+    if (!w) return fail(c, NESTGPU_ERR_TYPE, "unknown dtype %d", (int)dtype);
+    if (n < 0 || n >= (1ll << 31)) return fail(c, NESTGPU_ERR_INVALID, "column length %lld outside [0, 2^31)", (long long)n);
+    Column col{};
+    col.dtype = dtype;
+    col.scale = scale;
+    col.n = n;
+    col.off = c->lo;
+    col.d = palloc(c, (size_t)n * w);
+    if (!col.d) return fail(c, NESTGPU_ERR_OOM, "arena exhausted loading a %lld-row column", (long long)n);
+    if (with_valid) {
+        col.valid = (uint8_t *)palloc(c, (size_t)n);
+        if (!col.valid) {
+            c->lo = col.off;
+            return fail(c, NESTGPU_ERR_OOM, "arena exhausted (validity)");
+        }
+    }
+    col.alive = true;
+    c->cols.push_back(col);
+    *out = (int32_t)c->cols.size() - 1;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_load_column(nestgpu_ctx *c, nestgpu_dtype dtype, int32_t scale, const void *host_values,
+                                   const uint8_t *host_valid, int64_t n, int32_t *out_col)
+{
+    if (!c || !out_col || (n > 0 && !host_values)) return fail(c, NESTGPU_ERR_INVALID, "load_column: null argument");
+    cudaSetDevice(c->device);
+    int32_t id;
+    nestgpu_status s = new_column(c, dtype, scale, n, host_valid != nullptr, &id);
+    if (s) return s;
+    Column &col = c->cols[id];
+    const size_t bytes = (size_t)n * dtype_width(dtype);
+    if (n > 0) {
+        CUDA_TRY(c, cudaMemcpyAsync(col.d, host_values, bytes, cudaMemcpyHostToDevice, c->stream));
+        if (host_valid) CUDA_TRY(c, cudaMemcpyAsync(col.valid, host_valid, (size_t)n, cudaMemcpyHostToDevice, c->stream));
+        CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    }
+    *out_col = id;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_alloc_column(nestgpu_ctx *c, nestgpu_dtype dtype, int32_t scale, int64_t n, int32_t with_valid,
+                                    int32_t *out_col)
+{
+    if (!c || !out_col) return fail(c, NESTGPU_ERR_INVALID, "alloc_column: null argument");
+    return new_column(c, dtype, scale, n, with_valid != 0, out_col);
+}
+
+nestgpu_status nestgpu_column_info(const nestgpu_ctx *c, int32_t id, nestgpu_column_desc *out)
+{
+    if (!c || !out) return NESTGPU_ERR_INVALID;
+    const Column *col = col_get(c, id);
+    if (!col) return NESTGPU_ERR_INVALID;
+    out->dtype = col->dtype;
+    out->scale = col->scale;
+    out->n = col->n;
+    out->d_values = col->d;
+    out->d_valid = col->valid;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int32_t n_key_cols, int32_t payload_col,
+                                   const nestgpu_pred *inner_preds, int32_t n_inner_preds, int32_t *out_index)
+{
+    if (!c || !key_cols || !out_index) return fail(c, NESTGPU_ERR_INVALID, "build_index: null argument");
+    cudaSetDevice(c->device);
+    ng::KeySrc ks;
+    int64_t n;
+    nestgpu_status s = make_key(c, key_cols, n_key_cols, n, ks, "build_index");
+    if (s) return s;
+    ng::PredSet ps;
+    if ((s = make_preds(c, inner_preds, n_inner_preds, n, ps, "inner_preds"))) return s;
+    ng::ValSrc vs{nullptr, nullptr, 0};
+    const Column *pc = nullptr;
+    if (payload_col >= 0) {
+        pc = col_get(c, payload_col);
+        if (!pc) return fail(c, NESTGPU_ERR_INVALID, "build_index: unknown payload column %d", payload_col);
+        if (pc->n != n) return fail(c, NESTGPU_ERR_INVALID, "build_index: payload row count differs");
+        vs.c = pc->d;
+        vs.v = pc->valid;
+        vs.w = dtype_width(pc->dtype);
+    }
+    const int kb = key_bytes(c, key_cols, n_key_cols);
+    const int vb = pc ? vs.w : 0;
+    c->hi = c->size;  // scratch reset
+    for (int st = 0; st < NESTGPU_N_STAGES; st++) c->ran[st] = false;
+    void *tk = salloc(c, (size_t)n * kb), *tv = vb ? salloc(c, (size_t)n * vb) : nullptr;
+    void *uk = salloc(c, (size_t)n * kb), *uv = vb ? salloc(c, (size_t)n * vb) : nullptr;
+    void *fscr = salloc(c, ng::filter_scratch_bytes(n));
+    void *sscr = salloc(c, ng::sort_scratch_bytes(n));
+    unsigned *hist = (unsigned *)salloc(c, 8 * 256 * 4 + 64);
+    unsigned *dbase = (unsigned *)salloc(c, 8 * 256 * 4);
+    if (!tk || !uk || !fscr || !sscr || !hist || !dbase || (vb && (!tv || !uv)))
+        return fail(c, NESTGPU_ERR_OOM, "arena exhausted building an index over %lld rows", (long long)n);
+    long long *d_count = (long long *)(hist + 8 * 256);
+    CUDA_TRY(c, cudaMemsetAsync(hist, 0, 8 * 256 * 4, c->stream));
+    prof_begin(c, 1);
+    CUDA_TRY(c, ng::launch_filter(n, ps, ks, kb, vs, vb, 1, pc ? 1 : 0, nullptr, tk, nullptr, tv, hist, nullptr, fscr,
+                                  d_count, c->stream, &c->launches));
+    prof_end(c, 1);
+    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, hist, kb * 256 * 4, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaMemcpyAsync(c->pinned + 8 * 256, d_count, 8, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    long long nsp;
+    memcpy(&nsp, c->pinned + 8 * 256, 8);
+    // plan the passes: skip digits whose histogram has a single bucket
+    std::vector<int> passes;
+    for (int d = 0; d < kb; d++) {
+        bool trivial = false;
+        for (int b = 0; b < 256; b++)
+            if (c->pinned[d * 256 + b] == (unsigned)nsp) { trivial = true; break; }
+        if (!trivial) passes.push_back(d);
+    }
+    // digit bases for every pass (exclusive prefix over buckets)
+    for (size_t p = 0; p < passes.size(); p++) {
+        unsigned run = 0;
+        for (int b = 0; b < 256; b++) {
+            unsigned t = c->pinned[passes[p] * 256 + b];
+            c->pinned[p * 256 + b] = run;  // safe: p <= passes[p], rows read before overwritten
+            run += t;
+        }
+    }
+    if (!passes.empty())
+        CUDA_TRY(c, cudaMemcpyAsync(dbase, c->pinned, passes.size() * 256 * 4, cudaMemcpyHostToDevice, c->stream));
+
+    IndexRec ix{};
+    ix.off = c->lo;
+    ix.n = nsp;
+    ix.kb = kb;
+    ix.vb = vb;
+    ix.d_n = (long long *)palloc(c, 8);
+    ix.keys = palloc(c, (size_t)nsp * kb);
+    ix.payload = vb ? palloc(c, (size_t)nsp * vb) : nullptr;
+    if (!ix.d_n || !ix.keys || (vb && !ix.payload)) {
+        c->lo = ix.off;
+        return fail(c, NESTGPU_ERR_OOM, "arena exhausted storing an index of %lld rows", nsp);
+    }
+    c->pinned[8 * 256 + 4] = (unsigned)(nsp & 0xffffffffu);
+    c->pinned[8 * 256 + 5] = (unsigned)((unsigned long long)nsp >> 32);
+    CUDA_TRY(c, cudaMemcpyAsync(ix.d_n, c->pinned + 8 * 256 + 4, 8, cudaMemcpyHostToDevice, c->stream));
+    prof_begin(c, 2);
+    const int np = (int)passes.size();
+    if (np == 0) {
+        if (nsp > 0) {
+            CUDA_TRY(c, cudaMemcpyAsync(ix.keys, tk, (size_t)nsp * kb, cudaMemcpyDeviceToDevice, c->stream));
+            if (vb) CUDA_TRY(c, cudaMemcpyAsync(ix.payload, tv, (size_t)nsp * vb, cudaMemcpyDeviceToDevice, c->stream));
+        }
+    } else {
+        // T -> ... -> P with ping-pong so that the last pass writes P.
+        const void *ik = tk, *iv = tv;
+        for (int p = 0; p < np; p++) {
+            const bool to_final = ((np - 1 - p) % 2) == 0;
+            void *ok = to_final ? ix.keys : uk;
+            void *ov = to_final ? ix.payload : uv;
+            if (ok == ik) { ok = tk; ov = tv; }
+            CUDA_TRY(c, ng::launch_radix_pass(kb, vb, ik, ok, iv, ov, nsp, passes[p] * 8, dbase + p * 256, sscr,
+                                              c->stream, &c->launches));
+            ik = ok;
+            iv = ov;
+        }
+    }
+    prof_end(c, 2);
+    ix.key_cols[0] = key_cols[0];
+    ix.key_cols[1] = n_key_cols == 2 ? key_cols[1] : -1;
+    ix.n_key = n_key_cols;
+    ix.payload_col = payload_col;
+    ix.inner.assign(inner_preds, inner_preds + n_inner_preds);
+    ix.payload_nullable = pc && pc->valid;
+    ix.alive = true;
+    c->idx.push_back(ix);
+    *out_index = (int32_t)c->idx.size() - 1;
+    CUDA_TRY(c, cudaGetLastError());
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_drop_index(nestgpu_ctx *c, int32_t index)
+{
+    if (!c || index < 0 || index >= (int32_t)c->idx.size() || !c->idx[index].alive)
+        return fail(c, NESTGPU_ERR_INVALID, "drop_index: unknown index %d", index);
+    c->idx[index].alive = false;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_index_info(const nestgpu_ctx *c, int32_t index, nestgpu_index_desc *out)
+{
+    if (!c || !out || index < 0 || index >= (int32_t)c->idx.size() || !c->idx[index].alive) return NESTGPU_ERR_INVALID;
+    const IndexRec &ix = c->idx[index];
+    out->n = ix.n;
+    out->key_bytes = ix.kb;
+    out->payload_bytes = ix.vb;
+    out->d_keys = ix.keys;
+    out->d_payload = ix.payload;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_index_create_empty(nestgpu_ctx *c, int64_t n, int32_t key_bytes_, int32_t payload_bytes,
+                                          const int32_t *key_cols, int32_t n_key_cols, int32_t payload_col,
+                                          const nestgpu_pred *inner_preds, int32_t n_inner_preds,
+                                          nestgpu_index_desc *out, int32_t *out_index)
+{
+    if (!c || !out || !out_index || !key_cols) return fail(c, NESTGPU_ERR_INVALID, "index_create_empty: null argument");
+    if (n < 0 || n >= (1ll << 31) || (key_bytes_ != 4 && key_bytes_ != 8) ||
+        (payload_bytes != 0 && payload_bytes != 4 && payload_bytes != 8))
+        return fail(c, NESTGPU_ERR_INVALID, "index_create_empty: bad shape");
+    ng::KeySrc ks;
+    int64_t ns;
+    nestgpu_status s = make_key(c, key_cols, n_key_cols, ns, ks, "index_create_empty");
+    if (s) return s;
+    if (key_bytes(c, key_cols, n_key_cols) != key_bytes_)
+        return fail(c, NESTGPU_ERR_TYPE, "index_create_empty: key width does not match the key columns");
+    if (n_inner_preds < 0 || (n_inner_preds > 0 && !inner_preds)) return fail(c, NESTGPU_ERR_INVALID, "bad inner preds");
+    cudaSetDevice(c->device);
+    IndexRec ix{};
+    ix.off = c->lo;
+    ix.n = n;
+    ix.kb = key_bytes_;
+    ix.vb = payload_bytes;
+    ix.d_n = (long long *)palloc(c, 8);
+    ix.keys = palloc(c, (size_t)n * key_bytes_);
+    ix.payload = payload_bytes ? palloc(c, (size_t)n * payload_bytes) : nullptr;
+    if (!ix.d_n || !ix.keys || (payload_bytes && !ix.payload)) {
+        c->lo = ix.off;
+        return fail(c, NESTGPU_ERR_OOM, "arena exhausted (index_create_empty)");
+    }
+    long long nn = n;
+    memcpy(c->pinned, &nn, 8);
+    CUDA_TRY(c, cudaMemcpyAsync(ix.d_n, c->pinned, 8, cudaMemcpyHostToDevice, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    ix.key_cols[0] = key_cols[0];
+    ix.key_cols[1] = n_key_cols == 2 ? key_cols[1] : -1;
+    ix.n_key = n_key_cols;
+    ix.payload_col = payload_col;
+    ix.inner.assign(inner_preds, inner_preds + n_inner_preds);
+    const Column *pc = payload_col >= 0 ? col_get(c, payload_col) : nullptr;
+    ix.payload_nullable = pc && pc->valid;
+    ix.alive = true;
+    c->idx.push_back(ix);
+    *out_index = (int32_t)c->idx.size() - 1;
+    out->n = n;
+    out->key_bytes = key_bytes_;
+    out->payload_bytes = payload_bytes;
+    out->d_keys = ix.keys;
+    out->d_payload = ix.payload;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, nestgpu_result *out)
+{
+    if (!c || !P || !out) return fail(c, NESTGPU_ERR_INVALID, "exec: null argument");
+    cudaSetDevice(c->device);
+    memset(out, 0, sizeof *out);
+    // ------------------------------------------------------------ validation
+    if (P->agg < NG_MIN || P->agg > NG_NOT_EXISTS) return fail(c, NESTGPU_ERR_INVALID, "exec: bad aggregate");
+    if (!valid_op(P->corr_op)) return fail(c, NESTGPU_ERR_INVALID, "exec: bad correlated operator");
+    if (P->n_key_cols == 2 && P->corr_op != NG_EQ)
+        return fail(c, NESTGPU_ERR_UNSUPPORTED, "exec: composite correlation supports '=' only");
+    const bool is_exists = P->agg == NG_EXISTS || P->agg == NG_NOT_EXISTS;
+    const bool value_agg = P->agg == NG_MIN || P->agg == NG_MAX || P->agg == NG_SUM || P->agg == NG_AVG;
+    if (!is_exists && !valid_op(P->outer_op)) return fail(c, NESTGPU_ERR_INVALID, "exec: bad outer operator");
+    if (!is_exists && (P->lhs_mult < 1 || P->lhs_mult >= (1ll << 31) || P->rhs_mult < 1 || P->rhs_mult >= (1ll << 31)))
+        return fail(c, NESTGPU_ERR_INVALID, "exec: lhs_mult / rhs_mult must be in [1, 2^31)");
+    ng::KeySrc rks, sks;
+    int64_t nR, nS;
+    nestgpu_status s;
+    if ((s = make_key(c, P->outer_key_cols, P->n_key_cols, nR, rks, "outer key"))) return s;
+    if ((s = make_key(c, P->inner_key_cols, P->n_key_cols, nS, sks, "inner key"))) return s;
+    ng::PredSet ops, ips;
+    if ((s = make_preds(c, P->outer_preds, P->n_outer_preds, nR, ops, "outer_preds"))) return s;
+    if ((s = make_preds(c, P->inner_preds, P->n_inner_preds, nS, ips, "inner_preds"))) return s;
+    const Column *xc = nullptr;
+    if (!is_exists) {
+        xc = col_get(c, P->outer_cmp_col);
+        if (!xc) return fail(c, NESTGPU_ERR_INVALID, "exec: unknown outer comparison column %d", P->outer_cmp_col);
+        if (xc->n != nR) return fail(c, NESTGPU_ERR_INVALID, "exec: outer comparison column row count differs from R");
+    }
+    Column *ac = nullptr;
+    if (value_agg) {
+        ac = (P->agg_col >= 0 && P->agg_col < (int32_t)c->cols.size() && c->cols[P->agg_col].alive) ? &c->cols[P->agg_col] : nullptr;
+        if (!ac) return fail(c, NESTGPU_ERR_INVALID, "exec: unknown aggregate column %d", P->agg_col);
+        if (ac->n != nS) return fail(c, NESTGPU_ERR_INVALID, "exec: aggregate column row count differs from S");
+    }
+    const int rkb = key_bytes(c, P->outer_key_cols, P->n_key_cols);
+    const int skb = key_bytes(c, P->inner_key_cols, P->n_key_cols);
+    int kb = (rkb == 8 || skb == 8) ? 8 : 4;
+    const IndexRec *ix = nullptr;
+    if (P->index >= 0) {
+        if (P->index >= (int32_t)c->idx.size() || !c->idx[P->index].alive)
+            return fail(c, NESTGPU_ERR_INVALID, "exec: unknown index %d", P->index);
+        ix = &c->idx[P->index];
+        if (ix->n_key != P->n_key_cols || ix->key_cols[0] != P->inner_key_cols[0] ||
+            (P->n_key_cols == 2 && ix->key_cols[1] != P->inner_key_cols[1]))
+            return fail(c, NESTGPU_ERR_INVALID, "exec: index %d is on different key columns", P->index);
+        if (!same_preds(P->inner_preds, P->n_inner_preds, ix->inner))
+            return fail(c, NESTGPU_ERR_INVALID, "exec: index %d was built with different inner predicates", P->index);
+        if (value_agg && ix->payload_col != P->agg_col)
+            return fail(c, NESTGPU_ERR_INVALID, "exec: index %d carries column %d, plan aggregates %d", P->index, ix->payload_col, P->agg_col);
+        if (!value_agg && ix->payload_nullable)
+            return fail(c, NESTGPU_ERR_INVALID, "exec: index %d dropped NULL-payload rows; COUNT/EXISTS need an index without payload", P->index);
+        if (ix->kb != kb)
+            return fail(c, NESTGPU_ERR_UNSUPPORTED, "exec: outer key is 64-bit but index %d has 32-bit keys", P->index);
+    }
+    const int vb = value_agg ? dtype_width(ac->dtype) : 0;
+    if ((P->agg == NG_SUM || P->agg == NG_AVG) && vb == 8) {
+        if ((s = column_stats(c, *ac))) return s;
+        __int128 m = ac->mx > -(ac->mn) ? (__int128)ac->mx : -(__int128)ac->mn;
+        if ((__int128)nS * m >= ((__int128)1 << 63))
+            return fail(c, NESTGPU_ERR_OVERFLOW, "exec: |S| * max|payload| may exceed int64 (reading R5)");
+    }
+
+    // ------------------------------------------------------------ allocation
+    c->hi = c->size;  // scratch reset: previous results die here
+    for (int st = 0; st < NESTGPU_N_STAGES; st++) c->ran[st] = false;
+    const bool ravalid = rks.v0 || rks.v1;
+    int *ids = (int *)salloc(c, (size_t)nR * 4);
+    void *rkeys = salloc(c, (size_t)nR * kb);
+    uint8_t *rkvalid = ravalid ? (uint8_t *)salloc(c, (size_t)nR) : nullptr;
+    long long *acc = (long long *)salloc(c, (size_t)nR * 8);
+    long long *cnt = (long long *)salloc(c, (size_t)nR * 8);
+    long long *counts = (long long *)salloc(c, 64);  // [0] |R'| [1] |S'| [2] survivors; [4..5] extreme
+    size_t fsz = ng::filter_scratch_bytes(nR > nS ? nR : nS);
+    void *fscr = salloc(c, fsz);
+    void *kscr = salloc(c, ix ? ng::range_scratch_bytes(nR) : ng::bnl_scratch_bytes());
+    long long *o_ids = (long long *)salloc(c, (size_t)nR * 8);
+    long long *o_vals = (long long *)salloc(c, (size_t)nR * 8);
+    uint8_t *o_valid = (uint8_t *)salloc(c, (size_t)nR);
+    uint8_t *o_pass = (uint8_t *)salloc(c, (size_t)nR);
+    long long *o_sum = P->agg == NG_AVG ? (long long *)salloc(c, (size_t)nR * 8) : nullptr;
+    long long *o_cnt = P->agg == NG_AVG ? (long long *)salloc(c, (size_t)nR * 8) : nullptr;
+    void *skeys = nullptr, *svals = nullptr;
+    if (!ix) {
+        skeys = salloc(c, (size_t)nS * kb);
+        svals = vb ? salloc(c, (size_t)nS * vb) : nullptr;
+    }
+    if (!ids || !rkeys || (ravalid && !rkvalid) || !acc || !cnt || !counts || !fscr || !kscr || !o_ids || !o_vals ||
+        !o_valid || !o_pass || (P->agg == NG_AVG && (!o_sum || !o_cnt)) || (!ix && (!skeys || (vb && !svals))))
+        return fail(c, NESTGPU_ERR_OOM, "arena exhausted executing a plan over |R|=%lld |S|=%lld", (long long)nR, (long long)nS);
+    unsigned *extreme = (unsigned *)(counts + 4);
+    long long *d_nrp = counts, *d_nsp = counts + 1, *d_out = counts + 2;
+
+    // ------------------------------------------------------------ a2: R'
+    prof_begin(c, 5);
+    prof_begin(c, 0);
+    ng::ValSrc none{nullptr, nullptr, 0};
+    CUDA_TRY(c, cudaMemsetAsync(counts, 0, 64, c->stream));
+    CUDA_TRY(c, ng::launch_filter(nR, ops, rks, kb, none, 0, 0, 0, ids, rkeys, rkvalid, nullptr, nullptr, nullptr, fscr,
+                                  d_nrp, c->stream, &c->launches));
+    prof_end(c, 0);
+
+    // ------------------------------------------------------------ a3 / a5-a7
+    if (ix) {
+        prof_begin(c, 3);
+        CUDA_TRY(c, ng::launch_range_agg(kb, vb, P->corr_op, P->agg, nR, d_nrp, rkeys, ix->keys, ix->payload, ix->n,
+                                         acc, cnt, kscr, c->stream, &c->launches));
+        prof_end(c, 3);
+    } else {
+        prof_begin(c, 1);
+        ng::ValSrc vs{nullptr, nullptr, 0};
+        if (value_agg) { vs.c = ac->d; vs.v = ac->valid; vs.w = vb; }
+        CUDA_TRY(c, ng::launch_filter(nS, ips, sks, kb, vs, vb, 1, value_agg ? 1 : 0, nullptr, skeys, nullptr, svals,
+                                      nullptr, value_agg ? extreme : nullptr, fscr, d_nsp, c->stream, &c->launches));
+        CUDA_TRY(c, ng::launch_init_partials(nR, P->agg, acc, cnt, c->stream, &c->launches));
+        prof_end(c, 1);
+        prof_begin(c, 3);
+        CUDA_TRY(c, ng::launch_bnl(kb, vb, P->corr_op, P->agg, nR, d_nrp, rkeys, nS, d_nsp, skeys, svals, extreme, acc,
+                                   cnt, kscr, c->num_sms, c->stream, &c->launches));
+        prof_end(c, 3);
+    }
+
+    // ------------------------------------------------------------ a8 + a9
+    prof_begin(c, 4);
+    ng::FinalizeArgs fa{};
+    fa.n_rp_max = nR;
+    fa.d_nrp = d_nrp;
+    fa.ids = ids;
+    fa.kvalid = rkvalid;
+    fa.acc = acc;
+    fa.cnt = cnt;
+    fa.x_col = xc ? xc->d : nullptr;
+    fa.x_valid = xc ? xc->valid : nullptr;
+    fa.x_w = xc ? dtype_width(xc->dtype) : 4;
+    fa.agg = P->agg;
+    fa.outer_op = P->outer_op;
+    fa.a = P->lhs_mult;
+    fa.b = P->rhs_mult;
+    fa.row_id_base = P->row_id_base;
+    fa.emit_all = P->emit_all;
+    fa.out_ids = o_ids;
+    fa.out_vals = o_vals;
+    fa.out_sum = o_sum;
+    fa.out_cnt = o_cnt;
+    fa.out_valid = o_valid;
+    fa.out_passed = o_pass;
+    fa.out_count = d_out;
+    fa.scratch = fscr;
+    CUDA_TRY(c, ng::launch_finalize(fa, c->stream, &c->launches));
+    prof_end(c, 4);
+    prof_end(c, 5);
+    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, d_out, 8, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    long long nout;
+    memcpy(&nout, c->pinned, 8);
+    out->n_rows = nout;
+    out->d_row_ids = (const int64_t *)o_ids;
+    out->d_values = (const int64_t *)o_vals;
+    out->d_valid = o_valid;
+    out->d_passed = o_pass;
+    out->d_avg_sum = (const int64_t *)o_sum;
+    out->d_avg_cnt = (const int64_t *)o_cnt;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_result_to_host(nestgpu_ctx *c, const nestgpu_result *r, int64_t *row_ids, int64_t *values,
+                                      uint8_t *valid, uint8_t *passed, int64_t *avg_sum, int64_t *avg_cnt, int64_t cap)
+{
+    if (!c || !r) return fail(c, NESTGPU_ERR_INVALID, "result_to_host: null argument");
+    if (cap < r->n_rows) return fail(c, NESTGPU_ERR_BUFFER, "result_to_host: %lld rows, buffer holds %lld", (long long)r->n_rows, (long long)cap);
+    cudaSetDevice(c->device);
+    const size_t n = (size_t)r->n_rows;
+    if (n) {
+        if (row_ids) CUDA_TRY(c, cudaMemcpyAsync(row_ids, r->d_row_ids, n * 8, cudaMemcpyDeviceToHost, c->stream));
+        if (values) CUDA_TRY(c, cudaMemcpyAsync(values, r->d_values, n * 8, cudaMemcpyDeviceToHost, c->stream));
+        if (valid) CUDA_TRY(c, cudaMemcpyAsync(valid, r->d_valid, n, cudaMemcpyDeviceToHost, c->stream));
+        if (passed) CUDA_TRY(c, cudaMemcpyAsync(passed, r->d_passed, n, cudaMemcpyDeviceToHost, c->stream));
+        if (avg_sum && r->d_avg_sum) CUDA_TRY(c, cudaMemcpyAsync(avg_sum, r->d_avg_sum, n * 8, cudaMemcpyDeviceToHost, c->stream));
+        if (avg_cnt && r->d_avg_cnt) CUDA_TRY(c, cudaMemcpyAsync(avg_cnt, r->d_avg_cnt, n * 8, cudaMemcpyDeviceToHost, c->stream));
+    }
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_set_profiling(nestgpu_ctx *c, int32_t on)
+{
+    if (!c) return NESTGPU_ERR_INVALID;
+    c->profiling = on != 0;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_last_profile(const nestgpu_ctx *c, float *ms, int32_t n)
+{
+    if (!c || !ms) return NESTGPU_ERR_INVALID;
+    cudaSetDevice(c->device);
+    for (int s = 0; s < n && s < NESTGPU_N_STAGES; s++) {
+        ms[s] = NAN;
+        if (c->profiling && c->ran[s]) {
+            float t;
+            if (cudaEventSynchronize(c->ev[s][1]) == cudaSuccess &&
+                cudaEventElapsedTime(&t, c->ev[s][0], c->ev[s][1]) == cudaSuccess)
+                ms[s] = t;
+        }
+    }
+    return NESTGPU_OK;
+}
+
+}  // extern "C"

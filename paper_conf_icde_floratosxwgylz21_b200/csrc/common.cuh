@@ -1,0 +1,189 @@
+// common.cuh -- device-side helpers shared by the nestgpu kernels (sm_100a).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace ng {
+
+constexpr int MAX_PREDS = 8;
+constexpr unsigned FULL = 0xffffffffu;
+
+enum Op : int { EQ = 0, NE = 1, LT = 2, LE = 3, GT = 4, GE = 5 };
+enum Agg : int { MIN = 0, MAX = 1, SUM = 2, COUNT = 3, AVG = 4, EXISTS = 5, NOT_EXISTS = 6 };
+
+// One local predicate ("Selection(op, col, value)"), col OP literal or
+// col OP col; widths 4 or 8 bytes (int32 / int64 storage).
+struct DevPred {
+    const void *col;
+    const uint8_t *valid;
+    const void *rhs;
+    const uint8_t *rhs_valid;
+    long long lit;
+    int op;
+    int w;
+    int rhs_w;
+    int pad_;
+};
+struct PredSet {
+    int n;
+    DevPred p[MAX_PREDS];
+};
+
+// Source of the correlated key: one column (int32 or int64 storage) or two
+// int32-storage columns packed into an order-preserving 64-bit code
+// (reading R9).
+struct KeySrc {
+    const void *c0;
+    const uint8_t *v0;
+    const void *c1;
+    const uint8_t *v1;
+    int w0;      // 4 or 8
+    int n_key;   // 1 or 2
+};
+
+struct ValSrc {
+    const void *c;     // nullptr: no payload
+    const uint8_t *v;  // validity (nullptr: NOT NULL)
+    int w;             // 4 or 8
+};
+
+__device__ __forceinline__ long long load_w(const void *c, int w, long long i)
+{
+    return w == 4 ? (long long)__ldg((const int *)c + i) : __ldg((const long long *)c + i);
+}
+
+template <typename T>
+__device__ __forceinline__ bool cmp_rt(T x, int op, T y)
+{
+    switch (op) {
+    case EQ: return x == y;
+    case NE: return x != y;
+    case LT: return x < y;
+    case LE: return x <= y;
+    case GT: return x > y;
+    default: return x >= y;
+    }
+}
+
+// Compile-time operator: outer.key OP inner.key (reading R8).
+template <int OP, typename T>
+__device__ __forceinline__ bool cmp_ct(T x, T y)
+{
+    if constexpr (OP == EQ) return x == y;
+    else if constexpr (OP == NE) return x != y;
+    else if constexpr (OP == LT) return x < y;
+    else if constexpr (OP == LE) return x <= y;
+    else if constexpr (OP == GT) return x > y;
+    else return x >= y;
+}
+
+// Conjunction of local predicates; NULL operands make a predicate not TRUE.
+__device__ __forceinline__ bool eval_preds(const PredSet &P, long long row)
+{
+    bool ok = true;
+    for (int k = 0; k < P.n; k++) {
+        const DevPred &p = P.p[k];
+        if (p.valid && !__ldg(p.valid + row)) return false;
+        long long x = load_w(p.col, p.w, row);
+        long long y = p.lit;
+        if (p.rhs) {
+            if (p.rhs_valid && !__ldg(p.rhs_valid + row)) return false;
+            y = load_w(p.rhs, p.rhs_w, row);
+        }
+        ok = ok && cmp_rt(x, p.op, y);
+    }
+    return ok;
+}
+
+// Order-preserving unsigned encodings of signed keys.
+__device__ __forceinline__ uint32_t enc32(int32_t k) { return (uint32_t)k ^ 0x80000000u; }
+__device__ __forceinline__ uint64_t enc64(long long k) { return (uint64_t)k ^ 0x8000000000000000ull; }
+
+template <typename K>
+__device__ __forceinline__ K encode_key(const KeySrc &ks, long long row, bool &valid)
+{
+    valid = !(ks.v0 && !__ldg(ks.v0 + row));
+    if constexpr (sizeof(K) == 4) {
+        return enc32(__ldg((const int *)ks.c0 + row));
+    } else {
+        if (ks.n_key == 2) {
+            valid = valid && !(ks.v1 && !__ldg(ks.v1 + row));
+            uint64_t hi = enc32(__ldg((const int *)ks.c0 + row));
+            uint64_t lo = enc32(__ldg((const int *)ks.c1 + row));
+            return (hi << 32) | lo;
+        }
+        return ks.w0 == 4 ? enc64((long long)__ldg((const int *)ks.c0 + row))
+                          : enc64(__ldg((const long long *)ks.c0 + row));
+    }
+}
+
+__device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31; }
+__device__ __forceinline__ unsigned lanemask_lt()
+{
+    unsigned m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+// Device-scope relaxed loads/stores for decoupled look-back status words.
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long *p)
+{
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed_u64(unsigned long long *p, unsigned long long v)
+{
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned ld_relaxed_u32(const unsigned *p)
+{
+    unsigned v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed_u32(unsigned *p, unsigned v)
+{
+    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// ---------------------------------------------------------------------------
+// Single-pass ordered compaction offsets with decoupled look-back (the
+// paper's "0-1 vector -> prefix-sum -> materialize", fused into one
+// pass).  Status word: bits 62-63 flag (1 = aggregate, 2 = inclusive), low 62
+// bits the count.  `status` must be zeroed before the launch.
+constexpr unsigned long long ST_AGG = 1ull << 62;
+constexpr unsigned long long ST_INC = 2ull << 62;
+constexpr unsigned long long ST_VAL = (1ull << 62) - 1;
+
+// Called by all threads of warp 0 of a CTA.  Publishes `tile_total` for
+// `tile` and returns (in every lane) the exclusive prefix of the tile.
+__device__ __forceinline__ unsigned long long lookback_warp(unsigned long long *status, long long tile,
+                                                            unsigned long long tile_total)
+{
+    const unsigned lane = lane_id();
+    if (tile == 0) {
+        if (lane == 0) st_relaxed_u64(status, ST_INC | tile_total);
+        return 0;
+    }
+    if (lane == 0) st_relaxed_u64(status + tile, ST_AGG | tile_total);
+    unsigned long long excl = 0;
+    long long pred = tile - 1 - (long long)lane;
+    while (true) {
+        unsigned long long s = pred >= 0 ? ld_relaxed_u64(status + pred) : ST_INC;
+        while (__any_sync(FULL, (s >> 62) == 0)) {
+            if ((s >> 62) == 0) s = ld_relaxed_u64(status + pred);
+        }
+        unsigned inc = __ballot_sync(FULL, (s >> 62) == 2);
+        int stop = inc ? __ffs(inc) - 1 : 31;
+        unsigned long long v = (int)lane <= stop ? (s & ST_VAL) : 0;
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+        excl += v;
+        if (inc) break;
+        pred -= 32;
+    }
+    if (lane == 0) st_relaxed_u64(status + tile, ST_INC | (excl + tile_total));
+    return excl;
+}
+
+}  // namespace ng

@@ -1,0 +1,81 @@
+// internal.h -- host-side declarations shared by the C-ABI implementation
+// (api.cpp) and the kernel launchers (k_*.cu).  Not part of the ABI.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "common.cuh"
+
+namespace ng {
+
+// Every launcher returns the cudaError_t of its launch(es) and bumps *launches
+// by the number of kernels it launched.
+
+// a2 / a3: filter rows [0, n) by `preds`, compact survivors in row order.
+//   out_ids    : int32 row ids of survivors (nullable)
+//   out_keys   : encoded keys (K = uint32 when kb == 4, uint64 when 8) (nullable)
+//   out_kvalid : 1 byte per survivor, key not NULL (nullable)
+//   out_vals   : payload (vb = 4 or 8 bytes; nullable)
+//   drop_null_key / drop_null_val : NULL key / payload rows do not survive
+//   hist       : if non-null, kb*256 uint32 digit histograms of the encoded
+//                survivor keys (for the radix sort), accumulated atomically
+//   extreme    : if non-null, [0] |= any survivor payload == max of its type,
+//                [1] |= any == min (for the MIN/MAX identity check)
+//   scratch    : tile status + counter, from filter_scratch_bytes(n)
+//   out_count  : int64 survivor count (device)
+size_t filter_scratch_bytes(long long n);
+cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, int kb,
+                          const ValSrc &val, int vb, int drop_null_key, int drop_null_val,
+                          int *out_ids, void *out_keys, uint8_t *out_kvalid, void *out_vals,
+                          unsigned *hist, unsigned *extreme, void *scratch, long long *out_count,
+                          cudaStream_t st, long long *launches);
+
+// a4: one stable LSD radix pass on 8-bit digit `shift/8` of the encoded keys.
+//   digit_base: 256 uint32 global exclusive offsets of the digit (device)
+size_t sort_scratch_bytes(long long n);
+cudaError_t launch_radix_pass(int kb, int vb, const void *kin, void *kout, const void *vin, void *vout,
+                              long long n, int shift, const unsigned *digit_base, void *scratch,
+                              cudaStream_t st, long long *launches);
+
+// Partial aggregates per R' tuple: acc (int64) + cnt (int64); identity init.
+cudaError_t launch_init_partials(long long n, int agg, long long *acc, long long *cnt, cudaStream_t st,
+                                 long long *launches);
+
+// a5 + a6: per R' tuple binary search of the sorted index and fold of the
+// qualifying range(s).  d_nrp: device count of R'.  Long ranges go to a
+// warp-per-range second kernel.
+size_t range_scratch_bytes(long long n_rp_max);
+cudaError_t launch_range_agg(int kb, int vb, int op, int agg, long long n_rp_max, const long long *d_nrp,
+                             const void *rkeys, const void *skeys, const void *svals, long long ns,
+                             long long *acc, long long *cnt, void *scratch, cudaStream_t st,
+                             long long *launches);
+
+// a7: tiled block-nested-loop over R' x S'.  d_nrp / d_nsp: device counts.
+size_t bnl_scratch_bytes();
+cudaError_t launch_bnl(int kb, int vb, int op, int agg, long long n_rp_max, const long long *d_nrp,
+                       const void *rkeys, long long ns_max, const long long *d_nsp, const void *skeys,
+                       const void *svals, const unsigned *extreme, long long *acc, long long *cnt,
+                       void *scratch, int num_sms, cudaStream_t st, long long *launches);
+
+// a8 + a9: aggregate finalize, outer comparison, ordered compaction.
+struct FinalizeArgs {
+    long long n_rp_max;
+    const long long *d_nrp;
+    const int *ids;          // R' row ids
+    const uint8_t *kvalid;   // R' key not NULL (nullable = all valid)
+    const long long *acc, *cnt;
+    const void *x_col;       // outer comparison column (nullable for EXISTS)
+    const uint8_t *x_valid;
+    int x_w;
+    int agg, outer_op;
+    long long a, b;
+    long long row_id_base;
+    int emit_all;
+    long long *out_ids, *out_vals, *out_sum, *out_cnt;  // sum/cnt: AVG only (nullable)
+    uint8_t *out_valid, *out_passed;
+    long long *out_count;
+    void *scratch;           // filter_scratch_bytes(n_rp_max)
+};
+cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *launches);
+
+}  // namespace ng

@@ -1,0 +1,318 @@
+// k_bnl.cuh -- a7: tiled block-nested-loop subquery kernel (non-equality
+// correlations and index-less plans).
+//
+// PAPER.md P:55 (§I): the nested method "iterat[es] all tuples of the
+// correlated columns from the outer query block and execut[es] the subquery
+// as many times as the number of the outer-loop tuples" -- O(|R'| x |S'|).
+// P:317 ("Vectorization"): evaluate many passed-in values in one kernel;
+// abstract P:31: "exploiting cache locality for loops".  The B200 design:
+//
+//  * persistent CTAs (grid = #SMs x occupancy) pull work units
+//    (R block of 2048 tuples) x (S' chunk) from an atomic counter;
+//  * each thread keeps RPT = 8 outer tuples' encoded keys and accumulators
+//    in registers, so every S' element read from shared memory is reused
+//    2048 times per CTA (the cache-locality loop);
+//  * S' (key, payload) tiles of 16 KB stream global -> shared through a
+//    4-stage ring of cp.async.bulk copies (TMA bulk engine, UBLKCP) completed
+//    on mbarriers by one elected thread; consumers read them with 128-bit
+//    broadcast LDS;
+//  * per (r, s) pair the work is one compare (ISETP) and one predicated
+//    combine (IMNMX / IADD3) on the integer ALU pipe -- the roofline of this
+//    kernel;
+//  * EXISTS stops streaming a unit once every tuple of the block has found a
+//    match (semi-join early exit);
+//  * partial aggregates of a unit are merged into per-tuple int64 partials
+//    with 64-bit atomics (MIN/MAX/ADD are associative and commutative on
+//    integers, so the merge order cannot change the result).
+#pragma once
+#include <type_traits>
+
+#include "internal.h"
+
+namespace ng {
+
+constexpr int B_THREADS = 256;
+constexpr int B_RPT = 8;
+constexpr int B_RBLOCK = B_THREADS * B_RPT;
+constexpr int B_STAGES = 4;
+constexpr int B_STAGE_BYTES = 16384;
+
+struct BnlArgs {
+    const long long *d_nrp;
+    const long long *d_nsp;
+    const void *rkeys;
+    const void *skeys;
+    const void *svals;
+    const unsigned *extreme;
+    long long *acc;
+    long long *cnt;
+    unsigned *unit_counter;
+    long long n_sc;
+    long long chunk;
+};
+
+template <typename K, int VB>
+struct BnlTile {
+    static constexpr int VSZ = VB;
+    // elements per stage, a multiple of 16 so every array stays 16-B aligned
+    static constexpr int TILE = (B_STAGE_BYTES / (int)(sizeof(K) + VSZ)) & ~15;
+    static constexpr int KBYTES = TILE * (int)sizeof(K);
+};
+
+__device__ __forceinline__ void mbar_init(unsigned long long *bar, unsigned count)
+{
+    unsigned a = (unsigned)__cvta_generic_to_shared(bar);
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long *bar, unsigned parity)
+{
+    unsigned a = (unsigned)__cvta_generic_to_shared(bar);
+    asm volatile(
+        "{\n\t.reg .pred P1;\n"
+        "NG_WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+        "@!P1 bra NG_WAIT_%=;\n}" ::"r"(a),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long *bar, unsigned bytes)
+{
+    unsigned a = (unsigned)__cvta_generic_to_shared(bar);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(a), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned bytes, unsigned long long *bar)
+{
+    unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+    unsigned b = (unsigned)__cvta_generic_to_shared(bar);
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(d),
+        "l"(src), "r"(bytes), "r"(b)
+        : "memory");
+}
+
+template <int AGG>
+struct AccKind {
+    static constexpr bool minmax = AGG == MIN || AGG == MAX;
+    static constexpr bool sum = AGG == SUM || AGG == AVG;
+    static constexpr bool count = AGG == COUNT;
+    static constexpr bool exists = AGG == EXISTS || AGG == NOT_EXISTS;
+};
+
+// One (r, s) pair: the whole nested-method inner step.
+template <int OP, int AGG, bool TRACK, typename K, typename V>
+__device__ __forceinline__ void pair_step(const K rk, const K sk, const V sv, V &mm, long long &sm, unsigned &c,
+                                          bool &found)
+{
+    const bool p = cmp_ct<OP>(rk, sk);
+    if constexpr (AccKind<AGG>::minmax) {
+        if (p) mm = (AGG == MIN) ? min(mm, sv) : max(mm, sv);
+        if constexpr (TRACK) found |= p;
+    } else if constexpr (AccKind<AGG>::sum) {
+        if (p) { sm += (long long)sv; c += 1; }
+    } else if constexpr (AccKind<AGG>::count) {
+        c += p ? 1u : 0u;
+    } else {
+        found |= p;
+    }
+}
+
+template <int OP, int AGG, bool TRACK, typename K, typename V, int VB>
+__device__ __forceinline__ void tile_full(const K *__restrict__ tk, const V *__restrict__ tv, const K (&rk)[B_RPT],
+                                          V (&mm)[B_RPT], long long (&sm)[B_RPT], unsigned (&c)[B_RPT],
+                                          bool (&found)[B_RPT])
+{
+    constexpr int TILE = BnlTile<K, VB>::TILE;
+    constexpr int KV = 16 / (int)sizeof(K);  // keys per 128-bit load
+#pragma unroll 2
+    for (int e = 0; e < TILE; e += KV) {
+        K kk[KV];
+        V vv[KV];
+        if constexpr (sizeof(K) == 4) {
+            const uint4 q = *reinterpret_cast<const uint4 *>(tk + e);
+            kk[0] = q.x; kk[1] = q.y; kk[2] = q.z; kk[3] = q.w;
+        } else {
+            const ulonglong2 q = *reinterpret_cast<const ulonglong2 *>(tk + e);
+            kk[0] = q.x; kk[1] = q.y;
+        }
+        if constexpr (VB == 4) {
+            if constexpr (KV == 4) {
+                const int4 q = *reinterpret_cast<const int4 *>(tv + e);
+                vv[0] = q.x; vv[1] = q.y; vv[2] = q.z; vv[3] = q.w;
+            } else {
+                const int2 q = *reinterpret_cast<const int2 *>(tv + e);
+                vv[0] = q.x; vv[1] = q.y;
+            }
+        } else if constexpr (VB == 8) {
+#pragma unroll
+            for (int q = 0; q < KV; q += 2) {
+                const longlong2 w = *reinterpret_cast<const longlong2 *>(tv + e + q);
+                vv[q] = w.x; vv[q + 1] = w.y;
+            }
+        } else {
+#pragma unroll
+            for (int q = 0; q < KV; q++) vv[q] = 0;
+        }
+#pragma unroll
+        for (int q = 0; q < KV; q++) {
+#pragma unroll
+            for (int i = 0; i < B_RPT; i++) pair_step<OP, AGG, TRACK>(rk[i], kk[q], vv[q], mm[i], sm[i], c[i], found[i]);
+        }
+    }
+}
+
+template <int OP, int AGG, bool TRACK, typename K, typename V, int VB>
+__device__ __forceinline__ void tile_part(const K *__restrict__ tk, const V *__restrict__ tv, int count,
+                                          const K (&rk)[B_RPT], V (&mm)[B_RPT], long long (&sm)[B_RPT],
+                                          unsigned (&c)[B_RPT], bool (&found)[B_RPT])
+{
+    for (int e = 0; e < count; e++) {
+        const K k = tk[e];
+        const V v = VB ? tv[e] : (V)0;
+#pragma unroll
+        for (int i = 0; i < B_RPT; i++) pair_step<OP, AGG, TRACK>(rk[i], k, v, mm[i], sm[i], c[i], found[i]);
+    }
+}
+
+template <typename K, int VB, int OP, int AGG>
+__global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
+{
+    using V = typename std::conditional<VB == 8, long long, int>::type;
+    constexpr int TILE = BnlTile<K, VB>::TILE;
+    constexpr int KBYTES = BnlTile<K, VB>::KBYTES;
+    constexpr V VMAX = VB == 8 ? (V)LLONG_MAX : (V)INT_MAX;
+    constexpr V VMIN = VB == 8 ? (V)LLONG_MIN : (V)INT_MIN;
+    constexpr V MM0 = AGG == MIN ? VMAX : VMIN;
+
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ __align__(8) unsigned long long full_bar[B_STAGES];
+    __shared__ long long s_unit;
+
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        for (int s = 0; s < B_STAGES; s++) mbar_init(&full_bar[s], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+
+    const long long nrp = *A.d_nrp, nsp = *A.d_nsp;
+    const long long n_rb = (nrp + B_RBLOCK - 1) / B_RBLOCK;
+    const long long n_units = n_rb * A.n_sc;
+    bool track = false;
+    if constexpr (AccKind<AGG>::minmax) track = A.extreme[AGG == MIN ? 0 : 1] != 0;
+    const K *rkeys = (const K *)A.rkeys;
+    const K *skeys = (const K *)A.skeys;
+    const V *svals = (const V *)A.svals;
+    unsigned g = 0;  // tiles consumed by this CTA so far (ring position / phase)
+
+    auto issue = [&](long long tile_start, long long s1, unsigned stage) {
+        const int cnt = (int)min((long long)TILE, s1 - tile_start);
+        const unsigned kb = ((unsigned)cnt * (unsigned)sizeof(K) + 15u) & ~15u;
+        const unsigned vb = VB ? (((unsigned)cnt * (unsigned)VB + 15u) & ~15u) : 0u;
+        unsigned char *base = smem + stage * B_STAGE_BYTES;
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        mbar_expect_tx(&full_bar[stage], kb + vb);
+        bulk_g2s(base, skeys + tile_start, kb, &full_bar[stage]);
+        if (VB) bulk_g2s(base + KBYTES, (const char *)svals + tile_start * VB, vb, &full_bar[stage]);
+    };
+
+    while (true) {
+        if (tid == 0) s_unit = (long long)atomicAdd(A.unit_counter, 1u);
+        __syncthreads();
+        const long long u = s_unit;
+        __syncthreads();
+        if (u >= n_units) break;
+        const long long sc = u / n_rb, rb = u - sc * n_rb;
+        const long long s0 = sc * A.chunk;
+        const long long s1 = min(nsp, s0 + A.chunk);
+        const int ntiles = s1 > s0 ? (int)((s1 - s0 + TILE - 1) / TILE) : 0;
+        if (ntiles == 0) continue;
+
+        K rk[B_RPT];
+        V mm[B_RPT];
+        long long sm[B_RPT];
+        unsigned c[B_RPT];
+        bool found[B_RPT];
+        const long long r0 = rb * B_RBLOCK + tid;
+#pragma unroll
+        for (int i = 0; i < B_RPT; i++) {
+            const long long r = r0 + (long long)i * B_THREADS;
+            rk[i] = r < nrp ? rkeys[r] : (K)0;
+            mm[i] = MM0;
+            sm[i] = 0;
+            c[i] = 0;
+            found[i] = false;
+        }
+        int issued = min(ntiles, B_STAGES);
+        if (tid == 0)
+            for (int t = 0; t < issued; t++) issue(s0 + (long long)t * TILE, s1, (g + t) % B_STAGES);
+        bool stop = false;
+        for (int t = 0; t < issued; t++) {
+            const unsigned stage = g % B_STAGES;
+            mbar_wait(&full_bar[stage], (g / B_STAGES) & 1u);
+            if (!stop) {
+                const unsigned char *base = smem + stage * B_STAGE_BYTES;
+                const K *tk = (const K *)base;
+                const V *tv = (const V *)(base + KBYTES);
+                const long long ts = s0 + (long long)t * TILE;
+                const int cnt = (int)min((long long)TILE, s1 - ts);
+                if (cnt == TILE) {
+                    if (track) tile_full<OP, AGG, true, K, V, VB>(tk, tv, rk, mm, sm, c, found);
+                    else tile_full<OP, AGG, false, K, V, VB>(tk, tv, rk, mm, sm, c, found);
+                } else {
+                    if (track) tile_part<OP, AGG, true, K, V, VB>(tk, tv, cnt, rk, mm, sm, c, found);
+                    else tile_part<OP, AGG, false, K, V, VB>(tk, tv, cnt, rk, mm, sm, c, found);
+                }
+            }
+            ++g;
+            if constexpr (AccKind<AGG>::exists) {
+                bool all = true;
+#pragma unroll
+                for (int i = 0; i < B_RPT; i++) all = all && (found[i] || r0 + (long long)i * B_THREADS >= nrp);
+                stop = __syncthreads_and(all) != 0;
+            } else {
+                __syncthreads();
+            }
+            if (!stop && t + B_STAGES < ntiles) {
+                if (tid == 0) issue(s0 + (long long)(t + B_STAGES) * TILE, s1, stage);
+                issued = t + B_STAGES + 1;
+            }
+        }
+        // merge this unit's partial aggregates
+#pragma unroll
+        for (int i = 0; i < B_RPT; i++) {
+            const long long r = r0 + (long long)i * B_THREADS;
+            if (r >= nrp) continue;
+            if constexpr (AccKind<AGG>::minmax) {
+                const bool f = track ? found[i] : (mm[i] != MM0);
+                if (f) {
+                    if (AGG == MIN) atomicMin(&A.acc[r], (long long)mm[i]);
+                    else atomicMax(&A.acc[r], (long long)mm[i]);
+                    A.cnt[r] = 1;
+                }
+            } else if constexpr (AccKind<AGG>::sum) {
+                if (c[i]) {
+                    atomicAdd((unsigned long long *)&A.acc[r], (unsigned long long)sm[i]);
+                    atomicAdd((unsigned long long *)&A.cnt[r], (unsigned long long)c[i]);
+                }
+            } else if constexpr (AccKind<AGG>::count) {
+                if (c[i]) atomicAdd((unsigned long long *)&A.cnt[r], (unsigned long long)c[i]);
+            } else {
+                if (found[i]) A.cnt[r] = 1;
+            }
+        }
+    }
+}
+
+// Host-side launchers, one per (key width, payload width) family, each in
+// its own translation unit (k_bnl_<key>_v<payload>.cu).
+#define NG_BNL_FAMILY_DECL(name) \
+    cudaError_t name(int op, int agg, const BnlArgs &a, long long n_rp_max, long long ns_max, void *scratch, \
+                     int num_sms, cudaStream_t st)
+NG_BNL_FAMILY_DECL(bnl_family_u32_v0);
+NG_BNL_FAMILY_DECL(bnl_family_u32_v4);
+NG_BNL_FAMILY_DECL(bnl_family_u32_v8);
+NG_BNL_FAMILY_DECL(bnl_family_u64_v0);
+NG_BNL_FAMILY_DECL(bnl_family_u64_v4);
+NG_BNL_FAMILY_DECL(bnl_family_u64_v8);
+
+}  // namespace ng

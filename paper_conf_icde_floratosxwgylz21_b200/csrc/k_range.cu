@@ -1,0 +1,218 @@
+// k_range.cu -- a5 + a6: the indexed, vectorised subquery.
+//
+// PAPER.md P:315 (§III-D "Indexing"): "locate a valid range of S.col1 by using
+// the binary search on the index and only scan a portion of table S";
+// P:317 ("Vectorization"): fuse the per-iteration kernels of many passed-in
+// values into one kernel.  One launch evaluates the subquery for every R'
+// tuple: each thread binary-searches the sorted S' keys for its tuple's
+// encoded key and derives the qualifying range(s) for the correlated operator
+// (S' ascending, N = |S'|, predicate r.key OP s.key):
+//     '='  [lb, ub)      '<'  [ub, N)     '<=' [lb, N)
+//     '>'  [0, lb)       '>=' [0, ub)     '!=' [0, lb) u [ub, N)
+// COUNT / EXISTS need only the range length; MIN/MAX/SUM/AVG fold the
+// co-sorted payload.  Short ranges are folded by the owning thread; long ones
+// are appended to a work list and folded warp-per-range with coalesced loads
+// and warp reductions (load balance for skewed / non-equality ranges).
+#include <type_traits>
+
+#include "internal.h"
+
+namespace ng {
+
+constexpr int R_THREADS = 256;
+constexpr int R_SHORT = 32;
+
+struct LongItem {
+    int r, lb, ub, pad;
+};
+
+size_t range_scratch_bytes(long long n_rp_max) { return 256 + (size_t)(n_rp_max > 0 ? n_rp_max : 1) * sizeof(LongItem); }
+
+template <typename K>
+__device__ __forceinline__ int lower_bound_g(const K *__restrict__ a, int lo, int hi, K k)
+{
+    while (lo < hi) {
+        int mid = (int)(((unsigned)lo + (unsigned)hi) >> 1);
+        if (__ldg(a + mid) < k) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+template <typename K>
+__device__ __forceinline__ int upper_bound_g(const K *__restrict__ a, int lo, int hi, K k)
+{
+    while (lo < hi) {
+        int mid = (int)(((unsigned)lo + (unsigned)hi) >> 1);
+        if (__ldg(a + mid) <= k) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+template <int OP>
+__device__ __forceinline__ void pieces(int lb, int ub, int N, int &a0, int &b0, int &a1, int &b1)
+{
+    a1 = b1 = 0;
+    if constexpr (OP == EQ) { a0 = lb; b0 = ub; }
+    else if constexpr (OP == LT) { a0 = ub; b0 = N; }
+    else if constexpr (OP == LE) { a0 = lb; b0 = N; }
+    else if constexpr (OP == GT) { a0 = 0; b0 = lb; }
+    else if constexpr (OP == GE) { a0 = 0; b0 = ub; }
+    else { a0 = 0; b0 = lb; a1 = ub; b1 = N; }
+}
+
+template <int AGG, typename V>
+__device__ __forceinline__ void fold(long long &acc, V v)
+{
+    if constexpr (AGG == MIN) acc = min(acc, (long long)v);
+    else if constexpr (AGG == MAX) acc = max(acc, (long long)v);
+    else acc += (long long)v;
+}
+
+template <typename K, int VB, int OP, int AGG>
+__global__ void __launch_bounds__(R_THREADS)
+range_short_kernel(const long long *__restrict__ d_nrp, const K *__restrict__ rkeys, const K *__restrict__ skeys,
+                   const void *__restrict__ svals_, int N, long long *__restrict__ acc, long long *__restrict__ cnt,
+                   LongItem *__restrict__ list, unsigned *__restrict__ list_n)
+{
+    using V = typename std::conditional<VB == 8, long long, int>::type;
+    const V *svals = (const V *)svals_;
+    const long long i = blockIdx.x * (long long)R_THREADS + threadIdx.x;
+    if (i >= *d_nrp) return;
+    const K k = rkeys[i];
+    int lb = 0, ub = 0;
+    if constexpr (OP == EQ || OP == NE) {
+        lb = lower_bound_g(skeys, 0, N, k);
+        ub = upper_bound_g(skeys, lb, N, k);
+    } else if constexpr (OP == LE || OP == GT) {
+        lb = lower_bound_g(skeys, 0, N, k);
+    } else {
+        ub = upper_bound_g(skeys, 0, N, k);
+    }
+    int a0, b0, a1, b1;
+    pieces<OP>(lb, ub, N, a0, b0, a1, b1);
+    const long long L = (long long)(b0 - a0) + (b1 - a1);
+    if constexpr (AGG == COUNT || AGG == EXISTS || AGG == NOT_EXISTS) {
+        cnt[i] = L;
+    } else {
+        if (L <= R_SHORT) {
+            long long a = AGG == MIN ? LLONG_MAX : (AGG == MAX ? LLONG_MIN : 0);
+            for (int s = a0; s < b0; s++) fold<AGG>(a, svals[s]);
+            for (int s = a1; s < b1; s++) fold<AGG>(a, svals[s]);
+            acc[i] = a;
+            cnt[i] = L;
+        } else {
+            unsigned slot = atomicAdd(list_n, 1u);
+            list[slot] = LongItem{(int)i, lb, ub, 0};
+        }
+    }
+}
+
+template <int AGG>
+__device__ __forceinline__ long long warp_reduce(long long a)
+{
+    for (int o = 16; o > 0; o >>= 1) {
+        long long b = __shfl_xor_sync(FULL, a, o);
+        if constexpr (AGG == MIN) a = min(a, b);
+        else if constexpr (AGG == MAX) a = max(a, b);
+        else a += b;
+    }
+    return a;
+}
+
+template <int VB, int OP, int AGG>
+__global__ void __launch_bounds__(R_THREADS)
+range_long_kernel(const void *__restrict__ svals_, int N, const LongItem *__restrict__ list,
+                  const unsigned *__restrict__ list_n, long long *__restrict__ acc, long long *__restrict__ cnt)
+{
+    using V = typename std::conditional<VB == 8, long long, int>::type;
+    const V *svals = (const V *)svals_;
+    const unsigned lane = threadIdx.x & 31;
+    const long long gw = (blockIdx.x * (long long)R_THREADS + threadIdx.x) >> 5;
+    const long long nw = ((long long)gridDim.x * R_THREADS) >> 5;
+    const long long items = *list_n;
+    for (long long it = gw; it < items; it += nw) {
+        const LongItem li = list[it];
+        int a0, b0, a1, b1;
+        pieces<OP>(li.lb, li.ub, N, a0, b0, a1, b1);
+        long long a = AGG == MIN ? LLONG_MAX : (AGG == MAX ? LLONG_MIN : 0);
+        for (int s = a0 + (int)lane; s < b0; s += 32) fold<AGG>(a, svals[s]);
+        for (int s = a1 + (int)lane; s < b1; s += 32) fold<AGG>(a, svals[s]);
+        a = warp_reduce<AGG>(a);
+        if (lane == 0) {
+            acc[li.r] = a;
+            cnt[li.r] = (long long)(b0 - a0) + (b1 - a1);
+        }
+    }
+}
+
+template <typename K, int VB, int OP, int AGG>
+static void launch_range_t(long long n_rp_max, const long long *d_nrp, const void *rkeys, const void *skeys,
+                           const void *svals, long long ns, long long *acc, long long *cnt, void *scratch,
+                           cudaStream_t st, long long *launches)
+{
+    unsigned *list_n = (unsigned *)scratch;
+    LongItem *list = (LongItem *)((char *)scratch + 256);
+    const unsigned blocks = (unsigned)((n_rp_max + R_THREADS - 1) / R_THREADS);
+    range_short_kernel<K, VB, OP, AGG><<<blocks, R_THREADS, 0, st>>>(d_nrp, (const K *)rkeys, (const K *)skeys,
+                                                                    svals, (int)ns, acc, cnt, list, list_n);
+    ++*launches;
+    if constexpr (AGG != COUNT && AGG != EXISTS && AGG != NOT_EXISTS) {
+        range_long_kernel<VB, OP, AGG><<<148 * 8, R_THREADS, 0, st>>>(svals, (int)ns, list, list_n, acc, cnt);
+        ++*launches;
+    }
+}
+
+template <typename K, int VB, int OP>
+static void dispatch_agg(int agg, long long n_rp_max, const long long *d_nrp, const void *rkeys, const void *skeys,
+                         const void *svals, long long ns, long long *acc, long long *cnt, void *scratch,
+                         cudaStream_t st, long long *launches)
+{
+#define NG_R(A) launch_range_t<K, VB, OP, A>(n_rp_max, d_nrp, rkeys, skeys, svals, ns, acc, cnt, scratch, st, launches)
+    switch (agg) {
+    case MIN: NG_R(MIN); break;
+    case MAX: NG_R(MAX); break;
+    case SUM: NG_R(SUM); break;
+    case AVG: NG_R(SUM); break;   // AVG = (sum, nn)
+    case COUNT: NG_R(COUNT); break;
+    default: NG_R(EXISTS); break; // EXISTS / NOT EXISTS: range length
+    }
+#undef NG_R
+}
+
+template <typename K, int VB>
+static void dispatch_op(int op, int agg, long long n_rp_max, const long long *d_nrp, const void *rkeys,
+                        const void *skeys, const void *svals, long long ns, long long *acc, long long *cnt,
+                        void *scratch, cudaStream_t st, long long *launches)
+{
+#define NG_O(O) dispatch_agg<K, VB, O>(agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, acc, cnt, scratch, st, launches)
+    switch (op) {
+    case EQ: NG_O(EQ); break;
+    case NE: NG_O(NE); break;
+    case LT: NG_O(LT); break;
+    case LE: NG_O(LE); break;
+    case GT: NG_O(GT); break;
+    default: NG_O(GE); break;
+    }
+#undef NG_O
+}
+
+cudaError_t launch_range_agg(int kb, int vb, int op, int agg, long long n_rp_max, const long long *d_nrp,
+                             const void *rkeys, const void *skeys, const void *svals, long long ns,
+                             long long *acc, long long *cnt, void *scratch, cudaStream_t st, long long *launches)
+{
+    if (n_rp_max <= 0) return cudaSuccess;
+    cudaError_t e = cudaMemsetAsync(scratch, 0, 256, st);
+    if (e != cudaSuccess) return e;
+    const bool noval = agg == COUNT || agg == EXISTS || agg == NOT_EXISTS;
+    if (kb == 4) {
+        if (noval || vb == 4) dispatch_op<uint32_t, 4>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, acc, cnt, scratch, st, launches);
+        else dispatch_op<uint32_t, 8>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, acc, cnt, scratch, st, launches);
+    } else {
+        if (noval || vb == 4) dispatch_op<uint64_t, 4>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, acc, cnt, scratch, st, launches);
+        else dispatch_op<uint64_t, 8>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, acc, cnt, scratch, st, launches);
+    }
+    return cudaGetLastError();
+}
+
+}  // namespace ng

@@ -1,0 +1,190 @@
+// k_sort.cu -- a4: index build = stable LSD radix sort of S' by the encoded
+// correlated key, carrying the aggregate payload.
+//
+// PAPER.md P:315 (§III-D "Indexing"): sort the correlated column
+// (O(N log N)) and keep "the sorted values and their original positions"
+// (O(2N)), then binary-search a valid range per passed-in value.  Here the
+// payload itself is carried through the sort instead of the positions, so the
+// per-tuple range scan of a6 reads contiguous memory.
+//
+// One kernel per 8-bit digit ("onesweep"): each 4096-key tile ranks its keys
+// with warp __match_any_sync (stable: warp-striped items, ranks in input
+// order), publishes per-digit tile counts, resolves its global per-digit
+// offset by decoupled look-back over preceding tiles (dynamic tile ids for
+// forward progress), reorders the tile in shared memory and writes each
+// digit run out coalesced.  Digit histograms come from the S' filter kernel
+// (fused), so a pass is exactly one read and one write of (key, payload);
+// digits whose histogram has a single bucket are skipped by the host.
+#include <type_traits>
+
+#include "internal.h"
+
+namespace ng {
+
+constexpr int S_THREADS = 256;
+constexpr int S_WARPS = S_THREADS / 32;
+constexpr int S_ITEMS = 16;
+constexpr int S_TILE = S_THREADS * S_ITEMS;
+constexpr unsigned D_AGG = 1u << 30, D_INC = 2u << 30, D_VAL = (1u << 30) - 1;
+
+size_t sort_scratch_bytes(long long n)
+{
+    long long tiles = (n + S_TILE - 1) / S_TILE;
+    return (size_t)tiles * 256 * 4 + 256;
+}
+
+template <typename K, int VB>
+__global__ void __launch_bounds__(S_THREADS)
+onesweep_kernel(const K *__restrict__ kin, K *__restrict__ kout, const void *__restrict__ vin_,
+                void *__restrict__ vout_, long long n, int shift, const unsigned *__restrict__ digit_base,
+                unsigned *__restrict__ status, unsigned *__restrict__ counter)
+{
+    using V = typename std::conditional<VB == 8, long long, int>::type;
+    const V *vin = (const V *)vin_;
+    V *vout = (V *)vout_;
+    extern __shared__ __align__(16) unsigned char smem[];
+    K *s_keys = (K *)smem;
+    V *s_vals = (V *)(smem + S_TILE * sizeof(K));
+    __shared__ unsigned s_whist[S_WARPS][256];
+    __shared__ unsigned s_tdig[256];
+    __shared__ unsigned s_gdig[256];
+    __shared__ unsigned s_wsum[S_WARPS];
+    __shared__ unsigned s_tile;
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    if (tid == 0) s_tile = atomicAdd(counter, 1u);
+    for (int i = tid; i < S_WARPS * 256; i += S_THREADS) (&s_whist[0][0])[i] = 0;
+    __syncthreads();
+    const long long tile = s_tile;
+    const long long base = tile * S_TILE;
+    const long long wbase = base + (long long)warp * 32 * S_ITEMS;
+
+    K key[S_ITEMS];
+    V val[S_ITEMS];
+    int dig[S_ITEMS];
+    unsigned rank[S_ITEMS];
+#pragma unroll
+    for (int j = 0; j < S_ITEMS; j++) {
+        const long long idx = wbase + j * 32 + lane;
+        const bool ok = idx < n;
+        key[j] = ok ? kin[idx] : (K)0;
+        if constexpr (VB > 0) val[j] = ok ? vin[idx] : (V)0;
+        dig[j] = ok ? (int)((key[j] >> shift) & 255) : 256;
+    }
+    const unsigned lt = lanemask_lt();
+#pragma unroll
+    for (int j = 0; j < S_ITEMS; j++) {
+        const unsigned peers = __match_any_sync(FULL, dig[j]);
+        const int leader = __ffs(peers) - 1;
+        unsigned b = 0;
+        if (lane == leader && dig[j] < 256) {
+            b = s_whist[warp][dig[j]];
+            s_whist[warp][dig[j]] = b + __popc(peers);
+        }
+        b = __shfl_sync(FULL, b, leader);
+        rank[j] = b + __popc(peers & lt);
+        __syncwarp();
+    }
+    __syncthreads();
+    // per digit (thread == digit): exclusive offsets across warps, tile count
+    const int d = tid;
+    unsigned cnt = 0;
+#pragma unroll
+    for (int w = 0; w < S_WARPS; w++) {
+        unsigned t = s_whist[w][d];
+        s_whist[w][d] = cnt;
+        cnt += t;
+    }
+    unsigned *my_status = status + tile * 256 + d;
+    if (tile == 0) st_relaxed_u32(my_status, D_INC | cnt);
+    else st_relaxed_u32(my_status, D_AGG | cnt);
+    // tile-local exclusive scan over digits
+    unsigned incl = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        unsigned t = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += t;
+    }
+    if (lane == 31) s_wsum[warp] = incl;
+    // decoupled look-back for digit d
+    unsigned excl = 0;
+    if (tile > 0) {
+        long long p = tile - 1;
+        while (true) {
+            unsigned s;
+            do { s = ld_relaxed_u32(status + p * 256 + d); } while ((s >> 30) == 0);
+            excl += s & D_VAL;
+            if ((s >> 30) == 2) break;
+            --p;
+        }
+        st_relaxed_u32(my_status, D_INC | (excl + cnt));
+    }
+    __syncthreads();
+    unsigned wpre = 0;
+    for (int w = 0; w < warp; w++) wpre += s_wsum[w];
+    s_tdig[d] = wpre + incl - cnt;
+    s_gdig[d] = digit_base[d] + excl;
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < S_ITEMS; j++) {
+        if (dig[j] < 256) {
+            const unsigned pos = s_tdig[dig[j]] + s_whist[warp][dig[j]] + rank[j];
+            s_keys[pos] = key[j];
+            if constexpr (VB > 0) s_vals[pos] = val[j];
+        }
+    }
+    __syncthreads();
+    const long long rem = n - base;
+    const int tile_n = rem < S_TILE ? (int)rem : S_TILE;
+    for (int p = tid; p < tile_n; p += S_THREADS) {
+        const K k = s_keys[p];
+        const int dd = (int)((k >> shift) & 255);
+        const long long dst = (long long)s_gdig[dd] + (p - (int)s_tdig[dd]);
+        kout[dst] = k;
+        if constexpr (VB > 0) vout[dst] = s_vals[p];
+    }
+}
+
+template <typename K, int VB>
+static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *vout, long long n, int shift,
+                            const unsigned *digit_base, void *scratch, cudaStream_t st)
+{
+    using V = typename std::conditional<VB == 8, long long, int>::type;
+    const long long tiles = (n + S_TILE - 1) / S_TILE;
+    const size_t smem = S_TILE * (sizeof(K) + (VB > 0 ? sizeof(V) : 0));
+    static bool attr_set = false;
+    if (!attr_set) {
+        cudaError_t e = cudaFuncSetAttribute(onesweep_kernel<K, VB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)smem);
+        if (e != cudaSuccess) return e;
+        attr_set = true;
+    }
+    cudaError_t e = cudaMemsetAsync(scratch, 0, sort_scratch_bytes(n), st);
+    if (e != cudaSuccess) return e;
+    onesweep_kernel<K, VB><<<(unsigned)tiles, S_THREADS, smem, st>>>(
+        (const K *)kin, (K *)kout, vin, vout, n, shift, digit_base, (unsigned *)((char *)scratch + 256),
+        (unsigned *)scratch);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_radix_pass(int kb, int vb, const void *kin, void *kout, const void *vin, void *vout,
+                              long long n, int shift, const unsigned *digit_base, void *scratch, cudaStream_t st,
+                              long long *launches)
+{
+    if (n <= 0) return cudaSuccess;
+    if (n >= (1ll << 30)) return cudaErrorInvalidValue;
+    cudaError_t e;
+    if (kb == 4) {
+        if (vb == 0) e = run_pass<uint32_t, 0>(kin, kout, vin, vout, n, shift, digit_base, scratch, st);
+        else if (vb == 4) e = run_pass<uint32_t, 4>(kin, kout, vin, vout, n, shift, digit_base, scratch, st);
+        else e = run_pass<uint32_t, 8>(kin, kout, vin, vout, n, shift, digit_base, scratch, st);
+    } else {
+        if (vb == 0) e = run_pass<uint64_t, 0>(kin, kout, vin, vout, n, shift, digit_base, scratch, st);
+        else if (vb == 4) e = run_pass<uint64_t, 4>(kin, kout, vin, vout, n, shift, digit_base, scratch, st);
+        else e = run_pass<uint64_t, 8>(kin, kout, vin, vout, n, shift, digit_base, scratch, st);
+    }
+    ++*launches;
+    return e;
+}
+
+}  // namespace ng

@@ -1,0 +1,273 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle,
+element by element, on the same seeded inputs.  Integer work -> bit-exact.
+
+Covers both subquery kernels (index path: sort + binary search + range
+aggregate; nested-loop path: tiled BNL) for every correlated operator and
+aggregate, NULLs and empty subqueries, local predicates, composite keys,
+64-bit keys / payloads, extreme values, ragged sizes spanning many tiles,
+the BASELINE configs (C1 full; C2 full with sampled oracle rows; C5-shaped),
+and the ABI's error paths.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from datagen import make_plan, PLAN_OPS, query1
+from tests import independent as ind
+from tests.gpu_helpers import run, assert_parity, make_engine
+
+pytestmark = pytest.mark.gpu
+
+AGGS = ("min", "max", "sum", "count", "avg", "exists", "not_exists")
+MODES = ("bnl", "index")
+
+
+@pytest.fixture(scope="module")
+def eng():
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    e = make_engine(16)
+    yield e
+    e.close()
+
+
+# ------------------------------------------------------------------ C1
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("corr_op", PLAN_OPS)
+def test_c1_all_aggs(eng, mode, corr_op):
+    t = query1.config("C1")
+    for agg in AGGS:
+        for outer_op in (("=",) if agg in ("exists", "not_exists") else ("=", "<", ">=")):
+            plan = make_plan(corr_op, agg, outer_op)
+            ref = oracle.evaluate(t, plan)
+            assert_parity(run(eng, t, plan, mode, emit_all=True), ref, plan, True, ctx=(mode, corr_op, agg, outer_op))
+            assert_parity(run(eng, t, plan, mode, emit_all=False), ref, plan, False, ctx=(mode, corr_op, agg, outer_op))
+
+
+# ------------------------------------------------------------------ NULLs, predicates, ragged
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("seed", [1, 2])
+def test_nulls_predicates_ragged(eng, mode, seed):
+    # |R| = 9001 and |S| = 13007 span several 4096-row filter tiles and
+    # 2048-element BNL tiles / R blocks with ragged tails.
+    t = query1.random_small(seed, n_r=9001, n_s=13007, key_hi=3000, val_lo=-50, val_hi=50, null_frac=0.1)
+    for corr_op in PLAN_OPS:
+        for agg in AGGS:
+            plan = make_plan(corr_op, agg, PLAN_OPS[(seed + len(agg)) % 6],
+                             outer_preds=[{"col": "col3", "op": "<=", "lit": 1}],
+                             inner_preds=[{"col": "col3", "op": "!=", "rhs": "col2"}],
+                             lhs_mult=2, rhs_mult=3)
+            ref = oracle.evaluate(t, plan)
+            assert_parity(run(eng, t, plan, mode, emit_all=True), ref, plan, True, ctx=(mode, corr_op, agg))
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_composite_key(eng, mode):
+    t = query1.random_small(5, n_r=7000, n_s=11000, key_hi=40, null_frac=0.05)
+    for agg in AGGS:
+        plan = make_plan("=", agg, "<=", outer_key=["col1", "col3"], inner_key=["col1", "col3"])
+        ref = oracle.evaluate(t, plan)
+        assert_parity(run(eng, t, plan, mode, emit_all=True), ref, plan, True, ctx=(mode, agg))
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_int64_keys_and_payloads(eng, mode):
+    rng = np.random.default_rng(8)
+    n_r, n_s = 5000, 9000
+    keys = rng.integers(-2 ** 40, 2 ** 40, size=600)
+    t = {"R": {"k": rng.choice(keys, n_r), "x": rng.integers(-10 ** 12, 10 ** 12, n_r)},
+         "S": {"k": rng.choice(keys, n_s), "v": rng.integers(-10 ** 12, 10 ** 12, n_s)}}
+    t["R"]["k"][:50] = rng.integers(-2 ** 62, 2 ** 62, 50)  # some keys absent from S
+    for corr_op in PLAN_OPS:
+        for agg in AGGS:
+            plan = make_plan(corr_op, agg, "<", outer_key=["k"], inner_key=["k"], agg_col="v", outer_cmp_col="x")
+            ref = oracle.evaluate(t, plan)
+            assert_parity(run(eng, t, plan, mode, emit_all=True), ref, plan, True, ctx=(mode, corr_op, agg))
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_mixed_key_widths(eng, mode):
+    # int32 outer key against int64 inner key (and decimals as int64)
+    rng = np.random.default_rng(9)
+    t = {"R": {"k": rng.integers(-100, 100, 3000).astype(np.int32), "x": rng.integers(0, 300, 3000)},
+         "S": {"k": rng.integers(-100, 100, 4000).astype(np.int64), "v": rng.integers(-500, 500, 4000)}}
+    for corr_op in ("=", "<", "!="):
+        for agg in ("min", "avg", "count"):
+            plan = make_plan(corr_op, agg, ">", outer_key=["k"], inner_key=["k"], agg_col="v", outer_cmp_col="x")
+            ref = oracle.evaluate(t, plan)
+            assert_parity(run(eng, t, plan, mode, emit_all=True,
+                              dtypes={"S": {"v": "decimal"}}), ref, plan, True, ctx=(mode, corr_op, agg))
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_extreme_values(eng, mode):
+    # INT32_MIN / INT32_MAX keys and payloads: exercises the order-preserving
+    # key encoding and the MIN/MAX identity tracking (payload == identity).
+    i32 = np.iinfo(np.int32)
+    rng = np.random.default_rng(10)
+    dom = np.array([i32.min, i32.min + 1, -1, 0, 1, i32.max - 1, i32.max], np.int32)
+    t = {"R": {"col1": rng.choice(dom, 3000), "col2": rng.choice(dom, 3000)},
+         "S": {"col1": rng.choice(dom, 5000), "col2": rng.choice(dom, 5000)}}
+    for corr_op in PLAN_OPS:
+        for agg in AGGS:
+            plan = make_plan(corr_op, agg, "=")
+            ref = oracle.evaluate(t, plan)
+            assert_parity(run(eng, t, plan, mode, emit_all=True), ref, plan, True, ctx=(mode, corr_op, agg))
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_degenerate(eng, mode):
+    e32 = np.zeros(0, np.int32)
+    one = np.array([3], np.int32)
+    cases = {
+        "empty_R": {"R": {"col1": e32, "col2": e32}, "S": {"col1": one, "col2": one}},
+        "empty_S": {"R": {"col1": one, "col2": np.array([0], np.int32)}, "S": {"col1": e32, "col2": e32}},
+        "single": {"R": {"col1": one, "col2": one}, "S": {"col1": one, "col2": one}},
+        "all_null_keys": {"R": {"col1": np.arange(100, dtype=np.int32), "col2": np.zeros(100, np.int32)},
+                          "R_valid": {"col1": np.zeros(100, np.uint8)},
+                          "S": {"col1": np.arange(50, dtype=np.int32), "col2": np.ones(50, np.int32)}},
+    }
+    for name, t in cases.items():
+        for corr_op in PLAN_OPS:
+            for agg in AGGS:
+                plan = make_plan(corr_op, agg, "=")
+                ref = oracle.evaluate(t, plan)
+                assert_parity(run(eng, t, plan, mode, emit_all=True), ref, plan, True, ctx=(name, mode, corr_op, agg))
+    # every outer row filtered out / every inner row filtered out
+    t = query1.config("C1")
+    for preds in ({"outer_preds": [{"col": "col2", "op": "<", "lit": -1}]},
+                  {"inner_preds": [{"col": "col2", "op": ">", "lit": 100}]}):
+        for agg in AGGS:
+            plan = make_plan(">", agg, "=", **preds)
+            ref = oracle.evaluate(t, plan)
+            assert_parity(run(eng, t, plan, mode, emit_all=True), ref, plan, True, ctx=(preds, agg))
+
+
+# ------------------------------------------------------------------ C2-shaped
+@pytest.mark.parametrize("zipf", [None, 1.0])
+def test_c2_shaped_reduced(eng, zipf):
+    """C2's distributions at 60,013 x 60,013: every row checked."""
+    t = query1.tables(n_r=60013, n_s=60013, key_hi=1 << 14, val_hi=16, seed=2, zipf=zipf)
+    for corr_op, agg in query1.C2_SWEEP:
+        plan = make_plan(corr_op, agg, "=")
+        ref = oracle.evaluate(t, plan)
+        modes = MODES if corr_op == "=" else ("bnl",)
+        for mode in modes:
+            assert_parity(run(eng, t, plan, mode, emit_all=True), ref, plan, True, ctx=(mode, corr_op, agg, zipf))
+            assert_parity(run(eng, t, plan, mode, emit_all=False), ref, plan, False, ctx=(mode, corr_op, agg, zipf))
+
+
+def test_c2_full_size(eng):
+    """BASELINE configs[1] at full size (|R|=|S|=1M), in the bench's launch
+    configuration ('=' on the index path, '<', '>', '!=' on the BNL path):
+    oracle on 1500 sampled rows, closed-form checker on every row."""
+    t = query1.config("C2")
+    rng = np.random.default_rng(0)
+    rows = np.unique(np.concatenate([[0, len(t["R"]["col1"]) - 1], rng.integers(0, len(t["R"]["col1"]), 1500)]))
+    for corr_op, agg in query1.C2_SWEEP:
+        plan = make_plan(corr_op, agg, "=")
+        mode = "index" if corr_op == "=" else "bnl"
+        g = run(eng, t, plan, mode, emit_all=True)
+        ref = oracle.evaluate(t, plan, rows=rows)
+        assert_parity(g, ref, plan, True, rows=rows, ctx=(corr_op, agg))
+        valid, value, _, _ = ind.closed_form(t["R"]["col1"], t["S"]["col1"], t["S"]["col2"], corr_op, agg)
+        assert np.array_equal(g["valid"].astype(bool), valid), (corr_op, agg)
+        assert np.array_equal(g["value"], value), (corr_op, agg)
+        s = run(eng, t, plan, mode, emit_all=False)
+        exp = np.nonzero(g["passed"])[0]
+        assert np.array_equal(s["row"], exp)
+
+
+def test_c5_shaped(eng):
+    """C5's distributions (keys U[0,2^31-1), values U[0,2^20)) with |S| = 16M
+    and |R| = 131,072: '>' min on the BNL path; oracle on sampled rows plus
+    the closed form on every row."""
+    t = query1.config("C5", n_r=131072)
+    rows = np.unique(np.random.default_rng(1).integers(0, 131072, 300))
+    for agg in ("min", "count"):
+        plan = make_plan(">", agg, "=")
+        g = run(eng, t, plan, "bnl", emit_all=True)
+        ref = oracle.evaluate(t, plan, rows=rows)
+        assert_parity(g, ref, plan, True, rows=rows, ctx=agg)
+        valid, value, _, _ = ind.closed_form(t["R"]["col1"], t["S"]["col1"], t["S"]["col2"], ">", agg)
+        assert np.array_equal(g["value"], value)
+        assert np.array_equal(g["valid"].astype(bool), valid)
+
+
+# ------------------------------------------------------------------ index content
+def test_index_is_stable_sort(eng):
+    import torch
+    rng = np.random.default_rng(4)
+    n = 300007
+    k = rng.integers(-2 ** 31, 2 ** 31, n, dtype=np.int64).astype(np.int32)
+    k[::3] = 7  # many duplicates: stability shows in the payload order
+    v = np.arange(n, dtype=np.int32)
+    m = eng.mark()
+    try:
+        S = eng.load_table({"k": k, "v": v})
+        ix = eng.build_index(S, ["k"], "v")
+        info = eng.index_info(ix)
+        assert info["n"] == n and info["key_bytes"] == 4 and info["payload_bytes"] == 4
+        keys = eng.arena_view(info["d_keys"], n * 4).view(torch.int32).cpu().numpy().view(np.uint32)
+        pay = eng.arena_view(info["d_payload"], n * 4).view(torch.int32).cpu().numpy()
+        order = np.argsort(k, kind="stable")
+        assert np.array_equal(keys, k[order].view(np.uint32) ^ np.uint32(0x80000000))
+        assert np.array_equal(pay, v[order])
+    finally:
+        eng.release(m)
+
+
+# ------------------------------------------------------------------ errors
+def test_error_paths(eng):
+    from paper_conf_icde_floratosxwgylz21_b200 import NestGPUError, Engine
+    t = query1.config("C1")
+    m = eng.mark()
+    try:
+        R, S = eng.load_table(t["R"]), eng.load_table(t["S"])
+        bad = dict(make_plan("<", "min", "="), outer_key=["col1", "col2"], inner_key=["col1", "col2"])
+        with pytest.raises(NestGPUError) as ei:
+            eng.exec(bad, R, S)
+        assert ei.value.code == -4  # composite non-equality: UNSUPPORTED
+        with pytest.raises(NestGPUError) as ei:
+            eng.exec(make_plan("=", "min", "=", lhs_mult=0), R, S)
+        assert ei.value.code == -1
+        ix = eng.build_index(S, ["col1"], "col2")
+        with pytest.raises(NestGPUError) as ei:
+            eng.exec(make_plan("=", "min", "=", inner_preds=[{"col": "col2", "op": ">", "lit": 3}]), R, S, index=ix)
+        assert ei.value.code == -1  # index built with other inner predicates
+        res = eng.exec(make_plan("=", "count", "="), R, S, index=ix, emit_all=True)
+        import ctypes
+        buf = np.empty(1, np.int64)
+        st = eng.lib.nestgpu_result_to_host(eng.ctx, ctypes.byref(res), ctypes.c_void_p(buf.ctypes.data),
+                                            None, None, None, None, None, 1)
+        assert st == -7  # BUFFER
+        big = {"k": np.zeros(4, np.int64), "v": np.full(4, 2 ** 62, np.int64)}
+        S2 = eng.load_table(big, dtypes={"v": "decimal"})
+        R2 = eng.load_table({"k": np.zeros(2, np.int64), "x": np.zeros(2, np.int64)})
+        with pytest.raises(NestGPUError) as ei:
+            eng.exec(make_plan("=", "sum", "=", outer_key=["k"], inner_key=["k"], agg_col="v", outer_cmp_col="x"), R2, S2)
+        assert ei.value.code == -5  # OVERFLOW pre-check
+    finally:
+        eng.release(m)
+    small = Engine(0, arena_bytes=1 << 20)
+    with pytest.raises(NestGPUError) as ei:
+        small.load_column(np.zeros(1 << 20, np.int32))
+    assert ei.value.code == -2  # OOM
+    small.close()
+
+
+def test_launch_count_and_profile(eng):
+    t = query1.config("C1")
+    m = eng.mark()
+    try:
+        R, S = eng.load_table(t["R"]), eng.load_table(t["S"])
+        eng.set_profiling(True)
+        before = eng.launch_count()
+        eng.exec(make_plan(">", "min", "="), R, S)
+        assert eng.launch_count() - before >= 4  # R' filter, S' filter, init, BNL, finalize
+        prof = eng.last_profile()
+        assert prof["subquery"] > 0 and prof["total"] >= prof["subquery"]
+        eng.set_profiling(False)
+    finally:
+        eng.release(m)
