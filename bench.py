@@ -165,6 +165,49 @@ def ncu_traffic(workload_name):
         return None
 
 
+# Pipe-bound pair rate of each nested-loop variant (pairs / clk / SM), from its
+# SASS: MIN/MAX issue ISETP + predicated VIMNMX, both on
+# the ALU pipe (64 lanes/clk/SM) -> 32 pairs/clk; COUNT issues ISETP (ALU) +
+# predicated IMAD (FMA-heavy, 64 lanes/clk/SM) -> 64 pairs/clk.
+PAIRS_PER_SM_CLK = {"min": 32.0, "max": 32.0, "count": 64.0}
+OPS_PER_PAIR = 2.0   # algorithmic: one compare + one combine per (r, s) pair
+
+
+def bnl_roofline(profs, n_r, n_s, sm_max_mhz, workload_name):
+    """Aggregate roofline of the nested-loop kernel over the timed launches:
+    frac = sum(pipe-bound time) / sum(measured time), per-launch times from
+    CUDA events on the engine stream around the kernel."""
+    t_act = t_ideal = ops = 0.0
+    per = {}
+    for plan, mode, prof in profs:
+        agg = plan["agg"]
+        if mode != "bnl" or agg not in PAIRS_PER_SM_CLK:
+            continue
+        pairs = float(n_r) * n_s
+        ideal = pairs / (148 * PAIRS_PER_SM_CLK[agg] * sm_max_mhz * 1e6)
+        act = prof["subquery"] / 1000.0
+        t_act += act
+        t_ideal += ideal
+        ops += OPS_PER_PAIR * pairs
+        d = per.setdefault(agg, {"launches": 0, "ms": 0.0, "ideal_ms": 0.0})
+        d["launches"] += 1
+        d["ms"] += act * 1000
+        d["ideal_ms"] += ideal * 1000
+    if not t_act:
+        return None
+    for d in per.values():
+        d["frac"] = d["ideal_ms"] / d["ms"]
+        d["ms_per_launch"] = d["ms"] / d["launches"]
+    return {"bound": "alu", "achieved": ops / t_act / 1e12, "peak": ops / t_ideal / 1e12, "unit": "Tops/s",
+            "frac": t_ideal / t_act, "traffic": ncu_traffic(workload_name),
+            "kernel": "bnl_kernel (tiled block-nested loop), MIN and COUNT launches",
+            "algorithmic": "2 integer ops (compare + combine) per (r,s) pair x |R'| x |S'| per launch",
+            "peak_source": ("integer pipes: 148 SMs x %.0f MHz (sm_max_mhz, MEASURED_PEAKS.json) x "
+                            "ALU 64 lanes/clk (MIN: 2 ALU ops/pair) | ALU+FMA-heavy 64 lanes/clk each "
+                            "(COUNT: 1+1 ops/pair); B300_MICROARCH pipe rates" % sm_max_mhz),
+            "per_agg": per}
+
+
 def peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -308,28 +351,7 @@ def main():
     # ---- dominant kernel: the nested loop (min / count plans; EXISTS stops early)
     pk = peaks()
     sm_max = pk.get("sm_max_mhz") or clocks.summary().get("sm_max_mhz") or 1965.0
-    alu_peak = 148 * ALU_LANES_PER_SM_CLK * sm_max * 1e6 / 1e12   # T lane-ops/s
-    bnl_ms, bnl_ops, bnl_launch = 0.0, 0.0, 0
-    stages = {}
-    for plan, mode, prof in profs:
-        for k, v in prof.items():
-            if v == v:  # not NaN
-                stages[k] = stages.get(k, 0.0) + v / args.steps
-        if mode == "bnl" and plan["agg"] in ("min", "count"):
-            bnl_ms += prof["subquery"]
-            bnl_ops += 2.0 * n_r * n_s          # ISETP + predicated IMNMX / IADD3 per (r, s) pair
-            bnl_launch += 1
-    roofline = None
-    if bnl_launch:
-        achieved = bnl_ops / (bnl_ms / 1000.0) / 1e12
-        roofline = {"bound": "alu", "achieved": achieved, "peak": alu_peak, "unit": "Tops/s",
-                    "frac": achieved / alu_peak, "traffic": ncu_traffic(args.workload),
-                    "kernel": "bnl_kernel (tiled block-nested loop)",
-                    "per_launch_ms": bnl_ms / bnl_launch,
-                    "algorithmic": "2 int ALU ops per (r,s) pair x |R'| x |S'| per launch",
-                    "peak_source": "148 SMs x 64 ALU lanes/clk x %.0f MHz (sm_max_mhz, MEASURED_PEAKS.json)" % sm_max}
-    else:  # index-only workload (C1 '=' ...): report the HBM view of the whole step
-        roofline = None
+    roofline = bnl_roofline(profs, n_r, n_s, sm_max, args.workload)
 
     # ---- e2e through the public API with host buffers
     e2e = None

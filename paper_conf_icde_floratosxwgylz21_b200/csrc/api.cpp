@@ -434,8 +434,8 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     long long *d_count = (long long *)(hist + 8 * 256);
     CUDA_TRY(c, cudaMemsetAsync(hist, 0, 8 * 256 * 4, c->stream));
     prof_begin(c, 1);
-    CUDA_TRY(c, ng::launch_filter(n, ps, ks, kb, vs, vb, 1, pc ? 1 : 0, nullptr, tk, nullptr, tv, hist, nullptr, fscr,
-                                  d_count, c->stream, &c->launches));
+    CUDA_TRY(c, ng::launch_filter(n, ps, ks, kb, vs, vb, 1, pc ? 1 : 0, nullptr, tk, nullptr, tv, hist, nullptr,
+                                  fscr, d_count, c->stream, &c->launches));
     prof_end(c, 1);
     CUDA_TRY(c, cudaMemcpyAsync(c->pinned, hist, kb * 256 * 4, cudaMemcpyDeviceToHost, c->stream));
     CUDA_TRY(c, cudaMemcpyAsync(c->pinned + 8 * 256, d_count, 8, cudaMemcpyDeviceToHost, c->stream));
@@ -658,7 +658,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     long long *counts = (long long *)salloc(c, 64);  // [0] |R'| [1] |S'| [2] survivors; [4..5] extreme
     size_t fsz = ng::filter_scratch_bytes(nR > nS ? nR : nS);
     void *fscr = salloc(c, fsz);
-    void *kscr = salloc(c, ix ? ng::range_scratch_bytes(nR) : ng::bnl_scratch_bytes());
+    void *kscr = salloc(c, ix ? ng::range_scratch_bytes(nR) : ng::bnl_scratch_bytes(nR));
     long long *o_ids = (long long *)salloc(c, (size_t)nR * 8);
     long long *o_vals = (long long *)salloc(c, (size_t)nR * 8);
     uint8_t *o_valid = (uint8_t *)salloc(c, (size_t)nR);
@@ -673,7 +673,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     if (!ids || !rkeys || (ravalid && !rkvalid) || !acc || !cnt || !counts || !fscr || !kscr || !o_ids || !o_vals ||
         !o_valid || !o_pass || (P->agg == NG_AVG && (!o_sum || !o_cnt)) || (!ix && (!skeys || (vb && !svals))))
         return fail(c, NESTGPU_ERR_OOM, "arena exhausted executing a plan over |R|=%lld |S|=%lld", (long long)nR, (long long)nS);
-    unsigned *extreme = (unsigned *)(counts + 4);
+    unsigned *extreme = (unsigned *)(counts + 4);   // [2]
     long long *d_nrp = counts, *d_nsp = counts + 1, *d_out = counts + 2;
 
     // ------------------------------------------------------------ a2: R'
@@ -681,8 +681,8 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     prof_begin(c, 0);
     ng::ValSrc none{nullptr, nullptr, 0};
     CUDA_TRY(c, cudaMemsetAsync(counts, 0, 64, c->stream));
-    CUDA_TRY(c, ng::launch_filter(nR, ops, rks, kb, none, 0, 0, 0, ids, rkeys, rkvalid, nullptr, nullptr, nullptr, fscr,
-                                  d_nrp, c->stream, &c->launches));
+    CUDA_TRY(c, ng::launch_filter(nR, ops, rks, kb, none, 0, 0, 0, ids, rkeys, rkvalid, nullptr, nullptr, nullptr,
+                                  fscr, d_nrp, c->stream, &c->launches));
     prof_end(c, 0);
 
     // ------------------------------------------------------------ a3 / a5-a7
@@ -696,7 +696,8 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         ng::ValSrc vs{nullptr, nullptr, 0};
         if (value_agg) { vs.c = ac->d; vs.v = ac->valid; vs.w = vb; }
         CUDA_TRY(c, ng::launch_filter(nS, ips, sks, kb, vs, vb, 1, value_agg ? 1 : 0, nullptr, skeys, nullptr, svals,
-                                      nullptr, value_agg ? extreme : nullptr, fscr, d_nsp, c->stream, &c->launches));
+                                      nullptr, value_agg ? extreme : nullptr, fscr, d_nsp, c->stream,
+                                      &c->launches));
         CUDA_TRY(c, ng::launch_init_partials(nR, P->agg, acc, cnt, c->stream, &c->launches));
         prof_end(c, 1);
         prof_begin(c, 3);

@@ -27,8 +27,8 @@ size_t filter_scratch_bytes(long long n);
 cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, int kb,
                           const ValSrc &val, int vb, int drop_null_key, int drop_null_val,
                           int *out_ids, void *out_keys, uint8_t *out_kvalid, void *out_vals,
-                          unsigned *hist, unsigned *extreme, void *scratch, long long *out_count,
-                          cudaStream_t st, long long *launches);
+                          unsigned *hist, unsigned *extreme, void *scratch,
+                          long long *out_count, cudaStream_t st, long long *launches);
 
 // a4: one stable LSD radix pass on 8-bit digit `shift/8` of the encoded keys.
 //   digit_base: 256 uint32 global exclusive offsets of the digit (device)
@@ -51,7 +51,7 @@ cudaError_t launch_range_agg(int kb, int vb, int op, int agg, long long n_rp_max
                              long long *launches);
 
 // a7: tiled block-nested-loop over R' x S'.  d_nrp / d_nsp: device counts.
-size_t bnl_scratch_bytes();
+size_t bnl_scratch_bytes(long long n_rp_max);
 cudaError_t launch_bnl(int kb, int vb, int op, int agg, long long n_rp_max, const long long *d_nrp,
                        const void *rkeys, long long ns_max, const long long *d_nsp, const void *skeys,
                        const void *svals, const unsigned *extreme, long long *acc, long long *cnt,

@@ -3,7 +3,7 @@
 
 namespace ng {
 
-size_t bnl_scratch_bytes() { return 256; }
+size_t bnl_scratch_bytes(long long n_rp_max) { return 256 + (size_t)((n_rp_max + B_RBLOCK - 1) / B_RBLOCK + 1) * 4; }
 
 cudaError_t launch_bnl(int kb, int vb, int op, int agg, long long n_rp_max, const long long *d_nrp, const void *rkeys,
                        long long ns_max, const long long *d_nsp, const void *skeys, const void *svals,
@@ -18,6 +18,7 @@ cudaError_t launch_bnl(int kb, int vb, int op, int agg, long long n_rp_max, cons
     a.skeys = skeys;
     a.svals = svals;
     a.extreme = extreme;
+    a.one = 1u;
     a.acc = acc;
     a.cnt = cnt;
     const bool noval = agg == COUNT || agg == EXISTS || agg == NOT_EXISTS;

@@ -44,9 +44,11 @@ struct BnlArgs {
     const void *skeys;
     const void *svals;
     const unsigned *extreme;
+    unsigned one;              // runtime 1 (keeps the IMAD multiplier opaque to ptxas)
     long long *acc;
     long long *cnt;
     unsigned *unit_counter;
+    unsigned *rb_done;         // EXISTS: per R block, set once every tuple of the block found a match
     long long n_sc;
     long long chunk;
 };
@@ -98,28 +100,101 @@ struct AccKind {
     static constexpr bool exists = AGG == EXISTS || AGG == NOT_EXISTS;
 };
 
+// PTX spelling of the correlated operator (r.key OP s.key, reading R8).
+template <int OP>
+struct OpName;
+template <> struct OpName<EQ> { static constexpr const char *s = "eq"; };
+template <> struct OpName<NE> { static constexpr const char *s = "ne"; };
+template <> struct OpName<LT> { static constexpr const char *s = "lt"; };
+template <> struct OpName<LE> { static constexpr const char *s = "le"; };
+template <> struct OpName<GT> { static constexpr const char *s = "gt"; };
+template <> struct OpName<GE> { static constexpr const char *s = "ge"; };
+
+#define NG_SETP_U32(OPS) "setp." OPS ".u32 p, %1, %2;"
+#define NG_SETP_U64(OPS) "setp." OPS ".u64 p, %1, %2;"
+#define NG_SETP2_U32(OPS) "setp." OPS ".u32 p, %2, %3;"
+#define NG_SETP2_U64(OPS) "setp." OPS ".u64 p, %2, %3;"
+
+// c += (r OP s): one ISETP on the ALU pipe + one predicated IMAD (c = c*one +
+// one, `one` a runtime 1 so ptxas cannot turn it into an ALU add) on the FMA
+// pipe -- the two pipes split the pair's work evenly.
+template <int OP, typename K>
+__device__ __forceinline__ void count_if(const K rk, const K sk, unsigned &c, const unsigned one)
+{
+#define NG_CNT(OPS)                                                                                   \
+    if constexpr (sizeof(K) == 4)                                                                     \
+        asm("{.reg .pred p;\n\t" NG_SETP_U32(OPS) "\n\t@p mad.lo.u32 %0, %0, %3, %3;}"                \
+            : "+r"(c) : "r"((uint32_t)rk), "r"((uint32_t)sk), "r"(one));                              \
+    else                                                                                              \
+        asm("{.reg .pred p;\n\t" NG_SETP_U64(OPS) "\n\t@p mad.lo.u32 %0, %0, %3, %3;}"                \
+            : "+r"(c) : "l"((uint64_t)rk), "l"((uint64_t)sk), "r"(one));
+    if constexpr (OP == EQ) { NG_CNT("eq") } else if constexpr (OP == NE) { NG_CNT("ne") }
+    else if constexpr (OP == LT) { NG_CNT("lt") } else if constexpr (OP == LE) { NG_CNT("le") }
+    else if constexpr (OP == GT) { NG_CNT("gt") } else { NG_CNT("ge") }
+#undef NG_CNT
+}
+
+// c += (r OP s); sum += (r OP s) ? v : 0 -- ISETP + predicated IMAD (count)
+// + predicated IMAD.WIDE (sum = v*one + sum, 32-bit payload) on the FMA pipe;
+// 64-bit payloads add on the ALU pipe.
+#define NG_SUM_BODY(SETP, KCON, VADD, VCON)                                                           \
+    asm("{.reg .pred p;\n\t" SETP "\n\t@p mad.lo.u32 %0, %0, %4, %4;\n\t" VADD "}"                    \
+        : "+r"(c), "+l"(sm) : KCON((rk)), KCON((sk)), "r"(one), VCON(v));
+#define NG_K32(x) "r"((uint32_t)x)
+#define NG_K64(x) "l"((uint64_t)x)
+#define NG_V32(x) "r"((int)x)
+#define NG_V64(x) "l"((long long)x)
+#define NG_ADD32 "@p mad.wide.s32 %1, %5, %4, %1;"
+#define NG_ADD64 "@p add.s64 %1, %1, %5;"
+#define NG_SUM_OP(OPS)                                                                                \
+    if constexpr (sizeof(K) == 4 && sizeof(V) == 4) { NG_SUM_BODY(NG_SETP2_U32(OPS), NG_K32, NG_ADD32, NG_V32) } \
+    else if constexpr (sizeof(K) == 4) { NG_SUM_BODY(NG_SETP2_U32(OPS), NG_K32, NG_ADD64, NG_V64) }  \
+    else if constexpr (sizeof(V) == 4) { NG_SUM_BODY(NG_SETP2_U64(OPS), NG_K64, NG_ADD32, NG_V32) }  \
+    else { NG_SUM_BODY(NG_SETP2_U64(OPS), NG_K64, NG_ADD64, NG_V64) }
+template <int OP, typename K, typename V>
+__device__ __forceinline__ void sum_if(const K rk, const K sk, const V v, long long &sm, unsigned &c,
+                                       const unsigned one)
+{
+    if constexpr (OP == EQ) { NG_SUM_OP("eq") } else if constexpr (OP == NE) { NG_SUM_OP("ne") }
+    else if constexpr (OP == LT) { NG_SUM_OP("lt") } else if constexpr (OP == LE) { NG_SUM_OP("le") }
+    else if constexpr (OP == GT) { NG_SUM_OP("gt") } else { NG_SUM_OP("ge") }
+}
+#undef NG_SUM_OP
+#undef NG_ADD64
+#undef NG_ADD32
+#undef NG_V64
+#undef NG_V32
+#undef NG_K64
+#undef NG_K32
+#undef NG_SUM_BODY
+
 // One (r, s) pair: the whole nested-method inner step.
+//   MIN/MAX: ISETP + predicated IMNMX (both ALU pipe); with TRACK also
+//            "found" (only when some payload equals the MIN/MAX identity).
+//   COUNT:   ISETP (ALU) + predicated IMAD (FMA).
+//   SUM/AVG: ISETP (ALU) + predicated IMAD + IMAD.WIDE (FMA).
+//   EXISTS:  predicate OR.
 template <int OP, int AGG, bool TRACK, typename K, typename V>
 __device__ __forceinline__ void pair_step(const K rk, const K sk, const V sv, V &mm, long long &sm, unsigned &c,
-                                          bool &found)
+                                          bool &found, const unsigned one)
 {
-    const bool p = cmp_ct<OP>(rk, sk);
     if constexpr (AccKind<AGG>::minmax) {
+        const bool p = cmp_ct<OP>(rk, sk);
         if (p) mm = (AGG == MIN) ? min(mm, sv) : max(mm, sv);
         if constexpr (TRACK) found |= p;
     } else if constexpr (AccKind<AGG>::sum) {
-        if (p) { sm += (long long)sv; c += 1; }
+        sum_if<OP>(rk, sk, sv, sm, c, one);
     } else if constexpr (AccKind<AGG>::count) {
-        c += p ? 1u : 0u;
+        count_if<OP>(rk, sk, c, one);
     } else {
-        found |= p;
+        found |= cmp_ct<OP>(rk, sk);
     }
 }
 
 template <int OP, int AGG, bool TRACK, typename K, typename V, int VB>
 __device__ __forceinline__ void tile_full(const K *__restrict__ tk, const V *__restrict__ tv, const K (&rk)[B_RPT],
                                           V (&mm)[B_RPT], long long (&sm)[B_RPT], unsigned (&c)[B_RPT],
-                                          bool (&found)[B_RPT])
+                                          bool (&found)[B_RPT], const unsigned mul)
 {
     constexpr int TILE = BnlTile<K, VB>::TILE;
     constexpr int KV = 16 / (int)sizeof(K);  // keys per 128-bit load
@@ -155,7 +230,7 @@ __device__ __forceinline__ void tile_full(const K *__restrict__ tk, const V *__r
 #pragma unroll
         for (int q = 0; q < KV; q++) {
 #pragma unroll
-            for (int i = 0; i < B_RPT; i++) pair_step<OP, AGG, TRACK>(rk[i], kk[q], vv[q], mm[i], sm[i], c[i], found[i]);
+            for (int i = 0; i < B_RPT; i++) pair_step<OP, AGG, TRACK>(rk[i], kk[q], vv[q], mm[i], sm[i], c[i], found[i], mul);
         }
     }
 }
@@ -163,13 +238,13 @@ __device__ __forceinline__ void tile_full(const K *__restrict__ tk, const V *__r
 template <int OP, int AGG, bool TRACK, typename K, typename V, int VB>
 __device__ __forceinline__ void tile_part(const K *__restrict__ tk, const V *__restrict__ tv, int count,
                                           const K (&rk)[B_RPT], V (&mm)[B_RPT], long long (&sm)[B_RPT],
-                                          unsigned (&c)[B_RPT], bool (&found)[B_RPT])
+                                          unsigned (&c)[B_RPT], bool (&found)[B_RPT], const unsigned mul)
 {
     for (int e = 0; e < count; e++) {
         const K k = tk[e];
         const V v = VB ? tv[e] : (V)0;
 #pragma unroll
-        for (int i = 0; i < B_RPT; i++) pair_step<OP, AGG, TRACK>(rk[i], k, v, mm[i], sm[i], c[i], found[i]);
+        for (int i = 0; i < B_RPT; i++) pair_step<OP, AGG, TRACK>(rk[i], k, v, mm[i], sm[i], c[i], found[i], mul);
     }
 }
 
@@ -197,8 +272,11 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
     const long long nrp = *A.d_nrp, nsp = *A.d_nsp;
     const long long n_rb = (nrp + B_RBLOCK - 1) / B_RBLOCK;
     const long long n_units = n_rb * A.n_sc;
+    // MIN/MAX: if some S' payload equals the identity, track "found"
+    // explicitly (uniform per launch, flag from the S' filter kernel).
     bool track = false;
     if constexpr (AccKind<AGG>::minmax) track = A.extreme[AGG == MIN ? 0 : 1] != 0;
+    const unsigned mul = A.one;
     const K *rkeys = (const K *)A.rkeys;
     const K *skeys = (const K *)A.skeys;
     const V *svals = (const V *)A.svals;
@@ -226,6 +304,12 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
         const long long s1 = min(nsp, s0 + A.chunk);
         const int ntiles = s1 > s0 ? (int)((s1 - s0 + TILE - 1) / TILE) : 0;
         if (ntiles == 0) continue;
+        if constexpr (AccKind<AGG>::exists) {
+            // semi-join early exit across units: another S' chunk already
+            // satisfied every tuple of this R block (flag read by one thread,
+            // decision made uniform through the barrier)
+            if (__syncthreads_or(tid == 0 && ld_relaxed_u32(A.rb_done + rb) != 0)) continue;
+        }
 
         K rk[B_RPT];
         V mm[B_RPT];
@@ -256,11 +340,11 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
                 const long long ts = s0 + (long long)t * TILE;
                 const int cnt = (int)min((long long)TILE, s1 - ts);
                 if (cnt == TILE) {
-                    if (track) tile_full<OP, AGG, true, K, V, VB>(tk, tv, rk, mm, sm, c, found);
-                    else tile_full<OP, AGG, false, K, V, VB>(tk, tv, rk, mm, sm, c, found);
+                    if (track) tile_full<OP, AGG, true, K, V, VB>(tk, tv, rk, mm, sm, c, found, mul);
+                    else tile_full<OP, AGG, false, K, V, VB>(tk, tv, rk, mm, sm, c, found, mul);
                 } else {
-                    if (track) tile_part<OP, AGG, true, K, V, VB>(tk, tv, cnt, rk, mm, sm, c, found);
-                    else tile_part<OP, AGG, false, K, V, VB>(tk, tv, cnt, rk, mm, sm, c, found);
+                    if (track) tile_part<OP, AGG, true, K, V, VB>(tk, tv, cnt, rk, mm, sm, c, found, mul);
+                    else tile_part<OP, AGG, false, K, V, VB>(tk, tv, cnt, rk, mm, sm, c, found, mul);
                 }
             }
             ++g;
@@ -269,6 +353,7 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
 #pragma unroll
                 for (int i = 0; i < B_RPT; i++) all = all && (found[i] || r0 + (long long)i * B_THREADS >= nrp);
                 stop = __syncthreads_and(all) != 0;
+                if (stop && tid == 0) st_relaxed_u32(A.rb_done + rb, 1u);
             } else {
                 __syncthreads();
             }

@@ -163,8 +163,7 @@ filter_kernel(long long n, PredSet preds, KeySrc ks, ValSrc vs, int drop_null_ke
 
 cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, int kb, const ValSrc &val,
                           int vb, int drop_null_key, int drop_null_val, int *out_ids, void *out_keys,
-                          uint8_t *out_kvalid, void *out_vals, unsigned *hist, unsigned *extreme, void *scratch,
-                          long long *out_count, cudaStream_t st, long long *launches)
+                          uint8_t *out_kvalid, void *out_vals, unsigned *hist, unsigned *extreme, void *scratch, long long *out_count, cudaStream_t st, long long *launches)
 {
     cudaError_t e = cudaMemsetAsync(out_count, 0, sizeof(long long), st);
     if (e != cudaSuccess || n <= 0) return e;
