@@ -1,0 +1,128 @@
+"""GPU parity on the TPC-H-shaped configs (BASELINE.json configs[2], [3]):
+C3 = SF1 Q2 + Q17, C4 = SF10 Q4 + Q20, at full size, through the C ABI, on
+both subquery kernels (index path and tiled nested loop).
+
+Oracle: every R' row where |R'| x |S| is small enough (Q2, Q17), sampled R'
+rows otherwise (Q4, Q20); plus, at every row, the independent unnested
+checkers that hold for '=' (semi-join for EXISTS, GROUP BY for MIN / AVG /
+SUM -- Query 2's form)."""
+import numpy as np
+import pytest
+
+import oracle
+from datagen import tpch
+from tests.gpu_helpers import run, assert_parity, make_engine
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def eng():
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    e = make_engine(40)
+    yield e
+    e.close()
+
+
+@pytest.fixture(scope="module")
+def c3():
+    sf, _, seed = tpch.CONFIGS["C3"]
+    return tpch.base_tables(sf, seed)
+
+
+@pytest.fixture(scope="module")
+def c4():
+    sf, _, seed = tpch.CONFIGS["C4"]
+    return tpch.base_tables(sf, seed)
+
+
+def _outer_rows(tables, plan):
+    """R' row numbers (numpy evaluation of the outer local predicates; used
+    only to pick the oracle's sample)."""
+    R = tables["R"]
+    m = np.ones(len(next(iter(R.values()))), bool)
+    for p in plan["outer_preds"]:
+        rhs = R[p["rhs"]] if p.get("rhs") else p["lit"]
+        x = R[p["col"]]
+        m &= {"=": x == rhs, "!=": x != rhs, "<": x < rhs, "<=": x <= rhs, ">": x > rhs, ">=": x >= rhs}[p["op"]]
+    return np.nonzero(m)[0]
+
+
+def _inner_mask(tables, plan):
+    S = tables["S"]
+    m = np.ones(len(next(iter(S.values()))), bool)
+    for p in plan["inner_preds"]:
+        rhs = S[p["rhs"]] if p.get("rhs") else p["lit"]
+        x = S[p["col"]]
+        m &= {"=": x == rhs, "!=": x != rhs, "<": x < rhs, "<=": x <= rhs, ">": x > rhs, ">=": x >= rhs}[p["op"]]
+    return m
+
+
+def _pack(cols):
+    if len(cols) == 1:
+        return cols[0].astype(np.int64)
+    return (cols[0].astype(np.int64) << 32) | (cols[1].astype(np.int64) & 0xffffffff)
+
+
+def _groupby_check(tables, plan, g):
+    """Unnested GROUP BY checker (Query 2 form) for '=' plans, every R' row."""
+    S, R = tables["S"], tables["R"]
+    m = _inner_mask(tables, plan)
+    sk = _pack([S[c][m] for c in plan["inner_key"]])
+    rk = _pack([R[c][g["row"]] for c in plan["outer_key"]])
+    agg = plan["agg"]
+    if agg == "exists":
+        hit = np.isin(rk, sk)
+        assert np.array_equal(g["passed"].astype(bool), hit)
+        return
+    v = S[plan["agg_col"]][m].astype(np.int64)
+    o = np.argsort(sk, kind="stable")
+    sk, v = sk[o], v[o]
+    uk, first, cnt = np.unique(sk, return_index=True, return_counts=True)
+    gi = np.searchsorted(uk, rk)
+    gi_c = np.minimum(gi, len(uk) - 1)
+    hit = (gi < len(uk)) & (uk[gi_c] == rk)
+    a, b = plan["lhs_mult"], plan["rhs_mult"]
+    x = R[plan["outer_cmp_col"]][g["row"]].astype(np.int64)
+    if agg == "min":
+        gv = np.minimum.reduceat(v, first)[gi_c]
+        exp = hit & (a * x == b * gv)
+    elif agg == "sum":
+        gv = np.add.reduceat(v, first)[gi_c]
+        exp = hit & (a * x > b * gv)
+    elif agg == "avg":
+        gs = np.add.reduceat(v, first)[gi_c]
+        exp = hit & (a * x * cnt[gi_c] < b * gs)
+    assert np.array_equal(g["valid"].astype(bool), hit)
+    assert np.array_equal(g["passed"].astype(bool), exp)
+
+
+@pytest.mark.parametrize("mode", ["index", "bnl"])
+@pytest.mark.parametrize("query", ["q2", "q17"])
+def test_c3(eng, c3, query, mode):
+    tables, plan = tpch.QUERIES[query](c3)
+    g = run(eng, tables, plan, mode, emit_all=True)
+    ref = oracle.evaluate(tables, plan)          # |R'| x |S| <= ~4e10 pair checks
+    assert_parity(g, ref, plan, True, ctx=(query, mode))
+    _groupby_check(tables, plan, g)
+    s = run(eng, tables, plan, mode, emit_all=False)
+    assert_parity(s, ref, plan, False, ctx=(query, mode, "survivors"))
+    assert len(s["row"]) > 0
+
+
+@pytest.mark.parametrize("mode", ["index", "bnl"])
+@pytest.mark.parametrize("query", ["q4", "q20"])
+def test_c4(eng, c4, query, mode):
+    tables, plan = tpch.QUERIES[query](c4)
+    g = run(eng, tables, plan, mode, emit_all=True)
+    rp = _outer_rows(tables, plan)
+    assert np.array_equal(g["row"], rp)
+    rng = np.random.default_rng(0)
+    rows = np.unique(np.concatenate([rp[:2], rp[-2:], rng.choice(rp, 40, replace=False)]))
+    ref = oracle.evaluate(tables, plan, rows=rows)
+    assert_parity(g, ref, plan, True, rows=rows, ctx=(query, mode))
+    _groupby_check(tables, plan, g)
+    s = run(eng, tables, plan, mode, emit_all=False)
+    assert np.array_equal(s["row"], g["row"][g["passed"].astype(bool)])
