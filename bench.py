@@ -352,6 +352,11 @@ def main():
     pk = peaks()
     sm_max = pk.get("sm_max_mhz") or clocks.summary().get("sm_max_mhz") or 1965.0
     roofline = bnl_roofline(profs, n_r, n_s, sm_max, args.workload)
+    stages = {}
+    for _, _, prof in profs:
+        for k, v in prof.items():
+            if v == v:  # not NaN
+                stages[k] = stages.get(k, 0.0) + v / args.steps
 
     # ---- e2e through the public API with host buffers
     e2e = None

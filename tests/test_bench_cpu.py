@@ -1,0 +1,58 @@
+"""CPU checks of bench.py: the reference arm end to end (it times the CPU
+oracle, no GPU involved) and the roofline arithmetic."""
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import bench  # noqa: E402
+
+
+def test_reference_arm_prints_one_json_line():
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--steps", "1",
+                        "--warmup", "0", "--workload", "C1", "--cpu-seconds", "0.3"],
+                       capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stderr
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["metric"] == "outer tuples/s" and d["value"] > 0
+    assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["cpu_baseline"]["kind"] == "oracle"
+
+
+def test_bnl_roofline_arithmetic():
+    from datagen import make_plan
+    n = 1_000_000
+    # a MIN launch exactly at the ALU bound and a COUNT launch at half its bound
+    t_min = n * n / (148 * 32 * 1965e6) * 1000
+    t_cnt = 2 * n * n / (148 * 64 * 1965e6) * 1000
+    profs = [(make_plan(">", "min", "="), "bnl", {"subquery": t_min}),
+             (make_plan(">", "count", "="), "bnl", {"subquery": t_cnt}),
+             (make_plan("=", "min", "="), "index", {"subquery": 0.1})]
+    r = bench.bnl_roofline(profs, n, n, 1965.0, "C2")
+    ideal = t_min + t_cnt / 2
+    assert abs(r["frac"] - ideal / (t_min + t_cnt)) < 1e-9
+    assert abs(r["per_agg"]["min"]["frac"] - 1.0) < 1e-9
+    assert abs(r["per_agg"]["count"]["frac"] - 0.5) < 1e-9
+    assert r["bound"] == "alu" and abs(r["achieved"] / r["peak"] - r["frac"]) < 1e-9
+
+
+import pytest  # noqa: E402
+
+
+@pytest.mark.gpu
+def test_bench_our_arm_c1_json_contract():
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--workload", "C1", "--steps", "3",
+                        "--warmup", "3", "--cpu-seconds", "0.5"], capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
+              "vs_baseline", "dtype", "data", "config", "roofline", "cpu_baseline", "e2e", "gpu_launches", "clocks"):
+        assert k in d, k
+    assert d["value"] > 0 and d["gpu_launches"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0
+    assert d["roofline"]["bound"] == "alu" and 0 < d["roofline"]["frac"]
