@@ -160,6 +160,20 @@ def q2(T):
     return {"R": R, "S": S}, plan
 
 
+def q5(T):
+    """The paper's Query 5 (Fig. 11): TPC-H Q2 (+ Query 4's
+    p_brand = 'Brand#41') with the subquery predicate changed to
+    ps_supplycost > (...) and the correlation to p_partkey != ps_partkey --
+    "cannot be unnested".  The diff in the paper is garbled
+    (R13); this reading keeps Q2's other predicates."""
+    tables, plan = q2(T)
+    part = T["part"]
+    tables["R"]["p_brand"] = part["p_brand"][T["partsupp"]["ps_partkey"] - 1]
+    plan = dict(plan, corr_op="!=", outer_op=">",
+                outer_preds=plan["outer_preds"] + [{"col": "p_brand", "op": "=", "lit": brand_code(4, 1)}])
+    return tables, plan
+
+
 def q17(T):
     """TPC-H Q17: outer = lineitem x part with p_brand = 'Brand#23'
     and p_container = 'MED BOX'; l_quantity < 0.2 * AVG(l_quantity) over the
@@ -213,7 +227,7 @@ def q20(T):
     return {"R": R, "S": S}, plan
 
 
-QUERIES = {"q2": q2, "q17": q17, "q4": q4, "q20": q20}
+QUERIES = {"q2": q2, "q5": q5, "q17": q17, "q4": q4, "q20": q20}
 # BASELINE.json configs[2] = C3 (SF1 Q2, Q17), configs[3] = C4 (SF10 Q4, Q20)
 CONFIGS = {"C3": (1.0, ("q2", "q17"), 3), "C4": (10.0, ("q4", "q20"), 5)}
 

@@ -427,40 +427,36 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     void *uk = salloc(c, (size_t)n * kb), *uv = vb ? salloc(c, (size_t)n * vb) : nullptr;
     void *fscr = salloc(c, ng::filter_scratch_bytes(n));
     void *sscr = salloc(c, ng::sort_scratch_bytes(n));
-    unsigned *hist = (unsigned *)salloc(c, 8 * 256 * 4 + 64);
+    unsigned *hist = (unsigned *)salloc(c, 8 * 256 * 4);
     unsigned *dbase = (unsigned *)salloc(c, 8 * 256 * 4);
-    if (!tk || !uk || !fscr || !sscr || !hist || !dbase || (vb && (!tv || !uv)))
+    long long *dsmall = (long long *)salloc(c, 64);   // [0] |S'|, [2] key AND, [3] key OR
+    if (!tk || !uk || !fscr || !sscr || !hist || !dbase || !dsmall || (vb && (!tv || !uv)))
         return fail(c, NESTGPU_ERR_OOM, "arena exhausted building an index over %lld rows", (long long)n);
-    long long *d_count = (long long *)(hist + 8 * 256);
-    CUDA_TRY(c, cudaMemsetAsync(hist, 0, 8 * 256 * 4, c->stream));
+    long long *d_count = dsmall;
+    unsigned long long *keymask = (unsigned long long *)(dsmall + 2);
+    CUDA_TRY(c, cudaMemsetAsync(dsmall, 0, 64, c->stream));
+    CUDA_TRY(c, cudaMemsetAsync(keymask, 0xff, 8, c->stream));   // AND identity
     prof_begin(c, 1);
-    CUDA_TRY(c, ng::launch_filter(n, ps, ks, kb, vs, vb, 1, pc ? 1 : 0, nullptr, tk, nullptr, tv, hist, nullptr,
+    CUDA_TRY(c, ng::launch_filter(n, ps, ks, kb, vs, vb, 1, pc ? 1 : 0, nullptr, tk, nullptr, tv, keymask, nullptr,
                                   fscr, d_count, c->stream, &c->launches));
     prof_end(c, 1);
-    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, hist, kb * 256 * 4, cudaMemcpyDeviceToHost, c->stream));
-    CUDA_TRY(c, cudaMemcpyAsync(c->pinned + 8 * 256, d_count, 8, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, dsmall, 32, cudaMemcpyDeviceToHost, c->stream));
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
     long long nsp;
-    memcpy(&nsp, c->pinned + 8 * 256, 8);
-    // plan the passes: skip digits whose histogram has a single bucket
+    unsigned long long kand, kor;
+    memcpy(&nsp, c->pinned, 8);
+    memcpy(&kand, c->pinned + 4, 8);
+    memcpy(&kor, c->pinned + 6, 8);
+    // plan the passes: a digit on which every key agrees needs no pass
     std::vector<int> passes;
-    for (int d = 0; d < kb; d++) {
-        bool trivial = false;
-        for (int b = 0; b < 256; b++)
-            if (c->pinned[d * 256 + b] == (unsigned)nsp) { trivial = true; break; }
-        if (!trivial) passes.push_back(d);
-    }
-    // digit bases for every pass (exclusive prefix over buckets)
-    for (size_t p = 0; p < passes.size(); p++) {
-        unsigned run = 0;
-        for (int b = 0; b < 256; b++) {
-            unsigned t = c->pinned[passes[p] * 256 + b];
-            c->pinned[p * 256 + b] = run;  // safe: p <= passes[p], rows read before overwritten
-            run += t;
-        }
-    }
-    if (!passes.empty())
-        CUDA_TRY(c, cudaMemcpyAsync(dbase, c->pinned, passes.size() * 256 * 4, cudaMemcpyHostToDevice, c->stream));
+    if (nsp > 1)
+        for (int d = 0; d < kb; d++)
+            if (((kand ^ kor) >> (8 * d)) & 0xff) passes.push_back(d);
+    int shifts[8];
+    for (size_t p = 0; p < passes.size(); p++) shifts[p] = passes[p] * 8;
+    prof_begin(c, 2);
+    CUDA_TRY(c, ng::launch_digit_hist(kb, tk, nsp, shifts, (int)passes.size(), hist, dbase, c->num_sms, c->stream,
+                                      &c->launches));
 
     IndexRec ix{};
     ix.off = c->lo;
@@ -477,7 +473,6 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     c->pinned[8 * 256 + 4] = (unsigned)(nsp & 0xffffffffu);
     c->pinned[8 * 256 + 5] = (unsigned)((unsigned long long)nsp >> 32);
     CUDA_TRY(c, cudaMemcpyAsync(ix.d_n, c->pinned + 8 * 256 + 4, 8, cudaMemcpyHostToDevice, c->stream));
-    prof_begin(c, 2);
     const int np = (int)passes.size();
     if (np == 0) {
         if (nsp > 0) {
@@ -492,7 +487,7 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
             void *ok = to_final ? ix.keys : uk;
             void *ov = to_final ? ix.payload : uv;
             if (ok == ik) { ok = tk; ov = tv; }
-            CUDA_TRY(c, ng::launch_radix_pass(kb, vb, ik, ok, iv, ov, nsp, passes[p] * 8, dbase + p * 256, sscr,
+            CUDA_TRY(c, ng::launch_radix_pass(kb, vb, ik, ok, iv, ov, nsp, shifts[p], dbase + p * 256, sscr,
                                               c->stream, &c->launches));
             ik = ok;
             iv = ov;

@@ -77,45 +77,9 @@ __device__ __forceinline__ bool cmp_ct(T x, T y)
     else return x >= y;
 }
 
-// Conjunction of local predicates; NULL operands make a predicate not TRUE.
-__device__ __forceinline__ bool eval_preds(const PredSet &P, long long row)
-{
-    bool ok = true;
-    for (int k = 0; k < P.n; k++) {
-        const DevPred &p = P.p[k];
-        if (p.valid && !__ldg(p.valid + row)) return false;
-        long long x = load_w(p.col, p.w, row);
-        long long y = p.lit;
-        if (p.rhs) {
-            if (p.rhs_valid && !__ldg(p.rhs_valid + row)) return false;
-            y = load_w(p.rhs, p.rhs_w, row);
-        }
-        ok = ok && cmp_rt(x, p.op, y);
-    }
-    return ok;
-}
-
 // Order-preserving unsigned encodings of signed keys.
 __device__ __forceinline__ uint32_t enc32(int32_t k) { return (uint32_t)k ^ 0x80000000u; }
 __device__ __forceinline__ uint64_t enc64(long long k) { return (uint64_t)k ^ 0x8000000000000000ull; }
-
-template <typename K>
-__device__ __forceinline__ K encode_key(const KeySrc &ks, long long row, bool &valid)
-{
-    valid = !(ks.v0 && !__ldg(ks.v0 + row));
-    if constexpr (sizeof(K) == 4) {
-        return enc32(__ldg((const int *)ks.c0 + row));
-    } else {
-        if (ks.n_key == 2) {
-            valid = valid && !(ks.v1 && !__ldg(ks.v1 + row));
-            uint64_t hi = enc32(__ldg((const int *)ks.c0 + row));
-            uint64_t lo = enc32(__ldg((const int *)ks.c1 + row));
-            return (hi << 32) | lo;
-        }
-        return ks.w0 == 4 ? enc64((long long)__ldg((const int *)ks.c0 + row))
-                          : enc64(__ldg((const long long *)ks.c0 + row));
-    }
-}
 
 __device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31; }
 __device__ __forceinline__ unsigned lanemask_lt()
@@ -155,35 +119,5 @@ __device__ __forceinline__ void st_relaxed_u32(unsigned *p, unsigned v)
 constexpr unsigned long long ST_AGG = 1ull << 62;
 constexpr unsigned long long ST_INC = 2ull << 62;
 constexpr unsigned long long ST_VAL = (1ull << 62) - 1;
-
-// Called by all threads of warp 0 of a CTA.  Publishes `tile_total` for
-// `tile` and returns (in every lane) the exclusive prefix of the tile.
-__device__ __forceinline__ unsigned long long lookback_warp(unsigned long long *status, long long tile,
-                                                            unsigned long long tile_total)
-{
-    const unsigned lane = lane_id();
-    if (tile == 0) {
-        if (lane == 0) st_relaxed_u64(status, ST_INC | tile_total);
-        return 0;
-    }
-    if (lane == 0) st_relaxed_u64(status + tile, ST_AGG | tile_total);
-    unsigned long long excl = 0;
-    long long pred = tile - 1 - (long long)lane;
-    while (true) {
-        unsigned long long s = pred >= 0 ? ld_relaxed_u64(status + pred) : ST_INC;
-        while (__any_sync(FULL, (s >> 62) == 0)) {
-            if ((s >> 62) == 0) s = ld_relaxed_u64(status + pred);
-        }
-        unsigned inc = __ballot_sync(FULL, (s >> 62) == 2);
-        int stop = inc ? __ffs(inc) - 1 : 31;
-        unsigned long long v = (int)lane <= stop ? (s & ST_VAL) : 0;
-        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
-        excl += v;
-        if (inc) break;
-        pred -= 32;
-    }
-    if (lane == 0) st_relaxed_u64(status + tile, ST_INC | (excl + tile_total));
-    return excl;
-}
 
 }  // namespace ng

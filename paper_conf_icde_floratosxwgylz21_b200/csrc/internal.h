@@ -17,8 +17,8 @@ namespace ng {
 //   out_kvalid : 1 byte per survivor, key not NULL (nullable)
 //   out_vals   : payload (vb = 4 or 8 bytes; nullable)
 //   drop_null_key / drop_null_val : NULL key / payload rows do not survive
-//   hist       : if non-null, kb*256 uint32 digit histograms of the encoded
-//                survivor keys (for the radix sort), accumulated atomically
+//   keymask    : if non-null, [0] &= and [1] |= every survivor's encoded key
+//                (radix digits where they agree need no sort pass)
 //   extreme    : if non-null, [0] |= any survivor payload == max of its type,
 //                [1] |= any == min (for the MIN/MAX identity check)
 //   scratch    : tile status + counter, from filter_scratch_bytes(n)
@@ -27,8 +27,13 @@ size_t filter_scratch_bytes(long long n);
 cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, int kb,
                           const ValSrc &val, int vb, int drop_null_key, int drop_null_val,
                           int *out_ids, void *out_keys, uint8_t *out_kvalid, void *out_vals,
-                          unsigned *hist, unsigned *extreme, void *scratch,
+                          unsigned long long *keymask, unsigned *extreme, void *scratch,
                           long long *out_count, cudaStream_t st, long long *launches);
+
+// a4: histograms of the digits at `shifts` (np of them) over n encoded keys,
+// and their exclusive scans into digit_base[np][256].
+cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *shifts, int np, unsigned *hist,
+                              unsigned *digit_base, int num_sms, cudaStream_t st, long long *launches);
 
 // a4: one stable LSD radix pass on 8-bit digit `shift/8` of the encoded keys.
 //   digit_base: 256 uint32 global exclusive offsets of the digit (device)

@@ -12,9 +12,9 @@
 // order), publishes per-digit tile counts, resolves its global per-digit
 // offset by decoupled look-back over preceding tiles (dynamic tile ids for
 // forward progress), reorders the tile in shared memory and writes each
-// digit run out coalesced.  Digit histograms come from the S' filter kernel
-// (fused), so a pass is exactly one read and one write of (key, payload);
-// digits whose histogram has a single bucket are skipped by the host.
+// digit run out coalesced, so a pass is one read and one write of (key,
+// payload).  The S' filter kernel also reduces AND / OR over the keys: digits
+// on which all keys agree are skipped; one histogram kernel covers the rest.
 #include <type_traits>
 
 #include "internal.h"
@@ -109,13 +109,22 @@ onesweep_kernel(const K *__restrict__ kin, K *__restrict__ kout, const void *__r
     // decoupled look-back for digit d
     unsigned excl = 0;
     if (tile > 0) {
+        // walk back 4 predecessors per round trip (loads issued together)
         long long p = tile - 1;
-        while (true) {
-            unsigned s;
-            do { s = ld_relaxed_u32(status + p * 256 + d); } while ((s >> 30) == 0);
-            excl += s & D_VAL;
-            if ((s >> 30) == 2) break;
-            --p;
+        bool done = false;
+        while (!done) {
+            unsigned sv[4];
+#pragma unroll
+            for (int q = 0; q < 4; q++) sv[q] = p - q >= 0 ? ld_relaxed_u32(status + (p - q) * 256 + d) : D_INC;
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                if (done) break;
+                unsigned s = sv[q];
+                while ((s >> 30) == 0) s = ld_relaxed_u32(status + (p - q) * 256 + d);
+                excl += s & D_VAL;
+                done = (s >> 30) == 2;
+            }
+            p -= 4;
         }
         st_relaxed_u32(my_status, D_INC | (excl + cnt));
     }
@@ -143,6 +152,72 @@ onesweep_kernel(const K *__restrict__ kin, K *__restrict__ kout, const void *__r
         kout[dst] = k;
         if constexpr (VB > 0) vout[dst] = s_vals[p];
     }
+}
+
+// Histograms of the 8-bit digits that vary (the others were dropped using
+// the AND / OR masks the S' filter computed): one pass over the keys, per-CTA
+// shared-memory bins, one global atomic per bin per CTA.
+struct DigitList {
+    int n;
+    int shift[8];
+};
+
+template <typename K>
+__global__ void __launch_bounds__(256) digit_hist_kernel(const K *__restrict__ keys, long long n, DigitList dl,
+                                                         unsigned *__restrict__ hist)
+{
+    __shared__ unsigned s_hist[8 * 256];
+    for (int i = threadIdx.x; i < dl.n * 256; i += 256) s_hist[i] = 0;
+    __syncthreads();
+    const long long stride = (long long)gridDim.x * 256;
+    for (long long i = blockIdx.x * 256LL + threadIdx.x; i < n; i += stride) {
+        const K k = keys[i];
+#pragma unroll
+        for (int p = 0; p < 8; p++)
+            if (p < dl.n) atomicAdd(&s_hist[p * 256 + (unsigned)((k >> dl.shift[p]) & 255)], 1u);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < dl.n * 256; i += 256)
+        if (s_hist[i]) atomicAdd(&hist[i], s_hist[i]);
+}
+
+// Exclusive scan of each pass's 256 bins -> global digit base offsets.
+__global__ void __launch_bounds__(256) digit_scan_kernel(const unsigned *__restrict__ hist, unsigned *__restrict__ base)
+{
+    __shared__ unsigned s_w[8];
+    const unsigned *h = hist + blockIdx.x * 256;
+    const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+    const unsigned c = h[t];
+    unsigned incl = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        unsigned v = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += v;
+    }
+    if (lane == 31) s_w[warp] = incl;
+    __syncthreads();
+    unsigned pre = 0;
+    for (int w = 0; w < warp; w++) pre += s_w[w];
+    base[blockIdx.x * 256 + t] = pre + incl - c;
+}
+
+cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *shifts, int np, unsigned *hist,
+                              unsigned *digit_base, int num_sms, cudaStream_t st, long long *launches)
+{
+    if (np <= 0) return cudaSuccess;
+    cudaError_t e = cudaMemsetAsync(hist, 0, (size_t)np * 256 * 4, st);
+    if (e != cudaSuccess) return e;
+    DigitList dl{};
+    dl.n = np;
+    for (int p = 0; p < np; p++) dl.shift[p] = shifts[p];
+    long long blocks = (n + 255) / 256;
+    if (blocks > (long long)num_sms * 8) blocks = (long long)num_sms * 8;
+    if (blocks < 1) blocks = 1;
+    if (kb == 4) digit_hist_kernel<uint32_t><<<(unsigned)blocks, 256, 0, st>>>((const uint32_t *)keys, n, dl, hist);
+    else digit_hist_kernel<uint64_t><<<(unsigned)blocks, 256, 0, st>>>((const uint64_t *)keys, n, dl, hist);
+    digit_scan_kernel<<<np, 256, 0, st>>>(hist, digit_base);
+    *launches += 2;
+    return cudaGetLastError();
 }
 
 template <typename K, int VB>

@@ -100,13 +100,14 @@ def _groupby_check(tables, plan, g):
 
 
 @pytest.mark.parametrize("mode", ["index", "bnl"])
-@pytest.mark.parametrize("query", ["q2", "q17"])
+@pytest.mark.parametrize("query", ["q2", "q5", "q17"])
 def test_c3(eng, c3, query, mode):
     tables, plan = tpch.QUERIES[query](c3)
     g = run(eng, tables, plan, mode, emit_all=True)
     ref = oracle.evaluate(tables, plan)          # |R'| x |S| <= ~4e10 pair checks
     assert_parity(g, ref, plan, True, ctx=(query, mode))
-    _groupby_check(tables, plan, g)
+    if plan["corr_op"] == "=":
+        _groupby_check(tables, plan, g)
     s = run(eng, tables, plan, mode, emit_all=False)
     assert_parity(s, ref, plan, False, ctx=(query, mode, "survivors"))
     assert len(s["row"]) > 0

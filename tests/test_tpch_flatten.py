@@ -78,6 +78,46 @@ def test_q2(base, db):
     assert got == exp and len(exp) > 0
 
 
+@pytest.mark.parametrize("with_brand", [True, False])
+def test_q5_non_unnestable(with_brand):
+    """Query 5: Q2 (+ Brand#41) with ps_supplycost > MIN and the
+    correlation p_partkey != ps_partkey.  SF 0.2 without lineitem/orders;
+    the brand-less variant keeps ~100 outer rows."""
+    T = tpch.base_tables(0.2, seed=12)
+    con = sqlite3.connect(":memory:")
+    for name, cols in (("supplier", T["supplier"]), ("partsupp", T["partsupp"])):
+        con.execute("CREATE TABLE %s (%s)" % (name, ", ".join(cols)))
+        con.executemany("INSERT INTO %s VALUES (%s)" % (name, ",".join("?" * len(cols))),
+                        zip(*[c.tolist() for c in cols.values()]))
+    con.execute("CREATE TABLE nation (n_nationkey, n_regionkey)")
+    con.executemany("INSERT INTO nation VALUES (?,?)", zip(range(25), [r for _, r in tpch.NATIONS]))
+    con.execute("CREATE TABLE region (r_regionkey, r_name)")
+    con.executemany("INSERT INTO region VALUES (?,?)", enumerate(tpch.REGIONS))
+    p = T["part"]
+    con.execute("CREATE TABLE part (p_partkey, p_size, p_type_s, p_brand_s)")
+    con.executemany("INSERT INTO part VALUES (?,?,?,?)", zip(
+        p["p_partkey"].tolist(), p["p_size"].tolist(),
+        ["%s %s %s" % (tpch.TYPE_S1[t // 25], tpch.TYPE_S2[(t // 5) % 5], tpch.TYPE_S3[t % 5]) for t in p["p_type"].tolist()],
+        ["Brand#%d%d" % (b // 5 + 1, b % 5 + 1) for b in p["p_brand"].tolist()]))
+    con.execute("CREATE INDEX s_k ON supplier(s_suppkey)")
+    tables, plan = tpch.q5(T)
+    if not with_brand:
+        plan = dict(plan, outer_preds=[q for q in plan["outer_preds"] if q["col"] != "p_brand"])
+    rows = _oracle_rows(tables, plan)
+    got = sorted(zip(T["partsupp"]["ps_partkey"][rows].tolist(), T["partsupp"]["ps_suppkey"][rows].tolist()))
+    sql = """
+      SELECT p_partkey, s_suppkey FROM part, supplier, partsupp, nation, region
+      WHERE p_partkey = ps_partkey AND s_suppkey = ps_suppkey AND p_size = 15 AND p_type_s LIKE '%%BRASS'
+        %s
+        AND s_nationkey = n_nationkey AND n_regionkey = r_regionkey AND r_name = 'EUROPE'
+        AND ps_supplycost > (SELECT min(ps_supplycost) FROM partsupp, supplier, nation, region
+                             WHERE p_partkey != ps_partkey AND s_suppkey = ps_suppkey
+                               AND s_nationkey = n_nationkey AND n_regionkey = r_regionkey
+                               AND r_name = 'EUROPE')""" % ("AND p_brand_s = 'Brand#41'" if with_brand else "")
+    exp = sorted(con.execute(sql).fetchall())
+    assert got == exp and len(exp) > 0
+
+
 def test_q17(base, db):
     tables, plan = tpch.q17(base)
     rows = _oracle_rows(tables, plan)
