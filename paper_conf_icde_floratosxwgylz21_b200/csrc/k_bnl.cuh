@@ -61,37 +61,6 @@ struct BnlTile {
     static constexpr int KBYTES = TILE * (int)sizeof(K);
 };
 
-__device__ __forceinline__ void mbar_init(unsigned long long *bar, unsigned count)
-{
-    unsigned a = (unsigned)__cvta_generic_to_shared(bar);
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(unsigned long long *bar, unsigned parity)
-{
-    unsigned a = (unsigned)__cvta_generic_to_shared(bar);
-    asm volatile(
-        "{\n\t.reg .pred P1;\n"
-        "NG_WAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
-        "@!P1 bra NG_WAIT_%=;\n}" ::"r"(a),
-        "r"(parity)
-        : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(unsigned long long *bar, unsigned bytes)
-{
-    unsigned a = (unsigned)__cvta_generic_to_shared(bar);
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(a), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned bytes, unsigned long long *bar)
-{
-    unsigned d = (unsigned)__cvta_generic_to_shared(dst);
-    unsigned b = (unsigned)__cvta_generic_to_shared(bar);
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(d),
-        "l"(src), "r"(bytes), "r"(b)
-        : "memory");
-}
-
 template <int AGG>
 struct AccKind {
     static constexpr bool minmax = AGG == MIN || AGG == MAX;

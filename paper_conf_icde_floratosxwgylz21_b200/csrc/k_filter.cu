@@ -1,276 +1,265 @@
-// k_filter.cu -- a2/a3 (outer / inner local predicates -> compacted R', S')
-// and a8/a9 (aggregate finalize + outer comparison + ordered compaction).
+// k_filter.cu -- a2 / a3: local predicates over R (outer) or S (inner), and
+// compaction of the surviving rows into R' (row ids + encoded keys) or
+// S' (encoded keys + payload).
 //
 // PAPER.md P:235 (§III-C): a Selection is "scan -> 0-1 vector -> prefix-sum ->
 // materialize" over several primitive kernels with inter-kernel results in a
-// pool.  On B200 this is ONE pass per relation: each CTA evaluates the
-// predicates for a 4096-row tile with coalesced column loads, builds the 0-1
-// vector in registers (warp __ballot_sync), ranks survivors with __popc, gets
-// its global offset by decoupled look-back (no second pass over HBM), and
-// writes the compacted (row id | encoded key | payload) directly.  The same
-// tile machinery compacts the survivors of the outer comparison (the final
-// "Selection(=, R.col1, Res)" + Materialize of P:183), fused with the
-// aggregate finalisation.
+// memory pool.  On B200 it is ONE pass:
+//  * persistent CTAs take 256*ITEMS-row tiles from an atomic counter;
+//  * every column segment the tile needs (predicate operands, validity
+//    bytes, key, payload) is staged global -> shared by cp.async.bulk (TMA
+//    bulk engine) into a double-buffered stage, completed on an mbarrier --
+//    the next tile's copies are in flight while this tile is compacted;
+//  * predicates are evaluated from shared memory (conflict-free), the 0-1
+//    vector lives in a register bitmask, warp ballots + popc give ranks,
+//    and a CTA-wide decoupled look-back gives the tile's global offset;
+//  * survivors are written in row order.
+// The S' pass also reduces AND / OR over the encoded keys (radix digits on
+// which all keys agree need no sort pass) and flags payloads equal to the
+// MIN/MAX identity.
 #include <climits>
+#include <cstring>
 #include <type_traits>
 
 #include "internal.h"
+#include "scan.cuh"
 
 namespace ng {
 
-constexpr int F_THREADS = 256;
-constexpr int F_WARPS = F_THREADS / 32;
-constexpr int F_ITEMS = 16;
-constexpr int F_TILE = F_THREADS * F_ITEMS;
+constexpr int T_THREADS = 256;
+constexpr int T_WARPS = T_THREADS / 32;
+constexpr int MAX_SRC = 40;
+constexpr int STAGE_MAX = 49152;  // bytes per stage (2 stages per CTA)
 
-size_t filter_scratch_bytes(long long n)
-{
-    long long tiles = (n + F_TILE - 1) / F_TILE;
-    return (size_t)(tiles + 1) * 8 + 256;
-}
+struct SrcCols {
+    int n;
+    int stage_bytes;
+    const void *ptr[MAX_SRC];
+    int w[MAX_SRC];    // 1, 4 or 8 bytes per row
+    int off[MAX_SRC];  // byte offset of the column's segment inside a stage
+};
 
-// Shared scan of the per-(item, warp) survivor counts in row order
-// (item-major, then warp) + the tile's global offset.  Called by all threads.
-// s_cnt holds counts on entry and exclusive offsets on exit.  The decoupled
-// look-back is done by the whole CTA (the other warps would only wait at the
-// barrier): thread t inspects predecessor tile-1-t, so one L2 round trip
-// covers 256 predecessors; the nearest inclusive prefix ends the walk.
-__device__ __forceinline__ unsigned long long tile_offsets(unsigned (*s_cnt)[F_WARPS], unsigned long long *status,
-                                                           long long tile, long long num_tiles,
-                                                           long long *out_count,
-                                                           unsigned long long *s_base)
-{
-    __shared__ unsigned s_total;
-    __shared__ int s_stop;
-    __shared__ unsigned long long s_wsum[F_WARPS];
-    __syncthreads();
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    if (tid < 32) {
-        unsigned *flat = &s_cnt[0][0];
-        unsigned c[4], s = 0;
-#pragma unroll
-        for (int q = 0; q < 4; q++) { c[q] = flat[4 * lane + q]; s += c[q]; }
-        unsigned incl = s;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            unsigned t = __shfl_up_sync(FULL, incl, o);
-            if (lane >= o) incl += t;
-        }
-        unsigned run = incl - s;
-        const unsigned total = __shfl_sync(FULL, incl, 31);
-#pragma unroll
-        for (int q = 0; q < 4; q++) { unsigned t = c[q]; flat[4 * lane + q] = run; run += t; }
-        if (lane == 0) {
-            s_total = total;
-            st_relaxed_u64(status + tile, (tile == 0 ? ST_INC : ST_AGG) | total);
-            s_stop = 0x7fffffff;
-        }
+struct TPred {
+    int col, valid, rhs, rhs_valid;  // source indices, -1 = none
+    int op;
+    long long lit;
+};
+
+struct TPlan {
+    int n_preds;
+    TPred p[MAX_PREDS];
+    int key0, key0v, key1, key1v, n_key;
+    int val, valv;
+    int drop_null_key, drop_null_val;
+};
+
+size_t filter_scratch_bytes(long long n) { return (size_t)(n / T_THREADS + 2) * 8 + 256; }
+
+template <int ITEMS>
+struct Stage {
+    const unsigned char *base;
+    const SrcCols *sc;
+    template <typename T>
+    __device__ __forceinline__ T at(int c, int li) const
+    {
+        return reinterpret_cast<const T *>(base + sc->off[c])[li];
     }
-    __syncthreads();
-    const unsigned long long total = s_total;
-    unsigned long long excl = 0;
-    if (tile > 0) {
-        for (long long round = 0;; round += F_THREADS) {
-            const long long pred = tile - 1 - round - tid;
-            unsigned long long sv = pred >= 0 ? ld_relaxed_u64(status + pred) : ST_INC;
-            while ((sv >> 62) == 0) sv = ld_relaxed_u64(status + pred);
-            if ((sv >> 62) == 2) atomicMin(&s_stop, tid);
-            __syncthreads();
-            const int stop = s_stop;                       // nearest inclusive predecessor
-            unsigned long long v = tid <= stop ? (sv & ST_VAL) : 0;
-#pragma unroll
-            for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
-            if (lane == 0) s_wsum[warp] = v;
-            __syncthreads();
-#pragma unroll
-            for (int w = 0; w < F_WARPS; w++) excl += s_wsum[w];
-            if (stop != 0x7fffffff) break;
-            __syncthreads();                               // s_wsum reuse
-        }
-        if (tid == 0) st_relaxed_u64(status + tile, ST_INC | (excl + total));
+    __device__ __forceinline__ long long val(int c, int li) const
+    {
+        const int w = sc->w[c];
+        return w == 4 ? (long long)at<int>(c, li) : (w == 8 ? at<long long>(c, li) : (long long)at<uint8_t>(c, li));
     }
-    if (tid == 0 && tile == num_tiles - 1) *out_count = (long long)(excl + total);
-    (void)s_base;
-    __syncthreads();
-    return excl;
-}
-
-// Load items j = 0..F_ITEMS-1 of one column for the rows still alive in
-// `live` (bit j), all loads issued before any use (memory-level parallelism:
-// 16 independent coalesced loads per thread).
-template <int W>
-__device__ __forceinline__ void load_items(const void *__restrict__ col, long long base, int tid, unsigned live,
-                                           long long (&x)[F_ITEMS])
-{
+    __device__ __forceinline__ unsigned nonnull(int c, unsigned live, int tid) const
+    {
+        if (c < 0) return live;
+        unsigned out = 0;
 #pragma unroll
-    for (int j = 0; j < F_ITEMS; j++) {
-        const long long row = base + (long long)j * F_THREADS + tid;
-        x[j] = 0;
-        if (live >> j & 1u) {
-            if constexpr (W == 4) x[j] = __ldg((const int *)col + row);
-            else x[j] = __ldg((const long long *)col + row);
-        }
+        for (int j = 0; j < ITEMS; j++)
+            if ((live >> j & 1u) && at<uint8_t>(c, j * T_THREADS + tid)) out |= 1u << j;
+        return out;
     }
-}
+};
 
-__device__ __forceinline__ unsigned valid_bits(const uint8_t *__restrict__ v, long long base, int tid, unsigned live)
-{
-    if (!v) return live;
-    unsigned out = 0;
-#pragma unroll
-    for (int j = 0; j < F_ITEMS; j++) {
-        const long long row = base + (long long)j * F_THREADS + tid;
-        if ((live >> j & 1u) && __ldg(v + row)) out |= 1u << j;
-    }
-    return out;
-}
-
-template <int OP>
-__device__ __forceinline__ unsigned cmp_bits(const long long (&x)[F_ITEMS], const long long (&y)[F_ITEMS])
+template <int ITEMS, int OP>
+__device__ __forceinline__ unsigned cmp_items(const Stage<ITEMS> &S, const TPred &p, unsigned live, int tid)
 {
     unsigned m = 0;
 #pragma unroll
-    for (int j = 0; j < F_ITEMS; j++)
-        if (cmp_ct<OP>(x[j], y[j])) m |= 1u << j;
+    for (int j = 0; j < ITEMS; j++) {
+        const int li = j * T_THREADS + tid;
+        const long long x = S.val(p.col, li);
+        const long long y = p.rhs >= 0 ? S.val(p.rhs, li) : p.lit;
+        if ((live >> j & 1u) && cmp_ct<OP>(x, y)) m |= 1u << j;
+    }
     return m;
 }
 
-// Conjunction of the local predicates for this thread's 16 rows, evaluated
-// predicate by predicate (column-major) so each predicate's 16 loads are in
-// flight together.  NULL operands make a predicate not TRUE (reading R2).
-__device__ __forceinline__ unsigned eval_preds_tile(const PredSet &P, long long base, int tid, unsigned live)
-{
-    for (int k = 0; k < P.n && live; k++) {
-        const DevPred &p = P.p[k];
-        live = valid_bits(p.valid, base, tid, live);
-        long long x[F_ITEMS], y[F_ITEMS];
-        if (p.w == 4) load_items<4>(p.col, base, tid, live, x);
-        else load_items<8>(p.col, base, tid, live, x);
-        if (p.rhs) {
-            live = valid_bits(p.rhs_valid, base, tid, live);
-            if (p.rhs_w == 4) load_items<4>(p.rhs, base, tid, live, y);
-            else load_items<8>(p.rhs, base, tid, live, y);
-        } else {
-#pragma unroll
-            for (int j = 0; j < F_ITEMS; j++) y[j] = p.lit;
-        }
-        unsigned m;
-        switch (p.op) {
-        case EQ: m = cmp_bits<EQ>(x, y); break;
-        case NE: m = cmp_bits<NE>(x, y); break;
-        case LT: m = cmp_bits<LT>(x, y); break;
-        case LE: m = cmp_bits<LE>(x, y); break;
-        case GT: m = cmp_bits<GT>(x, y); break;
-        default: m = cmp_bits<GE>(x, y); break;
-        }
-        live &= m;
-    }
-    return live;
-}
-
-template <int KB, int VB>
-__global__ void __launch_bounds__(F_THREADS, 2)
-filter_kernel(long long n, PredSet preds, KeySrc ks, ValSrc vs, int drop_null_key, int drop_null_val,
-              int *__restrict__ out_ids, void *__restrict__ out_keys, uint8_t *__restrict__ out_kvalid,
-              void *__restrict__ out_vals, unsigned long long *__restrict__ keymask,
-              unsigned *__restrict__ extreme, unsigned long long *__restrict__ status,
-              unsigned *__restrict__ counter, long long *__restrict__ out_count)
+// ORDERED: survivors keep row order (R', whose order is the result's order)
+// via the decoupled look-back; otherwise (S', re-ordered by the sort anyway
+// and order-free for the nested loop) a tile claims its output range with
+// one atomicAdd on the survivor counter -- no dependency between tiles.
+template <int KB, int VB, int ITEMS, bool ORDERED>
+__global__ void __launch_bounds__(T_THREADS)
+filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, void *__restrict__ out_keys,
+                  uint8_t *__restrict__ out_kvalid, void *__restrict__ out_vals,
+                  unsigned long long *__restrict__ keymask, unsigned *__restrict__ extreme,
+                  unsigned long long *__restrict__ status, unsigned *__restrict__ counter,
+                  long long *__restrict__ out_count)
 {
     using K = typename std::conditional<KB == 8, uint64_t, uint32_t>::type;
     using V = typename std::conditional<VB == 8, long long, int>::type;
-    __shared__ unsigned s_tile;
-    __shared__ unsigned s_cnt[F_ITEMS][F_WARPS];
-    __shared__ unsigned long long s_base;
+    constexpr int TILE = T_THREADS * ITEMS;
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ __align__(8) unsigned long long bar[2];
+    __shared__ unsigned s_cnt[ITEMS][T_WARPS];
+    __shared__ long long s_tile[2];
+    __shared__ unsigned long long s_claim;
+
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    if (tid == 0) s_tile = atomicAdd(counter, 1u);
+    const long long num_tiles = (n + TILE - 1) / TILE;
+
+    auto issue = [&](long long tile, int stage) {
+        const long long rows = min((long long)TILE, n - tile * TILE);
+        unsigned total = 0;
+        for (int c = 0; c < sc.n; c++) total += ((unsigned)rows * sc.w[c] + 15u) & ~15u;
+        unsigned char *dst = smem + stage * sc.stage_bytes;
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        mbar_expect_tx(&bar[stage], total);
+        for (int c = 0; c < sc.n; c++)
+            bulk_g2s(dst + sc.off[c], (const char *)sc.ptr[c] + tile * TILE * sc.w[c],
+                     ((unsigned)rows * sc.w[c] + 15u) & ~15u, &bar[stage]);
+    };
+
+    if (tid == 0) {
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        const long long t0 = atomicAdd(counter, 1u);
+        s_tile[0] = t0;
+        if (t0 < num_tiles) issue(t0, 0);
+    }
     __syncthreads();
-    const long long tile = s_tile;
-    const long long num_tiles = (n + F_TILE - 1) / F_TILE;
-    const long long base = tile * F_TILE;
 
-    // rows of this thread: base + j*256 + tid (coalesced per warp)
-    unsigned live = 0;
-#pragma unroll
-    for (int j = 0; j < F_ITEMS; j++)
-        if (base + (long long)j * F_THREADS + tid < n) live |= 1u << j;
-    live = eval_preds_tile(preds, base, tid, live);
-
-    K key[F_ITEMS];
-    unsigned kvalid = live;
-    if constexpr (KB > 0) {
-        // encoded correlated key (order-preserving unsigned)
-        kvalid = valid_bits(ks.v0, base, tid, live);
-        if (ks.n_key == 2) {
-            kvalid = valid_bits(ks.v1, base, tid, kvalid);
-            long long a[F_ITEMS], b[F_ITEMS];
-            load_items<4>(ks.c0, base, tid, live, a);
-            load_items<4>(ks.c1, base, tid, live, b);
-#pragma unroll
-            for (int j = 0; j < F_ITEMS; j++)
-                key[j] = (K)(((uint64_t)enc32((int)a[j]) << 32) | (uint64_t)enc32((int)b[j]));
-        } else {
-            long long a[F_ITEMS];
-            if (ks.w0 == 4) load_items<4>(ks.c0, base, tid, live, a);
-            else load_items<8>(ks.c0, base, tid, live, a);
-#pragma unroll
-            for (int j = 0; j < F_ITEMS; j++) {
-                if constexpr (KB == 4) key[j] = (K)enc32((int)a[j]);
-                else key[j] = (K)enc64(a[j]);
-            }
-        }
-        if (drop_null_key) live = kvalid;
-    }
-    V val[F_ITEMS];
+    unsigned phase = 0u;  // bit s: parity of the next completion of stage s
+    int stage = 0;
     bool ext_max = false, ext_min = false;
-    if constexpr (VB > 0) {
-        const unsigned vv = valid_bits(vs.v, base, tid, live);
-        if (drop_null_val) live = vv;
-        long long a[F_ITEMS];
-        if (vs.w == 4) load_items<4>(vs.c, base, tid, live, a);
-        else load_items<8>(vs.c, base, tid, live, a);
-#pragma unroll
-        for (int j = 0; j < F_ITEMS; j++) {
-            val[j] = (V)a[j];
-            if (live >> j & 1u) {
-                ext_max |= val[j] == (VB == 8 ? (V)LLONG_MAX : (V)INT_MAX);
-                ext_min |= val[j] == (VB == 8 ? (V)LLONG_MIN : (V)INT_MIN);
-            }
-        }
-    }
-    unsigned rank[F_ITEMS];
     unsigned long long kand = ~0ull, kor = 0ull;
+    while (true) {
+        const long long tile = s_tile[stage];
+        if (tile >= num_tiles) break;
+        if (tid == 0) {  // prefetch the next tile into the other stage
+            const long long nt = atomicAdd(counter, 1u);
+            s_tile[stage ^ 1] = nt;
+            if (nt < num_tiles) issue(nt, stage ^ 1);
+        }
+        mbar_wait(&bar[stage], (phase >> stage) & 1u);
+        phase ^= 1u << stage;
+        const Stage<ITEMS> S{smem + stage * sc.stage_bytes, &sc};
+        const long long base = tile * TILE;
+        const long long rows = min((long long)TILE, n - base);
+
+        unsigned live = 0;
 #pragma unroll
-    for (int j = 0; j < F_ITEMS; j++) {
-        const bool f = live >> j & 1u;
-        const unsigned m = __ballot_sync(FULL, f);
-        if (lane == 0) s_cnt[j][warp] = __popc(m);
-        rank[j] = __popc(m & lanemask_lt());
-        if constexpr (KB > 0) {
-            if (f) {
-                kand &= (unsigned long long)key[j];
-                kor |= (unsigned long long)key[j];
+        for (int j = 0; j < ITEMS; j++)
+            if (j * T_THREADS + tid < rows) live |= 1u << j;
+        // local predicates (NULL operands are not TRUE, reading R2)
+        for (int k = 0; k < tp.n_preds; k++) {
+            const TPred &p = tp.p[k];
+            live = S.nonnull(p.valid, live, tid);
+            live = S.nonnull(p.rhs_valid, live, tid);
+            switch (p.op) {
+            case EQ: live &= cmp_items<ITEMS, EQ>(S, p, live, tid); break;
+            case NE: live &= cmp_items<ITEMS, NE>(S, p, live, tid); break;
+            case LT: live &= cmp_items<ITEMS, LT>(S, p, live, tid); break;
+            case LE: live &= cmp_items<ITEMS, LE>(S, p, live, tid); break;
+            case GT: live &= cmp_items<ITEMS, GT>(S, p, live, tid); break;
+            default: live &= cmp_items<ITEMS, GE>(S, p, live, tid); break;
             }
         }
-    }
-    const unsigned long long tb = tile_offsets(s_cnt, status, tile, num_tiles, out_count, &s_base);
-#pragma unroll
-    for (int j = 0; j < F_ITEMS; j++) {
-        if (!(live >> j & 1u)) continue;
-        const long long pos = (long long)tb + s_cnt[j][warp] + rank[j];
-        const long long row = base + (long long)j * F_THREADS + tid;
-        if (out_ids) out_ids[pos] = (int)row;
+        unsigned kvalid = live;
         if constexpr (KB > 0) {
-            if (out_keys) ((K *)out_keys)[pos] = key[j];
-            if (out_kvalid) out_kvalid[pos] = (kvalid >> j) & 1u;
+            kvalid = S.nonnull(tp.key1v, S.nonnull(tp.key0v, live, tid), tid);
+            if (tp.drop_null_key) live = kvalid;
         }
         if constexpr (VB > 0) {
-            if (out_vals) ((V *)out_vals)[pos] = val[j];
+            const unsigned vv = S.nonnull(tp.valv, live, tid);
+            if (tp.drop_null_val) live = vv;
         }
+        unsigned rank[ITEMS];
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            const unsigned m = __ballot_sync(FULL, live >> j & 1u);
+            if (lane == 0) s_cnt[j][warp] = __popc(m);
+            rank[j] = __popc(m & lanemask_lt());
+        }
+        unsigned long long tb;
+        if constexpr (ORDERED) {
+            tb = tile_offsets<ITEMS, T_THREADS>(s_cnt, status, tile, num_tiles, out_count);
+        } else {
+            __syncthreads();
+            if (tid < 32) {  // exclusive scan of the (item, warp) counts + one atomic claim
+                unsigned *flat = &s_cnt[0][0];
+                constexpr int E = ITEMS * T_WARPS, PER = (E + 31) / 32;
+                unsigned c[PER], sum = 0;
+#pragma unroll
+                for (int q = 0; q < PER; q++) {
+                    c[q] = PER * lane + q < E ? flat[PER * lane + q] : 0u;
+                    sum += c[q];
+                }
+                unsigned incl = sum;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const unsigned t = __shfl_up_sync(FULL, incl, o);
+                    if (lane >= o) incl += t;
+                }
+                unsigned run = incl - sum;
+#pragma unroll
+                for (int q = 0; q < PER; q++) {
+                    if (PER * lane + q < E) flat[PER * lane + q] = run;
+                    run += c[q];
+                }
+                if (lane == 31)
+                    s_claim = incl ? atomicAdd((unsigned long long *)out_count, (unsigned long long)incl) : 0ull;
+            }
+            __syncthreads();
+            tb = s_claim;
+        }
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            if (!(live >> j & 1u)) continue;
+            const int li = j * T_THREADS + tid;
+            const long long pos = (long long)tb + s_cnt[j][warp] + rank[j];
+            if (out_ids) out_ids[pos] = (int)(base + li);
+            if constexpr (KB > 0) {
+                K key;
+                if (tp.n_key == 2)
+                    key = (K)(((uint64_t)enc32(S.template at<int>(tp.key0, li)) << 32) |
+                              enc32(S.template at<int>(tp.key1, li)));
+                else if constexpr (KB == 4)
+                    key = (K)enc32(S.template at<int>(tp.key0, li));
+                else
+                    key = (K)enc64(S.val(tp.key0, li));
+                if (out_keys) ((K *)out_keys)[pos] = key;
+                if (out_kvalid) out_kvalid[pos] = (kvalid >> j) & 1u;
+                kand &= (unsigned long long)key;
+                kor |= (unsigned long long)key;
+            }
+            if constexpr (VB > 0) {
+                const V v = (V)S.val(tp.val, li);
+                if (out_vals) ((V *)out_vals)[pos] = v;
+                ext_max |= v == (VB == 8 ? (V)LLONG_MAX : (V)INT_MAX);
+                ext_min |= v == (VB == 8 ? (V)LLONG_MIN : (V)INT_MIN);
+            }
+        }
+        __syncthreads();  // stage fully read before it is refilled; s_tile visible
+        stage ^= 1;
     }
     if constexpr (KB > 0) {
-        if (keymask) {  // bits shared by every survivor key: which radix digits are constant
-            const unsigned alo = __reduce_and_sync(FULL, (unsigned)kand), ahi = __reduce_and_sync(FULL, (unsigned)(kand >> 32));
-            const unsigned olo = __reduce_or_sync(FULL, (unsigned)kor), ohi = __reduce_or_sync(FULL, (unsigned)(kor >> 32));
+        if (keymask) {  // bits shared by every survivor key
+            const unsigned alo = __reduce_and_sync(FULL, (unsigned)kand);
+            const unsigned ahi = __reduce_and_sync(FULL, (unsigned)(kand >> 32));
+            const unsigned olo = __reduce_or_sync(FULL, (unsigned)kor);
+            const unsigned ohi = __reduce_or_sync(FULL, (unsigned)(kor >> 32));
             if (lane == 0) {
                 atomicAnd(&keymask[0], ((unsigned long long)ahi << 32) | alo);
                 atomicOr(&keymask[1], ((unsigned long long)ohi << 32) | olo);
@@ -285,203 +274,136 @@ filter_kernel(long long n, PredSet preds, KeySrc ks, ValSrc vs, int drop_null_ke
     }
 }
 
-cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, int kb, const ValSrc &val,
-                          int vb, int drop_null_key, int drop_null_val, int *out_ids, void *out_keys,
-                          uint8_t *out_kvalid, void *out_vals, unsigned long long *keymask, unsigned *extreme,
-                          void *scratch, long long *out_count, cudaStream_t st, long long *launches)
+// ------------------------------------------------------------------ host side
+namespace {
+
+int add_src(SrcCols &sc, const void *p, int w)
+{
+    if (!p) return -1;
+    for (int c = 0; c < sc.n; c++)
+        if (sc.ptr[c] == p && sc.w[c] == w) return c;
+    sc.ptr[sc.n] = p;
+    sc.w[sc.n] = w;
+    return sc.n++;
+}
+
+template <int KB, int VB, int ITEMS, bool ORDERED>
+cudaError_t launch_t(long long n, const SrcCols &sc, const TPlan &tp, int *out_ids, void *out_keys,
+                     uint8_t *out_kvalid, void *out_vals, unsigned long long *keymask, unsigned *extreme,
+                     void *scratch, long long *out_count, int num_sms, cudaStream_t st)
+{
+    auto kern = filter_tma_kernel<KB, VB, ITEMS, ORDERED>;
+    const int smem = 2 * sc.stage_bytes;
+    static int occ_for = -1, occ = 0;
+    if (occ_for != smem) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * STAGE_MAX);
+        if (e != cudaSuccess) return e;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, T_THREADS, smem);
+        if (e != cudaSuccess) return e;
+        occ_for = smem;
+    }
+    const long long tiles = (n + T_THREADS * ITEMS - 1) / (T_THREADS * ITEMS);
+    long long grid = (long long)num_sms * (occ > 0 ? occ : 1);
+    if (grid > tiles) grid = tiles;
+    unsigned *counter = (unsigned *)scratch;
+    unsigned long long *status = (unsigned long long *)((char *)scratch + 256);
+    kern<<<(unsigned)grid, T_THREADS, smem, st>>>(n, sc, tp, out_ids, out_keys, out_kvalid, out_vals, keymask,
+                                                  extreme, status, counter, out_count);
+    return cudaGetLastError();
+}
+
+template <int KB, int VB, bool ORDERED>
+cudaError_t launch_items(int items, long long n, const SrcCols &sc, const TPlan &tp, int *out_ids, void *out_keys,
+                         uint8_t *out_kvalid, void *out_vals, unsigned long long *keymask, unsigned *extreme,
+                         void *scratch, long long *out_count, int num_sms, cudaStream_t st)
+{
+#define NG_LT(I) launch_t<KB, VB, I, ORDERED>(n, sc, tp, out_ids, out_keys, out_kvalid, out_vals, keymask, extreme, scratch, \
+                                     out_count, num_sms, st)
+    switch (items) {
+    case 16: return NG_LT(16);
+    case 8: return NG_LT(8);
+    case 4: return NG_LT(4);
+    case 2: return NG_LT(2);
+    default: return NG_LT(1);
+    }
+#undef NG_LT
+}
+
+}  // namespace
+
+cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, int kb, const ValSrc &val, int vb,
+                          int drop_null_key, int drop_null_val, int *out_ids, void *out_keys, uint8_t *out_kvalid,
+                          void *out_vals, unsigned long long *keymask, unsigned *extreme, void *scratch,
+                          long long *out_count, cudaStream_t st, long long *launches)
 {
     cudaError_t e = cudaMemsetAsync(out_count, 0, sizeof(long long), st);
     if (e != cudaSuccess || n <= 0) return e;
-    const long long tiles = (n + F_TILE - 1) / F_TILE;
-    e = cudaMemsetAsync(scratch, 0, filter_scratch_bytes(n), st);
-    if (e != cudaSuccess) return e;
-    unsigned *counter = (unsigned *)scratch;
-    unsigned long long *status = (unsigned long long *)((char *)scratch + 256);
-    dim3 grid((unsigned)tiles), block(F_THREADS);
-#define NG_FILTER(KB_, VB_)                                                                             \
-    filter_kernel<KB_, VB_><<<grid, block, 0, st>>>(n, preds, key, val, drop_null_key, drop_null_val,   \
-                                                    out_ids, out_keys, out_kvalid, out_vals, keymask,   \
-                                                    extreme, status, counter, out_count)
+    // the column segments a tile needs, deduplicated
+    SrcCols sc;
+    memset(&sc, 0, sizeof sc);
+    TPlan tp;
+    memset(&tp, 0, sizeof tp);
+    tp.n_preds = preds.n;
+    for (int k = 0; k < preds.n; k++) {
+        const DevPred &p = preds.p[k];
+        tp.p[k].col = add_src(sc, p.col, p.w);
+        tp.p[k].valid = add_src(sc, p.valid, 1);
+        tp.p[k].rhs = add_src(sc, p.rhs, p.rhs_w);
+        tp.p[k].rhs_valid = add_src(sc, p.rhs_valid, 1);
+        tp.p[k].op = p.op;
+        tp.p[k].lit = p.lit;
+    }
     const int k = kb == 8 ? 8 : (kb == 4 ? 4 : 0);
     const int v = val.c ? (vb == 8 ? 8 : 4) : 0;
-    if (k == 0 && v == 0) NG_FILTER(0, 0);
-    else if (k == 4 && v == 0) NG_FILTER(4, 0);
-    else if (k == 4 && v == 4) NG_FILTER(4, 4);
-    else if (k == 4 && v == 8) NG_FILTER(4, 8);
-    else if (k == 8 && v == 0) NG_FILTER(8, 0);
-    else if (k == 8 && v == 4) NG_FILTER(8, 4);
-    else NG_FILTER(8, 8);
-#undef NG_FILTER
-    ++*launches;
-    return cudaGetLastError();
-}
-
-// ------------------------------------------------------------------ a8 + a9
-// round_half_away_from_zero(num / den), den > 0 (reading R6).
-__device__ __forceinline__ long long div_round_half_away(__int128 num, long long den)
-{
-    __int128 mag = num < 0 ? -num : num;
-    __int128 q = (2 * mag + den) / (2 * (__int128)den);
-    return (long long)(num < 0 ? -q : q);
-}
-
-__global__ void __launch_bounds__(F_THREADS) finalize_kernel(FinalizeArgs A, unsigned long long *__restrict__ status,
-                                                             unsigned *__restrict__ counter)
-{
-    __shared__ unsigned s_tile;
-    __shared__ unsigned s_cnt[F_ITEMS][F_WARPS];
-    __shared__ unsigned long long s_base;
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const long long n = *A.d_nrp;
-    const long long num_tiles = (n + F_TILE - 1) / F_TILE;
-    if (tid == 0) s_tile = atomicAdd(counter, 1u);
-    __syncthreads();
-    const long long tile = s_tile;
-    if (tile >= num_tiles) return;  // grid sized for the R' upper bound
-    const long long base = tile * F_TILE;
-
-    bool flag[F_ITEMS];
-    unsigned rank[F_ITEMS];
-    long long value[F_ITEMS];
-    uint8_t valid[F_ITEMS], pass[F_ITEMS];
-#pragma unroll
-    for (int j = 0; j < F_ITEMS; j++) {
-        const long long i = base + (long long)j * F_THREADS + tid;
-        bool in = i < n;
-        value[j] = 0;
-        valid[j] = 0;
-        pass[j] = 0;
-        if (in) {
-            const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
-            const long long c = kval ? A.cnt[i] : 0;     // NULL key: empty subquery (R2)
-            const long long acc = A.acc[i];
-            bool vv = true;
-            long long v = 0;
-            switch (A.agg) {
-            case MIN: case MAX: case SUM: vv = c > 0; v = acc; break;
-            case COUNT: v = c; break;
-            case AVG: vv = c > 0; if (vv) v = div_round_half_away((__int128)acc * 1000000, c); break;
-            case EXISTS: v = c > 0; break;
-            default: v = c == 0; break;
-            }
-            bool p;
-            if (A.agg == EXISTS || A.agg == NOT_EXISTS) {
-                p = v != 0;
-            } else {
-                const int row = A.ids[i];
-                const bool xv = !(A.x_valid && !A.x_valid[row]);
-                p = false;
-                if (vv && xv) {
-                    const __int128 x = load_w(A.x_col, A.x_w, row);
-                    if (A.agg == AVG)
-                        p = cmp_rt<__int128>((__int128)A.a * x * c, A.outer_op, (__int128)A.b * acc);
-                    else
-                        p = cmp_rt<__int128>((__int128)A.a * x, A.outer_op, (__int128)A.b * v);
-                }
-            }
-            value[j] = vv ? v : 0;
-            valid[j] = vv;
-            pass[j] = p;
-            in = A.emit_all ? true : p;
-        }
-        flag[j] = in;
-        const unsigned m = __ballot_sync(FULL, in);
-        if (lane == 0) s_cnt[j][warp] = __popc(m);
-        rank[j] = __popc(m & lanemask_lt());
-    }
-    const unsigned long long tb = tile_offsets(s_cnt, status, tile, num_tiles, A.out_count, &s_base);
-#pragma unroll
-    for (int j = 0; j < F_ITEMS; j++) {
-        if (!flag[j]) continue;
-        const long long i = base + (long long)j * F_THREADS + tid;
-        const long long pos = (long long)tb + s_cnt[j][warp] + rank[j];
-        A.out_ids[pos] = A.row_id_base + A.ids[i];
-        A.out_vals[pos] = value[j];
-        A.out_valid[pos] = valid[j];
-        A.out_passed[pos] = pass[j];
-        if (A.out_sum) {
-            const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
-            A.out_sum[pos] = kval ? A.acc[i] : 0;
-            A.out_cnt[pos] = kval ? A.cnt[i] : 0;
+    tp.key0 = tp.key0v = tp.key1 = tp.key1v = tp.val = tp.valv = -1;
+    tp.n_key = key.n_key;
+    if (k) {
+        tp.key0 = add_src(sc, key.c0, key.n_key == 2 ? 4 : key.w0);
+        tp.key0v = add_src(sc, key.v0, 1);
+        if (key.n_key == 2) {
+            tp.key1 = add_src(sc, key.c1, 4);
+            tp.key1v = add_src(sc, key.v1, 1);
         }
     }
-}
-
-cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *launches)
-{
-    cudaError_t e = cudaMemsetAsync(a.out_count, 0, sizeof(long long), st);
-    if (e != cudaSuccess || a.n_rp_max <= 0) return e;
-    e = cudaMemsetAsync(a.scratch, 0, filter_scratch_bytes(a.n_rp_max), st);
+    if (v) {
+        tp.val = add_src(sc, val.c, val.w);
+        tp.valv = add_src(sc, val.v, 1);
+    }
+    tp.drop_null_key = drop_null_key;
+    tp.drop_null_val = drop_null_val;
+    // tile size: the largest 256*ITEMS whose stage fits STAGE_MAX bytes
+    int row_bytes = 0;
+    for (int c = 0; c < sc.n; c++) row_bytes += sc.w[c];
+    int items = 16;
+    while (items > 1 && T_THREADS * items * row_bytes + 16 * sc.n > STAGE_MAX) items >>= 1;
+    if (T_THREADS * items * row_bytes + 16 * sc.n > STAGE_MAX) return cudaErrorInvalidValue;
+    int off = 0;
+    for (int c = 0; c < sc.n; c++) {
+        sc.off[c] = off;
+        off += (T_THREADS * items * sc.w[c] + 15) & ~15;
+    }
+    sc.stage_bytes = (off + 127) & ~127;
+    if (sc.stage_bytes == 0) sc.stage_bytes = 128;
+    e = cudaMemsetAsync(scratch, 0, filter_scratch_bytes(n), st);
     if (e != cudaSuccess) return e;
-    const long long tiles = (a.n_rp_max + F_TILE - 1) / F_TILE;
-    finalize_kernel<<<(unsigned)tiles, F_THREADS, 0, st>>>(a, (unsigned long long *)((char *)a.scratch + 256),
-                                                         (unsigned *)a.scratch);
+    int dev = 0, num_sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&num_sms, cudaDevAttrMultiProcessorCount, dev);
+#define NG_F(KB_, VB_) e = out_ids ? launch_items<KB_, VB_, true>(items, n, sc, tp, out_ids, out_keys, out_kvalid,  \
+                                                                   out_vals, keymask, extreme, scratch, out_count, \
+                                                                   num_sms, st)                                     \
+                              : launch_items<KB_, VB_, false>(items, n, sc, tp, out_ids, out_keys, out_kvalid, out_vals, keymask, \
+                                                 extreme, scratch, out_count, num_sms, st)
+    if (k == 0 && v == 0) NG_F(0, 0);
+    else if (k == 4 && v == 0) NG_F(4, 0);
+    else if (k == 4 && v == 4) NG_F(4, 4);
+    else if (k == 4 && v == 8) NG_F(4, 8);
+    else if (k == 8 && v == 0) NG_F(8, 0);
+    else if (k == 8 && v == 4) NG_F(8, 4);
+    else NG_F(8, 8);
+#undef NG_F
     ++*launches;
-    return cudaGetLastError();
-}
-
-// ------------------------------------------------------------------ partials
-__global__ void init_partials_kernel(long long n, long long acc0, long long *__restrict__ acc,
-                                     long long *__restrict__ cnt)
-{
-    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
-        acc[i] = acc0;
-        cnt[i] = 0;
-    }
-}
-
-cudaError_t launch_init_partials(long long n, int agg, long long *acc, long long *cnt, cudaStream_t st,
-                                 long long *launches)
-{
-    if (n <= 0) return cudaSuccess;
-    long long acc0 = agg == MIN ? LLONG_MAX : (agg == MAX ? LLONG_MIN : 0);
-    long long blocks = (n + 255) / 256;
-    if (blocks > 148 * 16) blocks = 148 * 16;
-    init_partials_kernel<<<(unsigned)blocks, 256, 0, st>>>(n, acc0, acc, cnt);
-    ++*launches;
-    return cudaGetLastError();
-}
-
-// ------------------------------------------------------------------ column min / max
-// (for the SUM/AVG overflow pre-check, reading R5)
-__global__ void minmax_init_kernel(long long *out)
-{
-    out[0] = LLONG_MAX;
-    out[1] = LLONG_MIN;
-}
-
-__global__ void minmax_kernel(const void *__restrict__ col, int w, const uint8_t *__restrict__ valid, long long n,
-                              long long *__restrict__ out)
-{
-    long long mn = LLONG_MAX, mx = LLONG_MIN;
-    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
-        if (valid && !valid[i]) continue;
-        const long long v = load_w(col, w, i);
-        mn = min(mn, v);
-        mx = max(mx, v);
-    }
-    for (int o = 16; o > 0; o >>= 1) {
-        mn = min(mn, __shfl_xor_sync(FULL, mn, o));
-        mx = max(mx, __shfl_xor_sync(FULL, mx, o));
-    }
-    if ((threadIdx.x & 31) == 0) {
-        atomicMin(&out[0], mn);
-        atomicMax(&out[1], mx);
-    }
-}
-
-cudaError_t launch_minmax(const void *col, int w, const uint8_t *valid, long long n, long long *out2, cudaStream_t st,
-                          long long *launches)
-{
-    minmax_init_kernel<<<1, 1, 0, st>>>(out2);
-    ++*launches;
-    if (n > 0) {
-        long long blocks = (n + 255) / 256;
-        if (blocks > 148 * 8) blocks = 148 * 8;
-        minmax_kernel<<<(unsigned)blocks, 256, 0, st>>>(col, w, valid, n, out2);
-        ++*launches;
-    }
-    return cudaGetLastError();
+    return e;
 }
 
 }  // namespace ng

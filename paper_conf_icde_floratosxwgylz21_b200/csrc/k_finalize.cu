@@ -1,0 +1,196 @@
+// k_finalize.cu -- a8 (aggregate finalize + outer comparison) and a9
+// (ordered compaction of the survivors), plus the partial-aggregate init and
+// the column min/max used by the SUM/AVG overflow pre-check.
+//
+// PAPER.md P:183 (§III-B, Fig. 4): after the subquery loop fills Res[i], the
+// drive program runs "Selection(=, R.col1, Res)" and materialises the result
+// (0-1 vector -> prefix sum -> materialize).  Here one kernel computes
+// Res[i] from the per-tuple partial aggregates with the SQL empty-set rules
+// (readings R1, R2), evaluates a*x OP b*v exactly in int128 (R6, R7) and
+// compacts the survivors in row order with a decoupled look-back.
+#include <climits>
+
+#include "internal.h"
+#include "scan.cuh"
+
+namespace ng {
+
+constexpr int F_THREADS = 256;
+constexpr int F_WARPS = F_THREADS / 32;
+constexpr int F_ITEMS = 16;
+constexpr int F_TILE = F_THREADS * F_ITEMS;
+
+size_t finalize_scratch_bytes(long long n)
+{
+    long long tiles = (n + F_TILE - 1) / F_TILE;
+    return (size_t)(tiles + 1) * 8 + 256;
+}
+
+// ------------------------------------------------------------------ a8 + a9
+// round_half_away_from_zero(num / den), den > 0 (reading R6).
+__device__ __forceinline__ long long div_round_half_away(__int128 num, long long den)
+{
+    __int128 mag = num < 0 ? -num : num;
+    __int128 q = (2 * mag + den) / (2 * (__int128)den);
+    return (long long)(num < 0 ? -q : q);
+}
+
+__global__ void __launch_bounds__(F_THREADS) finalize_kernel(FinalizeArgs A, unsigned long long *__restrict__ status,
+                                                             unsigned *__restrict__ counter)
+{
+    __shared__ unsigned s_tile;
+    __shared__ unsigned s_cnt[F_ITEMS][F_WARPS];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const long long n = *A.d_nrp;
+    const long long num_tiles = (n + F_TILE - 1) / F_TILE;
+    if (tid == 0) s_tile = atomicAdd(counter, 1u);
+    __syncthreads();
+    const long long tile = s_tile;
+    if (tile >= num_tiles) return;  // grid sized for the R' upper bound
+    const long long base = tile * F_TILE;
+
+    bool flag[F_ITEMS];
+    unsigned rank[F_ITEMS];
+    long long value[F_ITEMS];
+    uint8_t valid[F_ITEMS], pass[F_ITEMS];
+#pragma unroll
+    for (int j = 0; j < F_ITEMS; j++) {
+        const long long i = base + (long long)j * F_THREADS + tid;
+        bool in = i < n;
+        value[j] = 0;
+        valid[j] = 0;
+        pass[j] = 0;
+        if (in) {
+            const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
+            const long long c = kval ? A.cnt[i] : 0;     // NULL key: empty subquery (R2)
+            const long long acc = A.acc[i];
+            bool vv = true;
+            long long v = 0;
+            switch (A.agg) {
+            case MIN: case MAX: case SUM: vv = c > 0; v = acc; break;
+            case COUNT: v = c; break;
+            case AVG: vv = c > 0; if (vv) v = div_round_half_away((__int128)acc * 1000000, c); break;
+            case EXISTS: v = c > 0; break;
+            default: v = c == 0; break;
+            }
+            bool p;
+            if (A.agg == EXISTS || A.agg == NOT_EXISTS) {
+                p = v != 0;
+            } else {
+                const int row = A.ids[i];
+                const bool xv = !(A.x_valid && !A.x_valid[row]);
+                p = false;
+                if (vv && xv) {
+                    const __int128 x = load_w(A.x_col, A.x_w, row);
+                    if (A.agg == AVG)
+                        p = cmp_rt<__int128>((__int128)A.a * x * c, A.outer_op, (__int128)A.b * acc);
+                    else
+                        p = cmp_rt<__int128>((__int128)A.a * x, A.outer_op, (__int128)A.b * v);
+                }
+            }
+            value[j] = vv ? v : 0;
+            valid[j] = vv;
+            pass[j] = p;
+            in = A.emit_all ? true : p;
+        }
+        flag[j] = in;
+        const unsigned m = __ballot_sync(FULL, in);
+        if (lane == 0) s_cnt[j][warp] = __popc(m);
+        rank[j] = __popc(m & lanemask_lt());
+    }
+    const unsigned long long tb = tile_offsets<F_ITEMS, F_THREADS>(s_cnt, status, tile, num_tiles, A.out_count);
+#pragma unroll
+    for (int j = 0; j < F_ITEMS; j++) {
+        if (!flag[j]) continue;
+        const long long i = base + (long long)j * F_THREADS + tid;
+        const long long pos = (long long)tb + s_cnt[j][warp] + rank[j];
+        A.out_ids[pos] = A.row_id_base + A.ids[i];
+        A.out_vals[pos] = value[j];
+        A.out_valid[pos] = valid[j];
+        A.out_passed[pos] = pass[j];
+        if (A.out_sum) {
+            const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
+            A.out_sum[pos] = kval ? A.acc[i] : 0;
+            A.out_cnt[pos] = kval ? A.cnt[i] : 0;
+        }
+    }
+}
+
+cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *launches)
+{
+    cudaError_t e = cudaMemsetAsync(a.out_count, 0, sizeof(long long), st);
+    if (e != cudaSuccess || a.n_rp_max <= 0) return e;
+    e = cudaMemsetAsync(a.scratch, 0, finalize_scratch_bytes(a.n_rp_max), st);
+    if (e != cudaSuccess) return e;
+    const long long tiles = (a.n_rp_max + F_TILE - 1) / F_TILE;
+    finalize_kernel<<<(unsigned)tiles, F_THREADS, 0, st>>>(a, (unsigned long long *)((char *)a.scratch + 256),
+                                                         (unsigned *)a.scratch);
+    ++*launches;
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------ partials
+__global__ void init_partials_kernel(long long n, long long acc0, long long *__restrict__ acc,
+                                     long long *__restrict__ cnt)
+{
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+        acc[i] = acc0;
+        cnt[i] = 0;
+    }
+}
+
+cudaError_t launch_init_partials(long long n, int agg, long long *acc, long long *cnt, cudaStream_t st,
+                                 long long *launches)
+{
+    if (n <= 0) return cudaSuccess;
+    long long acc0 = agg == MIN ? LLONG_MAX : (agg == MAX ? LLONG_MIN : 0);
+    long long blocks = (n + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    init_partials_kernel<<<(unsigned)blocks, 256, 0, st>>>(n, acc0, acc, cnt);
+    ++*launches;
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------ column min / max
+// (for the SUM/AVG overflow pre-check, reading R5)
+__global__ void minmax_init_kernel(long long *out)
+{
+    out[0] = LLONG_MAX;
+    out[1] = LLONG_MIN;
+}
+
+__global__ void minmax_kernel(const void *__restrict__ col, int w, const uint8_t *__restrict__ valid, long long n,
+                              long long *__restrict__ out)
+{
+    long long mn = LLONG_MAX, mx = LLONG_MIN;
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+        if (valid && !valid[i]) continue;
+        const long long v = load_w(col, w, i);
+        mn = min(mn, v);
+        mx = max(mx, v);
+    }
+    for (int o = 16; o > 0; o >>= 1) {
+        mn = min(mn, __shfl_xor_sync(FULL, mn, o));
+        mx = max(mx, __shfl_xor_sync(FULL, mx, o));
+    }
+    if ((threadIdx.x & 31) == 0) {
+        atomicMin(&out[0], mn);
+        atomicMax(&out[1], mx);
+    }
+}
+
+cudaError_t launch_minmax(const void *col, int w, const uint8_t *valid, long long n, long long *out2, cudaStream_t st,
+                          long long *launches)
+{
+    minmax_init_kernel<<<1, 1, 0, st>>>(out2);
+    ++*launches;
+    if (n > 0) {
+        long long blocks = (n + 255) / 256;
+        if (blocks > 148 * 8) blocks = 148 * 8;
+        minmax_kernel<<<(unsigned)blocks, 256, 0, st>>>(col, w, valid, n, out2);
+        ++*launches;
+    }
+    return cudaGetLastError();
+}
+
+}  // namespace ng
