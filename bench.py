@@ -52,6 +52,9 @@ def parse_args():
     ap.add_argument("--impl", choices=("ours", "reference"), default="ours")
     ap.add_argument("--workload", default="C2", choices=("C2", "C1", "C5"))
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--dedup", action="store_true",
+                    help="headline with P:331 caching (one subquery evaluation per distinct correlated value)")
+    ap.add_argument("--no-variants", action="store_true", help="skip the with/without-caching side measurement")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="CPU oracle sample budget")
     ap.add_argument("--out", default=None, help="also append the JSON line to this file")
@@ -179,11 +182,11 @@ def bnl_roofline(profs, n_r, n_s, sm_max_mhz, workload_name):
     CUDA events on the engine stream around the kernel."""
     t_act = t_ideal = ops = 0.0
     per = {}
-    for plan, mode, prof in profs:
+    for plan, mode, prof, n_eval in profs:
         agg = plan["agg"]
         if mode != "bnl" or agg not in PAIRS_PER_SM_CLK:
             continue
-        pairs = float(n_r) * n_s
+        pairs = float(n_eval) * n_s   # outer keys evaluated (distinct ones with caching) x |S'|
         ideal = pairs / (148 * PAIRS_PER_SM_CLK[agg] * sm_max_mhz * 1e6)
         act = prof["subquery"] / 1000.0
         t_act += act
@@ -287,7 +290,7 @@ def main():
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     row_base = ngd.shard_range(n_r * world, rank, world)[0]
 
-    def step(profile_sink=None):
+    def step(profile_sink=None, dedup=args.dedup):
         """One pass of the hot path over the batch (all plans)."""
         m = eng.mark()
         need_index = any(mode == "index" for _, mode in plans)
@@ -303,12 +306,14 @@ def main():
                 ngd.broadcast_tensors([eng.arena_view(info["d_keys"], n_idx * 4),
                                        eng.arena_view(info["d_payload"], n_idx * 4)])
         surv = []
+        evals.clear()
         gathered = []
         for plan, mode in plans:
-            res = eng.exec(plan, Rc, Sc, index=idx if mode == "index" else -1, row_id_base=row_base)
+            res = eng.exec(plan, Rc, Sc, index=idx if mode == "index" else -1, row_id_base=row_base, dedup=dedup)
             surv.append(res.n_rows)
+            evals.append(res.n_evaluated)
             if profile_sink is not None:
-                profile_sink.append((plan, mode, eng.last_profile()))
+                profile_sink.append((plan, mode, eng.last_profile(), res.n_evaluated))
             if world > 1:
                 t = eng.result_tensors(res)
                 gathered.append((t["row"].clone(), t["value"].clone()))
@@ -319,6 +324,7 @@ def main():
         eng.release(m)
         return surv
 
+    evals = []
     eng.set_profiling(True)
     for _ in range(args.warmup):
         step()
@@ -341,6 +347,7 @@ def main():
             step_ms.append(e0.elapsed_time(e1))
     torch.cuda.synchronize()
     launches = eng.launch_count() - launches0
+    evals_main = list(evals)
     if world > 1:
         dist.barrier()
     total_ms = ngd.max_over_ranks(sum(step_ms), device=dev)
@@ -353,10 +360,27 @@ def main():
     sm_max = pk.get("sm_max_mhz") or clocks.summary().get("sm_max_mhz") or 1965.0
     roofline = bnl_roofline(profs, n_r, n_s, sm_max, args.workload)
     stages = {}
-    for _, _, prof in profs:
+    for _, _, prof, _ in profs:
         for k, v in prof.items():
             if v == v:  # not NaN
                 stages[k] = stages.get(k, 0.0) + v / args.steps
+
+    # ---- side measurement: the same step with the other caching setting
+    variant = None
+    if not args.no_variants:
+        vms = []
+        for _ in range(max(1, args.steps)):
+            flush.zero_()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            step(dedup=not args.dedup)
+            e1.record(stream)
+            e1.synchronize()
+            vms.append(e0.elapsed_time(e1))
+        v_ms = ngd.max_over_ranks(sum(vms), device=dev) / len(vms)
+        variant = {"dedup": not args.dedup, "value": outer_per_step / (v_ms / 1000.0), "ms_per_step": v_ms,
+                   "subquery_evaluations_per_plan": list(evals)}
 
     # ---- e2e through the public API with host buffers
     e2e = None
@@ -376,7 +400,8 @@ def main():
             idx = eng.build_index(Sx, ["col1"], "col2") if any(md == "index" for _, md in plans) else -1
             nb = 0
             for plan, mode in plans:
-                res = eng.exec(plan, Rx, Sx, index=idx if mode == "index" else -1, row_id_base=row_base)
+                res = eng.exec(plan, Rx, Sx, index=idx if mode == "index" else -1, row_id_base=row_base,
+                           dedup=args.dedup)
                 out = eng.result_to_numpy(res)
                 nb += sum(a.nbytes for a in out.values())
             eng.release(m)
@@ -404,7 +429,7 @@ def main():
         if not args.no_cpu_baseline:
             cpu = time_oracle({"R": R, "S": S_host}, plans, args.cpu_seconds)
         latency = {}
-        for plan, mode, prof in profs:
+        for plan, mode, prof, _ in profs:
             key = "%s %s (%s)" % (plan["corr_op"], plan["agg"], mode)
             latency.setdefault(key, []).append(prof["total"])
         line = {
@@ -424,6 +449,9 @@ def main():
             "query_latency_ms": {k: statistics.median(v) for k, v in latency.items()},
             "stages_ms_per_step": stages,
             "survivors_per_plan": surv,
+            "dedup": args.dedup,
+            "subquery_evaluations_per_plan": evals_main,
+            "variant": variant,
             "step_ms": step_ms,
         }
         emit(line, args)

@@ -47,7 +47,7 @@
 extern "C" {
 #endif
 
-#define NESTGPU_ABI_VERSION 1
+#define NESTGPU_ABI_VERSION 2
 
 typedef int32_t nestgpu_status;
 enum {
@@ -207,10 +207,16 @@ typedef struct {
     int32_t index;                                            /* -1: tiled nested loop over S'; else index id */
     int64_t row_id_base;                                      /* added to emitted row ids (R shard offset) */
     int32_t emit_all;                                         /* 0: survivors only; 1: every R' tuple */
+    int32_t dedup;                                            /* 1: evaluate the subquery once per distinct
+                                                                 correlated value and reuse the result for
+                                                                 duplicates ("Caching"); 0: once per
+                                                                 R' tuple.  Same result either way. */
 } nestgpu_plan;
 
 typedef struct {
     int64_t n_rows;               /* survivors, or |R'| if emit_all */
+    int64_t n_evaluated;          /* subquery evaluations performed: |R'|, or the number of
+                                     distinct correlated values with dedup */
     const int64_t *d_row_ids;     /* ascending R row ids (+ row_id_base) */
     const int64_t *d_values;      /* Res[i]: MIN/MAX/SUM value, COUNT, AVG rounded at
                                      scale+6 (reading R6), EXISTS 0/1 */
@@ -226,7 +232,8 @@ typedef struct {
  * and inner predicates must match the plan: INVALID otherwise); index == -1:
  * S is filtered here and the tiled block-nested-loop kernel runs.  Work is
  * enqueued on the context stream; the call synchronises once at the end to
- * read the survivor count.  Errors: INVALID, TYPE, UNSUPPORTED, OVERFLOW,
+ * read the survivor count (dedup adds two synchronisations: to plan the sort
+ * of R' keys and to size the evaluation of the distinct keys).  Errors: INVALID, TYPE, UNSUPPORTED, OVERFLOW,
  * OOM, CUDA.  Nothing is launched when validation fails. */
 nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *ctx, const nestgpu_plan *plan,
                                        nestgpu_result *out);

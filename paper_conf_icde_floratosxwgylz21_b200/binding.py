@@ -63,11 +63,12 @@ class Plan(ctypes.Structure):
                 ("outer_cmp_col", ctypes.c_int32), ("outer_op", ctypes.c_int32),
                 ("lhs_mult", ctypes.c_int64), ("rhs_mult", ctypes.c_int64),
                 ("index", ctypes.c_int32), ("row_id_base", ctypes.c_int64),
-                ("emit_all", ctypes.c_int32)]
+                ("emit_all", ctypes.c_int32), ("dedup", ctypes.c_int32)]
 
 
 class Result(ctypes.Structure):
-    _fields_ = [("n_rows", ctypes.c_int64), ("d_row_ids", ctypes.c_void_p), ("d_values", ctypes.c_void_p),
+    _fields_ = [("n_rows", ctypes.c_int64), ("n_evaluated", ctypes.c_int64),
+                ("d_row_ids", ctypes.c_void_p), ("d_values", ctypes.c_void_p),
                 ("d_valid", ctypes.c_void_p), ("d_passed", ctypes.c_void_p),
                 ("d_avg_sum", ctypes.c_void_p), ("d_avg_cnt", ctypes.c_void_p)]
 
@@ -289,8 +290,9 @@ class Engine:
         return out.value, {"n": d.n, "key_bytes": d.key_bytes, "payload_bytes": d.payload_bytes,
                            "d_keys": d.d_keys, "d_payload": d.d_payload}
 
-    def exec(self, plan, R, S, index=-1, emit_all=False, row_id_base=0):
-        """Run one plan (datagen.plans dict).  R / S map column names to ids."""
+    def exec(self, plan, R, S, index=-1, emit_all=False, row_id_base=0, dedup=False):
+        """Run one plan (datagen.plans dict).  R / S map column names to ids.
+        dedup: evaluate each distinct correlated value once (P:331 caching)."""
         p = Plan()
         opa, p.n_outer_preds = self._preds(plan["outer_preds"], R)
         ipa, p.n_inner_preds = self._preds(plan["inner_preds"], S)
@@ -311,6 +313,7 @@ class Engine:
         p.index = int(index)
         p.row_id_base = int(row_id_base)
         p.emit_all = 1 if emit_all else 0
+        p.dedup = 1 if dedup else 0
         res = Result()
         self._keep = (opa, ipa)
         self._check(self.lib.nestgpu_exec_correlated(self.ctx, ctypes.byref(p), ctypes.byref(res)))

@@ -18,6 +18,7 @@
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <utility>
 #include <vector>
 
 #include "../../include/nestgpu.h"
@@ -668,23 +669,84 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     if (!ids || !rkeys || (ravalid && !rkvalid) || !acc || !cnt || !counts || !fscr || !kscr || !o_ids || !o_vals ||
         !o_valid || !o_pass || (P->agg == NG_AVG && (!o_sum || !o_cnt)) || (!ix && (!skeys || (vb && !svals))))
         return fail(c, NESTGPU_ERR_OOM, "arena exhausted executing a plan over |R|=%lld |S|=%lld", (long long)nR, (long long)nS);
-    unsigned *extreme = (unsigned *)(counts + 4);   // [2]
-    long long *d_nrp = counts, *d_nsp = counts + 1, *d_out = counts + 2;
+    // counts: [0] |R'| [1] |S'| [2] survivors [3] distinct keys [4] extreme flags (2 x u32)
+    //         [6] AND / [7] OR of the R' keys (dedup sort planning)
+    unsigned *extreme = (unsigned *)(counts + 4);
+    long long *d_nrp = counts, *d_nsp = counts + 1, *d_out = counts + 2, *d_u = counts + 3;
+    unsigned long long *rmask = (unsigned long long *)(counts + 6);
+    // caching: sort buffers, distinct keys and the R' -> distinct map
+    int *pos = nullptr, *tpos = nullptr, *map = nullptr;
+    void *tkeys = nullptr, *ukeys = nullptr, *sscr = nullptr, *gscr = nullptr;
+    unsigned *hist = nullptr, *dbase = nullptr;
+    if (P->dedup) {
+        pos = (int *)salloc(c, (size_t)nR * 4);
+        tpos = (int *)salloc(c, (size_t)nR * 4);
+        map = (int *)salloc(c, (size_t)nR * 4);
+        tkeys = salloc(c, (size_t)nR * kb);
+        ukeys = salloc(c, (size_t)nR * kb);
+        sscr = salloc(c, ng::sort_scratch_bytes(nR));
+        gscr = salloc(c, ng::group_scratch_bytes(nR));
+        hist = (unsigned *)salloc(c, 8 * 256 * 4);
+        dbase = (unsigned *)salloc(c, 8 * 256 * 4);
+        if (!pos || !tpos || !map || !tkeys || !ukeys || !sscr || !gscr || !hist || !dbase)
+            return fail(c, NESTGPU_ERR_OOM, "arena exhausted (dedup buffers for |R|=%lld)", (long long)nR);
+    }
 
     // ------------------------------------------------------------ a2: R'
     prof_begin(c, 5);
     prof_begin(c, 0);
     ng::ValSrc none{nullptr, nullptr, 0};
     CUDA_TRY(c, cudaMemsetAsync(counts, 0, 64, c->stream));
-    CUDA_TRY(c, ng::launch_filter(nR, ops, rks, kb, none, 0, 0, 0, ids, rkeys, rkvalid, nullptr, nullptr, nullptr,
-                                  fscr, d_nrp, c->stream, &c->launches));
+    CUDA_TRY(c, cudaMemsetAsync(rmask, 0xff, 8, c->stream));   // AND identity
+    CUDA_TRY(c, ng::launch_filter(nR, ops, rks, kb, none, 0, 0, 0, ids, rkeys, rkvalid, nullptr,
+                                  P->dedup ? rmask : nullptr, nullptr, fscr, d_nrp, c->stream, &c->launches));
     prof_end(c, 0);
+
+    // The keys the subquery kernels evaluate: every R' key, or (dedup) each
+    // distinct R' key once -- P:331's cache keyed by the passed-in parameter.
+    const void *eval_keys = rkeys;
+    const long long *d_neval = d_nrp;
+    long long n_eval = nR;
+    long long n_distinct = -1;
+    if (P->dedup) {
+        prof_begin(c, 2);
+        CUDA_TRY(c, cudaMemcpyAsync(c->pinned, counts, 64, cudaMemcpyDeviceToHost, c->stream));
+        CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+        long long nrp;
+        unsigned long long kand, kor;
+        memcpy(&nrp, c->pinned, 8);
+        memcpy(&kand, c->pinned + 12, 8);
+        memcpy(&kor, c->pinned + 14, 8);
+        int shifts[8], np = 0;
+        if (nrp > 1)
+            for (int d = 0; d < kb; d++)
+                if (((kand ^ kor) >> (8 * d)) & 0xff) shifts[np++] = 8 * d;
+        CUDA_TRY(c, ng::launch_iota(pos, nrp, c->stream, &c->launches));
+        CUDA_TRY(c, ng::launch_digit_hist(kb, rkeys, nrp, shifts, np, hist, dbase, c->num_sms, c->stream,
+                                          &c->launches));
+        void *ck = rkeys, *ok = tkeys;
+        int *cv = pos, *ov = tpos;
+        for (int p = 0; p < np; p++) {
+            CUDA_TRY(c, ng::launch_radix_pass(kb, 4, ck, ok, cv, ov, nrp, shifts[p], dbase + p * 256, sscr,
+                                              c->stream, &c->launches));
+            std::swap(ck, ok);
+            std::swap(cv, ov);
+        }
+        CUDA_TRY(c, ng::launch_group(kb, ck, cv, nrp, ukeys, map, d_u, gscr, c->stream, &c->launches));
+        CUDA_TRY(c, cudaMemcpyAsync(c->pinned, d_u, 8, cudaMemcpyDeviceToHost, c->stream));
+        CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+        memcpy(&n_distinct, c->pinned, 8);
+        eval_keys = ukeys;
+        d_neval = d_u;
+        n_eval = n_distinct;
+        prof_end(c, 2);
+    }
 
     // ------------------------------------------------------------ a3 / a5-a7
     if (ix) {
         prof_begin(c, 3);
-        CUDA_TRY(c, ng::launch_range_agg(kb, vb, P->corr_op, P->agg, nR, d_nrp, rkeys, ix->keys, ix->payload, ix->n,
-                                         acc, cnt, kscr, c->stream, &c->launches));
+        CUDA_TRY(c, ng::launch_range_agg(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, ix->keys, ix->payload,
+                                         ix->n, acc, cnt, kscr, c->stream, &c->launches));
         prof_end(c, 3);
     } else {
         prof_begin(c, 1);
@@ -693,11 +755,11 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         CUDA_TRY(c, ng::launch_filter(nS, ips, sks, kb, vs, vb, 1, value_agg ? 1 : 0, nullptr, skeys, nullptr, svals,
                                       nullptr, value_agg ? extreme : nullptr, fscr, d_nsp, c->stream,
                                       &c->launches));
-        CUDA_TRY(c, ng::launch_init_partials(nR, P->agg, acc, cnt, c->stream, &c->launches));
+        CUDA_TRY(c, ng::launch_init_partials(n_eval, P->agg, acc, cnt, c->stream, &c->launches));
         prof_end(c, 1);
         prof_begin(c, 3);
-        CUDA_TRY(c, ng::launch_bnl(kb, vb, P->corr_op, P->agg, nR, d_nrp, rkeys, nS, d_nsp, skeys, svals, extreme, acc,
-                                   cnt, kscr, c->num_sms, c->stream, &c->launches));
+        CUDA_TRY(c, ng::launch_bnl(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, nS, d_nsp, skeys, svals,
+                                   extreme, acc, cnt, kscr, c->num_sms, c->stream, &c->launches));
         prof_end(c, 3);
     }
 
@@ -707,6 +769,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     fa.n_rp_max = nR;
     fa.d_nrp = d_nrp;
     fa.ids = ids;
+    fa.map = map;
     fa.kvalid = rkvalid;
     fa.acc = acc;
     fa.cnt = cnt;
@@ -730,11 +793,12 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     CUDA_TRY(c, ng::launch_finalize(fa, c->stream, &c->launches));
     prof_end(c, 4);
     prof_end(c, 5);
-    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, d_out, 8, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, counts, 32, cudaMemcpyDeviceToHost, c->stream));
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
-    long long nout;
-    memcpy(&nout, c->pinned, 8);
-    out->n_rows = nout;
+    long long cnts[4];
+    memcpy(cnts, c->pinned, 32);
+    out->n_rows = cnts[2];
+    out->n_evaluated = P->dedup ? n_distinct : cnts[0];
     out->d_row_ids = (const int64_t *)o_ids;
     out->d_values = (const int64_t *)o_vals;
     out->d_valid = o_valid;

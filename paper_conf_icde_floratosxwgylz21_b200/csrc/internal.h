@@ -62,11 +62,19 @@ cudaError_t launch_bnl(int kb, int vb, int op, int agg, long long n_rp_max, cons
                        const void *svals, const unsigned *extreme, long long *acc, long long *cnt,
                        void *scratch, int num_sms, cudaStream_t st, long long *launches);
 
+// Caching: R' positions 0..n-1; distinct keys of a sorted key run
+// and the map R' position -> distinct id.
+cudaError_t launch_iota(int *out, long long n, cudaStream_t st, long long *launches);
+size_t group_scratch_bytes(long long n);
+cudaError_t launch_group(int kb, const void *sorted_keys, const int *sorted_pos, long long n, void *uniq_keys, int *map,
+                         long long *d_u, void *scratch, cudaStream_t st, long long *launches);
+
 // a8 + a9: aggregate finalize, outer comparison, ordered compaction.
 struct FinalizeArgs {
     long long n_rp_max;
     const long long *d_nrp;
     const int *ids;          // R' row ids
+    const int *map;          // R' position -> partial-aggregate slot (nullable = identity)
     const uint8_t *kvalid;   // R' key not NULL (nullable = all valid)
     const long long *acc, *cnt;
     const void *x_col;       // outer comparison column (nullable for EXISTS)

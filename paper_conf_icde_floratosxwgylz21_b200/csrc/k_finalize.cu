@@ -62,8 +62,9 @@ __global__ void __launch_bounds__(F_THREADS) finalize_kernel(FinalizeArgs A, uns
         pass[j] = 0;
         if (in) {
             const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
-            const long long c = kval ? A.cnt[i] : 0;     // NULL key: empty subquery (R2)
-            const long long acc = A.acc[i];
+            const long long g = A.map ? (long long)A.map[i] : i;  // cached result slot
+            const long long c = kval ? A.cnt[g] : 0;     // NULL key: empty subquery (R2)
+            const long long acc = A.acc[g];
             bool vv = true;
             long long v = 0;
             switch (A.agg) {
@@ -110,8 +111,9 @@ __global__ void __launch_bounds__(F_THREADS) finalize_kernel(FinalizeArgs A, uns
         A.out_passed[pos] = pass[j];
         if (A.out_sum) {
             const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
-            A.out_sum[pos] = kval ? A.acc[i] : 0;
-            A.out_cnt[pos] = kval ? A.cnt[i] : 0;
+            const long long g = A.map ? (long long)A.map[i] : i;
+            A.out_sum[pos] = kval ? A.acc[g] : 0;
+            A.out_cnt[pos] = kval ? A.cnt[g] : 0;
         }
     }
 }

@@ -13,14 +13,17 @@ def load(eng, tables, dtypes=None):
     return R, S
 
 
-def run(eng, tables, plan, mode="bnl", emit_all=True, dtypes=None, row_id_base=0):
+def run(eng, tables, plan, mode="bnl", emit_all=True, dtypes=None, row_id_base=0, dedup=False, with_res=False):
     """mode: 'bnl' (index=-1) or 'index' (build the index first)."""
     m = eng.mark()
     try:
         R, S = load(eng, tables, dtypes)
         idx = eng.index_for_plan(plan, S) if mode == "index" else -1
-        res = eng.exec(plan, R, S, index=idx, emit_all=emit_all, row_id_base=row_id_base)
-        return eng.result_to_numpy(res)
+        res = eng.exec(plan, R, S, index=idx, emit_all=emit_all, row_id_base=row_id_base, dedup=dedup)
+        out = eng.result_to_numpy(res)
+        if with_res:
+            out["n_evaluated"] = res.n_evaluated
+        return out
     finally:
         eng.release(m)
 

@@ -29,9 +29,9 @@ def test_bnl_roofline_arithmetic():
     # a MIN launch exactly at the ALU bound and a COUNT launch at half its bound
     t_min = n * n / (148 * 32 * 1965e6) * 1000
     t_cnt = 2 * n * n / (148 * 64 * 1965e6) * 1000
-    profs = [(make_plan(">", "min", "="), "bnl", {"subquery": t_min}),
-             (make_plan(">", "count", "="), "bnl", {"subquery": t_cnt}),
-             (make_plan("=", "min", "="), "index", {"subquery": 0.1})]
+    profs = [(make_plan(">", "min", "="), "bnl", {"subquery": t_min}, n),
+             (make_plan(">", "count", "="), "bnl", {"subquery": t_cnt}, n),
+             (make_plan("=", "min", "="), "index", {"subquery": 0.1}, n)]
     r = bench.bnl_roofline(profs, n, n, 1965.0, "C2")
     ideal = t_min + t_cnt / 2
     assert abs(r["frac"] - ideal / (t_min + t_cnt)) < 1e-9

@@ -144,6 +144,33 @@ def test_degenerate(eng, mode):
             assert_parity(run(eng, t, plan, mode, emit_all=True), ref, plan, True, ctx=(preds, agg))
 
 
+# ------------------------------------------------------------------ caching
+@pytest.mark.parametrize("mode", MODES)
+def test_dedup_caching(eng, mode):
+    """dedup = evaluate each distinct correlated value once and reuse the
+    result: identical results to the oracle, and the number of
+    evaluations equals the number of distinct R' keys."""
+    cases = [("c1", query1.config("C1"), {}),
+             ("nulls", query1.random_small(3, n_r=9001, n_s=13007, key_hi=300, val_lo=-50, val_hi=50,
+                                           null_frac=0.1), {"outer_preds": [{"col": "col3", "op": "<=", "lit": 1}]}),
+             ("zipf", query1.tables(n_r=50000, n_s=40000, key_hi=1 << 12, val_hi=16, seed=5, zipf=1.0), {})]
+    for name, t, extra in cases:
+        for corr_op in PLAN_OPS:
+            for agg in AGGS:
+                plan = make_plan(corr_op, agg, "<=", **extra)
+                ref = oracle.evaluate(t, plan)
+                g = run(eng, t, plan, mode, emit_all=True, dedup=True, with_res=True)
+                assert_parity(g, ref, plan, True, ctx=(name, mode, corr_op, agg))
+                rp = ref["in_rp"].astype(bool)
+                assert g["n_evaluated"] == len(np.unique(t["R"]["col1"][rp]))
+    # composite keys
+    t = query1.random_small(6, n_r=7000, n_s=9000, key_hi=20, null_frac=0.0)
+    for agg in AGGS:
+        plan = make_plan("=", agg, ">", outer_key=["col1", "col3"], inner_key=["col1", "col3"])
+        ref = oracle.evaluate(t, plan)
+        assert_parity(run(eng, t, plan, mode, emit_all=True, dedup=True), ref, plan, True, ctx=("composite", agg))
+
+
 # ------------------------------------------------------------------ C2-shaped
 @pytest.mark.parametrize("zipf", [None, 1.0])
 def test_c2_shaped_reduced(eng, zipf):
