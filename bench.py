@@ -171,8 +171,9 @@ def ncu_traffic(workload_name):
 # Pipe-bound pair rate of each nested-loop variant (pairs / clk / SM), from its
 # SASS: MIN/MAX issue ISETP + predicated VIMNMX, both on
 # the ALU pipe (64 lanes/clk/SM) -> 32 pairs/clk; COUNT issues ISETP (ALU) +
-# predicated IMAD (FMA-heavy, 64 lanes/clk/SM) -> 64 pairs/clk.
-PAIRS_PER_SM_CLK = {"min": 32.0, "max": 32.0, "count": 64.0}
+# predicated IMAD (FMA-heavy, 64 lanes/clk/SM) -> 64 pairs/clk; SUM/AVG (small
+# payloads) ISETP + 2 predicated IMADs (FMA-heavy) -> 32 pairs/clk.
+PAIRS_PER_SM_CLK = {"min": 32.0, "max": 32.0, "count": 64.0, "sum": 32.0, "avg": 32.0}
 OPS_PER_PAIR = 2.0   # algorithmic: one compare + one combine per (r, s) pair
 
 

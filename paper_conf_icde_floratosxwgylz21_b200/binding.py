@@ -15,7 +15,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libnestgpu.so")
+LIB_PATH = os.environ.get("NESTGPU_LIB") or os.path.join(_HERE, "libnestgpu.so")
 
 OK, ERR_INVALID, ERR_OOM, ERR_TYPE, ERR_UNSUPPORTED, ERR_OVERFLOW, ERR_CUDA, ERR_BUFFER = 0, -1, -2, -3, -4, -5, -6, -7
 DT = {"int32": 0, "int64": 1, "decimal": 2, "date": 3, "decimal32": 4}

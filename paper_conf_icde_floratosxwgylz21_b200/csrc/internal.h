@@ -20,7 +20,8 @@ namespace ng {
 //   keymask    : if non-null, [0] &= and [1] |= every survivor's encoded key
 //                (radix digits where they agree need no sort pass)
 //   extreme    : if non-null, [0] |= any survivor payload == max of its type,
-//                [1] |= any == min (for the MIN/MAX identity check)
+//                [1] |= any == min (for the MIN/MAX identity check),
+//                (u64)[2..3] = max |payload| (atomicMax; 32-bit partial sums)
 //   scratch    : tile status + counter, from filter_scratch_bytes(n)
 //   out_count  : int64 survivor count (device)
 size_t filter_scratch_bytes(long long n);

@@ -31,10 +31,16 @@
 
 namespace ng {
 
+#ifndef NG_B_RPT
+#define NG_B_RPT 8
+#endif
+#ifndef NG_B_STAGES
+#define NG_B_STAGES 3
+#endif
 constexpr int B_THREADS = 256;
-constexpr int B_RPT = 8;
+constexpr int B_RPT = NG_B_RPT;        // outer tuples per thread (register blocking)
 constexpr int B_RBLOCK = B_THREADS * B_RPT;
-constexpr int B_STAGES = 4;
+constexpr int B_STAGES = NG_B_STAGES;  // shared-memory ring depth
 constexpr int B_STAGE_BYTES = 16384;
 
 struct BnlArgs {
@@ -43,7 +49,7 @@ struct BnlArgs {
     const void *rkeys;
     const void *skeys;
     const void *svals;
-    const unsigned *extreme;
+    const unsigned *extreme;   // [0] payload == max, [1] == min, (u64)[2..3] max |payload|
     unsigned one;              // runtime 1 (keeps the IMAD multiplier opaque to ptxas)
     long long *acc;
     long long *cnt;
@@ -137,6 +143,29 @@ __device__ __forceinline__ void sum_if(const K rk, const K sk, const V v, long l
 #undef NG_K32
 #undef NG_SUM_BODY
 
+// c += (r OP s); s32 += (r OP s) ? v : 0 -- ISETP + two predicated IMADs
+// (FMA pipe); s32 is a per-tile partial sum that cannot overflow (checked).
+#define NG_S32_BODY(SETP, KCON)                                                                       \
+    asm("{.reg .pred p;\n\t" SETP "\n\t@p mad.lo.u32 %0, %0, %4, %4;\n\t"                            \
+        "@p mad.lo.s32 %1, %5, %4, %1;}"                                                              \
+        : "+r"(c), "+r"(s32) : KCON((rk)), KCON((sk)), "r"(one), "r"((int)v));
+#define NG_K32(x) "r"((uint32_t)x)
+#define NG_K64(x) "l"((uint64_t)x)
+#define NG_S32_OP(OPS)                                                                                \
+    if constexpr (sizeof(K) == 4) { NG_S32_BODY(NG_SETP2_U32(OPS), NG_K32) }                          \
+    else { NG_S32_BODY(NG_SETP2_U64(OPS), NG_K64) }
+template <int OP, typename K, typename V>
+__device__ __forceinline__ void sum32_if(const K rk, const K sk, const V v, V &s32, unsigned &c, const unsigned one)
+{
+    if constexpr (OP == EQ) { NG_S32_OP("eq") } else if constexpr (OP == NE) { NG_S32_OP("ne") }
+    else if constexpr (OP == LT) { NG_S32_OP("lt") } else if constexpr (OP == LE) { NG_S32_OP("le") }
+    else if constexpr (OP == GT) { NG_S32_OP("gt") } else { NG_S32_OP("ge") }
+}
+#undef NG_S32_OP
+#undef NG_K64
+#undef NG_K32
+#undef NG_S32_BODY
+
 // One (r, s) pair: the whole nested-method inner step.
 //   MIN/MAX: ISETP + predicated IMNMX (both ALU pipe); with TRACK also
 //            "found" (only when some payload equals the MIN/MAX identity).
@@ -152,7 +181,8 @@ __device__ __forceinline__ void pair_step(const K rk, const K sk, const V sv, V 
         if (p) mm = (AGG == MIN) ? min(mm, sv) : max(mm, sv);
         if constexpr (TRACK) found |= p;
     } else if constexpr (AccKind<AGG>::sum) {
-        sum_if<OP>(rk, sk, sv, sm, c, one);
+        if constexpr (TRACK && sizeof(V) == 4) sum32_if<OP>(rk, sk, sv, mm, c, one);
+        else sum_if<OP>(rk, sk, sv, sm, c, one);
     } else if constexpr (AccKind<AGG>::count) {
         count_if<OP>(rk, sk, c, one);
     } else {
@@ -225,7 +255,7 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
     constexpr int KBYTES = BnlTile<K, VB>::KBYTES;
     constexpr V VMAX = VB == 8 ? (V)LLONG_MAX : (V)INT_MAX;
     constexpr V VMIN = VB == 8 ? (V)LLONG_MIN : (V)INT_MIN;
-    constexpr V MM0 = AGG == MIN ? VMAX : VMIN;
+    constexpr V MM0 = AGG == MIN ? VMAX : (AGG == MAX ? VMIN : (V)0);
 
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ __align__(8) unsigned long long full_bar[B_STAGES];
@@ -243,8 +273,13 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
     const long long n_units = n_rb * A.n_sc;
     // MIN/MAX: if some S' payload equals the identity, track "found"
     // explicitly (uniform per launch, flag from the S' filter kernel).
+    // SUM/AVG with 32-bit payloads: when max|payload| * TILE < 2^31 a tile's
+    // partial sum fits int32 -> "ALT" path accumulates it with a predicated
+    // 32-bit IMAD (FMA pipe) and widens once per tile.
     bool track = false;
     if constexpr (AccKind<AGG>::minmax) track = A.extreme[AGG == MIN ? 0 : 1] != 0;
+    if constexpr (AccKind<AGG>::sum && VB == 4)
+        track = *(const unsigned long long *)(A.extreme + 2) < (0x80000000ull / (unsigned long long)TILE);
     const unsigned mul = A.one;
     const K *rkeys = (const K *)A.rkeys;
     const K *skeys = (const K *)A.skeys;
@@ -317,6 +352,15 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
                 }
             }
             ++g;
+            if constexpr (AccKind<AGG>::sum && VB == 4) {
+                if (track) {  // widen the per-tile 32-bit partial sums
+#pragma unroll
+                    for (int i = 0; i < B_RPT; i++) {
+                        sm[i] += (long long)mm[i];
+                        mm[i] = 0;
+                    }
+                }
+            }
             if constexpr (AccKind<AGG>::exists) {
                 bool all = true;
 #pragma unroll

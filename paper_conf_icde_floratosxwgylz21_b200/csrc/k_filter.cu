@@ -143,6 +143,7 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
     unsigned phase = 0u;  // bit s: parity of the next completion of stage s
     int stage = 0;
     bool ext_max = false, ext_min = false;
+    unsigned long long vabs = 0;  // max |payload| over the survivors
     unsigned long long kand = ~0ull, kor = 0ull;
     while (true) {
         const long long tile = s_tile[stage];
@@ -249,6 +250,8 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
                 if (out_vals) ((V *)out_vals)[pos] = v;
                 ext_max |= v == (VB == 8 ? (V)LLONG_MAX : (V)INT_MAX);
                 ext_min |= v == (VB == 8 ? (V)LLONG_MIN : (V)INT_MIN);
+                const unsigned long long a = v < 0 ? 0ull - (unsigned long long)(long long)v : (unsigned long long)v;
+                vabs = a > vabs ? a : vabs;
             }
         }
         __syncthreads();  // stage fully read before it is refilled; s_tile visible
@@ -270,6 +273,12 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
         if (extreme) {
             if (__any_sync(FULL, ext_max) && lane == 0) atomicOr(&extreme[0], 1u);
             if (__any_sync(FULL, ext_min) && lane == 0) atomicOr(&extreme[1], 1u);
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                const unsigned long long b = __shfl_xor_sync(FULL, vabs, o);
+                vabs = b > vabs ? b : vabs;
+            }
+            if (lane == 0 && vabs) atomicMax((unsigned long long *)(extreme + 2), vabs);
         }
     }
 }
