@@ -268,25 +268,29 @@ def main():
     import torch.distributed as dist
     from paper_conf_icde_floratosxwgylz21_b200 import Engine, dist as ngd
 
-    torch.cuda.set_device(local_rank)
-    dev = torch.device("cuda", local_rank)
+    # one process per GPU (NCCL); NESTGPU_DIST_BACKEND=gloo lets several ranks
+    # share one device for functional runs of the multi-rank path
+    dev_idx = local_rank % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(dev_idx)
+    dev = torch.device("cuda", dev_idx)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if ngd.backend_name() == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(ngd.backend_name())
     R, S_host, plans, desc, cfg = workload(args.workload, rank)
     n_r, n_s = len(R["col1"]), len(S_host["col1"])
     stream = torch.cuda.Stream(dev)
     torch.cuda.set_stream(stream)
     need = (n_r + n_s) * 8 * 16 + (256 << 20)
-    eng = Engine(local_rank, arena_bytes=max(need, 1 << 30), stream=stream)
+    eng = Engine(dev_idx, arena_bytes=max(need, 1 << 30), stream=stream)
 
     # ---- resident inputs (untimed): R shard per rank, S on rank 0 then broadcast
     Rc = eng.load_table(R)
-    if rank == 0:
-        Sc = eng.load_table(S_host)
-    else:
-        Sc = {k: eng.alloc_column(n_s, "int32") for k in S_host}
     if world > 1:
-        ngd.broadcast_tensors([eng.arena_view(eng.column_info(Sc[k])["d_values"], n_s * 4) for k in ("col1", "col2")])
+        Sc = ngd.share_table(eng, S_host if rank == 0 else None, ["col1", "col2"], n_s, device=dev)
+    else:
+        Sc = eng.load_table(S_host)
     base_mark = eng.mark()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     row_base = ngd.shard_range(n_r * world, rank, world)[0]
@@ -296,16 +300,9 @@ def main():
         m = eng.mark()
         need_index = any(mode == "index" for _, mode in plans)
         idx = -1
-        if need_index:
-            if rank == 0:
-                idx = eng.build_index(Sc, ["col1"], "col2")
-            if world > 1:
-                n_idx = ngd.broadcast_int(eng.index_info(idx)["n"] if rank == 0 else -1, device=dev)
-                if rank != 0:
-                    idx, info = eng.index_create_empty(Sc, ["col1"], "col2", [], n_idx, 4, 4)
-                info = eng.index_info(idx)
-                ngd.broadcast_tensors([eng.arena_view(info["d_keys"], n_idx * 4),
-                                       eng.arena_view(info["d_payload"], n_idx * 4)])
+        if need_index:   # rank 0 sorts; the index is broadcast to the other ranks
+            idx = (ngd.share_index(eng, Sc, ["col1"], "col2", device=dev) if world > 1
+                   else eng.build_index(Sc, ["col1"], "col2"))
         surv = []
         evals.clear()
         gathered = []

@@ -36,6 +36,7 @@ def _worker(rank, world, port, q):
         s1 = torch.from_numpy(t["S"]["col1"].copy()) if rank == 0 else torch.zeros(len(t["S"]["col1"]), dtype=torch.int32)
         s2 = torch.from_numpy(t["S"]["col2"].copy()) if rank == 0 else torch.zeros(len(t["S"]["col2"]), dtype=torch.int32)
         nS = ngd.broadcast_int(len(s1) if rank == 0 else -1)
+        assert ngd.broadcast_ints([7, rank]) == [7, 0]
         assert nS == len(s1)
         ngd.broadcast_tensors([s1, s2])
         shard = {"R": {k: v[lo:hi] for k, v in t["R"].items()}, "S": {"col1": s1.numpy(), "col2": s2.numpy()}}
