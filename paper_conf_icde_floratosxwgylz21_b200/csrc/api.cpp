@@ -51,6 +51,11 @@ struct IndexRec {
     int32_t payload_col;
     std::vector<nestgpu_pred> inner;
     bool payload_nullable;
+    // index-pruned evaluation (NEXT 3): prefix / suffix aggregates of the
+    // payload per kind (0 MIN, 1 MAX, 2 SUM), built on first use
+    long long *aux_pre[3];
+    long long *aux_suf[3];
+    size_t aux_off[3];
 };
 
 constexpr int PIN_WORDS = 8 * 256 + 64;
@@ -321,8 +326,11 @@ nestgpu_status nestgpu_release(nestgpu_ctx *c, uint64_t m)
     c->hi = c->size;
     for (auto &col : c->cols)
         if (col.alive && col.off >= m) col.alive = false;
-    for (auto &ix : c->idx)
+    for (auto &ix : c->idx) {
         if (ix.alive && ix.off >= m) ix.alive = false;
+        for (int k = 0; k < 3; k++)
+            if (ix.aux_pre[k] && ix.aux_off[k] >= m) ix.aux_pre[k] = ix.aux_suf[k] = nullptr;
+    }
     return NESTGPU_OK;
 }
 
@@ -617,7 +625,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     const int rkb = key_bytes(c, P->outer_key_cols, P->n_key_cols);
     const int skb = key_bytes(c, P->inner_key_cols, P->n_key_cols);
     int kb = (rkb == 8 || skb == 8) ? 8 : 4;
-    const IndexRec *ix = nullptr;
+    IndexRec *ix = nullptr;
     if (P->index >= 0) {
         if (P->index >= (int32_t)c->idx.size() || !c->idx[P->index].alive)
             return fail(c, NESTGPU_ERR_INVALID, "exec: unknown index %d", P->index);
@@ -744,9 +752,34 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
 
     // ------------------------------------------------------------ a3 / a5-a7
     if (ix) {
+        // Index-pruned evaluation (NEXT 3): prefix / suffix aggregates of the
+        // payload make non-equality and SUM/AVG ranges O(1); built once per
+        // index and aggregate kind, kept with the index.
+        const long long *pre = nullptr, *suf = nullptr;
+        if (value_agg && (P->corr_op != NG_EQ || P->agg == NG_SUM || P->agg == NG_AVG)) {
+            const int kind = P->agg == NG_MIN ? 0 : (P->agg == NG_MAX ? 1 : 2);
+            const int akind = kind == 0 ? ng::MIN : (kind == 1 ? ng::MAX : ng::SUM);
+            if (!ix->aux_pre[kind]) {
+                const size_t off = c->lo;
+                long long *ap = (long long *)palloc(c, (size_t)(ix->n + 1) * 8);
+                long long *as = kind < 2 ? (long long *)palloc(c, (size_t)(ix->n + 1) * 8) : nullptr;
+                void *ascr = salloc(c, ng::index_aux_scratch_bytes(ix->n));
+                if (!ap || (kind < 2 && !as) || !ascr) {
+                    c->lo = off;
+                    return fail(c, NESTGPU_ERR_OOM, "arena exhausted (index prefix aggregates)");
+                }
+                CUDA_TRY(c, ng::launch_index_aux(akind, ix->vb, ix->payload, ix->n, ap, as, ascr, c->stream,
+                                                 &c->launches));
+                ix->aux_pre[kind] = ap;
+                ix->aux_suf[kind] = as;
+                ix->aux_off[kind] = off;
+            }
+            pre = ix->aux_pre[kind];
+            suf = ix->aux_suf[kind];
+        }
         prof_begin(c, 3);
         CUDA_TRY(c, ng::launch_range_agg(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, ix->keys, ix->payload,
-                                         ix->n, acc, cnt, kscr, c->stream, &c->launches));
+                                         ix->n, pre, suf, acc, cnt, kscr, c->stream, &c->launches));
         prof_end(c, 3);
     } else {
         prof_begin(c, 1);

@@ -51,10 +51,18 @@ cudaError_t launch_init_partials(long long n, int agg, long long *acc, long long
 // qualifying range(s).  d_nrp: device count of R'.  Long ranges go to a
 // warp-per-range second kernel.
 size_t range_scratch_bytes(long long n_rp_max);
+//   pre / suf: optional prefix / suffix aggregates of the index payload
+//   (launch_index_aux); non-equality and SUM/AVG ranges are then O(1).
 cudaError_t launch_range_agg(int kb, int vb, int op, int agg, long long n_rp_max, const long long *d_nrp,
                              const void *rkeys, const void *skeys, const void *svals, long long ns,
-                             long long *acc, long long *cnt, void *scratch, cudaStream_t st,
-                             long long *launches);
+                             const long long *pre, const long long *suf, long long *acc, long long *cnt,
+                             void *scratch, cudaStream_t st, long long *launches);
+
+// Index-pruned evaluation (NEXT 3): pre[0..n] / suf[0..n] aggregates (MIN,
+// MAX: both; SUM: pre only) of the co-sorted payload of an index.
+size_t index_aux_scratch_bytes(long long n);
+cudaError_t launch_index_aux(int agg, int vb, const void *payload, long long n, long long *pre, long long *suf,
+                             void *scratch, cudaStream_t st, long long *launches);
 
 // a7: tiled block-nested-loop over R' x S'.  d_nrp / d_nsp: device counts.
 size_t bnl_scratch_bytes(long long n_rp_max);

@@ -13,6 +13,14 @@
 // co-sorted payload.  Short ranges are folded by the owning thread; long ones
 // are appended to a work list and folded warp-per-range with coalesced loads
 // and warp reductions (load balance for skewed / non-equality ranges).
+//
+// Index-pruned evaluation (extending P:315's "only scan
+// a portion of table S"): when the index carries prefix / suffix aggregates
+// of its co-sorted payload (built once per index and aggregate kind), a
+// range that is a prefix or suffix of S' -- every non-equality operator --
+// and any SUM/AVG range is answered in O(1) from them instead of scanned:
+//   pre[p] = AGG(payload[0..p)),  suf[p] = AGG(payload[p..N)),  pre[0] =
+//   suf[N] = identity;  SUM uses pre only (sum[a,b) = pre[b] - pre[a]).
 #include <type_traits>
 
 #include "internal.h"
@@ -72,7 +80,8 @@ __device__ __forceinline__ void fold(long long &acc, V v)
 template <typename K, int VB, int OP, int AGG>
 __global__ void __launch_bounds__(R_THREADS)
 range_short_kernel(const long long *__restrict__ d_nrp, const K *__restrict__ rkeys, const K *__restrict__ skeys,
-                   const void *__restrict__ svals_, int N, long long *__restrict__ acc, long long *__restrict__ cnt,
+                   const void *__restrict__ svals_, int N, const long long *__restrict__ pre,
+                   const long long *__restrict__ suf, long long *__restrict__ acc, long long *__restrict__ cnt,
                    LongItem *__restrict__ list, unsigned *__restrict__ list_n)
 {
     using V = typename std::conditional<VB == 8, long long, int>::type;
@@ -95,7 +104,20 @@ range_short_kernel(const long long *__restrict__ d_nrp, const K *__restrict__ rk
     if constexpr (AGG == COUNT || AGG == EXISTS || AGG == NOT_EXISTS) {
         cnt[i] = L;
     } else {
-        if (L <= R_SHORT) {
+        if (pre && (AGG == SUM || OP != EQ)) {   // O(1) from the prefix / suffix aggregates
+            long long a;
+            if constexpr (AGG == SUM) {
+                a = (pre[b0] - pre[a0]) + (pre[b1] - pre[a1]);
+            } else if constexpr (OP == NE) {
+                a = AGG == MIN ? min(pre[lb], suf[ub]) : max(pre[lb], suf[ub]);
+            } else if constexpr (OP == GT || OP == GE) {
+                a = pre[b0];                       // [0, b0)
+            } else {
+                a = suf[a0];                       // [a0, N)
+            }
+            acc[i] = a;
+            cnt[i] = L;
+        } else if (L <= R_SHORT) {
             long long a = AGG == MIN ? LLONG_MAX : (AGG == MAX ? LLONG_MIN : 0);
             for (int s = a0; s < b0; s++) fold<AGG>(a, svals[s]);
             for (int s = a1; s < b1; s++) fold<AGG>(a, svals[s]);
@@ -148,14 +170,14 @@ range_long_kernel(const void *__restrict__ svals_, int N, const LongItem *__rest
 
 template <typename K, int VB, int OP, int AGG>
 static void launch_range_t(long long n_rp_max, const long long *d_nrp, const void *rkeys, const void *skeys,
-                           const void *svals, long long ns, long long *acc, long long *cnt, void *scratch,
-                           cudaStream_t st, long long *launches)
+                           const void *svals, long long ns, const long long *pre, const long long *suf,
+                           long long *acc, long long *cnt, void *scratch, cudaStream_t st, long long *launches)
 {
     unsigned *list_n = (unsigned *)scratch;
     LongItem *list = (LongItem *)((char *)scratch + 256);
     const unsigned blocks = (unsigned)((n_rp_max + R_THREADS - 1) / R_THREADS);
     range_short_kernel<K, VB, OP, AGG><<<blocks, R_THREADS, 0, st>>>(d_nrp, (const K *)rkeys, (const K *)skeys,
-                                                                    svals, (int)ns, acc, cnt, list, list_n);
+                                                                    svals, (int)ns, pre, suf, acc, cnt, list, list_n);
     ++*launches;
     if constexpr (AGG != COUNT && AGG != EXISTS && AGG != NOT_EXISTS) {
         range_long_kernel<VB, OP, AGG><<<148 * 8, R_THREADS, 0, st>>>(svals, (int)ns, list, list_n, acc, cnt);
@@ -165,10 +187,11 @@ static void launch_range_t(long long n_rp_max, const long long *d_nrp, const voi
 
 template <typename K, int VB, int OP>
 static void dispatch_agg(int agg, long long n_rp_max, const long long *d_nrp, const void *rkeys, const void *skeys,
-                         const void *svals, long long ns, long long *acc, long long *cnt, void *scratch,
-                         cudaStream_t st, long long *launches)
+                         const void *svals, long long ns, const long long *pre, const long long *suf, long long *acc,
+                         long long *cnt, void *scratch, cudaStream_t st, long long *launches)
 {
-#define NG_R(A) launch_range_t<K, VB, OP, A>(n_rp_max, d_nrp, rkeys, skeys, svals, ns, acc, cnt, scratch, st, launches)
+#define NG_R(A) launch_range_t<K, VB, OP, A>(n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, \
+                                             launches)
     switch (agg) {
     case MIN: NG_R(MIN); break;
     case MAX: NG_R(MAX); break;
@@ -182,10 +205,11 @@ static void dispatch_agg(int agg, long long n_rp_max, const long long *d_nrp, co
 
 template <typename K, int VB>
 static void dispatch_op(int op, int agg, long long n_rp_max, const long long *d_nrp, const void *rkeys,
-                        const void *skeys, const void *svals, long long ns, long long *acc, long long *cnt,
-                        void *scratch, cudaStream_t st, long long *launches)
+                        const void *skeys, const void *svals, long long ns, const long long *pre, const long long *suf,
+                        long long *acc, long long *cnt, void *scratch, cudaStream_t st, long long *launches)
 {
-#define NG_O(O) dispatch_agg<K, VB, O>(agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, acc, cnt, scratch, st, launches)
+#define NG_O(O) dispatch_agg<K, VB, O>(agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, \
+                                       launches)
     switch (op) {
     case EQ: NG_O(EQ); break;
     case NE: NG_O(NE); break;
@@ -199,19 +223,169 @@ static void dispatch_op(int op, int agg, long long n_rp_max, const long long *d_
 
 cudaError_t launch_range_agg(int kb, int vb, int op, int agg, long long n_rp_max, const long long *d_nrp,
                              const void *rkeys, const void *skeys, const void *svals, long long ns,
-                             long long *acc, long long *cnt, void *scratch, cudaStream_t st, long long *launches)
+                             const long long *pre, const long long *suf, long long *acc, long long *cnt,
+                             void *scratch, cudaStream_t st, long long *launches)
 {
     if (n_rp_max <= 0) return cudaSuccess;
     cudaError_t e = cudaMemsetAsync(scratch, 0, 256, st);
     if (e != cudaSuccess) return e;
     const bool noval = agg == COUNT || agg == EXISTS || agg == NOT_EXISTS;
     if (kb == 4) {
-        if (noval || vb == 4) dispatch_op<uint32_t, 4>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, acc, cnt, scratch, st, launches);
-        else dispatch_op<uint32_t, 8>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, acc, cnt, scratch, st, launches);
+        if (noval || vb == 4) dispatch_op<uint32_t, 4>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, launches);
+        else dispatch_op<uint32_t, 8>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, launches);
     } else {
-        if (noval || vb == 4) dispatch_op<uint64_t, 4>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, acc, cnt, scratch, st, launches);
-        else dispatch_op<uint64_t, 8>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, acc, cnt, scratch, st, launches);
+        if (noval || vb == 4) dispatch_op<uint64_t, 4>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, launches);
+        else dispatch_op<uint64_t, 8>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, launches);
     }
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------ index aggregates
+// pre[p] = AGG(v[0..p)) for p in [0, N]; with SUF, suf[p] = AGG(v[p..N)).
+// Three passes per direction: per-block aggregate, scan of the block
+// aggregates (one CTA), per-block inclusive scan offset by the block prefix.
+constexpr int P_THREADS = 256;
+constexpr int P_ITEMS = 16;
+constexpr int P_BLOCK = P_THREADS * P_ITEMS;
+
+template <int AGG>
+__device__ __forceinline__ long long comb(long long a, long long b)
+{
+    if constexpr (AGG == MIN) return min(a, b);
+    else if constexpr (AGG == MAX) return max(a, b);
+    else return a + b;
+}
+template <int AGG>
+constexpr long long ident() { return AGG == MIN ? LLONG_MAX : (AGG == MAX ? LLONG_MIN : 0); }
+
+// element e of the direction's sequence: forward v[e], backward v[N-1-e]
+template <typename V, bool BACK>
+__device__ __forceinline__ long long elem(const V *v, long long N, long long e)
+{
+    return (long long)v[BACK ? N - 1 - e : e];
+}
+
+template <typename V, int AGG, bool BACK>
+__global__ void __launch_bounds__(P_THREADS) block_agg_kernel(const V *__restrict__ v, long long N,
+                                                              long long *__restrict__ bagg)
+{
+    __shared__ long long s_w[P_THREADS / 32];
+    const long long b0 = blockIdx.x * (long long)P_BLOCK;
+    long long a = ident<AGG>();
+    for (int j = 0; j < P_ITEMS; j++) {
+        const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
+        if (e < N) a = comb<AGG>(a, elem<V, BACK>(v, N, e));
+    }
+    for (int o = 16; o > 0; o >>= 1) a = comb<AGG>(a, __shfl_xor_sync(FULL, a, o));
+    if ((threadIdx.x & 31) == 0) s_w[threadIdx.x >> 5] = a;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        long long t = ident<AGG>();
+        for (int w = 0; w < P_THREADS / 32; w++) t = comb<AGG>(t, s_w[w]);
+        bagg[blockIdx.x] = t;
+    }
+}
+
+template <int AGG>
+__global__ void __launch_bounds__(1024) block_scan_kernel(long long *__restrict__ bagg, long long nb)
+{
+    // exclusive scan, one CTA, sequential chunks of 1024
+    __shared__ long long s_carry;
+    __shared__ long long s_w[32];
+    if (threadIdx.x == 0) s_carry = ident<AGG>();
+    __syncthreads();
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (long long base = 0; base < nb; base += 1024) {
+        const long long i = base + threadIdx.x;
+        const long long x = i < nb ? bagg[i] : ident<AGG>();
+        long long incl = x;
+        for (int o = 1; o < 32; o <<= 1) {
+            const long long y = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl = comb<AGG>(incl, y);
+        }
+        if (lane == 31) s_w[warp] = incl;
+        __syncthreads();
+        long long wpre = ident<AGG>();
+        for (int w = 0; w < warp; w++) wpre = comb<AGG>(wpre, s_w[w]);
+        const long long carry = s_carry;
+        const long long up = __shfl_up_sync(FULL, incl, 1);
+        const long long ex_in_chunk = comb<AGG>(wpre, lane ? up : ident<AGG>());
+        __syncthreads();
+        if (i < nb) bagg[i] = comb<AGG>(carry, ex_in_chunk);
+        if (threadIdx.x == 1023) s_carry = comb<AGG>(carry, comb<AGG>(wpre, incl));
+        __syncthreads();
+    }
+}
+
+template <typename V, int AGG, bool BACK>
+__global__ void __launch_bounds__(P_THREADS) block_prefix_kernel(const V *__restrict__ v, long long N,
+                                                                 const long long *__restrict__ bpre,
+                                                                 long long *__restrict__ out)
+{
+    // out has N+1 entries: forward out[e+1] = AGG(v[0..e]); backward
+    // out[N-1-e] = AGG(v[N-1-e..N)); the identity entry is written by block 0.
+    __shared__ long long s_w[P_THREADS / 32];
+    __shared__ long long s_carry;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const long long b0 = blockIdx.x * (long long)P_BLOCK;
+    if (threadIdx.x == 0) s_carry = bpre[blockIdx.x];
+    if (blockIdx.x == 0 && threadIdx.x == 0) out[BACK ? N : 0] = ident<AGG>();
+    __syncthreads();
+    for (int j = 0; j < P_ITEMS; j++) {   // rows of the block in order, 256 at a time
+        const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
+        long long incl = e < N ? elem<V, BACK>(v, N, e) : ident<AGG>();
+        for (int o = 1; o < 32; o <<= 1) {
+            const long long y = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl = comb<AGG>(incl, y);
+        }
+        if (lane == 31) s_w[warp] = incl;
+        __syncthreads();
+        long long wpre = ident<AGG>();
+        for (int w = 0; w < warp; w++) wpre = comb<AGG>(wpre, s_w[w]);
+        const long long carry = s_carry;
+        const long long val = comb<AGG>(carry, comb<AGG>(wpre, incl));
+        if (e < N) out[BACK ? N - 1 - e : e + 1] = val;
+        __syncthreads();
+        if (threadIdx.x == P_THREADS - 1) s_carry = val;
+        __syncthreads();
+    }
+}
+
+template <typename V, int AGG, bool BACK>
+static void scan_dir(const void *v, long long N, long long *out, long long *bagg, cudaStream_t st, long long *launches)
+{
+    const long long nb = (N + P_BLOCK - 1) / P_BLOCK;
+    block_agg_kernel<V, AGG, BACK><<<(unsigned)nb, P_THREADS, 0, st>>>((const V *)v, N, bagg);
+    block_scan_kernel<AGG><<<1, 1024, 0, st>>>(bagg, nb);
+    block_prefix_kernel<V, AGG, BACK><<<(unsigned)nb, P_THREADS, 0, st>>>((const V *)v, N, bagg, out);
+    *launches += 3;
+}
+
+size_t index_aux_scratch_bytes(long long n) { return (size_t)((n + P_BLOCK - 1) / P_BLOCK + 1) * 8; }
+
+cudaError_t launch_index_aux(int agg, int vb, const void *payload, long long n, long long *pre, long long *suf,
+                             void *scratch, cudaStream_t st, long long *launches)
+{
+    if (n <= 0) {
+        const long long id = agg == MIN ? LLONG_MAX : (agg == MAX ? LLONG_MIN : 0);
+        cudaError_t e = cudaMemcpyAsync(pre, &id, 8, cudaMemcpyHostToDevice, st);
+        if (e == cudaSuccess && suf) e = cudaMemcpyAsync(suf, &id, 8, cudaMemcpyHostToDevice, st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);   // &id is a host stack value
+        return e;
+    }
+    long long *bagg = (long long *)scratch;
+#define NG_SCAN(V_)                                                                               \
+    if (agg == MIN) {                                                                             \
+        scan_dir<V_, MIN, false>(payload, n, pre, bagg, st, launches);                            \
+        scan_dir<V_, MIN, true>(payload, n, suf, bagg, st, launches);                             \
+    } else if (agg == MAX) {                                                                      \
+        scan_dir<V_, MAX, false>(payload, n, pre, bagg, st, launches);                            \
+        scan_dir<V_, MAX, true>(payload, n, suf, bagg, st, launches);                             \
+    } else {                                                                                      \
+        scan_dir<V_, SUM, false>(payload, n, pre, bagg, st, launches);                            \
+    }
+    if (vb == 8) { NG_SCAN(long long) } else { NG_SCAN(int) }
+#undef NG_SCAN
     return cudaGetLastError();
 }
 
