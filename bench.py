@@ -363,22 +363,36 @@ def main():
             if v == v:  # not NaN
                 stages[k] = stages.get(k, 0.0) + v / args.steps
 
-    # ---- side measurement: the same step with the other caching setting
-    variant = None
-    if not args.no_variants:
-        vms = []
-        for _ in range(max(1, args.steps)):
+    # ---- side measurements (not the headline): the same step with the other
+    # caching setting, and with every plan on the index path
+    # (index-pruned evaluation).
+    def time_steps(fn, k):
+        ms = []
+        for _ in range(k):
             flush.zero_()
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            step(dedup=not args.dedup)
+            fn()
             e1.record(stream)
             e1.synchronize()
-            vms.append(e0.elapsed_time(e1))
-        v_ms = ngd.max_over_ranks(sum(vms), device=dev) / len(vms)
+            ms.append(e0.elapsed_time(e1))
+        return ngd.max_over_ranks(sum(ms), device=dev) / len(ms)
+
+    variant = None
+    index_variant = None
+    if not args.no_variants:
+        v_ms = time_steps(lambda: step(dedup=not args.dedup), max(1, args.steps))
         variant = {"dedup": not args.dedup, "value": outer_per_step / (v_ms / 1000.0), "ms_per_step": v_ms,
                    "subquery_evaluations_per_plan": list(evals)}
+        saved = list(plans)
+        plans[:] = [(p, "index") for p, _ in saved]
+        step()
+        i_ms = time_steps(step, max(1, args.steps))
+        plans[:] = saved
+        index_variant = {"all_plans_on_index_path": True, "value": outer_per_step / (i_ms / 1000.0),
+                         "ms_per_step": i_ms,
+                         "note": "sorted index + binary search; non-equality ranges from prefix/suffix aggregates"}
 
     # ---- e2e through the public API with host buffers
     e2e = None
@@ -450,6 +464,7 @@ def main():
             "dedup": args.dedup,
             "subquery_evaluations_per_plan": evals_main,
             "variant": variant,
+            "variant_index_pruned": index_variant,
             "step_ms": step_ms,
         }
         emit(line, args)

@@ -1,0 +1,34 @@
+"""Time the index build (S' filter + digit histogram + radix passes) for the
+library in $NESTGPU_LIB: 16M int32 keys + int32 payload (C5 S), 38M int64
+keys (Q4-like), 60M int32 keys + payload."""
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+from paper_conf_icde_floratosxwgylz21_b200 import Engine  # noqa: E402
+
+eng = Engine(0, arena_bytes=8 << 30)
+eng.set_profiling(True)
+rng = np.random.default_rng(0)
+out = []
+for name, k, v in (("16M u32+v32", rng.integers(0, 2 ** 31 - 1, 16_000_000).astype(np.int32),
+                    rng.integers(0, 2 ** 20, 16_000_000).astype(np.int32)),
+                   ("38M u64", (rng.integers(0, 15_000_000, 38_000_000) // 8 * 32).astype(np.int64), None),
+                   ("60M u32+v32", rng.integers(0, 2 ** 26, 60_000_000).astype(np.int32),
+                    rng.integers(0, 5000, 60_000_000).astype(np.int32))):
+    m = eng.mark()
+    cols = {"k": eng.load_column(k)}
+    if v is not None:
+        cols["v"] = eng.load_column(v)
+    best = None
+    for _ in range(3):
+        eng.build_index(cols, ["k"], "v" if v is not None else None)
+        p = eng.last_profile()
+        t = (p["inner_filter"], p["sort"])
+        best = t if best is None or sum(t) < sum(best) else best
+    out.append("%s filter %.3f ms sort %.3f ms" % (name, best[0], best[1]))
+    eng.release(m)
+print(os.path.basename(os.environ.get("NESTGPU_LIB", "default")), " | ".join(out))
