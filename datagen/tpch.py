@@ -227,6 +227,29 @@ def q20(T):
     return {"R": R, "S": S}, plan
 
 
+def q20_levels(T):
+    """The full three-level TPC-H Q20 (subquery in subquery, Fig. 6):
+
+      level 2  p_partkey IN (part WHERE p_name LIKE 'forest%')   uncorrelated
+               -> a host flag column (R10), as in q20
+      level 1  partsupp rows with ps_availqty > 0.5*SUM(l_quantity) of their
+               (partkey, suppkey) lineitems shipped in 1994  -> q20's plan
+      level 0  supplier rows of nation CANADA with s_suppkey IN (level 1's
+               ps_suppkey) -- an IN over the level-1 result set, evaluated
+               as EXISTS(... WHERE ps_suppkey = s_suppkey) (R10b).
+
+    Returns (level1 tables, level1 plan, carry column name in level1's R --
+    the partsupp column level 0's subquery reads --, level0 R table,
+    level0 plan whose S is {"ps_suppkey": <level-1 survivors' ps_suppkey>})."""
+    tables1, plan1 = q20(T)
+    canada = [n for n, _ in NATIONS].index("CANADA")
+    R0 = {"s_suppkey": T["supplier"]["s_suppkey"],
+          "s_canada": (T["supplier"]["s_nationkey"] == canada).astype(np.int32)}
+    plan0 = _plan(corr_op="=", agg="exists", outer_key=["s_suppkey"], inner_key=["ps_suppkey"],
+                  outer_preds=[{"col": "s_canada", "op": "=", "lit": 1}])
+    return tables1, plan1, "ps_suppkey", R0, plan0
+
+
 QUERIES = {"q2": q2, "q5": q5, "q17": q17, "q4": q4, "q20": q20}
 # BASELINE.json configs[2] = C3 (SF1 Q2, Q17), configs[3] = C4 (SF10 Q4, Q20)
 CONFIGS = {"C3": (1.0, ("q2", "q17"), 3), "C4": (10.0, ("q4", "q20"), 5)}

@@ -145,6 +145,15 @@ typedef struct {
     uint8_t *d_valid;    /* n bytes or NULL */
 } nestgpu_column_desc;
 nestgpu_status nestgpu_column_info(const nestgpu_ctx *ctx, int32_t col, nestgpu_column_desc *out);
+/* Materialise a NOT NULL column of n values from row ids on the device:
+ * out[i] = src_col[d_row_ids[i] - row_id_base].  This is the data flow between
+ * the levels of a multi-level nested query (Fig. 6: a level's result
+ * vector feeds the block above it): pass a result's d_row_ids / n_rows and the
+ * row_id_base its plan used.  d_row_ids is borrowed for the call (it may be a
+ * result's pointer, valid until the next exec).  src_col must have no NULLs.
+ * Errors: INVALID, OOM, CUDA. */
+nestgpu_status nestgpu_gather_column(nestgpu_ctx *ctx, int32_t src_col, const int64_t *d_row_ids, int64_t n,
+                                     int64_t row_id_base, int32_t *out_col);
 
 /* ---------------------------------------------------------------- index */
 

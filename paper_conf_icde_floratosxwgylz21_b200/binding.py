@@ -27,7 +27,7 @@ STAGES = ("outer_filter", "inner_filter", "sort", "subquery", "finalize", "total
 # The exported C symbols (tests check that the library exports all of them).
 SYMBOLS = ("nestgpu_create", "nestgpu_destroy", "nestgpu_last_error", "nestgpu_launch_count",
            "nestgpu_set_stream", "nestgpu_mark", "nestgpu_release", "nestgpu_arena_usage",
-           "nestgpu_load_column", "nestgpu_alloc_column", "nestgpu_column_info",
+           "nestgpu_load_column", "nestgpu_alloc_column", "nestgpu_column_info", "nestgpu_gather_column",
            "nestgpu_build_index", "nestgpu_drop_index", "nestgpu_index_info",
            "nestgpu_index_create_empty", "nestgpu_exec_correlated", "nestgpu_result_to_host",
            "nestgpu_set_profiling", "nestgpu_last_profile")
@@ -99,6 +99,7 @@ def load_library(path=LIB_PATH):
         "nestgpu_load_column": (i32, [vp, i32, i32, vp, vp, i64, P(i32)]),
         "nestgpu_alloc_column": (i32, [vp, i32, i32, i64, i32, P(i32)]),
         "nestgpu_column_info": (i32, [vp, i32, P(ColumnDesc)]),
+        "nestgpu_gather_column": (i32, [vp, i32, vp, i64, i64, P(i32)]),
         "nestgpu_build_index": (i32, [vp, P(i32), i32, i32, vp, i32, P(i32)]),
         "nestgpu_drop_index": (i32, [vp, i32]),
         "nestgpu_index_info": (i32, [vp, i32, P(IndexDesc)]),
@@ -233,6 +234,14 @@ class Engine:
         d = ColumnDesc()
         self._check(self.lib.nestgpu_column_info(self.ctx, int(col), ctypes.byref(d)))
         return {"dtype": d.dtype, "scale": d.scale, "n": d.n, "d_values": d.d_values, "d_valid": d.d_valid}
+
+    def gather_column(self, src_col, res, row_id_base=0):
+        """New column = src_col at a result's row ids (multi-level nesting,
+        P:229: one level's survivors feed the block above)."""
+        out = ctypes.c_int32()
+        self._check(self.lib.nestgpu_gather_column(self.ctx, int(src_col), ctypes.c_void_p(res.d_row_ids),
+                                                   int(res.n_rows), int(row_id_base), ctypes.byref(out)))
+        return out.value
 
     def arena_view(self, ptr, nbytes):
         """torch uint8 view of arena bytes [ptr, ptr+nbytes) (for NCCL)."""

@@ -407,6 +407,26 @@ nestgpu_status nestgpu_column_info(const nestgpu_ctx *c, int32_t id, nestgpu_col
     return NESTGPU_OK;
 }
 
+nestgpu_status nestgpu_gather_column(nestgpu_ctx *c, int32_t src_col, const int64_t *d_row_ids, int64_t n,
+                                     int64_t row_id_base, int32_t *out_col)
+{
+    if (!c || !out_col || (n > 0 && !d_row_ids)) return fail(c, NESTGPU_ERR_INVALID, "gather_column: null argument");
+    const Column *src = col_get(c, src_col);
+    if (!src) return fail(c, NESTGPU_ERR_INVALID, "gather_column: unknown column %d", src_col);
+    if (src->valid) return fail(c, NESTGPU_ERR_UNSUPPORTED, "gather_column: source column has NULLs");
+    cudaSetDevice(c->device);
+    const nestgpu_dtype dt = src->dtype;
+    const int32_t scale = src->scale;
+    const void *sd = src->d;
+    int32_t id;
+    nestgpu_status s = new_column(c, dt, scale, n, false, &id);   // may reallocate c->cols
+    if (s) return s;
+    CUDA_TRY(c, ng::launch_gather(dtype_width(dt), sd, (const long long *)d_row_ids, n, row_id_base, c->cols[id].d,
+                                  c->stream, &c->launches));
+    *out_col = id;
+    return NESTGPU_OK;
+}
+
 nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int32_t n_key_cols, int32_t payload_col,
                                    const nestgpu_pred *inner_preds, int32_t n_inner_preds, int32_t *out_index)
 {

@@ -100,4 +100,8 @@ struct FinalizeArgs {
 };
 cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *launches);
 
+// out[i] = src[ids[i] - base] (w = 4 or 8 bytes per value).
+cudaError_t launch_gather(int w, const void *src, const long long *ids, long long n, long long base, void *out,
+                          cudaStream_t st, long long *launches);
+
 }  // namespace ng

@@ -196,3 +196,31 @@ cudaError_t launch_minmax(const void *col, int w, const uint8_t *valid, long lon
 }
 
 }  // namespace ng
+
+namespace ng {
+
+// ------------------------------------------------------------------ gather
+// out[i] = src[ids[i] - base]: materialises a column from a result's row ids
+// (multi-level nesting, Fig. 6 -- a level's survivors feed the next).
+template <typename T>
+__global__ void gather_kernel(const T *__restrict__ src, const long long *__restrict__ ids, long long n,
+                              long long base, T *__restrict__ out)
+{
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        out[i] = src[ids[i] - base];
+}
+
+cudaError_t launch_gather(int w, const void *src, const long long *ids, long long n, long long base, void *out,
+                          cudaStream_t st, long long *launches)
+{
+    if (n <= 0) return cudaSuccess;
+    long long blocks = (n + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    if (w == 4) gather_kernel<int><<<(unsigned)blocks, 256, 0, st>>>((const int *)src, ids, n, base, (int *)out);
+    else gather_kernel<long long><<<(unsigned)blocks, 256, 0, st>>>((const long long *)src, ids, n, base,
+                                                                   (long long *)out);
+    ++*launches;
+    return cudaGetLastError();
+}
+
+}  // namespace ng

@@ -127,3 +127,28 @@ def test_c4(eng, c4, query, mode):
     _groupby_check(tables, plan, g)
     s = run(eng, tables, plan, mode, emit_all=False)
     assert np.array_equal(s["row"], g["row"][g["passed"].astype(bool)])
+
+
+@pytest.mark.parametrize("mode", ["index", "bnl"])
+def test_q20_three_levels(eng, c3, mode):
+    """Full three-level Q20 (Fig. 6) on the GPU: level-1 survivors'
+    ps_suppkey are gathered on the device into level 0's subquery table
+    (nestgpu_gather_column) -- against the oracle run level by level."""
+    from paper_conf_icde_floratosxwgylz21_b200.nested import exec_levels
+    tables1, plan1, carry, R0, plan0 = tpch.q20_levels(c3)
+    r1 = oracle.evaluate(tables1, plan1)
+    rows1 = np.nonzero(r1["passed"])[0]
+    r0 = oracle.evaluate({"R": R0, "S": {"ps_suppkey": tables1["R"][carry][rows1]}}, plan0)
+    m = eng.mark()
+    try:
+        R1 = eng.load_table(tables1["R"])
+        S1 = eng.load_table(tables1["S"])
+        R0c = eng.load_table(R0)
+        res = exec_levels(eng, [
+            {"plan": plan1, "R": R1, "S": S1, "carry": carry, "as": "ps_suppkey", "mode": mode},
+            {"plan": plan0, "R": R0c, "mode": mode}], emit_all=True)
+        g = eng.result_to_numpy(res)
+    finally:
+        eng.release(m)
+    assert_parity(g, r0, plan0, True, ctx=("q20 three levels", mode))
+    assert g["passed"].sum() > 0

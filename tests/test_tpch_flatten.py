@@ -165,3 +165,26 @@ def test_base_table_shapes(base):
     assert np.all(li["l_receiptdate"] > li["l_shipdate"])
     assert set(zip(li["l_partkey"].tolist(), li["l_suppkey"].tolist())) <= pairs
     assert 1 <= len(li["l_orderkey"]) / len(T["orders"]["o_orderkey"]) <= 7
+
+
+def test_q20_three_levels(base, db):
+    """Full TPC-H Q20 (three nesting levels, Fig. 6) by the oracle,
+    level by level (level-1 survivors' ps_suppkey feed level 0's IN), against
+    SQLite running the original nested SQL."""
+    tables1, plan1, carry, R0, plan0 = tpch.q20_levels(base)
+    r1 = oracle.evaluate(tables1, plan1)
+    rows1 = np.nonzero(r1["passed"])[0]
+    S0 = {"ps_suppkey": tables1["R"][carry][rows1]}
+    r0 = oracle.evaluate({"R": R0, "S": S0}, plan0)
+    got = sorted(R0["s_suppkey"][np.nonzero(r0["passed"])[0]].tolist())
+    sql = """
+      SELECT s_suppkey FROM supplier, nation
+      WHERE s_suppkey IN (
+              SELECT ps_suppkey FROM partsupp
+              WHERE ps_partkey IN (SELECT p_partkey FROM part WHERE p_name LIKE 'forest%%')
+                AND 200 * ps_availqty > (SELECT sum(l_quantity) FROM lineitem
+                                         WHERE l_partkey = ps_partkey AND l_suppkey = ps_suppkey
+                                           AND l_shipdate >= %d AND l_shipdate < %d))
+        AND s_nationkey = n_nationkey AND n_name = 'CANADA'""" % (tpch.D_1994_01_01, tpch.D_1995_01_01)
+    exp = sorted(r for (r,) in db.execute(sql))
+    assert got == exp and len(exp) > 0
