@@ -1,0 +1,38 @@
+"""Small workload touching every kernel, for compute-sanitizer runs:
+filter (ordered / unordered), sort + histogram, range (short, long, prefix
+aggregates), nested loop (all agg kinds), dedup (iota / group), finalize,
+gather, minmax."""
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import oracle  # noqa: E402
+from datagen import make_plan, query1  # noqa: E402
+from paper_conf_icde_floratosxwgylz21_b200 import Engine  # noqa: E402
+
+eng = Engine(0, arena_bytes=512 << 20)
+t = query1.random_small(1, n_r=20011, n_s=30011, key_hi=600, val_lo=-50, val_hi=50, null_frac=0.1)
+R, S = eng.load_table(t["R"], t.get("R_valid")), eng.load_table(t["S"], t.get("S_valid"))
+bad = 0
+for mode in ("bnl", "index"):
+    for op in ("=", "!=", "<", ">="):
+        for agg in ("min", "max", "sum", "count", "avg", "exists"):
+            for dedup in (False, True):
+                plan = make_plan(op, agg, "<=", outer_preds=[{"col": "col3", "op": "<=", "lit": 1}],
+                                 inner_preds=[{"col": "col3", "op": "!=", "rhs": "col2"}])
+                idx = eng.index_for_plan(plan, S) if mode == "index" else -1
+                g = eng.result_to_numpy(eng.exec(plan, R, S, index=idx, emit_all=True, dedup=dedup))
+                ref = oracle.evaluate(t, plan)
+                m = ref["in_rp"].astype(bool)
+                ok = np.array_equal(g["row"], ref["row"][m]) and np.array_equal(g["value"], ref["value"][m])
+                bad += not ok
+big = {"k": np.zeros(8, np.int64), "v": np.arange(8, dtype=np.int64)}
+S2 = eng.load_table(big, dtypes={"v": "decimal"})
+R2 = eng.load_table({"k": np.zeros(3, np.int64), "x": np.zeros(3, np.int64)})
+res = eng.exec(make_plan("=", "sum", "<", outer_key=["k"], inner_key=["k"], agg_col="v", outer_cmp_col="x"), R2, S2)
+eng.gather_column(R2["x"], res)
+print("sanitize workload done, mismatches:", bad)
+sys.exit(1 if bad else 0)
