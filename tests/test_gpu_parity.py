@@ -325,3 +325,42 @@ def test_launch_count_and_profile(eng):
         eng.set_profiling(False)
     finally:
         eng.release(m)
+
+
+# ------------------------------------------------------------------ skew extremes
+@pytest.mark.parametrize("mode", MODES)
+def test_all_keys_equal_and_two_keys(eng, mode):
+    """Degenerate key distributions: every S key equal (every radix digit is
+    constant -> no sort pass; one '=' range spans all of S -> the long-range
+    path) and only two distinct keys (one populated digit)."""
+    rng = np.random.default_rng(12)
+    for name, sk in (("one_key", np.full(70001, 5, np.int32)),
+                     ("two_keys", rng.choice(np.array([5, 1 << 20], np.int32), 70001))):
+        t = {"R": {"col1": rng.choice(np.array([4, 5, 6, 1 << 20], np.int32), 5003),
+                   "col2": rng.integers(0, 40, 5003).astype(np.int32)},
+             "S": {"col1": sk, "col2": rng.integers(-100, 100, 70001).astype(np.int32)}}
+        for corr_op in PLAN_OPS:
+            for agg in AGGS:
+                plan = make_plan(corr_op, agg, ">")
+                ref = oracle.evaluate(t, plan)
+                for dedup in (False, True):
+                    assert_parity(run(eng, t, plan, mode, emit_all=True, dedup=dedup), ref, plan, True,
+                                  ctx=(name, mode, corr_op, agg, dedup))
+
+
+def test_c2_zipf_full_size_cached(eng):
+    """C2's Zipf(1.0) variant at full size (1M x 1M) with caching on: the
+    index path ('=') and the nested loop ('<', '>', '!='), oracle on sampled
+    rows + closed form on every row."""
+    t = query1.config("C2z")
+    rng = np.random.default_rng(3)
+    rows = np.unique(rng.integers(0, 1_000_000, 400))
+    for corr_op, agg in query1.C2_SWEEP:
+        plan = make_plan(corr_op, agg, "=")
+        mode = "index" if corr_op == "=" else "bnl"
+        g = run(eng, t, plan, mode, emit_all=True, dedup=True, with_res=True)
+        assert g["n_evaluated"] == len(np.unique(t["R"]["col1"]))
+        ref = oracle.evaluate(t, plan, rows=rows)
+        assert_parity(g, ref, plan, True, rows=rows, ctx=("zipf", corr_op, agg))
+        valid, value, _, _ = ind.closed_form(t["R"]["col1"], t["S"]["col1"], t["S"]["col2"], corr_op, agg)
+        assert np.array_equal(g["valid"].astype(bool), valid) and np.array_equal(g["value"], value)
