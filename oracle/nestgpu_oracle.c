@@ -230,6 +230,60 @@ int oracle_eval(const oplan *P, const int64_t *rows, int64_t n_eval,
     return status;
 }
 
+/*
+ * Type-J subquery results as two-level arrays (§III-B "For
+ * such subqueries, we use a two-level arrays to store the results of
+ * subquery evaluations.  The first level is to store the lengths of variable
+ * results for each subquery evaluation and the second is to store the
+ * results."): for every R row in row order, the multiset
+ *     SELECT S.<agg_col> FROM S WHERE <inner_preds> AND r.key OP s.key
+ * evaluated by a full scan of S in row order (Fig. 2's loop).
+ * Reading R17: the arrays hold the NON-NULL values of the select
+ * list -- their consumers are IN under WHERE semantics (a NULL element never
+ * makes IN TRUE, R10b) and equi-joins (NULL never joins).  A row that fails
+ * the outer predicates (not in R') gets length 0 and in_rp = 0.
+ *   lens   : level 1, one length per evaluated row (always written)
+ *   vals   : level 2, concatenated in row order; NULL => lengths only
+ *   cap    : capacity of vals; -7 if the total exceeds it
+ * Aggregate / outer-comparison fields of the plan are ignored.
+ * Returns 0, -1 (invalid plan) or -7 (vals too small).
+ */
+int oracle_collect(const oplan *P, uint8_t *in_rp, int64_t *lens, int64_t *vals, int64_t cap)
+{
+    if (P->n_corr < 1 || P->n_corr > 2 || P->agg_col < 0) return -1;
+    const ocol *vc = &P->S[P->agg_col];
+    int64_t pos = 0;
+    for (int64_t r = 0; r < P->nR; r++) {
+        int in = 1;
+        for (int k = 0; k < P->n_outer; k++)
+            if (!pred_true(P->R, &P->outer_preds[k], r)) { in = 0; break; }
+        int64_t len = 0;
+        if (in) {
+            for (int64_t s = 0; s < P->nS; s++) {
+                int ok = 1;
+                for (int k = 0; k < P->n_inner && ok; k++)
+                    ok = pred_true(P->S, &P->inner_preds[k], s);
+                for (int k = 0; k < P->n_corr && ok; k++) {
+                    const ocol *rc = &P->R[P->corr[k].outer_col];
+                    const ocol *sc = &P->S[P->corr[k].inner_col];
+                    ok = !is_null(rc, r) && !is_null(sc, s) &&
+                         cmp_i128(rc->v[r], P->corr[k].op, sc->v[s]);
+                }
+                if (!ok || is_null(vc, s)) continue;
+                if (vals) {
+                    if (pos >= cap) return -7;
+                    vals[pos] = vc->v[s];
+                }
+                pos += 1;
+                len += 1;
+            }
+        }
+        if (in_rp) in_rp[r] = (uint8_t)in;
+        lens[r] = len;
+    }
+    return 0;
+}
+
 int oracle_max_threads(void)
 {
 #ifdef _OPENMP

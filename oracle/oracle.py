@@ -89,18 +89,9 @@ def _ptr(a):
     return None if a is None else a.ctypes.data
 
 
-def evaluate(tables, plan, rows=None, s_window=None, threads=0):
-    """Evaluate ``plan`` over ``tables`` (datagen layout: {"R": {name: arr},
-    "S": {...}, optional "R_valid"/"S_valid"}).
-
-    rows     : optional int64 array of R row numbers to evaluate (a sample);
-               default all rows in order.
-    s_window : optional (lo, hi) int64 arrays, per evaluated row, restricting
-               S to rows [lo, hi) -- used to batch many tiny instances.
-    Returns a dict of numpy arrays, one entry per evaluated row:
-    row, in_rp, passed, valid, value, sum, cnt.
-    """
-    lib = _load()
+def _make_plan(tables, plan):
+    """Map (tables, plan dict) onto the C oplan (widening to int64).
+    Returns (oplan, objects to keep alive, nR)."""
     keep = []
 
     def table(name):
@@ -146,6 +137,7 @@ def evaluate(tables, plan, rows=None, s_window=None, threads=0):
     op_arr, n_op = preds(plan["outer_preds"], rnames)
     ip_arr, n_ip = preds(plan["inner_preds"], snames)
     corr = (_Corr * 2)()
+    keep.append(corr)
     for i, (oc, ic) in enumerate(zip(plan["outer_key"], plan["inner_key"])):
         corr[i].outer_col = rnames.index(oc)
         corr[i].inner_col = snames.index(ic)
@@ -165,6 +157,23 @@ def evaluate(tables, plan, rows=None, s_window=None, threads=0):
     P.cmp_col = rnames.index(plan["outer_cmp_col"]) if plan["outer_cmp_col"] else -1
     P.outer_op = OPS[plan["outer_op"]]
     P.a, P.b = plan["lhs_mult"], plan["rhs_mult"]
+
+    return P, keep, nR
+
+
+def evaluate(tables, plan, rows=None, s_window=None, threads=0):
+    """Evaluate ``plan`` over ``tables`` (datagen layout: {"R": {name: arr},
+    "S": {...}, optional "R_valid"/"S_valid"}).
+
+    rows     : optional int64 array of R row numbers to evaluate (a sample);
+               default all rows in order.
+    s_window : optional (lo, hi) int64 arrays, per evaluated row, restricting
+               S to rows [lo, hi) -- used to batch many tiny instances.
+    Returns a dict of numpy arrays, one entry per evaluated row:
+    row, in_rp, passed, valid, value, sum, cnt.
+    """
+    lib = _load()
+    P, keep, nR = _make_plan(tables, plan)
 
     if rows is None:
         rows_arr = None
@@ -197,6 +206,53 @@ def evaluate(tables, plan, rows=None, s_window=None, threads=0):
         raise ValueError("oracle rejected plan (%d)" % st)
     out["row"] = (np.arange(nR, dtype=np.int64) if rows_arr is None else rows_arr)
     return out
+
+
+def collect(tables, plan):
+    """Type-J subquery results as the paper's two-level arrays:
+    for every R row, the non-NULL values of plan["agg_col"] over the S rows
+    that satisfy the inner predicates and the correlation (reading R17).
+    Returns {"in_rp", "lens" (level 1), "offsets" (exclusive prefix of lens,
+    nR + 1 entries), "values" (level 2, per row in S row order)}.  Marshalling
+    only; the arithmetic is oracle_collect in nestgpu_oracle.c."""
+    lib = _load()
+    if not hasattr(lib, "_collect_ready"):
+        lib.oracle_collect.restype = ctypes.c_int
+        lib.oracle_collect.argtypes = [ctypes.c_void_p] * 4 + [ctypes.c_int64]
+        lib._collect_ready = True
+    P, keep, nR = _make_plan(tables, plan)
+    in_rp = np.zeros(nR, np.uint8)
+    lens = np.zeros(nR, np.int64)
+    st = lib.oracle_collect(ctypes.addressof(P), in_rp.ctypes.data, lens.ctypes.data, None, 0)
+    if st != 0:
+        raise ValueError("oracle rejected plan (%d)" % st)
+    total = int(lens.sum())
+    vals = np.zeros(max(total, 1), np.int64)
+    st = lib.oracle_collect(ctypes.addressof(P), None, lens.ctypes.data, vals.ctypes.data, total)
+    if st != 0:
+        raise ValueError("oracle collect failed (%d)" % st)
+    offsets = np.zeros(nR + 1, np.int64)
+    np.cumsum(lens, out=offsets[1:])
+    del keep
+    return {"in_rp": in_rp, "lens": lens, "offsets": offsets, "values": vals[:total]}
+
+
+def in_list(tables, plan, x_col):
+    """x IN (SELECT S.v FROM S WHERE ... correlated ...) per R row, read off
+    the two-level arrays of ``collect`` (the upper-level selection consuming a
+    type-J result).  SQL: TRUE iff x is not NULL and some element
+    equals it (NULL elements are never materialised, reading R17, and never
+    make IN TRUE).  Returns (in_rp, passed) uint8 arrays."""
+    c = collect(tables, plan)
+    x = np.asarray(tables["R"][x_col], dtype=np.int64)
+    xv = (tables.get("R_valid", {}) or {}).get(x_col)
+    passed = np.zeros(len(x), np.uint8)
+    for r in range(len(x)):
+        if not c["in_rp"][r] or (xv is not None and not xv[r]):
+            continue
+        lst = c["values"][c["offsets"][r]:c["offsets"][r + 1]]
+        passed[r] = 1 if any(int(v) == int(x[r]) for v in lst) else 0
+    return c["in_rp"], passed
 
 
 def survivors(res):

@@ -297,3 +297,51 @@ def test_overflow_detected(oracle_lib):
     with pytest.raises(oracle.OracleOverflow):
         oracle.evaluate(t, make_plan("=", "sum", "=", outer_key=["k"], inner_key=["k"],
                                      agg_col="v", outer_cmp_col="x"))
+
+
+# ---------------------------------------------------------------- type-J two-level arrays
+@pytest.mark.parametrize("seed", range(4))
+def test_collect_against_sqlite_join(oracle_lib, seed):
+    """oracle.collect (P:231 two-level arrays) vs SQLite running the unnested
+    JOIN form; NULL keys / payloads / local predicates included."""
+    t = query1.random_small(100 + seed, n_r=40, n_s=35)
+    con = ind._db(t)
+    for corr_op in PLAN_OPS:
+        plan = make_plan(corr_op, "min", "=",
+                         outer_preds=[{"col": "col3", "op": "<=", "lit": 1}],
+                         inner_preds=[{"col": "col3", "op": "!=", "lit": 0}])
+        c = oracle.collect(t, plan)
+        exp = ind.collect_sqlite(t, plan, con)
+        assert set(np.nonzero(c["in_rp"])[0].tolist()) == set(exp)
+        for r in range(len(c["lens"])):
+            got = sorted(c["values"][c["offsets"][r]:c["offsets"][r + 1]].tolist())
+            assert got == exp.get(r, []), (corr_op, r)
+
+
+def test_collect_consistent_with_aggregates(oracle_lib):
+    """Level 1 lengths == AVG's nn, and min / max / sum of each level-2 list ==
+    the (pinned) MIN / MAX / SUM evaluations of the same subquery."""
+    t = query1.random_small(7, n_r=60, n_s=80)
+    for corr_op in PLAN_OPS:
+        c = oracle.collect(t, make_plan(corr_op, "min", "="))
+        ev = {a: oracle.evaluate(t, make_plan(corr_op, a, "=")) for a in ("min", "max", "sum", "avg")}
+        assert np.array_equal(c["lens"], ev["avg"]["cnt"])
+        for r in range(len(c["lens"])):
+            lst = c["values"][c["offsets"][r]:c["offsets"][r + 1]]
+            if len(lst):
+                assert ev["min"]["value"][r] == lst.min() and ev["max"]["value"][r] == lst.max()
+                assert ev["sum"]["value"][r] == lst.sum()
+            else:
+                assert not ev["min"]["valid"][r] and not ev["sum"]["valid"][r]
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_in_list_against_sqlite(oracle_lib, seed):
+    """x IN (correlated type-J subquery) read off the two-level arrays vs
+    SQLite's literal IN (NULL x, NULL elements, empty lists)."""
+    t = query1.random_small(200 + seed, n_r=50, n_s=40)
+    con = ind._db(t)
+    for corr_op in PLAN_OPS:
+        plan = make_plan(corr_op, "min", "=", inner_preds=[{"col": "col3", "op": ">=", "lit": 1}])
+        in_rp, passed = oracle.in_list(t, plan, "col2")
+        assert np.nonzero(passed)[0].tolist() == ind.in_sqlite(t, plan, "col2", con), corr_op
