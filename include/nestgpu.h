@@ -47,7 +47,7 @@
 extern "C" {
 #endif
 
-#define NESTGPU_ABI_VERSION 2
+#define NESTGPU_ABI_VERSION 3
 
 typedef int32_t nestgpu_status;
 enum {
@@ -253,6 +253,65 @@ nestgpu_status nestgpu_result_to_host(nestgpu_ctx *ctx, const nestgpu_result *re
                                       int64_t *row_ids, int64_t *values, uint8_t *valid,
                                       uint8_t *passed, int64_t *avg_sum, int64_t *avg_cnt,
                                       int64_t cap);
+
+/* ---------------------------------------------------------------- type-J results */
+
+/* The result of a type-J (set-valued) correlated subquery
+ *     SELECT S.<agg_col> FROM S WHERE <inner_preds> AND R.key <corr_op> S.key
+ * for every R' tuple, stored as the paper's two-level arrays (§III-B:
+ * "The first level is to store the lengths of variable results for each
+ * subquery evaluation and the second is to store the results").  Level 1 is
+ * given as offsets (lengths = offsets[i+1] - offsets[i]).  Reading R17
+ * (DESIGN.md): level 2 holds the NON-NULL values of the select list (its
+ * consumers -- IN under WHERE semantics and equi-joins -- never match NULL).
+ * Within one list the order is the index order (ascending key); compare
+ * lists as multisets. */
+typedef struct {
+    int64_t n_outer;            /* level-1 entries = |R'| */
+    int64_t n_values;           /* level-2 entries */
+    const int64_t *d_row_ids;   /* [n_outer] R row ids (+ row_id_base), ascending */
+    const int64_t *d_offsets;   /* [n_outer + 1] exclusive prefix sums of the lengths */
+    const int64_t *d_values;    /* [n_values] S.<agg_col> widened to int64 */
+    const int64_t *d_owner;     /* [n_values] row id of the level-1 entry owning the slot */
+} nestgpu_collection;
+
+/* Evaluate a type-J subquery for every R' tuple into two-level arrays.  Uses
+ * the plan's outer_preds, key columns, corr_op, inner_preds, agg_col (the
+ * selected column), index and row_id_base; the aggregate and outer
+ * comparison fields are ignored.  The plan must name an index (index >= 0,
+ * built with payload_col == agg_col and the plan's inner predicates):
+ * with the sorted index every list is one run of the co-sorted payload (two
+ * for '!='), so the arrays are built by binary search + prefix sum + a
+ * load-balanced copy.  index == -1: UNSUPPORTED.  The arrays live in the
+ * scratch pool until the next exec / exec_collect / build_index / release.
+ * Synchronises once (to size level 2).  Errors: INVALID, UNSUPPORTED, OOM
+ * (level 2 does not fit the arena), CUDA. */
+nestgpu_status nestgpu_exec_collect(nestgpu_ctx *ctx, const nestgpu_plan *plan, nestgpu_collection *out);
+
+/* The upper-level selection over a type-J result: keep R' tuple i iff
+ * R.x_col[row] IN (list i) -- TRUE iff x is not NULL and some element equals
+ * it (SQL; "R.col1 IN (...)").  x_col is an R column; rows are
+ * d_row_ids[i] - row_id_base (pass the collection plan's row_id_base).
+ * Output as nestgpu_exec_correlated's (values = 1 for survivors; emit_all = 1:
+ * every level-1 entry with passed = the IN outcome).  The collection must
+ * still be valid; the result lives until the next exec.  NOT IN is not
+ * offered: its NULL semantics need the NULL elements R17 drops.
+ * Errors: INVALID, OOM, CUDA. */
+nestgpu_status nestgpu_collection_in(nestgpu_ctx *ctx, const nestgpu_collection *coll, int32_t x_col,
+                                     int64_t row_id_base, int32_t emit_all, nestgpu_result *out);
+
+/* Materialise a column from device int64 values: out[i] = src[i], valid[i] =
+ * d_valid ? d_valid[i] : 1 (no validity array if d_valid is NULL).  This is
+ * "Res[i] = Materialize(...)" (Fig. 4): it turns a result's d_values /
+ * d_row_ids or a collection's d_values / d_owner into a column that later
+ * plans, indexes and joins read (Fig. 5 join with a subquery;
+ * Fig. 6 levels).  dtype NG_INT32 / NG_DATE / NG_DECIMAL32 narrows: OVERFLOW
+ * (and no column) if a valid value is outside int32.  d_src / d_valid are
+ * borrowed for the call.  Synchronises once when narrowing.
+ * Errors: INVALID, TYPE, OVERFLOW, OOM, CUDA. */
+nestgpu_status nestgpu_column_from_device(nestgpu_ctx *ctx, nestgpu_dtype dtype, int32_t scale,
+                                          const int64_t *d_src, const uint8_t *d_valid, int64_t n,
+                                          int32_t *out_col);
 
 /* Per-stage device times (ms, CUDA events on the context stream) of the last
  * exec / build_index when profiling is on (nestgpu_set_profiling(ctx, 1)).

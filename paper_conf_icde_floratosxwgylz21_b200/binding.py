@@ -30,6 +30,7 @@ SYMBOLS = ("nestgpu_create", "nestgpu_destroy", "nestgpu_last_error", "nestgpu_l
            "nestgpu_load_column", "nestgpu_alloc_column", "nestgpu_column_info", "nestgpu_gather_column",
            "nestgpu_build_index", "nestgpu_drop_index", "nestgpu_index_info",
            "nestgpu_index_create_empty", "nestgpu_exec_correlated", "nestgpu_result_to_host",
+           "nestgpu_exec_collect", "nestgpu_collection_in", "nestgpu_column_from_device",
            "nestgpu_set_profiling", "nestgpu_last_profile")
 
 
@@ -73,6 +74,12 @@ class Result(ctypes.Structure):
                 ("d_avg_sum", ctypes.c_void_p), ("d_avg_cnt", ctypes.c_void_p)]
 
 
+class Collection(ctypes.Structure):
+    _fields_ = [("n_outer", ctypes.c_int64), ("n_values", ctypes.c_int64),
+                ("d_row_ids", ctypes.c_void_p), ("d_offsets", ctypes.c_void_p),
+                ("d_values", ctypes.c_void_p), ("d_owner", ctypes.c_void_p)]
+
+
 _lib = None
 
 
@@ -106,6 +113,9 @@ def load_library(path=LIB_PATH):
         "nestgpu_index_create_empty": (i32, [vp, i64, i32, i32, P(i32), i32, i32, vp, i32, P(IndexDesc), P(i32)]),
         "nestgpu_exec_correlated": (i32, [vp, P(Plan), P(Result)]),
         "nestgpu_result_to_host": (i32, [vp, P(Result), vp, vp, vp, vp, vp, vp, i64]),
+        "nestgpu_exec_collect": (i32, [vp, P(Plan), P(Collection)]),
+        "nestgpu_collection_in": (i32, [vp, P(Collection), i32, i64, i32, P(Result)]),
+        "nestgpu_column_from_device": (i32, [vp, i32, i32, vp, vp, i64, P(i32)]),
         "nestgpu_set_profiling": (i32, [vp, i32]),
         "nestgpu_last_profile": (i32, [vp, P(ctypes.c_float), i32]),
     }
@@ -237,10 +247,12 @@ class Engine:
 
     def gather_column(self, src_col, res, row_id_base=0):
         """New column = src_col at a result's row ids (multi-level nesting,
-        P:229: one level's survivors feed the block above)."""
+        P:229: one level's survivors feed the block above).  `res` is a Result
+        or a (device int64 pointer, n) pair, e.g. a collection's d_owner."""
+        ptr, n = (res.d_row_ids, res.n_rows) if isinstance(res, Result) else res
         out = ctypes.c_int32()
-        self._check(self.lib.nestgpu_gather_column(self.ctx, int(src_col), ctypes.c_void_p(res.d_row_ids),
-                                                   int(res.n_rows), int(row_id_base), ctypes.byref(out)))
+        self._check(self.lib.nestgpu_gather_column(self.ctx, int(src_col), ctypes.c_void_p(ptr), int(n),
+                                                   int(row_id_base), ctypes.byref(out)))
         return out.value
 
     def arena_view(self, ptr, nbytes):
@@ -299,9 +311,7 @@ class Engine:
         return out.value, {"n": d.n, "key_bytes": d.key_bytes, "payload_bytes": d.payload_bytes,
                            "d_keys": d.d_keys, "d_payload": d.d_payload}
 
-    def exec(self, plan, R, S, index=-1, emit_all=False, row_id_base=0, dedup=False):
-        """Run one plan (datagen.plans dict).  R / S map column names to ids.
-        dedup: evaluate each distinct correlated value once (P:331 caching)."""
+    def _plan(self, plan, R, S, index, emit_all, row_id_base, dedup):
         p = Plan()
         opa, p.n_outer_preds = self._preds(plan["outer_preds"], R)
         ipa, p.n_inner_preds = self._preds(plan["inner_preds"], S)
@@ -323,10 +333,53 @@ class Engine:
         p.row_id_base = int(row_id_base)
         p.emit_all = 1 if emit_all else 0
         p.dedup = 1 if dedup else 0
-        res = Result()
         self._keep = (opa, ipa)
+        return p
+
+    def exec(self, plan, R, S, index=-1, emit_all=False, row_id_base=0, dedup=False):
+        """Run one plan (datagen.plans dict).  R / S map column names to ids.
+        dedup: evaluate each distinct correlated value once (P:331 caching)."""
+        p = self._plan(plan, R, S, index, emit_all, row_id_base, dedup)
+        res = Result()
         self._check(self.lib.nestgpu_exec_correlated(self.ctx, ctypes.byref(p), ctypes.byref(res)))
         return res
+
+    # ------------------------------------------------------------ type-J (P:231)
+    def exec_collect(self, plan, R, S, index, row_id_base=0):
+        """Type-J subquery results as two-level arrays (nestgpu_collection);
+        plan["agg_col"] is the selected column, `index` must carry it."""
+        p = self._plan(plan, R, S, index, False, row_id_base, False)
+        coll = Collection()
+        self._check(self.lib.nestgpu_exec_collect(self.ctx, ctypes.byref(p), ctypes.byref(coll)))
+        return coll
+
+    def collection_to_numpy(self, coll):
+        torch = self._torch
+        n, m = coll.n_outer, coll.n_values
+
+        def dev(ptr, k):
+            if k == 0 or not ptr:
+                return np.zeros(0, np.int64)
+            return self.arena_view(ptr, k * 8).view(torch.int64).cpu().numpy()
+
+        return {"row": dev(coll.d_row_ids, n), "offsets": dev(coll.d_offsets, n + 1) if n else np.zeros(1, np.int64),
+                "values": dev(coll.d_values, m), "owner": dev(coll.d_owner, m)}
+
+    def collection_in(self, coll, x_col, row_id_base=0, emit_all=False):
+        """R.x IN (type-J list) for every level-1 entry (nestgpu_collection_in)."""
+        res = Result()
+        self._check(self.lib.nestgpu_collection_in(self.ctx, ctypes.byref(coll), int(x_col), int(row_id_base),
+                                                   1 if emit_all else 0, ctypes.byref(res)))
+        return res
+
+    def column_from_device(self, d_src, n, dtype="int64", d_valid=None, scale=0):
+        """Materialise a column from device int64 values (a result's / a
+        collection's arrays): Res[i] = Materialize(...) of Fig. 4."""
+        out = ctypes.c_int32()
+        self._check(self.lib.nestgpu_column_from_device(self.ctx, DT[dtype], int(scale), ctypes.c_void_p(d_src),
+                                                        ctypes.c_void_p(d_valid) if d_valid else None, int(n),
+                                                        ctypes.byref(out)))
+        return out.value
 
     def result_to_numpy(self, res, avg=None):
         n = res.n_rows

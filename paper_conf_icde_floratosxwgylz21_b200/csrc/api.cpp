@@ -880,6 +880,187 @@ nestgpu_status nestgpu_result_to_host(nestgpu_ctx *c, const nestgpu_result *r, i
     return NESTGPU_OK;
 }
 
+// ---------------------------------------------------------------- type-J results
+nestgpu_status nestgpu_exec_collect(nestgpu_ctx *c, const nestgpu_plan *P, nestgpu_collection *out)
+{
+    if (!c || !P || !out) return fail(c, NESTGPU_ERR_INVALID, "exec_collect: null argument");
+    cudaSetDevice(c->device);
+    memset(out, 0, sizeof *out);
+    if (!valid_op(P->corr_op)) return fail(c, NESTGPU_ERR_INVALID, "exec_collect: bad correlated operator");
+    if (P->n_key_cols == 2 && P->corr_op != NG_EQ)
+        return fail(c, NESTGPU_ERR_UNSUPPORTED, "exec_collect: composite correlation supports '=' only");
+    if (P->index < 0)
+        return fail(c, NESTGPU_ERR_UNSUPPORTED, "exec_collect: type-J results are built from an index (plan.index >= 0)");
+    ng::KeySrc rks, sks;
+    int64_t nR, nS;
+    nestgpu_status s;
+    if ((s = make_key(c, P->outer_key_cols, P->n_key_cols, nR, rks, "outer key"))) return s;
+    if ((s = make_key(c, P->inner_key_cols, P->n_key_cols, nS, sks, "inner key"))) return s;
+    ng::PredSet ops;
+    if ((s = make_preds(c, P->outer_preds, P->n_outer_preds, nR, ops, "outer_preds"))) return s;
+    if (P->index >= (int32_t)c->idx.size() || !c->idx[P->index].alive)
+        return fail(c, NESTGPU_ERR_INVALID, "exec_collect: unknown index %d", P->index);
+    IndexRec *ix = &c->idx[P->index];
+    if (ix->n_key != P->n_key_cols || ix->key_cols[0] != P->inner_key_cols[0] ||
+        (P->n_key_cols == 2 && ix->key_cols[1] != P->inner_key_cols[1]))
+        return fail(c, NESTGPU_ERR_INVALID, "exec_collect: index %d is on different key columns", P->index);
+    if (!same_preds(P->inner_preds, P->n_inner_preds, ix->inner))
+        return fail(c, NESTGPU_ERR_INVALID, "exec_collect: index %d was built with different inner predicates", P->index);
+    if (ix->vb == 0 || ix->payload_col != P->agg_col)
+        return fail(c, NESTGPU_ERR_INVALID, "exec_collect: index %d must carry the selected column %d as payload",
+                    P->index, P->agg_col);
+    const int rkb = key_bytes(c, P->outer_key_cols, P->n_key_cols);
+    const int kb = (rkb == 8 || ix->kb == 8) ? 8 : 4;
+    if (ix->kb != kb)
+        return fail(c, NESTGPU_ERR_UNSUPPORTED, "exec_collect: outer key is 64-bit but index %d has 32-bit keys", P->index);
+
+    c->hi = c->size;  // scratch reset
+    for (int st = 0; st < NESTGPU_N_STAGES; st++) c->ran[st] = false;
+    const bool ravalid = rks.v0 || rks.v1;
+    int *ids = (int *)salloc(c, (size_t)nR * 4);
+    void *rkeys = salloc(c, (size_t)nR * kb);
+    uint8_t *rkvalid = ravalid ? (uint8_t *)salloc(c, (size_t)nR) : nullptr;
+    long long *counts = (long long *)salloc(c, 64);   // [0] |R'| [1] level-2 total
+    void *fscr = salloc(c, ng::filter_scratch_bytes(nR));
+    void *cscr = salloc(c, ng::collect_scratch_bytes(nR));
+    long long *lens = (long long *)salloc(c, (size_t)nR * 8);
+    long long *row_ids = (long long *)salloc(c, (size_t)nR * 8);
+    long long *offsets = (long long *)salloc(c, (size_t)(nR + 1) * 8);
+    if (!ids || !rkeys || (ravalid && !rkvalid) || !counts || !fscr || !cscr || !lens || !row_ids || !offsets)
+        return fail(c, NESTGPU_ERR_OOM, "arena exhausted collecting over |R|=%lld", (long long)nR);
+    ng::ValSrc none{nullptr, nullptr, 0};
+    prof_begin(c, 5);
+    prof_begin(c, 0);
+    CUDA_TRY(c, cudaMemsetAsync(counts, 0, 64, c->stream));
+    CUDA_TRY(c, ng::launch_filter(nR, ops, rks, kb, none, 0, 0, 0, ids, rkeys, rkvalid, nullptr, nullptr, nullptr,
+                                  fscr, counts, c->stream, &c->launches));
+    prof_end(c, 0);
+    prof_begin(c, 3);
+    CUDA_TRY(c, ng::launch_collect_bounds(kb, P->corr_op, nR, counts, ids, rkeys, rkvalid, ix->keys, ix->n,
+                                          P->row_id_base, cscr, lens, row_ids, offsets, counts + 1, c->stream,
+                                          &c->launches));
+    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, counts, 16, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    long long nc[2];
+    memcpy(nc, c->pinned, 16);
+    long long *vals = (long long *)salloc(c, (size_t)(nc[1] > 0 ? nc[1] : 1) * 8);
+    long long *owner = (long long *)salloc(c, (size_t)(nc[1] > 0 ? nc[1] : 1) * 8);
+    if (!vals || !owner)
+        return fail(c, NESTGPU_ERR_OOM, "arena exhausted: the type-J result has %lld values", nc[1]);
+    CUDA_TRY(c, ng::launch_collect_fill(ix->vb, counts, offsets, cscr, row_ids, ix->payload, nc[1], vals, owner,
+                                        c->stream, &c->launches));
+    prof_end(c, 3);
+    prof_end(c, 5);
+    CUDA_TRY(c, cudaGetLastError());
+    out->n_outer = nc[0];
+    out->n_values = nc[1];
+    out->d_row_ids = (const int64_t *)row_ids;
+    out->d_offsets = (const int64_t *)offsets;
+    out->d_values = (const int64_t *)vals;
+    out->d_owner = (const int64_t *)owner;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_collection_in(nestgpu_ctx *c, const nestgpu_collection *coll, int32_t x_col,
+                                     int64_t row_id_base, int32_t emit_all, nestgpu_result *out)
+{
+    if (!c || !coll || !out) return fail(c, NESTGPU_ERR_INVALID, "collection_in: null argument");
+    cudaSetDevice(c->device);
+    memset(out, 0, sizeof *out);
+    const long long n = coll->n_outer;
+    if (n < 0 || coll->n_values < 0 || (n > 0 && (!coll->d_row_ids || !coll->d_offsets)) ||
+        (coll->n_values > 0 && !coll->d_values))
+        return fail(c, NESTGPU_ERR_INVALID, "collection_in: malformed collection");
+    const Column *xc = col_get(c, x_col);
+    if (!xc) return fail(c, NESTGPU_ERR_INVALID, "collection_in: unknown column %d", x_col);
+    // scratch grows below the collection (which must stay intact)
+    int *ids32 = (int *)salloc(c, (size_t)n * 4);
+    long long *cnt = (long long *)salloc(c, (size_t)n * 8);
+    long long *acc = (long long *)salloc(c, (size_t)n * 8);
+    long long *small = (long long *)salloc(c, 64);   // [0] n  [2] survivors
+    void *fscr = salloc(c, ng::filter_scratch_bytes(n));
+    long long *o_ids = (long long *)salloc(c, (size_t)n * 8);
+    long long *o_vals = (long long *)salloc(c, (size_t)n * 8);
+    uint8_t *o_valid = (uint8_t *)salloc(c, (size_t)n);
+    uint8_t *o_pass = (uint8_t *)salloc(c, (size_t)n);
+    if (!ids32 || !cnt || !acc || !small || !fscr || !o_ids || !o_vals || !o_valid || !o_pass)
+        return fail(c, NESTGPU_ERR_OOM, "arena exhausted (collection_in over %lld lists)", n);
+    memcpy(c->pinned + 8 * 256 + 8, &n, 8);
+    CUDA_TRY(c, cudaMemcpyAsync(small, c->pinned + 8 * 256 + 8, 8, cudaMemcpyHostToDevice, c->stream));
+    if (n > 0) CUDA_TRY(c, cudaMemsetAsync(acc, 0, (size_t)n * 8, c->stream));
+    CUDA_TRY(c, ng::launch_in_list(n, (const long long *)coll->d_row_ids, (const long long *)coll->d_offsets,
+                                   (const long long *)coll->d_values, xc->d, dtype_width(xc->dtype), xc->valid,
+                                   row_id_base, ids32, cnt, c->stream, &c->launches));
+    ng::FinalizeArgs fa{};
+    fa.n_rp_max = n;
+    fa.d_nrp = small;
+    fa.ids = ids32;
+    fa.acc = acc;
+    fa.cnt = cnt;
+    fa.x_w = 4;
+    fa.agg = NG_EXISTS;
+    fa.outer_op = NG_EQ;
+    fa.a = fa.b = 1;
+    fa.row_id_base = row_id_base;
+    fa.emit_all = emit_all;
+    fa.out_ids = o_ids;
+    fa.out_vals = o_vals;
+    fa.out_valid = o_valid;
+    fa.out_passed = o_pass;
+    fa.out_count = small + 2;
+    fa.scratch = fscr;
+    CUDA_TRY(c, ng::launch_finalize(fa, c->stream, &c->launches));
+    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, small + 2, 8, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    long long m;
+    memcpy(&m, c->pinned, 8);
+    out->n_rows = m;
+    out->n_evaluated = n;
+    out->d_row_ids = (const int64_t *)o_ids;
+    out->d_values = (const int64_t *)o_vals;
+    out->d_valid = o_valid;
+    out->d_passed = o_pass;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_column_from_device(nestgpu_ctx *c, nestgpu_dtype dtype, int32_t scale, const int64_t *d_src,
+                                          const uint8_t *d_valid, int64_t n, int32_t *out_col)
+{
+    if (!c || !out_col || (n > 0 && !d_src)) return fail(c, NESTGPU_ERR_INVALID, "column_from_device: null argument");
+    cudaSetDevice(c->device);
+    const int w = dtype_width(dtype);
+    const size_t off = c->lo;
+    int32_t id;
+    nestgpu_status s = new_column(c, dtype, scale, n, d_valid != nullptr, &id);
+    if (s) return s;
+    unsigned long long *bad = nullptr;
+    if (w == 4) {
+        bad = (unsigned long long *)salloc(c, 8);
+        if (!bad) {
+            c->cols.pop_back();
+            c->lo = off;
+            return fail(c, NESTGPU_ERR_OOM, "arena exhausted (column_from_device)");
+        }
+        CUDA_TRY(c, cudaMemsetAsync(bad, 0, 8, c->stream));
+    }
+    Column &col = c->cols[id];
+    CUDA_TRY(c, ng::launch_materialize(w, (const long long *)d_src, d_valid, n, col.d, col.valid, bad, c->stream,
+                                       &c->launches));
+    if (w == 4) {
+        CUDA_TRY(c, cudaMemcpyAsync(c->pinned, bad, 8, cudaMemcpyDeviceToHost, c->stream));
+        CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+        unsigned long long nb;
+        memcpy(&nb, c->pinned, 8);
+        if (nb) {
+            c->cols.pop_back();
+            c->lo = off;
+            return fail(c, NESTGPU_ERR_OVERFLOW, "column_from_device: %llu values do not fit a 4-byte column", nb);
+        }
+    }
+    *out_col = id;
+    return NESTGPU_OK;
+}
+
 nestgpu_status nestgpu_set_profiling(nestgpu_ctx *c, int32_t on)
 {
     if (!c) return NESTGPU_ERR_INVALID;

@@ -104,4 +104,25 @@ cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *l
 cudaError_t launch_gather(int w, const void *src, const long long *ids, long long n, long long base, void *out,
                           cudaStream_t st, long long *launches);
 
+// Type-J two-level arrays, k_collect.cu.
+//   bounds: per R' tuple the qualifying runs of the index, lens[i], int64
+//   row_ids[i] (+ base), offsets[0..n] = exclusive prefix of lens, *total =
+//   offsets[n] (all device).
+//   fill  : values[e] = payload of slot e (widened), owner[e] = its row id.
+size_t collect_scratch_bytes(long long n_rp_max);
+cudaError_t launch_collect_bounds(int kb, int op, long long n_rp_max, const long long *d_nrp, const int *ids,
+                                  const void *rkeys, const uint8_t *rkvalid, const void *skeys, long long ns,
+                                  long long base, void *scratch, long long *lens, long long *row_ids,
+                                  long long *offsets, long long *total, cudaStream_t st, long long *launches);
+cudaError_t launch_collect_fill(int vb, const long long *d_nrp, const long long *offsets, const void *scratch,
+                                const long long *row_ids, const void *payload, long long total, long long *values,
+                                long long *owner, cudaStream_t st, long long *launches);
+// IN over a two-level array: cnt[i] = x(row_ids[i]-base) in list i; ids32[i] = row_ids[i] - base.
+cudaError_t launch_in_list(long long n, const long long *row_ids, const long long *offsets, const long long *values,
+                           const void *x_col, int x_w, const uint8_t *x_valid, long long base, int *ids32,
+                           long long *cnt, cudaStream_t st, long long *launches);
+// out = (int32|int64) src with validity; *bad += valid values outside int32 (w == 4).
+cudaError_t launch_materialize(int w, const long long *src, const uint8_t *valid_in, long long n, void *out,
+                               uint8_t *valid_out, unsigned long long *bad, cudaStream_t st, long long *launches);
+
 }  // namespace ng
