@@ -313,6 +313,17 @@ nestgpu_status nestgpu_column_from_device(nestgpu_ctx *ctx, nestgpu_dtype dtype,
                                           const int64_t *d_src, const uint8_t *d_valid, int64_t n,
                                           int32_t *out_col);
 
+/* Ablation knobs -- NOT for production use; they exist to measure the
+ * paper's design claims against their baselines (tools/ablations.py).
+ *   NESTGPU_OPT_MALLOC_SCRATCH (value 0/1): per-exec scratch comes from one
+ *     cudaMalloc per allocation, freed (after a stream sync) at the next
+ *     exec / build_index / exec_collect / release -- the pool-less baseline
+ *     that P:147 ("calling malloc/free ... is unacceptable") and P:233-237
+ *     (memory pools) argue against.  Default 0: the arena pool.
+ * Errors: INVALID (unknown option). */
+enum { NESTGPU_OPT_MALLOC_SCRATCH = 1 };
+nestgpu_status nestgpu_set_option(nestgpu_ctx *ctx, int32_t option, int64_t value);
+
 /* Per-stage device times (ms, CUDA events on the context stream) of the last
  * exec / build_index when profiling is on (nestgpu_set_profiling(ctx, 1)).
  * Stage order: 0 outer filter, 1 inner filter, 2 sort, 3 subquery kernel

@@ -31,7 +31,8 @@ SYMBOLS = ("nestgpu_create", "nestgpu_destroy", "nestgpu_last_error", "nestgpu_l
            "nestgpu_build_index", "nestgpu_drop_index", "nestgpu_index_info",
            "nestgpu_index_create_empty", "nestgpu_exec_correlated", "nestgpu_result_to_host",
            "nestgpu_exec_collect", "nestgpu_collection_in", "nestgpu_column_from_device",
-           "nestgpu_set_profiling", "nestgpu_last_profile")
+           "nestgpu_set_option", "nestgpu_set_profiling", "nestgpu_last_profile")
+OPT_MALLOC_SCRATCH = 1
 
 
 class NestGPUError(RuntimeError):
@@ -116,6 +117,7 @@ def load_library(path=LIB_PATH):
         "nestgpu_exec_collect": (i32, [vp, P(Plan), P(Collection)]),
         "nestgpu_collection_in": (i32, [vp, P(Collection), i32, i64, i32, P(Result)]),
         "nestgpu_column_from_device": (i32, [vp, i32, i32, vp, vp, i64, P(i32)]),
+        "nestgpu_set_option": (i32, [vp, i32, i64]),
         "nestgpu_set_profiling": (i32, [vp, i32]),
         "nestgpu_last_profile": (i32, [vp, P(ctypes.c_float), i32]),
     }
@@ -202,6 +204,10 @@ class Engine:
         a, b = ctypes.c_size_t(), ctypes.c_size_t()
         self._check(self.lib.nestgpu_arena_usage(self.ctx, ctypes.byref(a), ctypes.byref(b)))
         return a.value, b.value
+
+    def set_option(self, option, value):
+        """Ablation knobs (nestgpu_set_option), e.g. OPT_MALLOC_SCRATCH."""
+        self._check(self.lib.nestgpu_set_option(self.ctx, int(option), int(value)))
 
     def set_profiling(self, on=True):
         self._check(self.lib.nestgpu_set_profiling(self.ctx, 1 if on else 0))

@@ -78,6 +78,11 @@ struct nestgpu_ctx {
     std::vector<IndexRec> idx;
     unsigned *pinned;  // host pinned words for small D2H / H2D
     bool profiling;
+    // Ablation knob (NESTGPU_OPT_MALLOC_SCRATCH): scratch comes from
+    // cudaMalloc per allocation, freed at the next scratch reset -- the
+    // pool-less baseline of P:147 / P:233.  Off by default.
+    bool malloc_scratch;
+    std::vector<void *> mallocs;
     cudaEvent_t ev[NESTGPU_N_STAGES][2];
     bool ran[NESTGPU_N_STAGES];
 };
@@ -105,6 +110,17 @@ nestgpu_status fail(nestgpu_ctx *c, nestgpu_status code, const char *fmt, ...)
 
 size_t align_up(size_t x) { return (x + ALIGN - 1) / ALIGN * ALIGN; }
 
+// Start a new scratch generation: everything salloc'd before dies here.
+void scratch_reset(nestgpu_ctx *c)
+{
+    c->hi = c->size;
+    if (!c->mallocs.empty()) {
+        cudaStreamSynchronize(c->stream);
+        for (void *p : c->mallocs) cudaFree(p);
+        c->mallocs.clear();
+    }
+}
+
 void *palloc(nestgpu_ctx *c, size_t bytes)
 {
     size_t b = align_up(bytes + 16);  // +16: bulk copies / vector loads may read a ragged tail
@@ -119,6 +135,12 @@ void *palloc(nestgpu_ctx *c, size_t bytes)
 void *salloc(nestgpu_ctx *c, size_t bytes)
 {
     size_t b = align_up(bytes + 16);
+    if (c->malloc_scratch) {
+        void *p = nullptr;
+        if (cudaMalloc(&p, b) != cudaSuccess) return nullptr;
+        c->mallocs.push_back(p);
+        return p;
+    }
     if (c->hi < c->lo + b) return nullptr;
     c->hi -= b;
     size_t used = c->lo + (c->size - c->hi);
@@ -270,6 +292,7 @@ nestgpu_status nestgpu_create(int device, void *d_arena, size_t arena_bytes, voi
     c->stream = (cudaStream_t)cuda_stream;
     c->launches = 0;
     c->profiling = false;
+    c->malloc_scratch = false;
     if (cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess ||
         cudaMallocHost((void **)&c->pinned, PIN_WORDS * sizeof(unsigned)) != cudaSuccess) {
         delete c;
@@ -289,6 +312,7 @@ nestgpu_status nestgpu_destroy(nestgpu_ctx *c)
     if (!c) return NESTGPU_OK;
     cudaSetDevice(c->device);
     cudaStreamSynchronize(c->stream);
+    scratch_reset(c);
     for (int s = 0; s < NESTGPU_N_STAGES; s++) {
         cudaEventDestroy(c->ev[s][0]);
         cudaEventDestroy(c->ev[s][1]);
@@ -323,7 +347,7 @@ nestgpu_status nestgpu_release(nestgpu_ctx *c, uint64_t m)
     // Work already enqueued may still read the released bytes.
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
     c->lo = m;
-    c->hi = c->size;
+    scratch_reset(c);
     for (auto &col : c->cols)
         if (col.alive && col.off >= m) col.alive = false;
     for (auto &ix : c->idx) {
@@ -450,7 +474,7 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     }
     const int kb = key_bytes(c, key_cols, n_key_cols);
     const int vb = pc ? vs.w : 0;
-    c->hi = c->size;  // scratch reset
+    scratch_reset(c);
     for (int st = 0; st < NESTGPU_N_STAGES; st++) c->ran[st] = false;
     void *tk = salloc(c, (size_t)n * kb), *tv = vb ? salloc(c, (size_t)n * vb) : nullptr;
     void *uk = salloc(c, (size_t)n * kb), *uv = vb ? salloc(c, (size_t)n * vb) : nullptr;
@@ -671,7 +695,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     }
 
     // ------------------------------------------------------------ allocation
-    c->hi = c->size;  // scratch reset: previous results die here
+    scratch_reset(c);  // previous results die here
     for (int st = 0; st < NESTGPU_N_STAGES; st++) c->ran[st] = false;
     const bool ravalid = rks.v0 || rks.v1;
     int *ids = (int *)salloc(c, (size_t)nR * 4);
@@ -914,7 +938,7 @@ nestgpu_status nestgpu_exec_collect(nestgpu_ctx *c, const nestgpu_plan *P, nestg
     if (ix->kb != kb)
         return fail(c, NESTGPU_ERR_UNSUPPORTED, "exec_collect: outer key is 64-bit but index %d has 32-bit keys", P->index);
 
-    c->hi = c->size;  // scratch reset
+    scratch_reset(c);
     for (int st = 0; st < NESTGPU_N_STAGES; st++) c->ran[st] = false;
     const bool ravalid = rks.v0 || rks.v1;
     int *ids = (int *)salloc(c, (size_t)nR * 4);
@@ -1059,6 +1083,19 @@ nestgpu_status nestgpu_column_from_device(nestgpu_ctx *c, nestgpu_dtype dtype, i
     }
     *out_col = id;
     return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_set_option(nestgpu_ctx *c, int32_t option, int64_t value)
+{
+    if (!c) return NESTGPU_ERR_INVALID;
+    switch (option) {
+    case NESTGPU_OPT_MALLOC_SCRATCH:
+        cudaSetDevice(c->device);
+        scratch_reset(c);
+        c->malloc_scratch = value != 0;
+        return NESTGPU_OK;
+    }
+    return fail(c, NESTGPU_ERR_INVALID, "set_option: unknown option %d", option);
 }
 
 nestgpu_status nestgpu_set_profiling(nestgpu_ctx *c, int32_t on)

@@ -364,3 +364,22 @@ def test_c2_zipf_full_size_cached(eng):
         assert_parity(g, ref, plan, True, rows=rows, ctx=("zipf", corr_op, agg))
         valid, value, _, _ = ind.closed_form(t["R"]["col1"], t["S"]["col1"], t["S"]["col2"], corr_op, agg)
         assert np.array_equal(g["valid"].astype(bool), valid) and np.array_equal(g["value"], value)
+
+
+# ------------------------------------------------------------------ ablation knob
+@pytest.mark.parametrize("mode", MODES)
+def test_malloc_scratch_option_same_result(eng, mode):
+    """NESTGPU_OPT_MALLOC_SCRATCH (the pool-less ablation baseline)
+    changes where scratch lives, never the result."""
+    from paper_conf_icde_floratosxwgylz21_b200.binding import OPT_MALLOC_SCRATCH
+    t = query1.config("C1")
+    for corr_op in ("=", ">", "!="):
+        for agg in ("min", "avg", "count"):
+            plan = make_plan(corr_op, agg, "=")
+            ref = oracle.evaluate(t, plan)
+            eng.set_option(OPT_MALLOC_SCRATCH, 1)
+            try:
+                got = run(eng, t, plan, mode, emit_all=True)
+            finally:
+                eng.set_option(OPT_MALLOC_SCRATCH, 0)
+            assert_parity(got, ref, plan, True, ctx=("malloc", mode, corr_op, agg))
