@@ -313,6 +313,86 @@ nestgpu_status nestgpu_column_from_device(nestgpu_ctx *ctx, nestgpu_dtype dtype,
                                           const int64_t *d_src, const uint8_t *d_valid, int64_t n,
                                           int32_t *out_col);
 
+/* ---------------------------------------------------------------- cost model */
+
+/* The paper's cost model (§IV), adapted to this engine's
+ * vectorised kernels, to predict the latency of one nestgpu_exec_correlated
+ * under each execution strategy and pick the fastest ("a cost model to
+ * guide subquery processing by selecting the most effective execution
+ * path").
+ *
+ *   Eq. (1)  T_op = sum_i K_i * ceil(D_i / Th_i) + M * D_r * sum(Rs) + C
+ *   Eq. (6)  N    = (S - Ch) * [per-evaluation cost] + invariant parts once
+ *   Eq. (7)  Nmem = memory-related cost per operation, once
+ *   Eq. (8)  U    = outer-block scans / aggregations
+ *   Eq. (9)  Q    = N + Nmem + U
+ *
+ * Every kernel here sizes its grid to its input, so K_i * ceil(D_i / Th_i)
+ * becomes a per-element cost K_i * D_i (per row, per sorted byte, per probe
+ * step, per (r,s) pair ...).  The K_i are MEASURED on this GPU by running the
+ * engine's own kernels once on synthetic data ("One method to estimate
+ * Ki is actually running the query once and reusing this value for all
+ * predictions").  Vectorisation turns the per-iteration constant C of
+ * Eq. (1) into one C per launch, not per outer tuple; caching makes
+ * S - Ch the number of distinct correlated values.  Nmem is zero: columns
+ * are preloaded and scratch comes from the pool, so there is no
+ * per-operation allocation or transfer.  Cardinalities (D_r) are inputs,
+ * known in advance as in the paper's evaluation. */
+typedef struct {
+    double launch_ms;                /* C: one kernel launch with a tiny input */
+    double filter_ms_per_row;        /* selection (a2/a3), per input row */
+    double hist_ms_per_key_digit;    /* index build digit histogram, per key per digit */
+    double sort_ms_per_key;          /* one radix pass: per key ...                      */
+    double sort_ms_per_byte;         /* ... plus per (key + payload) byte moved           */
+    double probe_ms_per_step;        /* a5 binary search, per outer tuple per log2|S'| step */
+    double range_ms_per_elem;        /* a6 fold, per qualifying element (only '=' MIN/MAX scans) */
+    double aux_ms_per_elem;          /* prefix/suffix aggregates of an index payload, per element */
+    double bnl_ms_per_pair[2][4];    /* a7 per (r,s) pair, [0] 4-byte / [1] 8-byte keys x
+                                        [0] MIN/MAX [1] COUNT [2] SUM/AVG [3] EXISTS (no early exit) */
+    double final_ms_per_row;         /* a8 aggregate finalize + outer comparison, per R' tuple */
+    double materialize_ms_per_byte;  /* M: a9 compaction, per survivor byte written */
+    double group_ms_per_key;         /* caching: grouping of sorted R' keys, per key */
+    double sync_ms;                  /* one host round trip (small D2H + stream sync): exec reads its
+                                        survivor count, an index build its |S'|, caching two more */
+} nestgpu_cost_params;
+
+typedef struct {
+    int64_t n_r, n_s;            /* |R|, |S| */
+    int64_t n_rp, n_sp;          /* |R'|, |S'| (after the local predicates) */
+    int64_t n_distinct;          /* distinct correlated values among R' (S - Ch of Eq. (6)) */
+    int64_t sum_k;               /* sum over R' tuples of their qualifying |S'| rows */
+    int64_t survivors;           /* result rows */
+    int32_t key_bytes;           /* 4 or 8 */
+    int32_t payload_bytes;       /* 0 (COUNT / EXISTS), 4 or 8 */
+    int32_t sort_passes;         /* radix passes of the index build (8-bit digits that vary) */
+    int32_t dedup_passes;        /* radix passes of the R' key sort when caching */
+    nestgpu_cmp corr_op;
+    nestgpu_agg agg;
+} nestgpu_cost_input;
+
+enum { NESTGPU_STRATEGY_NESTED_LOOP = 0, NESTGPU_STRATEGY_INDEX = 1,
+       NESTGPU_STRATEGY_NESTED_LOOP_CACHED = 2, NESTGPU_STRATEGY_INDEX_CACHED = 3 };
+
+typedef struct {
+    double ms[4];                /* predicted Q per strategy (index strategies include building it) */
+    double index_build_ms;       /* the index-build part of ms[1] / ms[3] (invariant, once) */
+    double outer_ms;             /* U, Eq. (8): outer selection + finalize + compaction */
+    double nested_ms[4];         /* N, Eq. (6), per strategy (index build excluded) */
+    int32_t best;                /* argmin of ms[] */
+} nestgpu_cost_estimate;
+
+/* Measure the K_i of nestgpu_cost_params on this GPU: runs the engine's
+ * filter, radix pass, digit histogram, binary-search range, prefix-aggregate,
+ * nested-loop (per aggregate class), finalize and grouping kernels once each
+ * (after a warm-up) on synthetic data in the scratch pool (~64 * n_rows bytes;
+ * n_rows <= 0 picks 4M and shrinks to fit the arena) and times them with CUDA
+ * events.  Invalidates results of earlier execs.  Errors: INVALID, OOM, CUDA. */
+nestgpu_status nestgpu_cost_calibrate(nestgpu_ctx *ctx, int64_t n_rows, nestgpu_cost_params *out);
+/* Evaluate Eqs. (1)-(9) for one plan shape.  Pure host arithmetic (no device
+ * work, no context).  Errors: INVALID (negative sizes, bad widths / enums). */
+nestgpu_status nestgpu_cost_estimate_plan(const nestgpu_cost_params *params, const nestgpu_cost_input *in,
+                                          nestgpu_cost_estimate *out);
+
 /* Ablation knobs -- NOT for production use; they exist to measure the
  * paper's design claims against their baselines (tools/ablations.py).
  *   NESTGPU_OPT_MALLOC_SCRATCH (value 0/1): per-exec scratch comes from one

@@ -31,7 +31,9 @@ SYMBOLS = ("nestgpu_create", "nestgpu_destroy", "nestgpu_last_error", "nestgpu_l
            "nestgpu_build_index", "nestgpu_drop_index", "nestgpu_index_info",
            "nestgpu_index_create_empty", "nestgpu_exec_correlated", "nestgpu_result_to_host",
            "nestgpu_exec_collect", "nestgpu_collection_in", "nestgpu_column_from_device",
-           "nestgpu_set_option", "nestgpu_set_profiling", "nestgpu_last_profile")
+           "nestgpu_set_option", "nestgpu_set_profiling", "nestgpu_last_profile",
+           "nestgpu_cost_calibrate", "nestgpu_cost_estimate_plan")
+STRATEGIES = ("nested_loop", "index", "nested_loop_cached", "index_cached")
 OPT_MALLOC_SCRATCH = 1
 
 
@@ -81,7 +83,66 @@ class Collection(ctypes.Structure):
                 ("d_values", ctypes.c_void_p), ("d_owner", ctypes.c_void_p)]
 
 
+class CostParams(ctypes.Structure):
+    _fields_ = [("launch_ms", ctypes.c_double), ("filter_ms_per_row", ctypes.c_double),
+                ("hist_ms_per_key_digit", ctypes.c_double), ("sort_ms_per_key", ctypes.c_double),
+                ("sort_ms_per_byte", ctypes.c_double),
+                ("probe_ms_per_step", ctypes.c_double), ("range_ms_per_elem", ctypes.c_double),
+                ("aux_ms_per_elem", ctypes.c_double), ("bnl_ms_per_pair", (ctypes.c_double * 4) * 2),
+                ("final_ms_per_row", ctypes.c_double), ("materialize_ms_per_byte", ctypes.c_double),
+                ("group_ms_per_key", ctypes.c_double), ("sync_ms", ctypes.c_double)]
+
+    def as_dict(self):
+        d = {k: getattr(self, k) for k, _ in self._fields_ if k != "bnl_ms_per_pair"}
+        d["bnl_ms_per_pair"] = [list(row) for row in self.bnl_ms_per_pair]
+        return d
+
+
+class CostInput(ctypes.Structure):
+    _fields_ = [("n_r", ctypes.c_int64), ("n_s", ctypes.c_int64), ("n_rp", ctypes.c_int64),
+                ("n_sp", ctypes.c_int64), ("n_distinct", ctypes.c_int64), ("sum_k", ctypes.c_int64),
+                ("survivors", ctypes.c_int64), ("key_bytes", ctypes.c_int32), ("payload_bytes", ctypes.c_int32),
+                ("sort_passes", ctypes.c_int32), ("dedup_passes", ctypes.c_int32), ("corr_op", ctypes.c_int32),
+                ("agg", ctypes.c_int32)]
+
+
+class CostEstimate(ctypes.Structure):
+    _fields_ = [("ms", ctypes.c_double * 4), ("index_build_ms", ctypes.c_double), ("outer_ms", ctypes.c_double),
+                ("nested_ms", ctypes.c_double * 4), ("best", ctypes.c_int32)]
+
+
 _lib = None
+
+
+def cost_estimate(params, n_r, n_s, n_rp, n_sp, n_distinct, sum_k, survivors, key_bytes, payload_bytes,
+                  sort_passes, dedup_passes, corr_op, agg):
+    """Eqs. (1)-(9) of the paper's cost model for one plan shape
+    (nestgpu_cost_estimate_plan; host arithmetic, no device).  params: a
+    CostParams (from Engine.cost_calibrate) or its as_dict().  Returns
+    {strategy: predicted ms, "best": strategy, "index_build_ms", "outer_ms"}."""
+    lib = load_library()
+    if isinstance(params, dict):
+        p = CostParams()
+        for k, v in params.items():
+            if k == "bnl_ms_per_pair":
+                for w, row in enumerate(v):
+                    for i, x in enumerate(row):
+                        p.bnl_ms_per_pair[w][i] = x
+            else:
+                setattr(p, k, v)
+        params = p
+    ci = CostInput(int(n_r), int(n_s), int(n_rp), int(n_sp), int(n_distinct), int(sum_k), int(survivors),
+                   int(key_bytes), int(payload_bytes), int(sort_passes), int(dedup_passes), CMP[corr_op], AGG[agg])
+    e = CostEstimate()
+    st = lib.nestgpu_cost_estimate_plan(ctypes.byref(params), ctypes.byref(ci), ctypes.byref(e))
+    if st != OK:
+        raise NestGPUError(st, "cost_estimate_plan rejected its input")
+    out = {name: e.ms[i] for i, name in enumerate(STRATEGIES)}
+    out["nested"] = {name: e.nested_ms[i] for i, name in enumerate(STRATEGIES)}
+    out["best"] = STRATEGIES[e.best]
+    out["index_build_ms"] = e.index_build_ms
+    out["outer_ms"] = e.outer_ms
+    return out
 
 
 def load_library(path=LIB_PATH):
@@ -118,6 +179,8 @@ def load_library(path=LIB_PATH):
         "nestgpu_collection_in": (i32, [vp, P(Collection), i32, i64, i32, P(Result)]),
         "nestgpu_column_from_device": (i32, [vp, i32, i32, vp, vp, i64, P(i32)]),
         "nestgpu_set_option": (i32, [vp, i32, i64]),
+        "nestgpu_cost_calibrate": (i32, [vp, i64, P(CostParams)]),
+        "nestgpu_cost_estimate_plan": (i32, [P(CostParams), P(CostInput), P(CostEstimate)]),
         "nestgpu_set_profiling": (i32, [vp, i32]),
         "nestgpu_last_profile": (i32, [vp, P(ctypes.c_float), i32]),
     }
@@ -204,6 +267,12 @@ class Engine:
         a, b = ctypes.c_size_t(), ctypes.c_size_t()
         self._check(self.lib.nestgpu_arena_usage(self.ctx, ctypes.byref(a), ctypes.byref(b)))
         return a.value, b.value
+
+    def cost_calibrate(self, n_rows=0):
+        """Measure the cost model's K_i on this GPU (nestgpu_cost_calibrate)."""
+        p = CostParams()
+        self._check(self.lib.nestgpu_cost_calibrate(self.ctx, int(n_rows), ctypes.byref(p)))
+        return p
 
     def set_option(self, option, value):
         """Ablation knobs (nestgpu_set_option), e.g. OPT_MALLOC_SCRATCH."""

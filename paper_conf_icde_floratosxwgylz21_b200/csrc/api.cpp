@@ -274,6 +274,18 @@ nestgpu_status column_stats(nestgpu_ctx *c, Column &col)
 }
 }  // namespace
 
+// Context accessors for the host-side modules (cost.cpp) -- internal.h.
+namespace ng {
+void *ctx_scratch_alloc(nestgpu_ctx *c, size_t bytes) { return salloc(c, bytes); }
+void ctx_scratch_reset(nestgpu_ctx *c) { scratch_reset(c); }
+cudaStream_t ctx_stream(nestgpu_ctx *c) { return c->stream; }
+int ctx_num_sms(nestgpu_ctx *c) { return c->num_sms; }
+long long *ctx_launches(nestgpu_ctx *c) { return &c->launches; }
+unsigned *ctx_pinned(nestgpu_ctx *c) { return c->pinned; }
+int ctx_device(nestgpu_ctx *c) { return c->device; }
+nestgpu_status ctx_fail(nestgpu_ctx *c, nestgpu_status code, const char *msg) { return fail(c, code, "%s", msg); }
+}  // namespace ng
+
 extern "C" {
 
 nestgpu_status nestgpu_create(int device, void *d_arena, size_t arena_bytes, void *cuda_stream, nestgpu_ctx **out)

@@ -6,7 +6,26 @@
 
 #include "common.cuh"
 
+struct nestgpu_ctx;
+
 namespace ng {
+
+// Context accessors (api.cpp) for host-side modules such as cost.cpp.
+void *ctx_scratch_alloc(nestgpu_ctx *c, size_t bytes);   // nullptr when the arena is exhausted
+void ctx_scratch_reset(nestgpu_ctx *c);
+cudaStream_t ctx_stream(nestgpu_ctx *c);
+int ctx_num_sms(nestgpu_ctx *c);
+long long *ctx_launches(nestgpu_ctx *c);
+unsigned *ctx_pinned(nestgpu_ctx *c);
+int ctx_device(nestgpu_ctx *c);
+int32_t ctx_fail(nestgpu_ctx *c, int32_t code, const char *msg);
+
+// out[i] = hash(seed, i) % mod (+ lo), for synthetic calibration inputs; w = 4 or 8.
+cudaError_t launch_fill_hash(void *out, int w, long long n, unsigned seed, unsigned long long mod, long long lo,
+                             cudaStream_t st, long long *launches);
+// out[i] = lo + i / div (ascending runs), w = 4 or 8.
+cudaError_t launch_fill_runs(void *out, int w, long long n, long long div, long long lo, cudaStream_t st,
+                             long long *launches);
 
 // Every launcher returns the cudaError_t of its launch(es) and bumps *launches
 // by the number of kernels it launched.

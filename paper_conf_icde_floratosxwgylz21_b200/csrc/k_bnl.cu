@@ -3,7 +3,8 @@
 
 namespace ng {
 
-size_t bnl_scratch_bytes(long long n_rp_max) { return 256 + (size_t)((n_rp_max + B_RBLOCK - 1) / B_RBLOCK + 1) * 4; }
+// rb_done: one word per R block of the smallest block size (B_THREADS tuples)
+size_t bnl_scratch_bytes(long long n_rp_max) { return 256 + (size_t)((n_rp_max + B_THREADS - 1) / B_THREADS + 1) * 4; }
 
 cudaError_t launch_bnl(int kb, int vb, int op, int agg, long long n_rp_max, const long long *d_nrp, const void *rkeys,
                        long long ns_max, const long long *d_nsp, const void *skeys, const void *svals,

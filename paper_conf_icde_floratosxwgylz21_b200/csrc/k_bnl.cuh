@@ -37,6 +37,12 @@ namespace ng {
 #ifndef NG_B_STAGES
 #define NG_B_STAGES 3
 #endif
+#ifndef NG_B_UNROLL
+#define NG_B_UNROLL 2      // element groups per inner iteration (DESIGN.md §8 tuning log)
+#endif
+#ifndef NG_B_UNROLL_V0
+#define NG_B_UNROLL_V0 4   // ... for COUNT / EXISTS / SUM with 32-bit keys
+#endif
 constexpr int B_THREADS = 256;
 constexpr int B_RPT = NG_B_RPT;        // outer tuples per thread (register blocking)
 constexpr int B_RBLOCK = B_THREADS * B_RPT;
@@ -55,8 +61,7 @@ struct BnlArgs {
     long long *cnt;
     unsigned *unit_counter;
     unsigned *rb_done;         // EXISTS: per R block, set once every tuple of the block found a match
-    long long n_sc;
-    long long chunk;
+    long long target_units;    // work units to aim for (grid x 16)
 };
 
 template <typename K, int VB>
@@ -190,65 +195,92 @@ __device__ __forceinline__ void pair_step(const K rk, const K sk, const V sv, V 
     }
 }
 
-template <int OP, int AGG, bool TRACK, typename K, typename V, int VB>
-__device__ __forceinline__ void tile_full(const K *__restrict__ tk, const V *__restrict__ tv, const K (&rk)[B_RPT],
-                                          V (&mm)[B_RPT], long long (&sm)[B_RPT], unsigned (&c)[B_RPT],
-                                          bool (&found)[B_RPT], const unsigned mul)
+// SPLIT: the CTA's 8 warps hold the SAME outer tuples and each warp scans
+// every 8th group of the tile (small-R' mode); otherwise every warp scans the
+// whole tile for its own tuples.
+template <int RPT, bool SPLIT, int OP, int AGG, bool TRACK, typename K, typename V, int VB>
+__device__ __forceinline__ void tile_full(const K *__restrict__ tk, const V *__restrict__ tv, const K (&rk)[RPT],
+                                          V (&mm)[RPT], long long (&sm)[RPT], unsigned (&c)[RPT],
+                                          bool (&found)[RPT], const unsigned mul)
 {
     constexpr int TILE = BnlTile<K, VB>::TILE;
     constexpr int KV = 16 / (int)sizeof(K);  // keys per 128-bit load
-#pragma unroll 2
-    for (int e = 0; e < TILE; e += KV) {
-        K kk[KV];
-        V vv[KV];
-        if constexpr (sizeof(K) == 4) {
-            const uint4 q = *reinterpret_cast<const uint4 *>(tk + e);
-            kk[0] = q.x; kk[1] = q.y; kk[2] = q.z; kk[3] = q.w;
-        } else {
-            const ulonglong2 q = *reinterpret_cast<const ulonglong2 *>(tk + e);
-            kk[0] = q.x; kk[1] = q.y;
-        }
-        if constexpr (VB == 4) {
-            if constexpr (KV == 4) {
-                const int4 q = *reinterpret_cast<const int4 *>(tv + e);
-                vv[0] = q.x; vv[1] = q.y; vv[2] = q.z; vv[3] = q.w;
+    constexpr int STEP = SPLIT ? KV * (B_THREADS / 32) : KV;
+    // U groups of KV elements per iteration, all loaded up front (no
+    // cross-iteration software pipelining: ptxas would add register moves)
+    // (MIN/MAX or 64-bit keys: 2 groups -- MIN stays at 3 CTAs/SM; COUNT /
+    // EXISTS / SUM with 32-bit keys: 4, measured fastest)
+    constexpr int U = (AccKind<AGG>::minmax || sizeof(K) == 8) ? NG_B_UNROLL : NG_B_UNROLL_V0;
+    const int e0 = SPLIT ? (int)(threadIdx.x >> 5) * KV : 0;
+#pragma unroll 1
+    for (int e = e0; e < TILE; e += STEP * U) {
+        K kk[U][KV];
+        V vv[U][KV];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const int eu = min(e + u * STEP, TILE - KV);   // clamped: the ragged tail is skipped below
+            if constexpr (sizeof(K) == 4) {
+                const uint4 q = *reinterpret_cast<const uint4 *>(tk + eu);
+                kk[u][0] = q.x; kk[u][1] = q.y; kk[u][2] = q.z; kk[u][3] = q.w;
             } else {
-                const int2 q = *reinterpret_cast<const int2 *>(tv + e);
-                vv[0] = q.x; vv[1] = q.y;
+                const ulonglong2 q = *reinterpret_cast<const ulonglong2 *>(tk + eu);
+                kk[u][0] = q.x; kk[u][1] = q.y;
             }
-        } else if constexpr (VB == 8) {
+            if constexpr (VB == 4) {
+                if constexpr (KV == 4) {
+                    const int4 q = *reinterpret_cast<const int4 *>(tv + eu);
+                    vv[u][0] = q.x; vv[u][1] = q.y; vv[u][2] = q.z; vv[u][3] = q.w;
+                } else {
+                    const int2 q = *reinterpret_cast<const int2 *>(tv + eu);
+                    vv[u][0] = q.x; vv[u][1] = q.y;
+                }
+            } else if constexpr (VB == 8) {
 #pragma unroll
-            for (int q = 0; q < KV; q += 2) {
-                const longlong2 w = *reinterpret_cast<const longlong2 *>(tv + e + q);
-                vv[q] = w.x; vv[q + 1] = w.y;
+                for (int q = 0; q < KV; q += 2) {
+                    const longlong2 w = *reinterpret_cast<const longlong2 *>(tv + eu + q);
+                    vv[u][q] = w.x; vv[u][q + 1] = w.y;
+                }
+            } else {
+#pragma unroll
+                for (int q = 0; q < KV; q++) vv[u][q] = 0;
             }
-        } else {
-#pragma unroll
-            for (int q = 0; q < KV; q++) vv[q] = 0;
         }
 #pragma unroll
-        for (int q = 0; q < KV; q++) {
+        for (int u = 0; u < U; u++) {
+            // whole iterations cover the tile unless TILE / KV is not a
+            // multiple of the per-iteration stride (uniform per warp)
+            if ((TILE % (STEP * U)) != 0 && e + u * STEP >= TILE) break;
 #pragma unroll
-            for (int i = 0; i < B_RPT; i++) pair_step<OP, AGG, TRACK>(rk[i], kk[q], vv[q], mm[i], sm[i], c[i], found[i], mul);
+            for (int q = 0; q < KV; q++) {
+#pragma unroll
+                for (int i = 0; i < RPT; i++)
+                    pair_step<OP, AGG, TRACK>(rk[i], kk[u][q], vv[u][q], mm[i], sm[i], c[i], found[i], mul);
+            }
         }
     }
 }
 
-template <int OP, int AGG, bool TRACK, typename K, typename V, int VB>
+template <int RPT, bool SPLIT, int OP, int AGG, bool TRACK, typename K, typename V, int VB>
 __device__ __forceinline__ void tile_part(const K *__restrict__ tk, const V *__restrict__ tv, int count,
-                                          const K (&rk)[B_RPT], V (&mm)[B_RPT], long long (&sm)[B_RPT],
-                                          unsigned (&c)[B_RPT], bool (&found)[B_RPT], const unsigned mul)
+                                          const K (&rk)[RPT], V (&mm)[RPT], long long (&sm)[RPT],
+                                          unsigned (&c)[RPT], bool (&found)[RPT], const unsigned mul)
 {
-    for (int e = 0; e < count; e++) {
+    for (int e = SPLIT ? (int)(threadIdx.x >> 5) : 0; e < count; e += SPLIT ? B_THREADS / 32 : 1) {
         const K k = tk[e];
         const V v = VB ? tv[e] : (V)0;
 #pragma unroll
-        for (int i = 0; i < B_RPT; i++) pair_step<OP, AGG, TRACK>(rk[i], k, v, mm[i], sm[i], c[i], found[i], mul);
+        for (int i = 0; i < RPT; i++) pair_step<OP, AGG, TRACK>(rk[i], k, v, mm[i], sm[i], c[i], found[i], mul);
     }
 }
 
-template <typename K, int VB, int OP, int AGG>
-__global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
+// The whole loop: RPT outer tuples per thread; R blocks of B_THREADS * RPT
+// tuples (every warp its own tuples), or with SPLIT of 32 * RPT tuples held
+// by all 8 warps, each scanning 1/8 of every S' tile -- 8x more R blocks for
+// an |R'| so small that full blocks would leave CTAs idle (Q2 / Q5 / cached
+// Q17 have a few hundred R' tuples).  Same ILP and registers either way.
+template <int RPT, bool SPLIT, typename K, int VB, int OP, int AGG>
+__device__ __forceinline__ void bnl_body(const BnlArgs &A, unsigned char *smem, unsigned long long *full_bar,
+                                         long long &s_unit, const long long nrp, const long long nsp)
 {
     using V = typename std::conditional<VB == 8, long long, int>::type;
     constexpr int TILE = BnlTile<K, VB>::TILE;
@@ -256,21 +288,27 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
     constexpr V VMAX = VB == 8 ? (V)LLONG_MAX : (V)INT_MAX;
     constexpr V VMIN = VB == 8 ? (V)LLONG_MIN : (V)INT_MIN;
     constexpr V MM0 = AGG == MIN ? VMAX : (AGG == MAX ? VMIN : (V)0);
-
-    extern __shared__ __align__(128) unsigned char smem[];
-    __shared__ __align__(8) unsigned long long full_bar[B_STAGES];
-    __shared__ long long s_unit;
-
+    constexpr long long RSTRIDE = SPLIT ? 32 : B_THREADS;   // tuple stride within a block
+    constexpr long long RBLOCK = RSTRIDE * RPT;
+    static_assert(!SPLIT || RBLOCK * 20 <= (long long)B_STAGES * B_STAGE_BYTES, "split merge area");
     const int tid = threadIdx.x;
-    if (tid == 0) {
-        for (int s = 0; s < B_STAGES; s++) mbar_init(&full_bar[s], 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
+    const int rlane = SPLIT ? (tid & 31) : tid;
 
-    const long long nrp = *A.d_nrp, nsp = *A.d_nsp;
-    const long long n_rb = (nrp + B_RBLOCK - 1) / B_RBLOCK;
-    const long long n_units = n_rb * A.n_sc;
+    // Work decomposition from the ACTUAL |R'| and |S'| (device counts; the
+    // host only knows upper bounds): (R block) x (S' chunk of whole tiles)
+    // units, about target_units of them, chunks down to a single tile so a
+    // small R' (few R blocks) still spreads over every CTA.
+    const long long n_rb = (nrp + RBLOCK - 1) / RBLOCK;
+    const long long n_ts = (nsp + TILE - 1) / TILE;
+    long long n_sc = n_rb > 0 ? (A.target_units + n_rb - 1) / n_rb : 1;
+    // chunks of at least one tile; in the warp-split shape at least 4 tiles, so
+    // the TMA fill latency and the per-unit merge amortise over a unit
+    const long long max_sc = SPLIT ? (n_ts + 3) / 4 : n_ts;
+    n_sc = n_sc < 1 ? 1 : (n_sc > max_sc ? max_sc : n_sc);
+    const long long chunk_tiles = n_sc > 0 ? (n_ts + n_sc - 1) / n_sc : 1;
+    const long long chunk = chunk_tiles * TILE;
+    n_sc = chunk_tiles > 0 ? (n_ts + chunk_tiles - 1) / chunk_tiles : 0;
+    const long long n_units = n_rb * n_sc;
     // MIN/MAX: if some S' payload equals the identity, track "found"
     // explicitly (uniform per launch, flag from the S' filter kernel).
     // SUM/AVG with 32-bit payloads: when max|payload| * TILE < 2^31 a tile's
@@ -304,8 +342,8 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
         __syncthreads();
         if (u >= n_units) break;
         const long long sc = u / n_rb, rb = u - sc * n_rb;
-        const long long s0 = sc * A.chunk;
-        const long long s1 = min(nsp, s0 + A.chunk);
+        const long long s0 = sc * chunk;
+        const long long s1 = min(nsp, s0 + chunk);
         const int ntiles = s1 > s0 ? (int)((s1 - s0 + TILE - 1) / TILE) : 0;
         if (ntiles == 0) continue;
         if constexpr (AccKind<AGG>::exists) {
@@ -315,15 +353,15 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
             if (__syncthreads_or(tid == 0 && ld_relaxed_u32(A.rb_done + rb) != 0)) continue;
         }
 
-        K rk[B_RPT];
-        V mm[B_RPT];
-        long long sm[B_RPT];
-        unsigned c[B_RPT];
-        bool found[B_RPT];
-        const long long r0 = rb * B_RBLOCK + tid;
+        K rk[RPT];
+        V mm[RPT];
+        long long sm[RPT];
+        unsigned c[RPT];
+        bool found[RPT];
+        const long long r0 = rb * RBLOCK + rlane;
 #pragma unroll
-        for (int i = 0; i < B_RPT; i++) {
-            const long long r = r0 + (long long)i * B_THREADS;
+        for (int i = 0; i < RPT; i++) {
+            const long long r = r0 + (long long)i * RSTRIDE;
             rk[i] = r < nrp ? rkeys[r] : (K)0;
             mm[i] = MM0;
             sm[i] = 0;
@@ -344,18 +382,18 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
                 const long long ts = s0 + (long long)t * TILE;
                 const int cnt = (int)min((long long)TILE, s1 - ts);
                 if (cnt == TILE) {
-                    if (track) tile_full<OP, AGG, true, K, V, VB>(tk, tv, rk, mm, sm, c, found, mul);
-                    else tile_full<OP, AGG, false, K, V, VB>(tk, tv, rk, mm, sm, c, found, mul);
+                    if (track) tile_full<RPT, SPLIT, OP, AGG, true, K, V, VB>(tk, tv, rk, mm, sm, c, found, mul);
+                    else tile_full<RPT, SPLIT, OP, AGG, false, K, V, VB>(tk, tv, rk, mm, sm, c, found, mul);
                 } else {
-                    if (track) tile_part<OP, AGG, true, K, V, VB>(tk, tv, cnt, rk, mm, sm, c, found, mul);
-                    else tile_part<OP, AGG, false, K, V, VB>(tk, tv, cnt, rk, mm, sm, c, found, mul);
+                    if (track) tile_part<RPT, SPLIT, OP, AGG, true, K, V, VB>(tk, tv, cnt, rk, mm, sm, c, found, mul);
+                    else tile_part<RPT, SPLIT, OP, AGG, false, K, V, VB>(tk, tv, cnt, rk, mm, sm, c, found, mul);
                 }
             }
             ++g;
             if constexpr (AccKind<AGG>::sum && VB == 4) {
                 if (track) {  // widen the per-tile 32-bit partial sums
 #pragma unroll
-                    for (int i = 0; i < B_RPT; i++) {
+                    for (int i = 0; i < RPT; i++) {
                         sm[i] += (long long)mm[i];
                         mm[i] = 0;
                     }
@@ -364,7 +402,10 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
             if constexpr (AccKind<AGG>::exists) {
                 bool all = true;
 #pragma unroll
-                for (int i = 0; i < B_RPT; i++) all = all && (found[i] || r0 + (long long)i * B_THREADS >= nrp);
+                // (SPLIT: a warp only saw 1/8 of the tile, so this stops only
+                // once every warp found a match for every tuple -- later than
+                // necessary, never too early)
+                for (int i = 0; i < RPT; i++) all = all && (found[i] || r0 + (long long)i * RSTRIDE >= nrp);
                 stop = __syncthreads_and(all) != 0;
                 if (stop && tid == 0) st_relaxed_u32(A.rb_done + rb, 1u);
             } else {
@@ -376,29 +417,115 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
             }
         }
         // merge this unit's partial aggregates
+        if constexpr (SPLIT) {
+            // the 8 warps hold partials of the SAME 256 tuples: combine them
+            // in shared memory (the ring is idle: every issued tile has been
+            // consumed), then one global atomic per tuple instead of eight
+            long long *s_acc = (long long *)smem;
+            unsigned long long *s_cnt = (unsigned long long *)(smem + RBLOCK * 8);
+            int *s_found = (int *)(smem + RBLOCK * 16);
+            for (int t = tid; t < RBLOCK; t += B_THREADS) {
+                s_acc[t] = AccKind<AGG>::minmax ? (long long)MM0 : 0;
+                s_cnt[t] = 0;
+                s_found[t] = 0;
+            }
+            __syncthreads();
 #pragma unroll
-        for (int i = 0; i < B_RPT; i++) {
-            const long long r = r0 + (long long)i * B_THREADS;
-            if (r >= nrp) continue;
-            if constexpr (AccKind<AGG>::minmax) {
-                const bool f = track ? found[i] : (mm[i] != MM0);
-                if (f) {
-                    if (AGG == MIN) atomicMin(&A.acc[r], (long long)mm[i]);
-                    else atomicMax(&A.acc[r], (long long)mm[i]);
-                    A.cnt[r] = 1;
+            for (int i = 0; i < RPT; i++) {
+                const int t = rlane + i * (int)RSTRIDE;
+                if (r0 + (long long)i * RSTRIDE >= nrp) continue;
+                if constexpr (AccKind<AGG>::minmax) {
+                    if (track ? found[i] : (mm[i] != MM0)) {
+                        if (AGG == MIN) atomicMin(&s_acc[t], (long long)mm[i]);
+                        else atomicMax(&s_acc[t], (long long)mm[i]);
+                        s_found[t] = 1;
+                    }
+                } else if constexpr (AccKind<AGG>::sum) {
+                    if (c[i]) {
+                        atomicAdd((unsigned long long *)&s_acc[t], (unsigned long long)sm[i]);
+                        atomicAdd(&s_cnt[t], (unsigned long long)c[i]);
+                    }
+                } else if constexpr (AccKind<AGG>::count) {
+                    if (c[i]) atomicAdd(&s_cnt[t], (unsigned long long)c[i]);
+                } else {
+                    if (found[i]) s_found[t] = 1;
                 }
-            } else if constexpr (AccKind<AGG>::sum) {
-                if (c[i]) {
-                    atomicAdd((unsigned long long *)&A.acc[r], (unsigned long long)sm[i]);
-                    atomicAdd((unsigned long long *)&A.cnt[r], (unsigned long long)c[i]);
+            }
+            __syncthreads();
+            for (int t = tid; t < RBLOCK; t += B_THREADS) {
+                const long long r = rb * RBLOCK + t;
+                if (r >= nrp) continue;
+                if constexpr (AccKind<AGG>::minmax) {
+                    if (s_found[t]) {
+                        if (AGG == MIN) atomicMin(&A.acc[r], s_acc[t]);
+                        else atomicMax(&A.acc[r], s_acc[t]);
+                        A.cnt[r] = 1;
+                    }
+                } else if constexpr (AccKind<AGG>::sum) {
+                    if (s_cnt[t]) {
+                        atomicAdd((unsigned long long *)&A.acc[r], (unsigned long long)s_acc[t]);
+                        atomicAdd((unsigned long long *)&A.cnt[r], s_cnt[t]);
+                    }
+                } else if constexpr (AccKind<AGG>::count) {
+                    if (s_cnt[t]) atomicAdd((unsigned long long *)&A.cnt[r], s_cnt[t]);
+                } else {
+                    if (s_found[t]) A.cnt[r] = 1;
                 }
-            } else if constexpr (AccKind<AGG>::count) {
-                if (c[i]) atomicAdd((unsigned long long *)&A.cnt[r], (unsigned long long)c[i]);
-            } else {
-                if (found[i]) A.cnt[r] = 1;
+            }
+            __syncthreads();   // the ring is refilled by the next unit
+        } else {
+#pragma unroll
+            for (int i = 0; i < RPT; i++) {
+                const long long r = r0 + (long long)i * RSTRIDE;
+                if (r >= nrp) continue;
+                if constexpr (AccKind<AGG>::minmax) {
+                    const bool f = track ? found[i] : (mm[i] != MM0);
+                    if (f) {
+                        if (AGG == MIN) atomicMin(&A.acc[r], (long long)mm[i]);
+                        else atomicMax(&A.acc[r], (long long)mm[i]);
+                        A.cnt[r] = 1;
+                    }
+                } else if constexpr (AccKind<AGG>::sum) {
+                    if (c[i]) {
+                        atomicAdd((unsigned long long *)&A.acc[r], (unsigned long long)sm[i]);
+                        atomicAdd((unsigned long long *)&A.cnt[r], (unsigned long long)c[i]);
+                    }
+                } else if constexpr (AccKind<AGG>::count) {
+                    if (c[i]) atomicAdd((unsigned long long *)&A.cnt[r], (unsigned long long)c[i]);
+                } else {
+                    if (found[i]) A.cnt[r] = 1;
+                }
             }
         }
     }
+}
+
+template <typename K, int VB, int OP, int AGG>
+__global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
+{
+    constexpr int TILE = BnlTile<K, VB>::TILE;
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ __align__(8) unsigned long long full_bar[B_STAGES];
+    __shared__ long long s_unit;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < B_STAGES; s++) mbar_init(&full_bar[s], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const long long nrp = *A.d_nrp, nsp = *A.d_nsp;
+    // Uniform choice of the R-block shape.  Full blocks (2048 tuples) unless
+    // they (a) leave fewer than two (R block x S' tile) units per CTA, or (b)
+    // pad |R'| by more than 20 % over the warp-split blocks (256 tuples): the
+    // padded tuple slots are compared against every S' element like real
+    // ones (SF1 Q17 cached: 210 tuples in a 2048-slot block).
+    constexpr long long FULL = (long long)B_THREADS * B_RPT, SPL = 32LL * B_RPT;
+    const long long n_rb_full = (nrp + FULL - 1) / FULL;
+    const long long units_big = n_rb_full * ((nsp + TILE - 1) / TILE);
+    const long long slots_full = n_rb_full * FULL, slots_split = (nrp + SPL - 1) / SPL * SPL;
+    if (units_big < 2LL * gridDim.x || 5 * slots_full > 6 * slots_split)
+        bnl_body<B_RPT, true, K, VB, OP, AGG>(A, smem, full_bar, s_unit, nrp, nsp);
+    else
+        bnl_body<B_RPT, false, K, VB, OP, AGG>(A, smem, full_bar, s_unit, nrp, nsp);
 }
 
 // Host-side launchers, one per (key width, payload width) family, each in

@@ -224,3 +224,55 @@ cudaError_t launch_gather(int w, const void *src, const long long *ids, long lon
 }
 
 }  // namespace ng
+
+namespace ng {
+
+// ------------------------------------------------------------------ synthetic fills
+// Inputs for the cost model's calibration runs (cost.cpp): a counter-based
+// hash (splitmix64 finaliser) and ascending runs.
+__device__ __forceinline__ unsigned long long mix64(unsigned long long z)
+{
+    z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ull;
+    z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
+    return z ^ (z >> 31);
+}
+
+template <typename T>
+__global__ void fill_hash_kernel(T *__restrict__ out, long long n, unsigned seed, unsigned long long mod, long long lo)
+{
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        out[i] = (T)(lo + (long long)(mix64(((unsigned long long)seed << 40) + (unsigned long long)i) % mod));
+}
+
+template <typename T>
+__global__ void fill_runs_kernel(T *__restrict__ out, long long n, long long div, long long lo)
+{
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        out[i] = (T)(lo + i / div);
+}
+
+cudaError_t launch_fill_hash(void *out, int w, long long n, unsigned seed, unsigned long long mod, long long lo,
+                             cudaStream_t st, long long *launches)
+{
+    if (n <= 0) return cudaSuccess;
+    long long blocks = (n + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    if (w == 4) fill_hash_kernel<int><<<(unsigned)blocks, 256, 0, st>>>((int *)out, n, seed, mod, lo);
+    else fill_hash_kernel<long long><<<(unsigned)blocks, 256, 0, st>>>((long long *)out, n, seed, mod, lo);
+    ++*launches;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_fill_runs(void *out, int w, long long n, long long div, long long lo, cudaStream_t st,
+                             long long *launches)
+{
+    if (n <= 0) return cudaSuccess;
+    long long blocks = (n + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    if (w == 4) fill_runs_kernel<int><<<(unsigned)blocks, 256, 0, st>>>((int *)out, n, div, lo);
+    else fill_runs_kernel<long long><<<(unsigned)blocks, 256, 0, st>>>((long long *)out, n, div, lo);
+    ++*launches;
+    return cudaGetLastError();
+}
+
+}  // namespace ng

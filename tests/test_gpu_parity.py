@@ -383,3 +383,29 @@ def test_malloc_scratch_option_same_result(eng, mode):
             finally:
                 eng.set_option(OPT_MALLOC_SCRATCH, 0)
             assert_parity(got, ref, plan, True, ctx=("malloc", mode, corr_op, agg))
+
+
+# ------------------------------------------------------------------ both R-block shapes
+@pytest.mark.parametrize("shape", ["split", "full"])
+def test_bnl_block_shapes_ragged(eng, shape):
+    """The nested-loop kernel picks full R blocks (2048 tuples, every warp its
+    own) or the warp-split shape (256 tuples shared by 8 warps, each scanning
+    1/8 of every S' tile) from the device counts.  Both shapes, ragged R and S
+    tails, every operator x aggregate: closed form on every row + the oracle
+    on sampled rows."""
+    if shape == "split":
+        t = query1.tables(n_r=1999, n_s=250_001, key_hi=1 << 16, val_hi=1 << 12, seed=31)
+    else:
+        t = query1.tables(n_r=40_001, n_s=250_001, key_hi=1 << 16, val_hi=1 << 12, seed=32)
+    n_r = len(t["R"]["col1"])
+    rows = np.unique(np.random.default_rng(5).integers(0, n_r, 40))
+    for corr_op in PLAN_OPS:
+        for agg in ("min", "max", "sum", "count", "avg", "exists"):
+            plan = make_plan(corr_op, agg, "<")
+            g = run(eng, t, plan, "bnl", emit_all=True)
+            valid, value, _, _ = ind.closed_form(t["R"]["col1"], t["S"]["col1"], t["S"]["col2"], corr_op, agg)
+            assert np.array_equal(g["value"], value), (shape, corr_op, agg)
+            assert np.array_equal(g["valid"].astype(bool), valid), (shape, corr_op, agg)
+            if corr_op in ("<", "!=") and agg in ("min", "avg"):
+                ref = oracle.evaluate(t, plan, rows=rows)
+                assert_parity(g, ref, plan, True, rows=rows, ctx=(shape, corr_op, agg))

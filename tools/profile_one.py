@@ -2,6 +2,7 @@
 
   python tools/profile_one.py <op> <agg> <mode> [C1|C2|C5]     Query-1 family
   python tools/profile_one.py tpch <q2|q17|q4|q20> <mode> [SF]   TPC-H-shaped
+  NESTGPU_DEDUP=1 runs the plan with caching.
 """
 import os
 import sys
@@ -26,5 +27,5 @@ R, S = eng.load_table(t["R"]), eng.load_table(t["S"])
 eng.set_profiling(True)
 for _ in range(2):
     idx = eng.index_for_plan(plan, S) if mode == "index" else -1
-    res = eng.exec(plan, R, S, index=idx)
+    res = eng.exec(plan, R, S, index=idx, dedup=os.environ.get("NESTGPU_DEDUP") == "1")
 print("survivors", res.n_rows, "launches", eng.launch_count(), eng.last_profile())
