@@ -400,8 +400,11 @@ nestgpu_status nestgpu_cost_estimate_plan(const nestgpu_cost_params *params, con
  *     exec / build_index / exec_collect / release -- the pool-less baseline
  *     that P:147 ("calling malloc/free ... is unacceptable") and P:233-237
  *     (memory pools) argue against.  Default 0: the arena pool.
+ *   NESTGPU_OPT_BNL_SHAPE (value 0/1/2): the nested-loop kernel's R-block
+ *     shape -- 0 automatic (from |R'|, |S'|), 1 full blocks, 2 warp-split.
+ *     Results are identical; tests use it to cover both shapes on one input.
  * Errors: INVALID (unknown option). */
-enum { NESTGPU_OPT_MALLOC_SCRATCH = 1 };
+enum { NESTGPU_OPT_MALLOC_SCRATCH = 1, NESTGPU_OPT_BNL_SHAPE = 2 };
 nestgpu_status nestgpu_set_option(nestgpu_ctx *ctx, int32_t option, int64_t value);
 
 /* Per-stage device times (ms, CUDA events on the context stream) of the last

@@ -35,6 +35,7 @@ SYMBOLS = ("nestgpu_create", "nestgpu_destroy", "nestgpu_last_error", "nestgpu_l
            "nestgpu_cost_calibrate", "nestgpu_cost_estimate_plan")
 STRATEGIES = ("nested_loop", "index", "nested_loop_cached", "index_cached")
 OPT_MALLOC_SCRATCH = 1
+OPT_BNL_SHAPE = 2
 
 
 class NestGPUError(RuntimeError):

@@ -83,6 +83,7 @@ struct nestgpu_ctx {
     // pool-less baseline of P:147 / P:233.  Off by default.
     bool malloc_scratch;
     std::vector<void *> mallocs;
+    int bnl_shape;   // NESTGPU_OPT_BNL_SHAPE (test knob): 0 automatic, 1 full, 2 warp-split
     cudaEvent_t ev[NESTGPU_N_STAGES][2];
     bool ran[NESTGPU_N_STAGES];
 };
@@ -305,6 +306,7 @@ nestgpu_status nestgpu_create(int device, void *d_arena, size_t arena_bytes, voi
     c->launches = 0;
     c->profiling = false;
     c->malloc_scratch = false;
+    c->bnl_shape = 0;
     if (cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess ||
         cudaMallocHost((void **)&c->pinned, PIN_WORDS * sizeof(unsigned)) != cudaSuccess) {
         delete c;
@@ -848,7 +850,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         prof_end(c, 1);
         prof_begin(c, 3);
         CUDA_TRY(c, ng::launch_bnl(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, nS, d_nsp, skeys, svals,
-                                   extreme, acc, cnt, kscr, c->num_sms, c->stream, &c->launches));
+                                   extreme, acc, cnt, kscr, c->num_sms, c->bnl_shape, c->stream, &c->launches));
         prof_end(c, 3);
     }
 
@@ -1105,6 +1107,10 @@ nestgpu_status nestgpu_set_option(nestgpu_ctx *c, int32_t option, int64_t value)
         cudaSetDevice(c->device);
         scratch_reset(c);
         c->malloc_scratch = value != 0;
+        return NESTGPU_OK;
+    case NESTGPU_OPT_BNL_SHAPE:
+        if (value < 0 || value > 2) return fail(c, NESTGPU_ERR_INVALID, "set_option: BNL shape 0, 1 or 2");
+        c->bnl_shape = (int)value;
         return NESTGPU_OK;
     }
     return fail(c, NESTGPU_ERR_INVALID, "set_option: unknown option %d", option);

@@ -204,7 +204,7 @@ nestgpu_status nestgpu_cost_calibrate(nestgpu_ctx *c, int64_t n_rows, nestgpu_co
                 if (e != cudaSuccess) return e;
                 return ng::launch_bnl(kbw, cls_agg[k] == ng::COUNT || cls_agg[k] == ng::EXISTS ? 0 : 4, ng::GT,
                                       cls_agg[k], nbr, d_small + 1, k1, nbs, d_small + 2, k2, v1, extreme,
-                                      (long long *)acc, (long long *)cnt, bscr, sms, st, L);
+                                      (long long *)acc, (long long *)cnt, bscr, sms, 1, st, L);
             }, &t));
             out->bnl_ms_per_pair[kw][k] = pos(t - 2 * C) / ((double)nbr * nbs);
         }

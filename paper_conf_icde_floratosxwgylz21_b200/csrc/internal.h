@@ -88,7 +88,8 @@ size_t bnl_scratch_bytes(long long n_rp_max);
 cudaError_t launch_bnl(int kb, int vb, int op, int agg, long long n_rp_max, const long long *d_nrp,
                        const void *rkeys, long long ns_max, const long long *d_nsp, const void *skeys,
                        const void *svals, const unsigned *extreme, long long *acc, long long *cnt,
-                       void *scratch, int num_sms, cudaStream_t st, long long *launches);
+                       void *scratch, int num_sms, int shape /* 0 auto, 1 full, 2 warp-split */,
+                       cudaStream_t st, long long *launches);
 
 // Caching: R' positions 0..n-1; distinct keys of a sorted key run
 // and the map R' position -> distinct id.

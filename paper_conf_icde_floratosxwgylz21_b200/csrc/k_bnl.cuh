@@ -62,6 +62,7 @@ struct BnlArgs {
     unsigned *unit_counter;
     unsigned *rb_done;         // EXISTS: per R block, set once every tuple of the block found a match
     long long target_units;    // work units to aim for (grid x 16)
+    int shape;                 // R-block shape: 0 automatic, 1 full, 2 warp-split (test knob)
 };
 
 template <typename K, int VB>
@@ -522,7 +523,8 @@ __global__ void __launch_bounds__(B_THREADS, 2) bnl_kernel(BnlArgs A)
     const long long n_rb_full = (nrp + FULL - 1) / FULL;
     const long long units_big = n_rb_full * ((nsp + TILE - 1) / TILE);
     const long long slots_full = n_rb_full * FULL, slots_split = (nrp + SPL - 1) / SPL * SPL;
-    if (units_big < 2LL * gridDim.x || 5 * slots_full > 6 * slots_split)
+    const bool split = A.shape ? A.shape == 2 : (units_big < 2LL * gridDim.x || 5 * slots_full > 6 * slots_split);
+    if (split)
         bnl_body<B_RPT, true, K, VB, OP, AGG>(A, smem, full_bar, s_unit, nrp, nsp);
     else
         bnl_body<B_RPT, false, K, VB, OP, AGG>(A, smem, full_bar, s_unit, nrp, nsp);

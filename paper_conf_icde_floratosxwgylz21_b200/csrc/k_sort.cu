@@ -21,9 +21,15 @@
 
 namespace ng {
 
+#ifndef NG_S_ITEMS
+#define NG_S_ITEMS 16
+#endif
+#ifndef NG_S_MINB
+#define NG_S_MINB 1   // __launch_bounds__ min blocks per SM (register cap)
+#endif
 constexpr int S_THREADS = 256;
 constexpr int S_WARPS = S_THREADS / 32;
-constexpr int S_ITEMS = 16;
+constexpr int S_ITEMS = NG_S_ITEMS;
 constexpr int S_TILE = S_THREADS * S_ITEMS;
 constexpr unsigned D_AGG = 1u << 30, D_INC = 2u << 30, D_VAL = (1u << 30) - 1;
 
@@ -34,7 +40,7 @@ size_t sort_scratch_bytes(long long n)
 }
 
 template <typename K, int VB>
-__global__ void __launch_bounds__(S_THREADS)
+__global__ void __launch_bounds__(S_THREADS, NG_S_MINB)
 onesweep_kernel(const K *__restrict__ kin, K *__restrict__ kout, const void *__restrict__ vin_,
                 void *__restrict__ vout_, long long n, int shift, const unsigned *__restrict__ digit_base,
                 unsigned *__restrict__ status, unsigned *__restrict__ counter)
@@ -231,6 +237,10 @@ static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *
     if (!attr_set) {
         cudaError_t e = cudaFuncSetAttribute(onesweep_kernel<K, VB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              (int)smem);
+        if (e != cudaSuccess) return e;
+        // all of the unified L1 / shared array as shared memory: occupancy
+        // is then set by registers, not by the default carveout
+        e = cudaFuncSetAttribute(onesweep_kernel<K, VB>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
         if (e != cudaSuccess) return e;
         attr_set = true;
     }

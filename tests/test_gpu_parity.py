@@ -409,3 +409,22 @@ def test_bnl_block_shapes_ragged(eng, shape):
             if corr_op in ("<", "!=") and agg in ("min", "avg"):
                 ref = oracle.evaluate(t, plan, rows=rows)
                 assert_parity(g, ref, plan, True, rows=rows, ctx=(shape, corr_op, agg))
+
+
+@pytest.mark.parametrize("shape", [1, 2])
+def test_bnl_shape_knob(eng, shape):
+    """NESTGPU_OPT_BNL_SHAPE forces full or warp-split R blocks on the same
+    input (C1 + NULL-bearing random tables): identical to the oracle."""
+    from paper_conf_icde_floratosxwgylz21_b200.binding import OPT_BNL_SHAPE
+    tabs = [query1.config("C1"), query1.random_small(17, n_r=3001, n_s=5003, key_hi=500, val_lo=-9, val_hi=9,
+                                                      null_frac=0.1)]
+    eng.set_option(OPT_BNL_SHAPE, shape)
+    try:
+        for t in tabs:
+            for corr_op in PLAN_OPS:
+                for agg in AGGS:
+                    plan = make_plan(corr_op, agg, "<=")
+                    assert_parity(run(eng, t, plan, "bnl", emit_all=True), oracle.evaluate(t, plan), plan, True,
+                                  ctx=(shape, corr_op, agg))
+    finally:
+        eng.set_option(OPT_BNL_SHAPE, 0)

@@ -1,7 +1,8 @@
 """Small workload touching every kernel, for compute-sanitizer runs:
 filter (ordered / unordered), sort + histogram, range (short, long, prefix
-aggregates), nested loop (all agg kinds), dedup (iota / group), finalize,
-gather, minmax."""
+aggregates), nested loop (all agg kinds, both R-block shapes), dedup (iota /
+group), finalize, gather, minmax, type-J collections + IN + materialise,
+cost-model calibration (fills)."""
 import os
 import sys
 
@@ -12,18 +13,20 @@ sys.path.insert(0, ROOT)
 import oracle  # noqa: E402
 from datagen import make_plan, query1  # noqa: E402
 from paper_conf_icde_floratosxwgylz21_b200 import Engine  # noqa: E402
+from paper_conf_icde_floratosxwgylz21_b200.binding import OPT_BNL_SHAPE  # noqa: E402
 
 eng = Engine(0, arena_bytes=512 << 20)
 t = query1.random_small(1, n_r=20011, n_s=30011, key_hi=600, val_lo=-50, val_hi=50, null_frac=0.1)
 R, S = eng.load_table(t["R"], t.get("R_valid")), eng.load_table(t["S"], t.get("S_valid"))
 bad = 0
-for mode in ("bnl", "index"):
+for mode in ("bnl", "bnl_full", "index"):
     for op in ("=", "!=", "<", ">="):
         for agg in ("min", "max", "sum", "count", "avg", "exists"):
             for dedup in (False, True):
                 plan = make_plan(op, agg, "<=", outer_preds=[{"col": "col3", "op": "<=", "lit": 1}],
                                  inner_preds=[{"col": "col3", "op": "!=", "rhs": "col2"}])
                 idx = eng.index_for_plan(plan, S) if mode == "index" else -1
+                eng.set_option(OPT_BNL_SHAPE, 1 if mode == "bnl_full" else 0)
                 g = eng.result_to_numpy(eng.exec(plan, R, S, index=idx, emit_all=True, dedup=dedup))
                 ref = oracle.evaluate(t, plan)
                 m = ref["in_rp"].astype(bool)
@@ -34,5 +37,16 @@ S2 = eng.load_table(big, dtypes={"v": "decimal"})
 R2 = eng.load_table({"k": np.zeros(3, np.int64), "x": np.zeros(3, np.int64)})
 res = eng.exec(make_plan("=", "sum", "<", outer_key=["k"], inner_key=["k"], agg_col="v", outer_cmp_col="x"), R2, S2)
 eng.gather_column(R2["x"], res)
+eng.set_option(OPT_BNL_SHAPE, 0)
+# type-J collections, IN over them, materialisation
+plan = make_plan("=", "min", "=", inner_preds=[{"col": "col3", "op": ">=", "lit": 1}])
+idx = eng.build_index(S, ["col1"], payload="col2", inner_preds=plan["inner_preds"])
+coll = eng.exec_collect(plan, R, S, idx)
+c = eng.collection_to_numpy(coll)
+ref = oracle.collect(t, plan)
+bad += not np.array_equal(np.diff(c["offsets"]), ref["lens"][ref["in_rp"].astype(bool)])
+eng.result_to_numpy(eng.collection_in(coll, R["col2"], emit_all=True))
+col = eng.column_from_device(coll.d_values, coll.n_values, "int32")
+eng.cost_calibrate(1 << 16)
 print("sanitize workload done, mismatches:", bad)
 sys.exit(1 if bad else 0)
