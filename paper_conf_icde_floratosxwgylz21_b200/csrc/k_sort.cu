@@ -25,7 +25,10 @@ namespace ng {
 #define NG_S_ITEMS 16
 #endif
 #ifndef NG_S_MINB
-#define NG_S_MINB 1   // __launch_bounds__ min blocks per SM (register cap)
+#define NG_S_MINB 4   // __launch_bounds__ min blocks per SM (register cap; 1 lets ptxas take 160+)
+#endif
+#ifndef NG_S_CARVEOUT
+#define NG_S_CARVEOUT -1   // preferred shared-memory carveout (%); -1 = driver default
 #endif
 constexpr int S_THREADS = 256;
 constexpr int S_WARPS = S_THREADS / 32;
@@ -238,10 +241,11 @@ static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *
         cudaError_t e = cudaFuncSetAttribute(onesweep_kernel<K, VB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              (int)smem);
         if (e != cudaSuccess) return e;
-        // all of the unified L1 / shared array as shared memory: occupancy
-        // is then set by registers, not by the default carveout
-        e = cudaFuncSetAttribute(onesweep_kernel<K, VB>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-        if (e != cudaSuccess) return e;
+        if (NG_S_CARVEOUT >= 0) {
+            e = cudaFuncSetAttribute(onesweep_kernel<K, VB>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                     NG_S_CARVEOUT);
+            if (e != cudaSuccess) return e;
+        }
         attr_set = true;
     }
     cudaError_t e = cudaMemsetAsync(scratch, 0, sort_scratch_bytes(n), st);
