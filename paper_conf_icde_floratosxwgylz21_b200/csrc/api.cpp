@@ -548,14 +548,20 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
         }
     } else {
         // T -> ... -> P with ping-pong so that the last pass writes P.
+        // 64-bit keys whose high words all agree (AND == OR there, e.g. Q4's
+        // order keys) travel as 32-bit keys between the first and the last
+        // pass: the first pass drops the high word, the last re-attaches it.
+        const bool narrow = kb == 8 && np >= 2 && ((kand ^ kor) >> 32) == 0;
+        const unsigned hi = (unsigned)(kand >> 32);
         const void *ik = tk, *iv = tv;
         for (int p = 0; p < np; p++) {
             const bool to_final = ((np - 1 - p) % 2) == 0;
             void *ok = to_final ? ix.keys : uk;
             void *ov = to_final ? ix.payload : uv;
             if (ok == ik) { ok = tk; ov = tv; }
-            CUDA_TRY(c, ng::launch_radix_pass(kb, vb, ik, ok, iv, ov, nsp, shifts[p], dbase + p * 256, sscr,
-                                              c->stream, &c->launches));
+            const int kin = narrow && p > 0 ? 4 : kb, kout = narrow && p < np - 1 ? 4 : kb;
+            CUDA_TRY(c, ng::launch_radix_pass_x(kin, kout, vb, ik, ok, iv, ov, nsp, shifts[p], dbase + p * 256, sscr,
+                                                hi, c->stream, &c->launches));
             ik = ok;
             iv = ov;
         }
@@ -792,9 +798,11 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
                                           &c->launches));
         void *ck = rkeys, *ok = tkeys;
         int *cv = pos, *ov = tpos;
+        const bool narrow = kb == 8 && np >= 2 && ((kand ^ kor) >> 32) == 0;   // as in build_index
         for (int p = 0; p < np; p++) {
-            CUDA_TRY(c, ng::launch_radix_pass(kb, 4, ck, ok, cv, ov, nrp, shifts[p], dbase + p * 256, sscr,
-                                              c->stream, &c->launches));
+            const int kin = narrow && p > 0 ? 4 : kb, kout = narrow && p < np - 1 ? 4 : kb;
+            CUDA_TRY(c, ng::launch_radix_pass_x(kin, kout, 4, ck, ok, cv, ov, nrp, shifts[p], dbase + p * 256, sscr,
+                                                (unsigned)(kand >> 32), c->stream, &c->launches));
             std::swap(ck, ok);
             std::swap(cv, ov);
         }

@@ -61,6 +61,11 @@ size_t sort_scratch_bytes(long long n);
 cudaError_t launch_radix_pass(int kb, int vb, const void *kin, void *kout, const void *vin, void *vout,
                               long long n, int shift, const unsigned *digit_base, void *scratch,
                               cudaStream_t st, long long *launches);
+// The same with different key widths in and out: 8 -> 4 drops the high word
+// (all keys must share it), 4 -> 8 re-attaches `hi` as the high word.
+cudaError_t launch_radix_pass_x(int kb_in, int kb_out, int vb, const void *kin, void *kout, const void *vin,
+                                void *vout, long long n, int shift, const unsigned *digit_base, void *scratch,
+                                unsigned hi, cudaStream_t st, long long *launches);
 
 // Partial aggregates per R' tuple: acc (int64) + cnt (int64); identity init.
 cudaError_t launch_init_partials(long long n, int agg, long long *acc, long long *cnt, cudaStream_t st,

@@ -42,11 +42,14 @@ size_t sort_scratch_bytes(long long n)
     return (size_t)tiles * 256 * 4 + 256;
 }
 
-template <typename K, int VB>
+// K: the key type read; KO: the key type written.  KO narrower than K drops
+// the (constant) high word; KO wider than K re-attaches `hi` as the high word
+// -- 64-bit keys whose high 32 bits agree are sorted as 32-bit keys.
+template <typename K, int VB, typename KO = K>
 __global__ void __launch_bounds__(S_THREADS, NG_S_MINB)
-onesweep_kernel(const K *__restrict__ kin, K *__restrict__ kout, const void *__restrict__ vin_,
+onesweep_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *__restrict__ vin_,
                 void *__restrict__ vout_, long long n, int shift, const unsigned *__restrict__ digit_base,
-                unsigned *__restrict__ status, unsigned *__restrict__ counter)
+                unsigned *__restrict__ status, unsigned *__restrict__ counter, unsigned hi)
 {
     using V = typename std::conditional<VB == 8, long long, int>::type;
     const V *vin = (const V *)vin_;
@@ -158,7 +161,8 @@ onesweep_kernel(const K *__restrict__ kin, K *__restrict__ kout, const void *__r
         const K k = s_keys[p];
         const int dd = (int)((k >> shift) & 255);
         const long long dst = (long long)s_gdig[dd] + (p - (int)s_tdig[dd]);
-        kout[dst] = k;
+        if constexpr (sizeof(KO) > sizeof(K)) kout[dst] = ((KO)hi << 32) | (KO)k;
+        else kout[dst] = (KO)k;
         if constexpr (VB > 0) vout[dst] = s_vals[p];
     }
 }
@@ -229,20 +233,20 @@ cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *
     return cudaGetLastError();
 }
 
-template <typename K, int VB>
+template <typename K, int VB, typename KO>
 static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *vout, long long n, int shift,
-                            const unsigned *digit_base, void *scratch, cudaStream_t st)
+                            const unsigned *digit_base, void *scratch, unsigned hi, cudaStream_t st)
 {
     using V = typename std::conditional<VB == 8, long long, int>::type;
     const long long tiles = (n + S_TILE - 1) / S_TILE;
     const size_t smem = S_TILE * (sizeof(K) + (VB > 0 ? sizeof(V) : 0));
     static bool attr_set = false;
     if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(onesweep_kernel<K, VB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        cudaError_t e = cudaFuncSetAttribute(onesweep_kernel<K, VB, KO>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              (int)smem);
         if (e != cudaSuccess) return e;
         if (NG_S_CARVEOUT >= 0) {
-            e = cudaFuncSetAttribute(onesweep_kernel<K, VB>, cudaFuncAttributePreferredSharedMemoryCarveout,
+            e = cudaFuncSetAttribute(onesweep_kernel<K, VB, KO>, cudaFuncAttributePreferredSharedMemoryCarveout,
                                      NG_S_CARVEOUT);
             if (e != cudaSuccess) return e;
         }
@@ -250,30 +254,45 @@ static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *
     }
     cudaError_t e = cudaMemsetAsync(scratch, 0, sort_scratch_bytes(n), st);
     if (e != cudaSuccess) return e;
-    onesweep_kernel<K, VB><<<(unsigned)tiles, S_THREADS, smem, st>>>(
-        (const K *)kin, (K *)kout, vin, vout, n, shift, digit_base, (unsigned *)((char *)scratch + 256),
-        (unsigned *)scratch);
+    onesweep_kernel<K, VB, KO><<<(unsigned)tiles, S_THREADS, smem, st>>>(
+        (const K *)kin, (KO *)kout, vin, vout, n, shift, digit_base, (unsigned *)((char *)scratch + 256),
+        (unsigned *)scratch, hi);
     return cudaGetLastError();
+}
+
+template <typename K, typename KO>
+static cudaError_t run_pass_v(int vb, const void *kin, void *kout, const void *vin, void *vout, long long n, int shift,
+                              const unsigned *digit_base, void *scratch, unsigned hi, cudaStream_t st)
+{
+    if (vb == 0) return run_pass<K, 0, KO>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
+    if (vb == 4) return run_pass<K, 4, KO>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
+    return run_pass<K, 8, KO>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
+}
+
+cudaError_t launch_radix_pass_x(int kb_in, int kb_out, int vb, const void *kin, void *kout, const void *vin,
+                                void *vout, long long n, int shift, const unsigned *digit_base, void *scratch,
+                                unsigned hi, cudaStream_t st, long long *launches)
+{
+    if (n <= 0) return cudaSuccess;
+    if (n >= (1ll << 30)) return cudaErrorInvalidValue;
+    cudaError_t e;
+    if (kb_in == 4 && kb_out == 4)
+        e = run_pass_v<uint32_t, uint32_t>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
+    else if (kb_in == 8 && kb_out == 8)
+        e = run_pass_v<uint64_t, uint64_t>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
+    else if (kb_in == 8)
+        e = run_pass_v<uint64_t, uint32_t>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
+    else
+        e = run_pass_v<uint32_t, uint64_t>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
+    ++*launches;
+    return e;
 }
 
 cudaError_t launch_radix_pass(int kb, int vb, const void *kin, void *kout, const void *vin, void *vout,
                               long long n, int shift, const unsigned *digit_base, void *scratch, cudaStream_t st,
                               long long *launches)
 {
-    if (n <= 0) return cudaSuccess;
-    if (n >= (1ll << 30)) return cudaErrorInvalidValue;
-    cudaError_t e;
-    if (kb == 4) {
-        if (vb == 0) e = run_pass<uint32_t, 0>(kin, kout, vin, vout, n, shift, digit_base, scratch, st);
-        else if (vb == 4) e = run_pass<uint32_t, 4>(kin, kout, vin, vout, n, shift, digit_base, scratch, st);
-        else e = run_pass<uint32_t, 8>(kin, kout, vin, vout, n, shift, digit_base, scratch, st);
-    } else {
-        if (vb == 0) e = run_pass<uint64_t, 0>(kin, kout, vin, vout, n, shift, digit_base, scratch, st);
-        else if (vb == 4) e = run_pass<uint64_t, 4>(kin, kout, vin, vout, n, shift, digit_base, scratch, st);
-        else e = run_pass<uint64_t, 8>(kin, kout, vin, vout, n, shift, digit_base, scratch, st);
-    }
-    ++*launches;
-    return e;
+    return launch_radix_pass_x(kb, kb, vb, kin, kout, vin, vout, n, shift, digit_base, scratch, 0u, st, launches);
 }
 
 }  // namespace ng

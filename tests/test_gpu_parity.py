@@ -428,3 +428,21 @@ def test_bnl_shape_knob(eng, shape):
                                   ctx=(shape, corr_op, agg))
     finally:
         eng.set_option(OPT_BNL_SHAPE, 0)
+
+
+@pytest.mark.parametrize("base", [0, 5 << 40, -(3 << 40)])
+def test_int64_keys_narrowed_sort(eng, base):
+    """64-bit keys whose high 32 bits all agree are radix-sorted as 32-bit
+    keys between the first and the last pass (the high word re-attached at
+    the end): index path and caching (R' key sort), vs the oracle."""
+    rng = np.random.default_rng(abs(base) % 97 + 1)
+    t = {"R": {"col1": base + rng.integers(0, 1 << 20, 30001), "col2": rng.integers(-40, 40, 30001)},
+         "S": {"col1": base + rng.integers(0, 1 << 20, 40003), "col2": rng.integers(-40, 40, 40003)}}
+    dt = {"R": {"col1": "int64", "col2": "int64"}, "S": {"col1": "int64", "col2": "int64"}}
+    for corr_op in ("=", "<", "!="):
+        for agg in ("min", "count"):
+            plan = make_plan(corr_op, agg, ">=")
+            ref = oracle.evaluate(t, plan)
+            for dedup in (False, True):
+                g = run(eng, t, plan, "index", emit_all=True, dtypes=dt, dedup=dedup)
+                assert_parity(g, ref, plan, True, ctx=(base, corr_op, agg, dedup))
