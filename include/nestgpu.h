@@ -354,6 +354,10 @@ typedef struct {
     double group_ms_per_key;         /* caching: grouping of sorted R' keys, per key */
     double sync_ms;                  /* one host round trip (small D2H + stream sync): exec reads its
                                         survivor count, an index build its |S'|, caching two more */
+    double exec_overhead_ms;         /* host work of one exec beyond the above (validation, launch
+                                        calls): a tiny exec's wall time minus its modelled time */
+    double build_overhead_ms;        /* the same for one index build */
+    double dedup_overhead_ms;        /* the same for the caching steps of an exec */
 } nestgpu_cost_params;
 
 typedef struct {
@@ -366,6 +370,8 @@ typedef struct {
     int32_t payload_bytes;       /* 0 (COUNT / EXISTS), 4 or 8 */
     int32_t sort_passes;         /* radix passes of the index build (8-bit digits that vary) */
     int32_t dedup_passes;        /* radix passes of the R' key sort when caching */
+    int32_t narrow_keys;         /* 1: 8-byte keys whose high words all agree (sorted as 4-byte
+                                    keys between the first and the last pass) */
     nestgpu_cmp corr_op;
     nestgpu_agg agg;
 } nestgpu_cost_input;
@@ -386,7 +392,11 @@ typedef struct {
  * nested-loop (per aggregate class), finalize and grouping kernels once each
  * (after a warm-up) on synthetic data in the scratch pool (~64 * n_rows bytes;
  * n_rows <= 0 picks 4M and shrinks to fit the arena) and times them with CUDA
- * events.  Invalidates results of earlier execs.  Errors: INVALID, OOM, CUDA. */
+ * events; then runs a tiny exec (plain, cached) and index build through this
+ * API to measure their fixed host-side overheads (wall clock).  n_rows <= 0
+ * picks 16M rows (large sorts amortise their per-tile costs like real ones).
+ * Invalidates results of earlier execs; columns / indexes created after
+ * nestgpu_mark survive.  Errors: INVALID, OOM, CUDA. */
 nestgpu_status nestgpu_cost_calibrate(nestgpu_ctx *ctx, int64_t n_rows, nestgpu_cost_params *out);
 /* Evaluate Eqs. (1)-(9) for one plan shape.  Pure host arithmetic (no device
  * work, no context).  Errors: INVALID (negative sizes, bad widths / enums). */

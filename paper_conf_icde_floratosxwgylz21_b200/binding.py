@@ -91,7 +91,9 @@ class CostParams(ctypes.Structure):
                 ("probe_ms_per_step", ctypes.c_double), ("range_ms_per_elem", ctypes.c_double),
                 ("aux_ms_per_elem", ctypes.c_double), ("bnl_ms_per_pair", (ctypes.c_double * 4) * 2),
                 ("final_ms_per_row", ctypes.c_double), ("materialize_ms_per_byte", ctypes.c_double),
-                ("group_ms_per_key", ctypes.c_double), ("sync_ms", ctypes.c_double)]
+                ("group_ms_per_key", ctypes.c_double), ("sync_ms", ctypes.c_double),
+                ("exec_overhead_ms", ctypes.c_double), ("build_overhead_ms", ctypes.c_double),
+                ("dedup_overhead_ms", ctypes.c_double)]
 
     def as_dict(self):
         d = {k: getattr(self, k) for k, _ in self._fields_ if k != "bnl_ms_per_pair"}
@@ -103,8 +105,8 @@ class CostInput(ctypes.Structure):
     _fields_ = [("n_r", ctypes.c_int64), ("n_s", ctypes.c_int64), ("n_rp", ctypes.c_int64),
                 ("n_sp", ctypes.c_int64), ("n_distinct", ctypes.c_int64), ("sum_k", ctypes.c_int64),
                 ("survivors", ctypes.c_int64), ("key_bytes", ctypes.c_int32), ("payload_bytes", ctypes.c_int32),
-                ("sort_passes", ctypes.c_int32), ("dedup_passes", ctypes.c_int32), ("corr_op", ctypes.c_int32),
-                ("agg", ctypes.c_int32)]
+                ("sort_passes", ctypes.c_int32), ("dedup_passes", ctypes.c_int32),
+                ("narrow_keys", ctypes.c_int32), ("corr_op", ctypes.c_int32), ("agg", ctypes.c_int32)]
 
 
 class CostEstimate(ctypes.Structure):
@@ -116,7 +118,7 @@ _lib = None
 
 
 def cost_estimate(params, n_r, n_s, n_rp, n_sp, n_distinct, sum_k, survivors, key_bytes, payload_bytes,
-                  sort_passes, dedup_passes, corr_op, agg):
+                  sort_passes, dedup_passes, corr_op, agg, narrow_keys=0):
     """Eqs. (1)-(9) of the paper's cost model for one plan shape
     (nestgpu_cost_estimate_plan; host arithmetic, no device).  params: a
     CostParams (from Engine.cost_calibrate) or its as_dict().  Returns
@@ -133,7 +135,8 @@ def cost_estimate(params, n_r, n_s, n_rp, n_sp, n_distinct, sum_k, survivors, ke
                 setattr(p, k, v)
         params = p
     ci = CostInput(int(n_r), int(n_s), int(n_rp), int(n_sp), int(n_distinct), int(sum_k), int(survivors),
-                   int(key_bytes), int(payload_bytes), int(sort_passes), int(dedup_passes), CMP[corr_op], AGG[agg])
+                   int(key_bytes), int(payload_bytes), int(sort_passes), int(dedup_passes), int(narrow_keys),
+                   CMP[corr_op], AGG[agg])
     e = CostEstimate()
     st = lib.nestgpu_cost_estimate_plan(ctypes.byref(params), ctypes.byref(ci), ctypes.byref(e))
     if st != OK:

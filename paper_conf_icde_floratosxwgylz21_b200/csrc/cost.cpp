@@ -12,8 +12,10 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstring>
+#include <vector>
 
 #include "../../include/nestgpu.h"
 #include "internal.h"
@@ -69,7 +71,7 @@ nestgpu_status nestgpu_cost_calibrate(nestgpu_ctx *c, int64_t n_rows, nestgpu_co
     const cudaStream_t st = ng::ctx_stream(c);
     long long *L = ng::ctx_launches(c);
     const int sms = ng::ctx_num_sms(c);
-    long long n = n_rows > 0 ? n_rows : (4ll << 20);
+    long long n = n_rows > 0 ? n_rows : (16ll << 20);
     n = std::min<long long>(n, 1ll << 28);
 
     // ------------------------------------------------------------ buffers
@@ -270,6 +272,80 @@ nestgpu_status nestgpu_cost_calibrate(nestgpu_ctx *c, int64_t n_rows, nestgpu_co
     }
 #undef CC
     ng::ctx_scratch_reset(c);
+
+    // Fixed host-side overheads: tiny plans through the public API, wall
+    // clock, minus what the model already charges for them.
+    {
+        uint64_t mark;
+        nestgpu_status s = nestgpu_mark(c, &mark);
+        if (s) return s;
+        const int m = 256;
+        std::vector<int32_t> k(m), v(m);
+        for (int i = 0; i < m; i++) { k[i] = (i * 37) % 64; v[i] = (i * 11) % 16; }
+        int32_t rk, rv, sk, sv;
+        if ((s = nestgpu_load_column(c, NG_INT32, 0, k.data(), nullptr, m, &rk)) ||
+            (s = nestgpu_load_column(c, NG_INT32, 0, v.data(), nullptr, m, &rv)) ||
+            (s = nestgpu_load_column(c, NG_INT32, 0, k.data(), nullptr, m, &sk)) ||
+            (s = nestgpu_load_column(c, NG_INT32, 0, v.data(), nullptr, m, &sv)))
+            return s;
+        nestgpu_plan P;
+        memset(&P, 0, sizeof P);
+        P.outer_key_cols[0] = rk;
+        P.inner_key_cols[0] = sk;
+        P.n_key_cols = 1;
+        P.corr_op = NG_EQ;
+        P.agg = NG_MIN;
+        P.agg_col = sv;
+        P.outer_cmp_col = rv;
+        P.outer_op = NG_EQ;
+        P.lhs_mult = P.rhs_mult = 1;
+        P.index = -1;
+        nestgpu_result res;
+        auto wall = [&](auto fn, double *ms) -> nestgpu_status {
+            double t[7];
+            for (int r = 0; r < 8; r++) {
+                const auto a = std::chrono::steady_clock::now();
+                nestgpu_status e = fn();
+                if (e) return e;
+                cudaStreamSynchronize(st);
+                const auto b = std::chrono::steady_clock::now();
+                if (r) t[r - 1] = std::chrono::duration<double, std::milli>(b - a).count();
+            }
+            std::sort(t, t + 7);
+            *ms = t[3];
+            return NESTGPU_OK;
+        };
+        nestgpu_cost_input in;
+        memset(&in, 0, sizeof in);
+        in.n_r = in.n_s = in.n_rp = in.n_sp = m;
+        in.n_distinct = 64;
+        in.sum_k = (int64_t)m * 4;
+        in.key_bytes = 4;
+        in.payload_bytes = 4;
+        in.sort_passes = 1;
+        in.dedup_passes = 1;
+        in.corr_op = NG_EQ;
+        in.agg = NG_MIN;
+        nestgpu_cost_estimate est;
+        double t_exec, t_dedup, t_build;
+        if ((s = wall([&] { return nestgpu_exec_correlated(c, &P, &res); }, &t_exec))) return s;
+        P.dedup = 1;
+        if ((s = wall([&] { return nestgpu_exec_correlated(c, &P, &res); }, &t_dedup))) return s;
+        P.dedup = 0;
+        int32_t ix = -1;
+        const int32_t keyc[1] = {sk};
+        if ((s = wall([&] {
+                if (ix >= 0) nestgpu_drop_index(c, ix);
+                return nestgpu_build_index(c, keyc, 1, sv, nullptr, 0, &ix);
+            }, &t_build)))
+            return s;
+        nestgpu_cost_estimate_plan(out, &in, &est);
+        out->exec_overhead_ms = pos(t_exec - est.ms[NESTGPU_STRATEGY_NESTED_LOOP]);
+        out->dedup_overhead_ms = pos(t_dedup - t_exec - (est.ms[NESTGPU_STRATEGY_NESTED_LOOP_CACHED] -
+                                                         est.ms[NESTGPU_STRATEGY_NESTED_LOOP]));
+        out->build_overhead_ms = pos(t_build - est.index_build_ms);
+        if ((s = nestgpu_release(c, mark))) return s;
+    }
     return NESTGPU_OK;
 }
 
@@ -297,21 +373,30 @@ nestgpu_status nestgpu_cost_estimate_plan(const nestgpu_cost_params *p, const ne
     // U, Eq. (8): outer selection, then finalize + compaction (M * D_r * sum Rs)
     const double rs = 18.0 + (in->agg == NG_AVG ? 16.0 : 0.0);   // id + value + valid + passed (+ sum, nn)
     const double U = selection(nR) + C + p->final_ms_per_row * nRp +
-                     p->materialize_ms_per_byte * (double)in->survivors * rs + p->sync_ms;
+                     p->materialize_ms_per_byte * (double)in->survivors * rs + p->sync_ms + p->exec_overhead_ms;
     out->outer_ms = U;
 
+    // bytes per key moved by the passes: (key in + key out) / 2 + payload;
+    // narrowed 8-byte keys are 4 bytes wide between the first and last pass
+    auto pass_bytes = [&](double passes) {
+        if (passes <= 0) return 0.0;
+        if (!(in->narrow_keys && kb == 8 && passes >= 2)) return passes * (kb + vb);
+        return 2 * (6 + vb) + (passes - 2) * (4 + vb);
+    };
     // caching: S - Ch evaluations after sorting / grouping the R' keys
     const double dp = in->dedup_passes;
     const double dedup = 2 * C + p->hist_ms_per_key_digit * nRp * dp +
-                         dp * (2 * C + p->sort_ms_per_key * nRp + p->sort_ms_per_byte * nRp * (kb + 4)) + C +
+                         dp * (2 * C + p->sort_ms_per_key * nRp) +
+                         p->sort_ms_per_byte * nRp * (pass_bytes(dp) - dp * vb + dp * 4) + C +
                          p->group_ms_per_key * nRp +
-                         2 * p->sync_ms;
+                         2 * p->sync_ms + p->dedup_overhead_ms;
 
     // index build (invariant, once): S' selection + histogram + radix passes;
     // plus the payload prefix aggregates when the plan reads them (NEXT 3)
     const double sp = in->sort_passes;
-    double build = selection(nS) + p->sync_ms + (sp > 0 ? 2 * C + p->hist_ms_per_key_digit * nSp * sp : 0) +
-                   sp * (2 * C + p->sort_ms_per_key * nSp + p->sort_ms_per_byte * nSp * (kb + vb));
+    double build = selection(nS) + p->sync_ms + p->build_overhead_ms +
+                   (sp > 0 ? 2 * C + p->hist_ms_per_key_digit * nSp * sp : 0) +
+                   sp * (2 * C + p->sort_ms_per_key * nSp) + p->sort_ms_per_byte * nSp * pass_bytes(sp);
     if (value_agg && (in->corr_op != NG_EQ || sumavg)) build += (minmax ? 6 : 3) * C + p->aux_ms_per_elem * nSp;
     out->index_build_ms = build;
 

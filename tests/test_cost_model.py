@@ -20,7 +20,8 @@ P = {"launch_ms": 0.003, "filter_ms_per_row": 7e-9, "hist_ms_per_key_digit": 1e-
      "sort_ms_per_byte": 8e-10, "probe_ms_per_step": 5e-10, "range_ms_per_elem": 3e-10, "aux_ms_per_elem": 2e-8,
      "bnl_ms_per_pair": [[1.1e-10, 7e-11, 1.3e-10, 6e-11], [2.2e-10, 1.4e-10, 2.6e-10, 1.2e-10]],
      "final_ms_per_row": 2e-8,
-     "materialize_ms_per_byte": 2e-10, "group_ms_per_key": 1e-8, "sync_ms": 0.012}
+     "materialize_ms_per_byte": 2e-10, "group_ms_per_key": 1e-8, "sync_ms": 0.012,
+     "exec_overhead_ms": 0.02, "build_overhead_ms": 0.01, "dedup_overhead_ms": 0.01}
 
 
 def shape(**kw):

@@ -446,3 +446,17 @@ def test_int64_keys_narrowed_sort(eng, base):
             for dedup in (False, True):
                 g = run(eng, t, plan, "index", emit_all=True, dtypes=dt, dedup=dedup)
                 assert_parity(g, ref, plan, True, ctx=(base, corr_op, agg, dedup))
+
+
+def test_c5_full_size(eng):
+    """BASELINE configs[4] at its full size (|R| = |S| = 16M, '>' MIN on the
+    nested loop -- bench.py --workload C5's launch configuration): the closed
+    form on every one of the 16M rows, the oracle on 200 sampled rows."""
+    t = query1.config("C5")
+    plan = make_plan(">", "min", "=")
+    rows = np.unique(np.random.default_rng(9).integers(0, 16_000_000, 200))
+    g = run(eng, t, plan, "bnl", emit_all=True)
+    valid, value, _, _ = ind.closed_form(t["R"]["col1"], t["S"]["col1"], t["S"]["col2"], ">", "min")
+    assert np.array_equal(g["value"], value)
+    assert np.array_equal(g["valid"].astype(bool), valid)
+    assert_parity(g, oracle.evaluate(t, plan, rows=rows), plan, True, rows=rows, ctx="C5 full")

@@ -67,6 +67,13 @@ def _passes(keys, kb):
     return sum(1 for i in range(kb) if (d >> (8 * i)) & 0xff)
 
 
+def _narrow(keys, kb):
+    """8-byte keys whose high words agree (the engine sorts them as 4-byte keys)"""
+    if kb != 8 or len(keys) < 2:
+        return 0
+    return int(((int(np.bitwise_and.reduce(keys)) ^ int(np.bitwise_or.reduce(keys))) >> 32) == 0)
+
+
 def stats(tables, plan, survivors):
     R, S = tables["R"], tables["S"]
     rm = _mask(R, tables.get("R_valid"), plan["outer_preds"])
@@ -85,7 +92,7 @@ def stats(tables, plan, survivors):
     return dict(n_r=len(rm), n_s=len(sm), n_rp=int(rm.sum()), n_sp=int(sm.sum()),
                 n_distinct=int(len(np.unique(rk))), sum_k=int(k.sum()), survivors=int(survivors),
                 key_bytes=kb, payload_bytes=vb, sort_passes=_passes(sk, kb), dedup_passes=_passes(rk, kb),
-                corr_op=op, agg=plan["agg"])
+                narrow_keys=_narrow(sk, kb), corr_op=op, agg=plan["agg"])
 
 
 def measure(eng, tables, plan, reps=3):
