@@ -113,3 +113,18 @@ def join_subquery_both(eng, L, RT, S, join_on, l_rid, sub_plan, mode="index"):
     a = eng.gather_column(lid, res)
     b = eng.gather_column(rid, res)
     return _pairs_to_host(eng, eng.column_info(a)["d_values"], eng.column_info(b)["d_values"], res.n_rows)
+
+
+def exec_auto(eng, plan, R, S, params, stats, emit_all=False, row_id_base=0):
+    """Run a plan with the strategy the cost model predicts fastest (P:75,
+    §IV: the model "guide[s] subquery processing by selecting the most
+    effective execution path").  params: Engine.cost_calibrate(); stats: the
+    plan's cardinalities (nestgpu_cost_input fields, known in advance as in
+    the paper's evaluation).  Returns (result, strategy, predicted)."""
+    from .binding import cost_estimate
+    est = cost_estimate(params, **stats)
+    strategy = est["best"]
+    idx = eng.index_for_plan(plan, S) if strategy.startswith("index") else -1
+    res = eng.exec(plan, R, S, index=idx, emit_all=emit_all, row_id_base=row_id_base,
+                   dedup=strategy.endswith("cached"))
+    return res, strategy, est

@@ -101,3 +101,36 @@ def test_calibrate_and_choose_on_gpu():
     assert p["bnl_ms_per_pair"][0][0] > 1.2 * p["bnl_ms_per_pair"][0][1]
     assert p["bnl_ms_per_pair"][1][1] > 1.2 * p["bnl_ms_per_pair"][0][1]
     assert cost_estimate(p, **shape())["best"] in ("index", "index_cached")
+
+
+@pytest.mark.gpu
+def test_exec_auto_matches_oracle_and_picks_index_for_large_equality():
+    """nested.exec_auto runs the model's choice; the result is the oracle's
+    whatever the choice (C1 small: nested loop; C2-shaped '=': index)."""
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import numpy as np
+    import oracle
+    from datagen import make_plan, query1
+    from paper_conf_icde_floratosxwgylz21_b200 import Engine, nested
+    eng = Engine(0, arena_bytes=2 << 30)
+    try:
+        params = eng.cost_calibrate(1 << 20)
+        for t, want in ((query1.config("C1"), None), (query1.config("C2", n_r=50_000), "index")):
+            plan = make_plan("=", "min", "=")
+            n_r, n_s = len(t["R"]["col1"]), len(t["S"]["col1"])
+            stats = dict(n_r=n_r, n_s=n_s, n_rp=n_r, n_sp=n_s, n_distinct=len(np.unique(t["R"]["col1"])),
+                         sum_k=4 * n_r, survivors=n_r // 16, key_bytes=4, payload_bytes=4, sort_passes=3,
+                         dedup_passes=3, corr_op="=", agg="min")
+            m = eng.mark()
+            R, S = eng.load_table(t["R"]), eng.load_table(t["S"])
+            res, strategy, _ = nested.exec_auto(eng, plan, R, S, params, stats)
+            g = eng.result_to_numpy(res)
+            eng.release(m)
+            rows, vals = oracle.survivors(oracle.evaluate(t, plan))
+            assert np.array_equal(g["row"], rows) and np.array_equal(g["value"], vals), strategy
+            if want:
+                assert strategy.startswith(want), strategy
+    finally:
+        eng.close()
