@@ -109,6 +109,32 @@ nestgpu_status fail(nestgpu_ctx *c, nestgpu_status code, const char *fmt, ...)
                         __FILE__, __LINE__);                                                        \
     } while (0)
 
+// Radix-pass plan for n encoded keys of kb bytes whose AND / OR over all keys
+// are kand / kor: only bits that vary need sorting, so 8-bit digit windows
+// are placed greedily from the lowest varying bit (the fewest windows that
+// cover every varying bit), e.g. keys that are multiples of 32 below 2^26
+// take 3 passes instead of 4.  When every varying bit lies in the low word
+// of a 64-bit key the windows stay inside bits 0-31 (start <= 24; overlapping
+// a lower window is harmless for a stable LSD sort), so the passes can run
+// on 32-bit keys.  Returns the number of passes, shifts[] their bit offsets.
+static int plan_sort_passes(int kb, unsigned long long kand, unsigned long long kor, long long n, int *shifts)
+{
+    if (n < 2) return 0;
+    const unsigned long long var = kand ^ kor;
+    const bool low = (var >> 32) == 0;
+    int np = 0;
+    for (int b = 0; b < kb * 8 && np < 8;) {
+        if (!((var >> b) & 1ull)) {
+            b++;
+            continue;
+        }
+        const int s = low && b > 24 ? 24 : b;
+        shifts[np++] = s;
+        b = s + 8;
+    }
+    return np;
+}
+
 size_t align_up(size_t x) { return (x + ALIGN - 1) / ALIGN * ALIGN; }
 
 // Start a new scratch generation: everything salloc'd before dies here.
@@ -514,16 +540,10 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     memcpy(&nsp, c->pinned, 8);
     memcpy(&kand, c->pinned + 4, 8);
     memcpy(&kor, c->pinned + 6, 8);
-    // plan the passes: a digit on which every key agrees needs no pass
-    std::vector<int> passes;
-    if (nsp > 1)
-        for (int d = 0; d < kb; d++)
-            if (((kand ^ kor) >> (8 * d)) & 0xff) passes.push_back(d);
     int shifts[8];
-    for (size_t p = 0; p < passes.size(); p++) shifts[p] = passes[p] * 8;
+    const int np = plan_sort_passes(kb, kand, kor, nsp, shifts);
     prof_begin(c, 2);
-    CUDA_TRY(c, ng::launch_digit_hist(kb, tk, nsp, shifts, (int)passes.size(), hist, dbase, c->num_sms, c->stream,
-                                      &c->launches));
+    CUDA_TRY(c, ng::launch_digit_hist(kb, tk, nsp, shifts, np, hist, dbase, c->num_sms, c->stream, &c->launches));
 
     IndexRec ix{};
     ix.off = c->lo;
@@ -540,7 +560,6 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     c->pinned[8 * 256 + 4] = (unsigned)(nsp & 0xffffffffu);
     c->pinned[8 * 256 + 5] = (unsigned)((unsigned long long)nsp >> 32);
     CUDA_TRY(c, cudaMemcpyAsync(ix.d_n, c->pinned + 8 * 256 + 4, 8, cudaMemcpyHostToDevice, c->stream));
-    const int np = (int)passes.size();
     if (np == 0) {
         if (nsp > 0) {
             CUDA_TRY(c, cudaMemcpyAsync(ix.keys, tk, (size_t)nsp * kb, cudaMemcpyDeviceToDevice, c->stream));
@@ -789,10 +808,8 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         memcpy(&nrp, c->pinned, 8);
         memcpy(&kand, c->pinned + 12, 8);
         memcpy(&kor, c->pinned + 14, 8);
-        int shifts[8], np = 0;
-        if (nrp > 1)
-            for (int d = 0; d < kb; d++)
-                if (((kand ^ kor) >> (8 * d)) & 0xff) shifts[np++] = 8 * d;
+        int shifts[8];
+        const int np = plan_sort_passes(kb, kand, kor, nrp, shifts);
         CUDA_TRY(c, ng::launch_iota(pos, nrp, c->stream, &c->launches));
         CUDA_TRY(c, ng::launch_digit_hist(kb, rkeys, nrp, shifts, np, hist, dbase, c->num_sms, c->stream,
                                           &c->launches));

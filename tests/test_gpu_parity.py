@@ -460,3 +460,88 @@ def test_c5_full_size(eng):
     assert np.array_equal(g["value"], value)
     assert np.array_equal(g["valid"].astype(bool), valid)
     assert_parity(g, oracle.evaluate(t, plan, rows=rows), plan, True, rows=rows, ctx="C5 full")
+
+
+def _key_pattern(name, n, rng):
+    """Encoded-key bit patterns for the radix-pass planner (api.cpp
+    plan_sort_passes): which bits vary decides where the 8-bit windows go."""
+    if name == "mult32_lt2^26":       # varying bits 5..25 -> 3 windows (5, 13, 21)
+        return rng.integers(0, 1 << 21, n) * 32, "int32"
+    if name == "bits1_to_27":         # 27 varying bits from bit 1 -> windows 1, 9, 17, 24 (clamped)
+        return rng.integers(0, 1 << 27, n) * 2, "int32"
+    if name == "i64_low_word":        # 64-bit, high word constant, bits 3..31 vary (narrowed passes, clamp)
+        return (7 << 40) + rng.integers(0, 1 << 29, n) * 8, "int64"
+    if name == "i64_straddle":        # 64-bit, bits 20..44 vary (windows cross bit 32, no narrowing)
+        return -(1 << 50) + rng.integers(0, 1 << 25, n) * (1 << 20), "int64"
+    if name == "i64_full":            # all 64 bits vary
+        return rng.integers(-2 ** 63, 2 ** 63 - 1, n, dtype=np.int64), "int64"
+    if name == "i32_negative_dups":   # signed, heavy duplicates
+        k = rng.integers(-1000, 1000, n)
+        k[::5] = -7
+        return k, "int32"
+    raise KeyError(name)
+
+
+@pytest.mark.parametrize("pattern", ["mult32_lt2^26", "bits1_to_27", "i64_low_word", "i64_straddle",
+                                     "i64_full", "i32_negative_dups"])
+@pytest.mark.parametrize("n", [1, 2, 4095, 4097, 1_000_003])
+@pytest.mark.parametrize("pay", ["int32", "int64", None])
+def test_index_sort_digit_windows(eng, pattern, n, pay):
+    """a4 on key patterns whose varying bits sit at odd offsets, cross bit 32,
+    or span all 64 bits; 4/8-byte payloads or none (8- to 16-byte items, two
+    tile sizes); sizes below, at and across tile boundaries.  The index must
+    be the encoded keys ascending with every payload carried by its own key
+    (compared with numpy's sort of the same encoded keys)."""
+    import torch
+    rng = np.random.default_rng(hash((pattern, n)) % (1 << 32))
+    k, kdt = _key_pattern(pattern, n, rng)
+    k = np.asarray(k, dtype=np.int64)
+    cols, dts = {"k": k}, {"k": kdt}
+    if pay is not None:
+        cols["v"] = np.arange(n, dtype=np.int64) * (1 if pay == "int32" else (1 << 33) + 1)
+        dts["v"] = pay
+    m = eng.mark()
+    try:
+        S = eng.load_table(cols, dtypes=dts)
+        ix = eng.build_index(S, ["k"], "v" if pay else None)
+        info = eng.index_info(ix)
+        kb = 4 if kdt == "int32" else 8
+        assert info["n"] == n and info["key_bytes"] == kb
+        if kb == 4:
+            enc = k.astype(np.int32).view(np.uint32) ^ np.uint32(0x80000000)
+            keys = eng.arena_view(info["d_keys"], n * 4).view(torch.int32).cpu().numpy().view(np.uint32)
+        else:
+            enc = k.view(np.uint64) ^ np.uint64(1 << 63)
+            keys = eng.arena_view(info["d_keys"], n * 8).view(torch.int64).cpu().numpy().view(np.uint64)
+        assert np.array_equal(keys, np.sort(enc))
+        if pay is not None:
+            vb = 4 if pay == "int32" else 8
+            tdt = torch.int32 if vb == 4 else torch.int64
+            p = eng.arena_view(info["d_payload"], n * vb).view(tdt).cpu().numpy().astype(np.int64)
+            row = p if vb == 4 else p // ((1 << 33) + 1)
+            assert np.array_equal(np.sort(row), np.arange(n))       # every payload exactly once
+            assert np.array_equal(keys, enc[row])                   # carried with its own key
+    finally:
+        eng.release(m)
+
+
+@pytest.mark.parametrize("pattern", ["mult32_lt2^26", "bits1_to_27", "i64_low_word", "i64_straddle"])
+def test_dedup_sort_digit_windows(eng, pattern):
+    """The R' key sort of caching on the same key patterns: results
+    vs the oracle with and without caching, both subquery kernels."""
+    rng = np.random.default_rng(11)
+    kr, kdt = _key_pattern(pattern, 20011, rng)
+    ks, _ = _key_pattern(pattern, 9001, rng)
+    kr = np.asarray(kr, dtype=np.int64)
+    rep = np.arange(0, len(kr), 3)
+    kr[rep] = kr[(rep + 1) % len(kr)]              # repeated correlated values
+    ks = np.concatenate([np.asarray(ks, dtype=np.int64), kr[:3000]])
+    t = {"R": {"col1": kr, "col2": rng.integers(0, 5, len(kr))},
+         "S": {"col1": ks, "col2": rng.integers(0, 5, len(ks))}}
+    dt = {"R": {"col1": kdt, "col2": "int32"}, "S": {"col1": kdt, "col2": "int32"}}
+    for corr_op, agg, mode in (("=", "count", "index"), ("=", "min", "index"), ("<", "min", "bnl")):
+        plan = make_plan(corr_op, agg, "<=")
+        ref = oracle.evaluate(t, plan)
+        for dedup in (False, True):
+            g = run(eng, t, plan, mode, emit_all=True, dtypes=dt, dedup=dedup)
+            assert_parity(g, ref, plan, True, ctx=(pattern, corr_op, agg, dedup))

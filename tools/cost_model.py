@@ -64,7 +64,19 @@ def _passes(keys, kb):
     a = np.bitwise_and.reduce(keys)
     o = np.bitwise_or.reduce(keys)
     d = int(a ^ o)
-    return sum(1 for i in range(kb) if (d >> (8 * i)) & 0xff)
+    # the engine's plan (api.cpp plan_sort_passes): 8-bit windows placed
+    # greedily from the lowest varying bit, kept inside bits 0-31 when the
+    # high word does not vary
+    low = (d >> 32) == 0
+    n, b = 0, 0
+    while b < 8 * kb:
+        if not (d >> b) & 1:
+            b += 1
+            continue
+        s = 24 if low and b > 24 else b
+        n += 1
+        b = s + 8
+    return n
 
 
 def _narrow(keys, kb):
