@@ -27,6 +27,18 @@ namespace ng {
 #ifndef NG_S_MINB
 #define NG_S_MINB 4   // __launch_bounds__ min blocks per SM (register cap; 1 lets ptxas take 160+)
 #endif
+#ifndef NG_S_NBUF
+#define NG_S_NBUF 1   // persistent pass: tile buffers per CTA (2 = next tile prefetched)
+#endif
+#ifndef NG_S_LB_EARLY
+#define NG_S_LB_EARLY 0   // look-back before ranking (1) or after (0)
+#endif
+#ifndef NG_S_LB_BATCH
+#define NG_S_LB_BATCH 4  // look-back: predecessor tiles examined per round trip
+#endif
+#ifndef NG_S_PITEMS
+#define NG_S_PITEMS 24   // persistent pass: items per thread for <= 8-byte (key, payload) items
+#endif
 #ifndef NG_S_PMINB
 #define NG_S_PMINB 3  // persistent pass: CTAs per SM the register budget must allow
 #endif
@@ -42,7 +54,7 @@ constexpr unsigned D_AGG = 1u << 30, D_INC = 2u << 30, D_VAL = (1u << 30) - 1;
 size_t sort_scratch_bytes(long long n)
 {
     // status words for the smallest tile any pass uses (16-byte items)
-    long long tiles = (n + S_THREADS * 8 - 1) / (S_THREADS * 8);
+    long long tiles = (n + S_THREADS * (NG_S_PITEMS / 2) - 1) / (S_THREADS * (NG_S_PITEMS / 2));
     return (size_t)tiles * 256 * 4 + 256;
 }
 
@@ -218,11 +230,11 @@ __device__ __forceinline__ unsigned match_digit8(unsigned d)
 template <typename K, int VB>
 struct PassCfg {
     using V = typename std::conditional<VB == 8, long long, int>::type;
-    static constexpr int ITEMS = (sizeof(K) + VB) > 8 ? 8 : 16;
+    static constexpr int ITEMS = (sizeof(K) + VB) > 8 ? NG_S_PITEMS / 2 : NG_S_PITEMS;
     static constexpr int TILE = S_THREADS * ITEMS;
     static constexpr int KBYTES = TILE * (int)sizeof(K);
     static constexpr int BUF = KBYTES + (VB ? TILE * VB : 0);
-    static constexpr size_t SMEM = 2 * (size_t)BUF;
+    static constexpr size_t SMEM = NG_S_NBUF * (size_t)BUF;
 };
 
 template <typename K, int VB, typename KO = K>
@@ -240,8 +252,8 @@ onesweep_p_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *
     __shared__ unsigned s_cnt[S_WARPS][256];   // early counts, then running counters
     __shared__ unsigned s_off[256];            // global destination - tile start of the digit
     __shared__ unsigned s_wsum[S_WARPS];
-    __shared__ unsigned s_tile[2];
-    __shared__ __align__(8) unsigned long long bar[2];
+    __shared__ unsigned s_tile[NG_S_NBUF];
+    __shared__ __align__(8) unsigned long long bar[NG_S_NBUF];
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const long long tiles = (n + TILE - 1) / TILE;
@@ -261,10 +273,9 @@ onesweep_p_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *
 
     for (int i = tid; i < S_WARPS * 256; i += S_THREADS) (&s_cnt[0][0])[i] = 0;
     if (tid == 0) {
-        mbar_init(&bar[0], 1);
-        mbar_init(&bar[1], 1);
+        for (int b = 0; b < NG_S_NBUF; b++) mbar_init(&bar[b], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        for (int b = 0; b < 2; b++) {
+        for (int b = 0; b < NG_S_NBUF; b++) {
             const unsigned t = atomicAdd(counter, 1u);
             s_tile[b] = t;
             if (t < tiles) issue(t, b);
@@ -275,10 +286,10 @@ onesweep_p_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *
     const int d = tid;   // the digit this thread owns in the per-digit steps
 
     for (int it = 0;; it++) {
-        const int b = it & 1;
+        const int b = it % NG_S_NBUF;
         const long long tile = s_tile[b];
         if (tile >= tiles) break;
-        mbar_wait(&bar[b], (unsigned)(it >> 1) & 1u);
+        mbar_wait(&bar[b], (unsigned)(it / NG_S_NBUF) & 1u);
         K *s_k = (K *)(smem + b * C::BUF);
         V *s_v = (V *)(smem + b * C::BUF + C::KBYTES);
         const long long base = tile * TILE;
@@ -313,9 +324,39 @@ onesweep_p_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *
         }
         unsigned *my_status = status + tile * 256 + d;
         st_relaxed_u32(my_status, (tile == 0 ? D_INC : D_AGG) | cnt);
-        unsigned sv[4];
+        // decoupled look-back for digit d over the preceding tiles (their
+        // counts were published right after their early counts)
+        // first batch of predecessor statuses: loads in flight from here on
+        unsigned sv[NG_S_LB_BATCH];
 #pragma unroll
-        for (int q = 0; q < 4; q++) sv[q] = tile - 1 - q >= 0 ? ld_relaxed_u32(status + (tile - 1 - q) * 256 + d) : D_INC;
+        for (int q = 0; q < NG_S_LB_BATCH; q++)
+            sv[q] = tile - 1 - q >= 0 ? ld_relaxed_u32(status + (tile - 1 - q) * 256 + d) : D_INC;
+        auto lookback = [&]() -> unsigned {
+            unsigned ex = 0;
+            for (long long p = tile - 1; p >= 0; p -= NG_S_LB_BATCH) {
+                if (p != tile - 1) {
+#pragma unroll
+                    for (int q = 0; q < NG_S_LB_BATCH; q++)
+                        sv[q] = p - q >= 0 ? ld_relaxed_u32(status + (p - q) * 256 + d) : D_INC;
+                }
+                bool done = false;
+#pragma unroll
+                for (int q = 0; q < NG_S_LB_BATCH; q++) {
+                    if (!done) {
+                        unsigned sq = sv[q];
+                        while ((sq >> 30) == 0) sq = ld_relaxed_u32(status + (p - q) * 256 + d);
+                        ex += sq & D_VAL;
+                        done = (sq >> 30) == 2;
+                    }
+                }
+                if (done) break;
+            }
+            if (tile > 0) st_relaxed_u32(my_status, D_INC | (ex + cnt));
+            return ex;
+        };
+#if NG_S_LB_EARLY
+        const unsigned excl = lookback();   // INC published before ranking: successors find it at once
+#endif
         unsigned incl = cnt;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -354,29 +395,9 @@ onesweep_p_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *
             if constexpr (VB > 0) s_v[pos] = val[j];
             __syncwarp();
         }
-        // 5. finish the look-back for digit d (predecessors published their
-        // counts before ranking, so this rarely waits)
-        unsigned excl = 0;
-        if (tile > 0) {
-            long long p = tile - 1;
-            bool done = false;
-            while (!done) {
-#pragma unroll
-                for (int q = 0; q < 4; q++) {
-                    if (done) break;
-                    unsigned sq = sv[q];
-                    while ((sq >> 30) == 0) sq = ld_relaxed_u32(status + (p - q) * 256 + d);
-                    excl += sq & D_VAL;
-                    done = (sq >> 30) == 2;
-                }
-                p -= 4;
-                if (!done) {
-#pragma unroll
-                    for (int q = 0; q < 4; q++) sv[q] = p - q >= 0 ? ld_relaxed_u32(status + (p - q) * 256 + d) : D_INC;
-                }
-            }
-            st_relaxed_u32(my_status, D_INC | (excl + cnt));
-        }
+#if !NG_S_LB_EARLY
+        const unsigned excl = lookback();
+#endif
         s_off[d] = digit_base[d] + excl - tex;
         __syncthreads();
         for (int i = tid; i < S_WARPS * 256; i += S_THREADS) (&s_cnt[0][0])[i] = 0;
