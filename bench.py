@@ -139,18 +139,26 @@ class ClockSampler:
 # ---------------------------------------------------------------- CPU oracle
 def time_oracle(tables, plans, budget_s, calib_rows=8):
     """Time the oracle (as it stands) on a bounded sample: the first m rows of
-    R for every plan, m sized to ~budget_s seconds on this host."""
+    R for every plan, m sized to ~budget_s seconds on this host.  The size is
+    found by growing a calibration sample 4x until it runs >= budget/8 (a
+    handful of rows under-fills the oracle's OpenMP threads and would
+    overestimate the per-row cost), then scaled to the budget."""
     import oracle
     n_r = len(tables["R"]["col1"])
-    t0 = time.perf_counter()
-    for plan, _ in plans:
-        oracle.evaluate(tables, plan, rows=np.arange(min(calib_rows, n_r)))
-    per_row = max((time.perf_counter() - t0) / (len(plans) * min(calib_rows, n_r)), 1e-9)
-    m = int(max(calib_rows, min(n_r, budget_s / (per_row * len(plans)))))
-    t0 = time.perf_counter()
-    for plan, _ in plans:
-        oracle.evaluate(tables, plan, rows=np.arange(m))
-    dt = time.perf_counter() - t0
+
+    def run(m):
+        t0 = time.perf_counter()
+        for plan, _ in plans:
+            oracle.evaluate(tables, plan, rows=np.arange(m))
+        return time.perf_counter() - t0
+
+    m = min(calib_rows, n_r)
+    t = run(m)
+    while t < budget_s / 8 and m < n_r:
+        m = min(n_r, m * 4)
+        t = run(m)
+    m = int(max(1, min(n_r, m * budget_s / max(t, 1e-6))))
+    dt = run(m)
     return {"value": m * len(plans) / dt, "unit": "outer tuples/s", "cores": oracle.max_threads(),
             "kind": "oracle", "seconds": dt,
             "sample": "first %d R rows x all %d S rows for each of the %d plans (%d outer tuples)" % (

@@ -37,6 +37,9 @@ namespace ng {
 #ifndef NG_B_STAGES
 #define NG_B_STAGES 3
 #endif
+#ifndef NG_B_UNITS
+#define NG_B_UNITS 64      // work units per persistent CTA (tail granularity vs per-unit fill + merge)
+#endif
 #ifndef NG_B_UNROLL
 #define NG_B_UNROLL 2      // element groups per inner iteration (DESIGN.md §8 tuning log)
 #endif
@@ -219,7 +222,8 @@ __device__ __forceinline__ void tile_full(const K *__restrict__ tk, const V *__r
         V vv[U][KV];
 #pragma unroll
         for (int u = 0; u < U; u++) {
-            const int eu = min(e + u * STEP, TILE - KV);   // clamped: the ragged tail is skipped below
+            // clamped when whole iterations do not tile TILE: the ragged tail is skipped below
+            const int eu = (TILE % (STEP * U)) == 0 ? e + u * STEP : min(e + u * STEP, TILE - KV);
             if constexpr (sizeof(K) == 4) {
                 const uint4 q = *reinterpret_cast<const uint4 *>(tk + eu);
                 kk[u][0] = q.x; kk[u][1] = q.y; kk[u][2] = q.z; kk[u][3] = q.w;

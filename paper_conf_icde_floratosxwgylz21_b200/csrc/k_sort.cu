@@ -30,6 +30,12 @@ namespace ng {
 #ifndef NG_S_NBUF
 #define NG_S_NBUF 1   // persistent pass: tile buffers per CTA (2 = next tile prefetched)
 #endif
+#ifndef NG_S_LATE_PREFETCH
+#define NG_S_LATE_PREFETCH 0   // 1: two buffers, the next tile taken once this tile's offsets are known
+#endif
+#if NG_S_LATE_PREFETCH && NG_S_NBUF != 2
+#error "NG_S_LATE_PREFETCH needs NG_S_NBUF 2"
+#endif
 #ifndef NG_S_LB_EARLY
 #define NG_S_LB_EARLY 0   // look-back before ranking (1) or after (0)
 #endif
@@ -275,7 +281,7 @@ onesweep_p_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *
     if (tid == 0) {
         for (int b = 0; b < NG_S_NBUF; b++) mbar_init(&bar[b], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        for (int b = 0; b < NG_S_NBUF; b++) {
+        for (int b = 0; b < (NG_S_LATE_PREFETCH ? 1 : NG_S_NBUF); b++) {
             const unsigned t = atomicAdd(counter, 1u);
             s_tile[b] = t;
             if (t < tiles) issue(t, b);
@@ -400,6 +406,16 @@ onesweep_p_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *
 #endif
         s_off[d] = digit_base[d] + excl - tex;
         __syncthreads();
+#if NG_S_LATE_PREFETCH
+        // this tile's counts are published and its offsets resolved: take the
+        // next tile now (its predecessors wait for it only one write-out
+        // long) and let its bulk copy overlap the write-out
+        if (tid == 0) {
+            const unsigned t = atomicAdd(counter, 1u);
+            s_tile[b ^ 1] = t;
+            if (t < tiles) issue(t, b ^ 1);
+        }
+#endif
         for (int i = tid; i < S_WARPS * 256; i += S_THREADS) (&s_cnt[0][0])[i] = 0;
 #pragma unroll 4
         for (int p = tid; p < tile_n; p += S_THREADS) {
@@ -410,12 +426,14 @@ onesweep_p_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *
             if constexpr (VB > 0) vout[dst] = s_v[p];
         }
         __syncthreads();
+#if !NG_S_LATE_PREFETCH
         if (tid == 0) {
             const unsigned t = atomicAdd(counter, 1u);
             s_tile[b] = t;
             if (t < tiles) issue(t, b);
         }
         __syncthreads();
+#endif
     }
 }
 

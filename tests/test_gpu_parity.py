@@ -8,6 +8,8 @@ aggregate, NULLs and empty subqueries, local predicates, composite keys,
 the BASELINE configs (C1 full; C2 full with sampled oracle rows; C5-shaped),
 and the ABI's error paths.
 """
+import zlib
+
 import numpy as np
 import pytest
 
@@ -493,7 +495,7 @@ def test_index_sort_digit_windows(eng, pattern, n, pay):
     be the encoded keys ascending with every payload carried by its own key
     (compared with numpy's sort of the same encoded keys)."""
     import torch
-    rng = np.random.default_rng(hash((pattern, n)) % (1 << 32))
+    rng = np.random.default_rng([zlib.crc32(pattern.encode()), n])   # deterministic (str hash is salted)
     k, kdt = _key_pattern(pattern, n, rng)
     k = np.asarray(k, dtype=np.int64)
     cols, dts = {"k": k}, {"k": kdt}
@@ -523,6 +525,14 @@ def test_index_sort_digit_windows(eng, pattern, n, pay):
             assert np.array_equal(keys, enc[row])                   # carried with its own key
     finally:
         eng.release(m)
+
+
+@pytest.mark.parametrize("pattern", ["bits1_to_27", "i64_low_word", "i32_negative_dups"])
+@pytest.mark.parametrize("pay", ["int32", "int64"])
+def test_index_sort_large(eng, pattern, pay):
+    """3M keys: ~500-1000 tiles in flight across the persistent grid (deep
+    look-back walks)."""
+    test_index_sort_digit_windows(eng, pattern, 3_000_017, pay)
 
 
 @pytest.mark.parametrize("pattern", ["mult32_lt2^26", "bits1_to_27", "i64_low_word", "i64_straddle"])
