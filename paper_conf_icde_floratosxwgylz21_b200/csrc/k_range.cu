@@ -34,7 +34,65 @@ struct LongItem {
     int r, lb, ub, pad;
 };
 
-size_t range_scratch_bytes(long long n_rp_max) { return 256 + (size_t)(n_rp_max > 0 ? n_rp_max : 1) * sizeof(LongItem); }
+// Search samples: every stride-th key of the index, staged in shared memory
+// by each CTA, narrow a binary search to one stride-wide window of the keys
+// before it touches global memory (the top ~12 levels of the search come from
+// shared memory instead of ~12 dependent L2 round trips).
+constexpr int SAMP_BYTES = 16384;
+
+size_t range_scratch_bytes(long long n_rp_max)
+{
+    return 256 + (size_t)(n_rp_max > 0 ? n_rp_max : 1) * sizeof(LongItem) + SAMP_BYTES;
+}
+
+template <typename K>
+__global__ void __launch_bounds__(256) sample_kernel(const K *__restrict__ a, int stride, int M, K *__restrict__ samp)
+{
+    const int j = blockIdx.x * 256 + threadIdx.x;
+    if (j < M) samp[j] = a[(long long)j * stride];
+}
+
+// first i in [0, N) with a[i] >= k (LOWER) or a[i] > k (!LOWER): samples
+// s[j] = a[j * stride], j < M, locate the window ((J-1)*stride, J*stride].
+template <bool LOWER, typename K>
+__device__ __forceinline__ int bound_sampled(const K *__restrict__ a, int N, const K *s_samp, int M, int stride, K k)
+{
+    int lo = 0, hi = M;
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (LOWER ? s_samp[mid] < k : s_samp[mid] <= k) lo = mid + 1;
+        else hi = mid;
+    }
+    if (lo == 0) return 0;
+    int glo = (lo - 1) * stride + 1;
+    int ghi = lo < M ? lo * stride : N;
+    while (glo < ghi) {
+        const int mid = (int)(((unsigned)glo + (unsigned)ghi) >> 1);
+        if (LOWER ? __ldg(a + mid) < k : __ldg(a + mid) <= k) glo = mid + 1;
+        else ghi = mid;
+    }
+    return glo;
+}
+
+// upper bound of k given lb = its lower bound: gallop from lb (qualifying
+// ranges of '=' are short), then binary search the last doubling step
+template <typename K>
+__device__ __forceinline__ int upper_from(const K *__restrict__ a, int N, int lb, K k)
+{
+    if (lb >= N || __ldg(a + lb) > k) return lb;
+    int lo = lb + 1, step = 1;   // invariant: a[lo - 1] <= k
+    while (lo + step - 1 < N && __ldg(a + lo + step - 1) <= k) {
+        lo += step;
+        step <<= 1;
+    }
+    int hi = lo + step - 1 < N ? lo + step - 1 : N;   // a[hi] > k or hi == N
+    while (lo < hi) {
+        const int mid = (int)(((unsigned)lo + (unsigned)hi) >> 1);
+        if (__ldg(a + mid) <= k) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
 
 template <typename K>
 __device__ __forceinline__ int lower_bound_g(const K *__restrict__ a, int lo, int hi, K k)
@@ -80,52 +138,57 @@ __device__ __forceinline__ void fold(long long &acc, V v)
 template <typename K, int VB, int OP, int AGG>
 __global__ void __launch_bounds__(R_THREADS)
 range_short_kernel(const long long *__restrict__ d_nrp, const K *__restrict__ rkeys, const K *__restrict__ skeys,
-                   const void *__restrict__ svals_, int N, const long long *__restrict__ pre,
-                   const long long *__restrict__ suf, long long *__restrict__ acc, long long *__restrict__ cnt,
-                   LongItem *__restrict__ list, unsigned *__restrict__ list_n)
+                   const void *__restrict__ svals_, int N, const K *__restrict__ samp, int M, int stride,
+                   const long long *__restrict__ pre, const long long *__restrict__ suf, long long *__restrict__ acc,
+                   long long *__restrict__ cnt, LongItem *__restrict__ list, unsigned *__restrict__ list_n)
 {
     using V = typename std::conditional<VB == 8, long long, int>::type;
     const V *svals = (const V *)svals_;
-    const long long i = blockIdx.x * (long long)R_THREADS + threadIdx.x;
-    if (i >= *d_nrp) return;
-    const K k = rkeys[i];
-    int lb = 0, ub = 0;
-    if constexpr (OP == EQ || OP == NE) {
-        lb = lower_bound_g(skeys, 0, N, k);
-        ub = upper_bound_g(skeys, lb, N, k);
-    } else if constexpr (OP == LE || OP == GT) {
-        lb = lower_bound_g(skeys, 0, N, k);
-    } else {
-        ub = upper_bound_g(skeys, 0, N, k);
-    }
-    int a0, b0, a1, b1;
-    pieces<OP>(lb, ub, N, a0, b0, a1, b1);
-    const long long L = (long long)(b0 - a0) + (b1 - a1);
-    if constexpr (AGG == COUNT || AGG == EXISTS || AGG == NOT_EXISTS) {
-        cnt[i] = L;
-    } else {
-        if (pre && (AGG == SUM || OP != EQ)) {   // O(1) from the prefix / suffix aggregates
-            long long a;
-            if constexpr (AGG == SUM) {
-                a = (pre[b0] - pre[a0]) + (pre[b1] - pre[a1]);
-            } else if constexpr (OP == NE) {
-                a = AGG == MIN ? min(pre[lb], suf[ub]) : max(pre[lb], suf[ub]);
-            } else if constexpr (OP == GT || OP == GE) {
-                a = pre[b0];                       // [0, b0)
-            } else {
-                a = suf[a0];                       // [a0, N)
-            }
-            acc[i] = a;
-            cnt[i] = L;
-        } else if (L <= R_SHORT) {
-            long long a = AGG == MIN ? LLONG_MAX : (AGG == MAX ? LLONG_MIN : 0);
-            for (int s = a0; s < b0; s++) fold<AGG>(a, svals[s]);
-            for (int s = a1; s < b1; s++) fold<AGG>(a, svals[s]);
-            acc[i] = a;
+    __shared__ K s_samp[SAMP_BYTES / sizeof(K)];
+    for (int j = threadIdx.x; j < M; j += R_THREADS) s_samp[j] = samp[j];
+    __syncthreads();
+    const long long nrp = *d_nrp;
+    for (long long i = blockIdx.x * (long long)R_THREADS + threadIdx.x; i < nrp;
+         i += (long long)gridDim.x * R_THREADS) {
+        const K k = rkeys[i];
+        int lb = 0, ub = 0;
+        if constexpr (OP == EQ || OP == NE) {
+            lb = bound_sampled<true>(skeys, N, s_samp, M, stride, k);
+            ub = upper_from(skeys, N, lb, k);
+        } else if constexpr (OP == LE || OP == GT) {
+            lb = bound_sampled<true>(skeys, N, s_samp, M, stride, k);
+        } else {
+            ub = bound_sampled<false>(skeys, N, s_samp, M, stride, k);
+        }
+        int a0, b0, a1, b1;
+        pieces<OP>(lb, ub, N, a0, b0, a1, b1);
+        const long long L = (long long)(b0 - a0) + (b1 - a1);
+        if constexpr (AGG == COUNT || AGG == EXISTS || AGG == NOT_EXISTS) {
             cnt[i] = L;
         } else {
-            unsigned slot = atomicAdd(list_n, 1u);
-            list[slot] = LongItem{(int)i, lb, ub, 0};
+            if (pre && (AGG == SUM || OP != EQ)) {   // O(1) from the prefix / suffix aggregates
+                long long a;
+                if constexpr (AGG == SUM) {
+                    a = (pre[b0] - pre[a0]) + (pre[b1] - pre[a1]);
+                } else if constexpr (OP == NE) {
+                    a = AGG == MIN ? min(pre[lb], suf[ub]) : max(pre[lb], suf[ub]);
+                } else if constexpr (OP == GT || OP == GE) {
+                    a = pre[b0];                       // [0, b0)
+                } else {
+                    a = suf[a0];                       // [a0, N)
+                }
+                acc[i] = a;
+                cnt[i] = L;
+            } else if (L <= R_SHORT) {
+                long long a = AGG == MIN ? LLONG_MAX : (AGG == MAX ? LLONG_MIN : 0);
+                for (int s = a0; s < b0; s++) fold<AGG>(a, svals[s]);
+                for (int s = a1; s < b1; s++) fold<AGG>(a, svals[s]);
+                acc[i] = a;
+                cnt[i] = L;
+            } else {
+                unsigned slot = atomicAdd(list_n, 1u);
+                list[slot] = LongItem{(int)i, lb, ub, 0};
+            }
         }
     }
 }
@@ -175,9 +238,26 @@ static void launch_range_t(long long n_rp_max, const long long *d_nrp, const voi
 {
     unsigned *list_n = (unsigned *)scratch;
     LongItem *list = (LongItem *)((char *)scratch + 256);
-    const unsigned blocks = (unsigned)((n_rp_max + R_THREADS - 1) / R_THREADS);
-    range_short_kernel<K, VB, OP, AGG><<<blocks, R_THREADS, 0, st>>>(d_nrp, (const K *)rkeys, (const K *)skeys,
-                                                                    svals, (int)ns, pre, suf, acc, cnt, list, list_n);
+    K *samp = (K *)((char *)scratch + 256 + (size_t)n_rp_max * sizeof(LongItem));
+    constexpr int SMAX = SAMP_BYTES / (int)sizeof(K);
+    const int N = (int)ns;
+    const int stride = N > SMAX ? (N + SMAX - 1) / SMAX : 1;
+    const int M = N > 0 ? (N + stride - 1) / stride : 0;
+    if (M > 0) {
+        sample_kernel<K><<<(M + 255) / 256, 256, 0, st>>>((const K *)skeys, stride, M, samp);
+        ++*launches;
+    }
+    static int max_blocks = 0;   // persistent-ish grid: the samples are staged once per CTA
+    if (!max_blocks) {
+        int dev = 0, sms = 148;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        max_blocks = sms * 8;
+    }
+    long long blocks = (n_rp_max + R_THREADS - 1) / R_THREADS;
+    if (blocks > max_blocks) blocks = max_blocks;
+    range_short_kernel<K, VB, OP, AGG><<<(unsigned)blocks, R_THREADS, 0, st>>>(
+        d_nrp, (const K *)rkeys, (const K *)skeys, svals, N, samp, M, stride, pre, suf, acc, cnt, list, list_n);
     ++*launches;
     if constexpr (AGG != COUNT && AGG != EXISTS && AGG != NOT_EXISTS) {
         range_long_kernel<VB, OP, AGG><<<148 * 8, R_THREADS, 0, st>>>(svals, (int)ns, list, list_n, acc, cnt);
