@@ -159,6 +159,11 @@ def time_oracle(tables, plans, budget_s, calib_rows=8):
         t = run(m)
     m = int(max(1, min(n_r, m * budget_s / max(t, 1e-6))))
     dt = run(m)
+    for _ in range(2):   # per-call overhead makes the cost sub-linear in m: rescale until ~budget
+        if dt >= budget_s / 2 or m >= n_r:
+            break
+        m = int(max(1, min(n_r, m * budget_s / max(dt, 1e-6))))
+        dt = run(m)
     return {"value": m * len(plans) / dt, "unit": "outer tuples/s", "cores": oracle.max_threads(),
             "kind": "oracle", "seconds": dt,
             "sample": "first %d R rows x all %d S rows for each of the %d plans (%d outer tuples)" % (
@@ -233,7 +238,7 @@ def run_reference(args, rank, world):
         return
     R, S, plans, desc, cfg = workload(args.workload, 0)
     tables = {"R": R, "S": S}
-    per_step = max(1.0, args.cpu_seconds / 3.0)
+    per_step = max(1.0, args.cpu_seconds / 2.0)
     for _ in range(args.warmup):
         time_oracle(tables, plans, per_step / 4)
     vals, secs = [], []
