@@ -460,15 +460,25 @@ class Engine:
                                                         ctypes.byref(out)))
         return out.value
 
-    def result_to_numpy(self, res, avg=None):
+    def result_to_numpy(self, res, avg=None, out=None):
+        """Copy a result to host arrays.  out: optional dict of preallocated
+        host arrays ("row", "value" int64; "valid", "passed" uint8; "sum",
+        "cnt" int64 for AVG) with room for the rows -- e.g. views of pinned
+        memory reused across calls, so the copy runs at full PCIe speed;
+        the returned arrays are then views of them."""
         n = res.n_rows
-        out = {"row": np.empty(n, np.int64), "value": np.empty(n, np.int64),
-               "valid": np.empty(n, np.uint8), "passed": np.empty(n, np.uint8)}
-        s = c = None
-        if res.d_avg_sum:
-            out["sum"] = np.empty(n, np.int64)
-            out["cnt"] = np.empty(n, np.int64)
-            s, c = out["sum"], out["cnt"]
+        if out is None:
+            out = {"row": np.empty(n, np.int64), "value": np.empty(n, np.int64),
+                   "valid": np.empty(n, np.uint8), "passed": np.empty(n, np.uint8)}
+            if res.d_avg_sum:
+                out["sum"] = np.empty(n, np.int64)
+                out["cnt"] = np.empty(n, np.int64)
+        else:
+            keys = ("row", "value", "valid", "passed") + (("sum", "cnt") if res.d_avg_sum else ())
+            if min(len(out[k]) for k in keys) < n:
+                raise ValueError("result_to_numpy: %d rows do not fit the given buffers" % n)
+            out = {k: out[k][:n] for k in keys}
+        s, c = (out["sum"], out["cnt"]) if res.d_avg_sum else (None, None)
         self._check(self.lib.nestgpu_result_to_host(self.ctx, ctypes.byref(res), _np_ptr(out["row"]),
                                                     _np_ptr(out["value"]), _np_ptr(out["valid"]),
                                                     _np_ptr(out["passed"]), _np_ptr(s), _np_ptr(c), n))

@@ -3,8 +3,9 @@ record schema): C1 (both plans), C2 (the 12-plan sweep), C3a SF1 Q2, C3b SF1
 Q17, C4a SF10 Q4, C4b SF10 Q20, C5 16M '>' MIN.
 
 Latency = build_index (inner filter + sort; '=' plans) + exec_correlated +
-result_to_host, wall clock from a synchronised start until the survivors are
-in host memory, columns resident (the paper includes index build, and
+result_to_host (into pinned host buffers allocated once and reused), wall
+clock from a synchronised start until the survivors are in host memory,
+columns resident (the paper includes index build, and
 excludes disk I/O).  The strategy is the paper's: the index for '='
 correlations, the nested loop otherwise.  Per-stage device
 times come from one extra profiled run (nestgpu_last_profile).
@@ -62,9 +63,22 @@ def main():
     sm_mhz = float(peaks.get("sm_max_mhz", 1965))
     from paper_conf_icde_floratosxwgylz21_b200 import nested
     params = eng.cost_calibrate()
+    pinned = {}
+
+    def res_buffers(n):
+        # pinned host result buffers, allocated once (outside the timed region)
+        # and reused -- the copy then runs at PCIe speed (binding result_to_numpy(out=))
+        if not pinned or len(pinned["row"]) < n:
+            pinned.clear()
+            pinned.update({k: torch.empty(n, dtype=dt, pin_memory=True).numpy()
+                           for k, dt in (("row", torch.int64), ("value", torch.int64), ("valid", torch.uint8),
+                                         ("passed", torch.uint8), ("sum", torch.int64), ("cnt", torch.int64))})
+        return pinned
+
     for name, tabs, plan, seed in cases(args.skip_c5):
         m = eng.mark()
         R, S = load(eng, tabs)
+        out = res_buffers(len(next(iter(tabs["R"].values()))))
         use_index = plan["corr_op"] == "="
         reps = args.reps if name != "C5" else 2
         warm = 3 if name != "C5" else 1
@@ -76,7 +90,7 @@ def main():
             t0 = time.perf_counter()
             idx = eng.index_for_plan(plan, S) if use_index else -1
             res = eng.exec(plan, R, S, index=idx)
-            host = eng.result_to_numpy(res)
+            host = eng.result_to_numpy(res, out=out)
             t1 = time.perf_counter()
             if r >= warm:
                 lat.append(1e3 * (t1 - t0))
@@ -105,7 +119,7 @@ def main():
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             res, strategy, _ = nested.exec_auto(eng, plan, R, S, params, cin)
-            host = eng.result_to_numpy(res)
+            host = eng.result_to_numpy(res, out=out)
             t1 = time.perf_counter()
             if r >= warm:
                 alat.append(1e3 * (t1 - t0))
