@@ -555,3 +555,28 @@ def test_dedup_sort_digit_windows(eng, pattern):
         for dedup in (False, True):
             g = run(eng, t, plan, mode, emit_all=True, dtypes=dt, dedup=dedup)
             assert_parity(g, ref, plan, True, ctx=(pattern, corr_op, agg, dedup))
+
+
+def test_result_to_numpy_into_buffers(eng):
+    """result_to_numpy(out=): the copy into caller buffers (pinned in the
+    bench) equals the allocating copy; a buffer that is too small is refused."""
+    import torch
+    t = query1.config("C1")
+    m = eng.mark()
+    try:
+        R, S = eng.load_table(t["R"]), eng.load_table(t["S"])
+        plan = make_plan("=", "avg", "<=")
+        res = eng.exec(plan, R, S, index=eng.index_for_plan(plan, S), emit_all=True)
+        ref = eng.result_to_numpy(res)
+        bufs = {k: torch.empty(2000, dtype=dt, pin_memory=True).numpy()
+                for k, dt in (("row", torch.int64), ("value", torch.int64), ("valid", torch.uint8),
+                              ("passed", torch.uint8), ("sum", torch.int64), ("cnt", torch.int64))}
+        got = eng.result_to_numpy(res, out=bufs)
+        assert set(got) == set(ref)
+        for k in ref:
+            assert np.array_equal(got[k], ref[k]), k
+        small = {k: v[:10] for k, v in bufs.items()}
+        with pytest.raises(ValueError):
+            eng.result_to_numpy(res, out=small)
+    finally:
+        eng.release(m)
