@@ -871,7 +871,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         CUDA_TRY(c, ng::launch_filter(nS, ips, sks, kb, vs, vb, 1, value_agg ? 1 : 0, nullptr, skeys, nullptr, svals,
                                       nullptr, value_agg ? extreme : nullptr, fscr, d_nsp, c->stream,
                                       &c->launches));
-        CUDA_TRY(c, ng::launch_init_partials(n_eval, P->agg, acc, cnt, c->stream, &c->launches));
+        CUDA_TRY(c, ng::launch_init_partials(n_eval, d_neval, P->agg, acc, cnt, c->stream, &c->launches));
         prof_end(c, 1);
         prof_begin(c, 3);
         CUDA_TRY(c, ng::launch_bnl(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, nS, d_nsp, skeys, svals,

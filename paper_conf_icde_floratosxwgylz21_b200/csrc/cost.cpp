@@ -110,8 +110,8 @@ nestgpu_status nestgpu_cost_calibrate(nestgpu_ctx *c, int64_t n_rows, nestgpu_co
     // C: a kernel with a tiny input (20 back-to-back launches)
     CC(T.ms([&] {
         cudaError_t e = cudaSuccess;
-        for (int i = 0; i < 20 && e == cudaSuccess; i++) e = ng::launch_init_partials(1, ng::MIN, (long long *)acc,
-                                                                                     (long long *)cnt, st, L);
+        for (int i = 0; i < 20 && e == cudaSuccess; i++) e = ng::launch_init_partials(1, d_small, ng::MIN,
+                                                                                     (long long *)acc, (long long *)cnt, st, L);
         return e;
     }, &t));
     const double C = t / 20;
@@ -202,7 +202,8 @@ nestgpu_status nestgpu_cost_calibrate(nestgpu_ctx *c, int64_t n_rows, nestgpu_co
         for (int k = 0; k < 4; k++) {
             if (cls_agg[k] == ng::EXISTS) CC(cudaMemsetAsync(k1, 0, nbr * kbw, st));   // r.key = 0: no s < r
             CC(T.ms([&] {
-                cudaError_t e = ng::launch_init_partials(nbr, cls_agg[k], (long long *)acc, (long long *)cnt, st, L);
+                cudaError_t e = ng::launch_init_partials(nbr, d_small + 1, cls_agg[k], (long long *)acc, (long long *)cnt,
+                                                         st, L);
                 if (e != cudaSuccess) return e;
                 return ng::launch_bnl(kbw, cls_agg[k] == ng::COUNT || cls_agg[k] == ng::EXISTS ? 0 : 4, ng::GT,
                                       cls_agg[k], nbr, d_small + 1, k1, nbs, d_small + 2, k2, v1, extreme,
@@ -213,7 +214,6 @@ nestgpu_status nestgpu_cost_calibrate(nestgpu_ctx *c, int64_t n_rows, nestgpu_co
     }
 
     // finalize (+ compaction): nothing passes vs everything emitted
-    CC(ng::launch_init_partials(n, ng::MIN, (long long *)acc, (long long *)cnt, st, L));
     ng::FinalizeArgs fa{};
     fa.n_rp_max = n;
     fa.d_nrp = d_small;
@@ -233,6 +233,7 @@ nestgpu_status nestgpu_cost_calibrate(nestgpu_ctx *c, int64_t n_rows, nestgpu_co
     fa.scratch = fscr;
     memcpy(ng::ctx_pinned(c), &n, 8);
     CC(cudaMemcpyAsync(d_small, ng::ctx_pinned(c), 8, cudaMemcpyHostToDevice, st));
+    CC(ng::launch_init_partials(n, d_small, ng::MIN, (long long *)acc, (long long *)cnt, st, L));
     CC(ng::launch_fill_runs(ids, 4, n, 1, 0, st, L));
     double t_none, t_all;
     fa.emit_all = 0;

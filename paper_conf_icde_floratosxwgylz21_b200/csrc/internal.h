@@ -68,8 +68,9 @@ cudaError_t launch_radix_pass_x(int kb_in, int kb_out, int vb, const void *kin, 
                                 unsigned hi, cudaStream_t st, long long *launches);
 
 // Partial aggregates per R' tuple: acc (int64) + cnt (int64); identity init.
-cudaError_t launch_init_partials(long long n, int agg, long long *acc, long long *cnt, cudaStream_t st,
-                                 long long *launches);
+// n: host upper bound (grid size); d_n: the actual count (device)
+cudaError_t launch_init_partials(long long n, const long long *d_n, int agg, long long *acc, long long *cnt,
+                                 cudaStream_t st, long long *launches);
 
 // a5 + a6: per R' tuple binary search of the sorted index and fold of the
 // qualifying range(s).  d_nrp: device count of R'.  Long ranges go to a

@@ -17,7 +17,10 @@ namespace ng {
 
 constexpr int F_THREADS = 256;
 constexpr int F_WARPS = F_THREADS / 32;
-constexpr int F_ITEMS = 16;
+#ifndef NG_F_ITEMS
+#define NG_F_ITEMS 4   // rows per thread per tile (rolled loop: also the serial memory-latency chain)
+#endif
+constexpr int F_ITEMS = NG_F_ITEMS;
 constexpr int F_TILE = F_THREADS * F_ITEMS;
 
 size_t finalize_scratch_bytes(long long n)
@@ -35,86 +38,118 @@ __device__ __forceinline__ long long div_round_half_away(__int128 num, long long
     return (long long)(num < 0 ? -q : q);
 }
 
+// AVG as a scaled integer: round_half_away(acc * 10^6 / c), c > 0.  The
+// int128 quotient is a slow software routine (~67 us for SF1 Q17's 6.3k R'
+// rows at 16 rows per thread); split it instead: |acc| = q0 c + r0, so
+// |acc| 10^6 / c = q0 10^6 + r0 10^6 / c with r0 10^6 < c 10^6 < 2^53 --
+// identical result in 64-bit arithmetic whenever q0 10^6 fits.
+__device__ __forceinline__ long long avg_scaled(long long acc, long long c)
+{
+    const unsigned long long mag = acc < 0 ? 0ull - (unsigned long long)acc : (unsigned long long)acc;
+    const unsigned long long uc = (unsigned long long)c;
+    const unsigned long long q0 = mag / uc, r0 = mag - q0 * uc;
+    if (uc < (1ull << 32) && q0 < 9223372036854ull) {   // q0 10^6 + 10^6 <= INT64_MAX
+        const unsigned long long t = r0 * 1000000ull;
+        const unsigned long long q = q0 * 1000000ull + (2 * t + uc) / (2 * uc);
+        return acc < 0 ? -(long long)q : (long long)q;
+    }
+    return div_round_half_away((__int128)acc * 1000000, c);
+}
+
+// The per-row evaluation (int128 compares, the rare int128 division) is
+// large; unrolled over the tile's 16 rows per thread it made a ~175 KB kernel
+// whose instruction-cache misses dominated small R' (SF1 Q17: 69 us for 6.3k
+// rows).  Rows are therefore evaluated in a rolled loop and staged in shared
+// memory (value, valid|passed bits, one ballot per (row group, warp)).
 __global__ void __launch_bounds__(F_THREADS) finalize_kernel(FinalizeArgs A, unsigned long long *__restrict__ status,
                                                              unsigned *__restrict__ counter)
 {
     __shared__ unsigned s_tile;
     __shared__ unsigned s_cnt[F_ITEMS][F_WARPS];
+    __shared__ unsigned s_bal[F_ITEMS][F_WARPS];
+    __shared__ long long s_val[F_ITEMS][F_THREADS];
+    __shared__ uint8_t s_vp[F_ITEMS][F_THREADS];   // bit 0 valid, bit 1 passed
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const unsigned lt = lanemask_lt();
     const long long n = *A.d_nrp;
     const long long num_tiles = (n + F_TILE - 1) / F_TILE;
-    if (tid == 0) s_tile = atomicAdd(counter, 1u);
-    __syncthreads();
-    const long long tile = s_tile;
-    if (tile >= num_tiles) return;  // grid sized for the R' upper bound
-    const long long base = tile * F_TILE;
+    // persistent: the grid is sized for the host's upper bound of |R'| but
+    // capped; CTAs take tiles of the ACTUAL |R'| until none are left
+    for (;;) {
+        if (tid == 0) s_tile = atomicAdd(counter, 1u);
+        __syncthreads();
+        const long long tile = s_tile;
+        __syncthreads();
+        if (tile >= num_tiles) return;
+        const long long base = tile * F_TILE;
 
-    bool flag[F_ITEMS];
-    unsigned rank[F_ITEMS];
-    long long value[F_ITEMS];
-    uint8_t valid[F_ITEMS], pass[F_ITEMS];
-#pragma unroll
-    for (int j = 0; j < F_ITEMS; j++) {
-        const long long i = base + (long long)j * F_THREADS + tid;
-        bool in = i < n;
-        value[j] = 0;
-        valid[j] = 0;
-        pass[j] = 0;
-        if (in) {
-            const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
-            const long long g = A.map ? (long long)A.map[i] : i;  // cached result slot
-            const long long c = kval ? A.cnt[g] : 0;     // NULL key: empty subquery (R2)
-            const long long acc = A.acc[g];
-            bool vv = true;
-            long long v = 0;
-            switch (A.agg) {
-            case MIN: case MAX: case SUM: vv = c > 0; v = acc; break;
-            case COUNT: v = c; break;
-            case AVG: vv = c > 0; if (vv) v = div_round_half_away((__int128)acc * 1000000, c); break;
-            case EXISTS: v = c > 0; break;
-            default: v = c == 0; break;
-            }
-            bool p;
-            if (A.agg == EXISTS || A.agg == NOT_EXISTS) {
-                p = v != 0;
-            } else {
-                const int row = A.ids[i];
-                const bool xv = !(A.x_valid && !A.x_valid[row]);
-                p = false;
-                if (vv && xv) {
-                    const __int128 x = load_w(A.x_col, A.x_w, row);
-                    if (A.agg == AVG)
-                        p = cmp_rt<__int128>((__int128)A.a * x * c, A.outer_op, (__int128)A.b * acc);
-                    else
-                        p = cmp_rt<__int128>((__int128)A.a * x, A.outer_op, (__int128)A.b * v);
+#pragma unroll 1
+        for (int j = 0; j < F_ITEMS; j++) {
+            const long long i = base + (long long)j * F_THREADS + tid;
+            bool in = i < n;
+            long long value = 0;
+            uint8_t vp = 0;
+            if (in) {
+                const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
+                const long long g = A.map ? (long long)A.map[i] : i;  // cached result slot
+                const long long c = kval ? A.cnt[g] : 0;     // NULL key: empty subquery (R2)
+                const long long acc = A.acc[g];
+                bool vv = true;
+                long long v = 0;
+                switch (A.agg) {
+                case MIN: case MAX: case SUM: vv = c > 0; v = acc; break;
+                case COUNT: v = c; break;
+                case AVG: vv = c > 0; if (vv) v = avg_scaled(acc, c); break;
+                case EXISTS: v = c > 0; break;
+                default: v = c == 0; break;
                 }
+                bool p;
+                if (A.agg == EXISTS || A.agg == NOT_EXISTS) {
+                    p = v != 0;
+                } else {
+                    const int row = A.ids[i];
+                    const bool xv = !(A.x_valid && !A.x_valid[row]);
+                    p = false;
+                    if (vv && xv) {
+                        const __int128 x = load_w(A.x_col, A.x_w, row);
+                        if (A.agg == AVG)
+                            p = cmp_rt<__int128>((__int128)A.a * x * c, A.outer_op, (__int128)A.b * acc);
+                        else
+                            p = cmp_rt<__int128>((__int128)A.a * x, A.outer_op, (__int128)A.b * v);
+                    }
+                }
+                value = vv ? v : 0;
+                vp = (uint8_t)((vv ? 1 : 0) | (p ? 2 : 0));
+                in = A.emit_all ? true : p;
             }
-            value[j] = vv ? v : 0;
-            valid[j] = vv;
-            pass[j] = p;
-            in = A.emit_all ? true : p;
+            s_val[j][tid] = value;
+            s_vp[j][tid] = vp;
+            const unsigned m = __ballot_sync(FULL, in);
+            if (lane == 0) {
+                s_cnt[j][warp] = __popc(m);
+                s_bal[j][warp] = m;
+            }
         }
-        flag[j] = in;
-        const unsigned m = __ballot_sync(FULL, in);
-        if (lane == 0) s_cnt[j][warp] = __popc(m);
-        rank[j] = __popc(m & lanemask_lt());
-    }
-    const unsigned long long tb = tile_offsets<F_ITEMS, F_THREADS>(s_cnt, status, tile, num_tiles, A.out_count);
-#pragma unroll
-    for (int j = 0; j < F_ITEMS; j++) {
-        if (!flag[j]) continue;
-        const long long i = base + (long long)j * F_THREADS + tid;
-        const long long pos = (long long)tb + s_cnt[j][warp] + rank[j];
-        A.out_ids[pos] = A.row_id_base + A.ids[i];
-        A.out_vals[pos] = value[j];
-        A.out_valid[pos] = valid[j];
-        A.out_passed[pos] = pass[j];
-        if (A.out_sum) {
-            const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
-            const long long g = A.map ? (long long)A.map[i] : i;
-            A.out_sum[pos] = kval ? A.acc[g] : 0;
-            A.out_cnt[pos] = kval ? A.cnt[g] : 0;
+        const unsigned long long tb = tile_offsets<F_ITEMS, F_THREADS>(s_cnt, status, tile, num_tiles, A.out_count);
+#pragma unroll 1
+        for (int j = 0; j < F_ITEMS; j++) {
+            const unsigned m = s_bal[j][warp];
+            if (!((m >> lane) & 1u)) continue;
+            const long long i = base + (long long)j * F_THREADS + tid;
+            const long long pos = (long long)tb + s_cnt[j][warp] + __popc(m & lt);
+            const uint8_t vp = s_vp[j][tid];
+            A.out_ids[pos] = A.row_id_base + A.ids[i];
+            A.out_vals[pos] = s_val[j][tid];
+            A.out_valid[pos] = vp & 1;
+            A.out_passed[pos] = (vp >> 1) & 1;
+            if (A.out_sum) {
+                const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
+                const long long g = A.map ? (long long)A.map[i] : i;
+                A.out_sum[pos] = kval ? A.acc[g] : 0;
+                A.out_cnt[pos] = kval ? A.cnt[g] : 0;
+            }
         }
+        __syncthreads();   // shared staging is rewritten by the next tile
     }
 }
 
@@ -124,7 +159,15 @@ cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *l
     if (e != cudaSuccess || a.n_rp_max <= 0) return e;
     e = cudaMemsetAsync(a.scratch, 0, finalize_scratch_bytes(a.n_rp_max), st);
     if (e != cudaSuccess) return e;
-    const long long tiles = (a.n_rp_max + F_TILE - 1) / F_TILE;
+    long long tiles = (a.n_rp_max + F_TILE - 1) / F_TILE;
+    static int cap = 0;
+    if (!cap) {
+        int dev = 0, sms = 148;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cap = sms * 4;
+    }
+    if (tiles > cap) tiles = cap;
     finalize_kernel<<<(unsigned)tiles, F_THREADS, 0, st>>>(a, (unsigned long long *)((char *)a.scratch + 256),
                                                          (unsigned *)a.scratch);
     ++*launches;
@@ -132,23 +175,24 @@ cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *l
 }
 
 // ------------------------------------------------------------------ partials
-__global__ void init_partials_kernel(long long n, long long acc0, long long *__restrict__ acc,
+__global__ void init_partials_kernel(const long long *__restrict__ d_n, long long acc0, long long *__restrict__ acc,
                                      long long *__restrict__ cnt)
 {
+    const long long n = *d_n;   // the actual |R'| (the grid covers the host's upper bound)
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
         acc[i] = acc0;
         cnt[i] = 0;
     }
 }
 
-cudaError_t launch_init_partials(long long n, int agg, long long *acc, long long *cnt, cudaStream_t st,
-                                 long long *launches)
+cudaError_t launch_init_partials(long long n, const long long *d_n, int agg, long long *acc, long long *cnt,
+                                 cudaStream_t st, long long *launches)
 {
     if (n <= 0) return cudaSuccess;
     long long acc0 = agg == MIN ? LLONG_MAX : (agg == MAX ? LLONG_MIN : 0);
     long long blocks = (n + 255) / 256;
     if (blocks > 148 * 16) blocks = 148 * 16;
-    init_partials_kernel<<<(unsigned)blocks, 256, 0, st>>>(n, acc0, acc, cnt);
+    init_partials_kernel<<<(unsigned)blocks, 256, 0, st>>>(d_n, acc0, acc, cnt);
     ++*launches;
     return cudaGetLastError();
 }

@@ -580,3 +580,23 @@ def test_result_to_numpy_into_buffers(eng):
             eng.result_to_numpy(res, out=small)
     finally:
         eng.release(m)
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_avg_large_int64_payloads(eng, mode):
+    """AVG's scaled-integer division (round_half_away(sum * 10^6 / count),
+    reading R6) on int64 payloads up to ~9.2e12 in magnitude -- quotients
+    near the 64-bit limit and negative sums -- both kernels, vs the oracle."""
+    rng = np.random.default_rng(21)
+    lim = 9_000_000_000_000
+    t = {"R": {"col1": rng.integers(0, 40, 4000), "col2": rng.integers(-lim, lim, 4000)},
+         "S": {"col1": rng.integers(0, 40, 6001), "col2": rng.integers(-lim, lim, 6001)}}
+    t["S"]["col2"][::7] = lim                      # skewed groups: large positive / negative means
+    t["S"]["col2"][1::11] = -lim
+    dt = {"R": {"col1": "int32", "col2": "int64"}, "S": {"col1": "int32", "col2": "int64"}}
+    for corr_op in ("=", "<", "!="):
+        for outer in ("<", ">="):
+            plan = make_plan(corr_op, "avg", outer)
+            ref = oracle.evaluate(t, plan)
+            g = run(eng, t, plan, mode, emit_all=True, dtypes=dt)
+            assert_parity(g, ref, plan, True, ctx=(mode, corr_op, outer))
