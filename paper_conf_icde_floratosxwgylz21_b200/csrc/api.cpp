@@ -110,17 +110,17 @@ nestgpu_status fail(nestgpu_ctx *c, nestgpu_status code, const char *fmt, ...)
     } while (0)
 
 // Radix-pass plan for n encoded keys of kb bytes whose AND / OR over all keys
-// are kand / kor: only bits that vary need sorting, so 8-bit digit windows
+// are kand / kor: only bits that vary need sorting, so w-bit digit windows
 // are placed greedily from the lowest varying bit (the fewest windows that
 // cover every varying bit), e.g. keys that are multiples of 32 below 2^26
-// take 3 passes instead of 4.  When every varying bit lies in the low word
-// of a 64-bit key the windows stay inside bits 0-31 (start <= 24; overlapping
-// a lower window is harmless for a stable LSD sort), so the passes can run
-// on 32-bit keys.  Returns the number of passes, shifts[] their bit offsets.
-static int plan_sort_passes(int kb, unsigned long long kand, unsigned long long kor, long long n, int *shifts)
+// take 3 passes of 8 bits instead of 4.  9-bit windows (512 bins) are used
+// when they need at most 2/3 of the 8-bit passes (an 18-bit key: 2 instead
+// of 3; a 9-bit pass measured 1.3-1.4x an 8-bit one, so 4 -> 3 does not pay).  When every varying bit lies in the low word of a 64-bit key the
+// windows stay inside bits 0-31 (start <= 32 - w; overlapping a lower window
+// is harmless for a stable LSD sort), so the passes can run on 32-bit keys.
+// Returns the number of passes; shifts[] their bit offsets, *rb the width.
+static int plan_windows(int kb, unsigned long long var, int w, int *shifts)
 {
-    if (n < 2) return 0;
-    const unsigned long long var = kand ^ kor;
     const bool low = (var >> 32) == 0;
     int np = 0;
     for (int b = 0; b < kb * 8 && np < 8;) {
@@ -128,11 +128,28 @@ static int plan_sort_passes(int kb, unsigned long long kand, unsigned long long 
             b++;
             continue;
         }
-        const int s = low && b > 24 ? 24 : b;
+        const int s = low && b > 32 - w ? 32 - w : b;
         shifts[np++] = s;
-        b = s + 8;
+        b = s + w;
     }
     return np;
+}
+
+static int plan_sort_passes(int kb, unsigned long long kand, unsigned long long kor, long long n, int *shifts,
+                            int *rb)
+{
+    *rb = 8;
+    if (n < 2) return 0;
+    const unsigned long long var = kand ^ kor;
+    int s9[8];
+    const int np8 = plan_windows(kb, var, 8, shifts);
+    const int np9 = plan_windows(kb, var, 9, s9);
+    if (3 * np9 <= 2 * np8) {   // a 9-bit pass costs ~1.3-1.4x an 8-bit one (measured): 3 -> 2 pays, 4 -> 3 not
+        for (int p = 0; p < np9; p++) shifts[p] = s9[p];
+        *rb = 9;
+        return np9;
+    }
+    return np8;
 }
 
 size_t align_up(size_t x) { return (x + ALIGN - 1) / ALIGN * ALIGN; }
@@ -520,8 +537,8 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     void *uk = salloc(c, (size_t)n * kb), *uv = vb ? salloc(c, (size_t)n * vb) : nullptr;
     void *fscr = salloc(c, ng::filter_scratch_bytes(n));
     void *sscr = salloc(c, ng::sort_scratch_bytes(n));
-    unsigned *hist = (unsigned *)salloc(c, 8 * 256 * 4);
-    unsigned *dbase = (unsigned *)salloc(c, 8 * 256 * 4);
+    unsigned *hist = (unsigned *)salloc(c, 8 * 512 * 4);
+    unsigned *dbase = (unsigned *)salloc(c, 8 * 512 * 4);
     long long *dsmall = (long long *)salloc(c, 64);   // [0] |S'|, [2] key AND, [3] key OR
     if (!tk || !uk || !fscr || !sscr || !hist || !dbase || !dsmall || (vb && (!tv || !uv)))
         return fail(c, NESTGPU_ERR_OOM, "arena exhausted building an index over %lld rows", (long long)n);
@@ -540,10 +557,11 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     memcpy(&nsp, c->pinned, 8);
     memcpy(&kand, c->pinned + 4, 8);
     memcpy(&kor, c->pinned + 6, 8);
-    int shifts[8];
-    const int np = plan_sort_passes(kb, kand, kor, nsp, shifts);
+    int shifts[8], rb = 8;
+    const int np = plan_sort_passes(kb, kand, kor, nsp, shifts, &rb);
     prof_begin(c, 2);
-    CUDA_TRY(c, ng::launch_digit_hist(kb, tk, nsp, shifts, np, hist, dbase, c->num_sms, c->stream, &c->launches));
+    CUDA_TRY(c, ng::launch_digit_hist(kb, tk, nsp, shifts, np, hist, dbase, c->num_sms, c->stream, &c->launches,
+                                      rb));
 
     IndexRec ix{};
     ix.off = c->lo;
@@ -579,8 +597,8 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
             void *ov = to_final ? ix.payload : uv;
             if (ok == ik) { ok = tk; ov = tv; }
             const int kin = narrow && p > 0 ? 4 : kb, kout = narrow && p < np - 1 ? 4 : kb;
-            CUDA_TRY(c, ng::launch_radix_pass_x(kin, kout, vb, ik, ok, iv, ov, nsp, shifts[p], dbase + p * 256, sscr,
-                                                hi, c->stream, &c->launches));
+            CUDA_TRY(c, ng::launch_radix_pass_x(kin, kout, vb, ik, ok, iv, ov, nsp, shifts[p], dbase + p * (1 << rb),
+                                                sscr, hi, c->stream, &c->launches, rb));
             ik = ok;
             iv = ov;
         }
@@ -777,8 +795,8 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         ukeys = salloc(c, (size_t)nR * kb);
         sscr = salloc(c, ng::sort_scratch_bytes(nR));
         gscr = salloc(c, ng::group_scratch_bytes(nR));
-        hist = (unsigned *)salloc(c, 8 * 256 * 4);
-        dbase = (unsigned *)salloc(c, 8 * 256 * 4);
+        hist = (unsigned *)salloc(c, 8 * 512 * 4);
+        dbase = (unsigned *)salloc(c, 8 * 512 * 4);
         if (!pos || !tpos || !map || !tkeys || !ukeys || !sscr || !gscr || !hist || !dbase)
             return fail(c, NESTGPU_ERR_OOM, "arena exhausted (dedup buffers for |R|=%lld)", (long long)nR);
     }
@@ -808,18 +826,18 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         memcpy(&nrp, c->pinned, 8);
         memcpy(&kand, c->pinned + 12, 8);
         memcpy(&kor, c->pinned + 14, 8);
-        int shifts[8];
-        const int np = plan_sort_passes(kb, kand, kor, nrp, shifts);
+        int shifts[8], rb = 8;
+        const int np = plan_sort_passes(kb, kand, kor, nrp, shifts, &rb);
         CUDA_TRY(c, ng::launch_iota(pos, nrp, c->stream, &c->launches));
         CUDA_TRY(c, ng::launch_digit_hist(kb, rkeys, nrp, shifts, np, hist, dbase, c->num_sms, c->stream,
-                                          &c->launches));
+                                          &c->launches, rb));
         void *ck = rkeys, *ok = tkeys;
         int *cv = pos, *ov = tpos;
         const bool narrow = kb == 8 && np >= 2 && ((kand ^ kor) >> 32) == 0;   // as in build_index
         for (int p = 0; p < np; p++) {
             const int kin = narrow && p > 0 ? 4 : kb, kout = narrow && p < np - 1 ? 4 : kb;
-            CUDA_TRY(c, ng::launch_radix_pass_x(kin, kout, 4, ck, ok, cv, ov, nrp, shifts[p], dbase + p * 256, sscr,
-                                                (unsigned)(kand >> 32), c->stream, &c->launches));
+            CUDA_TRY(c, ng::launch_radix_pass_x(kin, kout, 4, ck, ok, cv, ov, nrp, shifts[p], dbase + p * (1 << rb),
+                                                sscr, (unsigned)(kand >> 32), c->stream, &c->launches, rb));
             std::swap(ck, ok);
             std::swap(cv, ov);
         }

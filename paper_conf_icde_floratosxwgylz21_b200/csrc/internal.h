@@ -52,20 +52,22 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
 
 // a4: histograms of the digits at `shifts` (np of them) over n encoded keys,
 // and their exclusive scans into digit_base[np][256].
+//   rb: digit bits (8 or 9); hist / digit_base hold np * 2^rb words
 cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *shifts, int np, unsigned *hist,
-                              unsigned *digit_base, int num_sms, cudaStream_t st, long long *launches);
+                              unsigned *digit_base, int num_sms, cudaStream_t st, long long *launches, int rb = 8);
 
-// a4: one stable LSD radix pass on 8-bit digit `shift/8` of the encoded keys.
-//   digit_base: 256 uint32 global exclusive offsets of the digit (device)
+// a4: one stable LSD radix pass on the rb-bit digit (rb = 8 or 9) at bit
+// `shift` of the encoded keys.
+//   digit_base: 2^rb uint32 global exclusive offsets of the digit (device)
 size_t sort_scratch_bytes(long long n);
 cudaError_t launch_radix_pass(int kb, int vb, const void *kin, void *kout, const void *vin, void *vout,
                               long long n, int shift, const unsigned *digit_base, void *scratch,
-                              cudaStream_t st, long long *launches);
+                              cudaStream_t st, long long *launches, int rb = 8);
 // The same with different key widths in and out: 8 -> 4 drops the high word
 // (all keys must share it), 4 -> 8 re-attaches `hi` as the high word.
 cudaError_t launch_radix_pass_x(int kb_in, int kb_out, int vb, const void *kin, void *kout, const void *vin,
                                 void *vout, long long n, int shift, const unsigned *digit_base, void *scratch,
-                                unsigned hi, cudaStream_t st, long long *launches);
+                                unsigned hi, cudaStream_t st, long long *launches, int rb = 8);
 
 // Partial aggregates per R' tuple: acc (int64) + cnt (int64); identity init.
 // n: host upper bound (grid size); d_n: the actual count (device)
