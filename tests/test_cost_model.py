@@ -134,3 +134,29 @@ def test_exec_auto_matches_oracle_and_picks_index_for_large_equality():
                 assert strategy.startswith(want), strategy
     finally:
         eng.close()
+
+
+@pytest.mark.parametrize("bits,lo,kb,want", [
+    (18, 0, 4, 2),    # C2 keys U[0, 2^18): two 9-bit passes instead of three 8-bit ones
+    (21, 5, 4, 3),    # multiples of 32 below 2^26: windows at 5, 13, 21
+    (26, 0, 4, 4),    # 4 x 8 bits (3 x 9 would not pay)
+    (31, 0, 4, 4),
+    (8, 0, 4, 1),
+    (1, 7, 4, 1),
+    (0, 0, 4, 0),     # all keys equal: nothing to sort
+    (25, 20, 8, 4),   # 64-bit keys, bits 20..44 vary (windows cross bit 32)
+    (64, 0, 8, 8),
+])
+def test_sort_pass_plan_mirror(bits, lo, kb, want):
+    """tools/cost_model._passes mirrors the engine's radix-pass planner
+    (api.cpp plan_sort_passes): greedy windows over the varying key bits,
+    9-bit windows only when they need <= 2/3 of the 8-bit passes."""
+    import numpy as np
+    from tools.cost_model import _passes
+    dt = np.uint32 if kb == 4 else np.uint64
+    if bits == 0:
+        keys = np.array([5, 5, 5], dtype=dt)
+    else:
+        top = (1 << bits) - 1
+        keys = np.array([0, top << lo], dtype=np.uint64).astype(dt)
+    assert _passes(keys, kb) == want
