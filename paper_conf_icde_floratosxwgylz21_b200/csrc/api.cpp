@@ -36,6 +36,7 @@ struct Column {
     bool alive;
     bool stats;         // host-side min/max known
     long long mn, mx;
+    bool caller_filled; // nestgpu_alloc_column: contents may change behind our back (stats not cached)
 };
 
 struct IndexRec {
@@ -472,7 +473,9 @@ nestgpu_status nestgpu_alloc_column(nestgpu_ctx *c, nestgpu_dtype dtype, int32_t
                                     int32_t *out_col)
 {
     if (!c || !out_col) return fail(c, NESTGPU_ERR_INVALID, "alloc_column: null argument");
-    return new_column(c, dtype, scale, n, with_valid != 0, out_col);
+    nestgpu_status st = new_column(c, dtype, scale, n, with_valid != 0, out_col);
+    if (st == NESTGPU_OK) c->cols[*out_col].caller_filled = true;
+    return st;
 }
 
 nestgpu_status nestgpu_column_info(const nestgpu_ctx *c, int32_t id, nestgpu_column_desc *out)
@@ -531,6 +534,25 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     }
     const int kb = key_bytes(c, key_cols, n_key_cols);
     const int vb = pc ? vs.w : 0;
+    // 64-bit keys of one column whose encoded min and max share the high word
+    // (column statistics, computed once per column): every key does, so the
+    // S' filter already writes 32-bit keys and the whole sort runs on them;
+    // the last pass re-attaches the word (Q4's order keys: 152 MB less to
+    // write, histogram and read again)
+    bool pre_narrow = false;
+    unsigned pre_hi = 0;
+    if (kb == 8 && n_key_cols == 1) {
+        Column &kc = c->cols[key_cols[0]];
+        if (kc.caller_filled) kc.stats = false;   // recomputed: the caller may have rewritten it
+        if ((s = column_stats(c, kc))) return s;
+        const unsigned long long emn = (unsigned long long)kc.mn ^ 0x8000000000000000ull;
+        const unsigned long long emx = (unsigned long long)kc.mx ^ 0x8000000000000000ull;
+        if (kc.mn <= kc.mx && (emn >> 32) == (emx >> 32)) {
+            pre_narrow = true;
+            pre_hi = (unsigned)(emn >> 32);
+        }
+    }
+    const int fkb = pre_narrow ? 4 : kb;   // key width the S' filter writes
     scratch_reset(c);
     for (int st = 0; st < NESTGPU_N_STAGES; st++) c->ran[st] = false;
     void *tk = salloc(c, (size_t)n * kb), *tv = vb ? salloc(c, (size_t)n * vb) : nullptr;
@@ -547,7 +569,7 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     CUDA_TRY(c, cudaMemsetAsync(dsmall, 0, 64, c->stream));
     CUDA_TRY(c, cudaMemsetAsync(keymask, 0xff, 8, c->stream));   // AND identity
     prof_begin(c, 1);
-    CUDA_TRY(c, ng::launch_filter(n, ps, ks, kb, vs, vb, 1, pc ? 1 : 0, nullptr, tk, nullptr, tv, keymask, nullptr,
+    CUDA_TRY(c, ng::launch_filter(n, ps, ks, fkb, vs, vb, 1, pc ? 1 : 0, nullptr, tk, nullptr, tv, keymask, nullptr,
                                   fscr, d_count, c->stream, &c->launches));
     prof_end(c, 1);
     CUDA_TRY(c, cudaMemcpyAsync(c->pinned, dsmall, 32, cudaMemcpyDeviceToHost, c->stream));
@@ -558,9 +580,13 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     memcpy(&kand, c->pinned + 4, 8);
     memcpy(&kor, c->pinned + 6, 8);
     int shifts[8], rb = 8;
-    const int np = plan_sort_passes(kb, kand, kor, nsp, shifts, &rb);
+    int np = plan_sort_passes(fkb, kand, kor, nsp, shifts, &rb);
+    if (pre_narrow && np == 0 && nsp > 0) {   // equal keys: one pass still widens them to 64 bits
+        np = 1;
+        shifts[0] = 0;
+    }
     prof_begin(c, 2);
-    CUDA_TRY(c, ng::launch_digit_hist(kb, tk, nsp, shifts, np, hist, dbase, c->num_sms, c->stream, &c->launches,
+    CUDA_TRY(c, ng::launch_digit_hist(fkb, tk, nsp, shifts, np, hist, dbase, c->num_sms, c->stream, &c->launches,
                                       rb));
 
     IndexRec ix{};
@@ -588,15 +614,15 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
         // 64-bit keys whose high words all agree (AND == OR there, e.g. Q4's
         // order keys) travel as 32-bit keys between the first and the last
         // pass: the first pass drops the high word, the last re-attaches it.
-        const bool narrow = kb == 8 && np >= 2 && ((kand ^ kor) >> 32) == 0;
-        const unsigned hi = (unsigned)(kand >> 32);
+        const bool narrow = pre_narrow || (kb == 8 && np >= 2 && ((kand ^ kor) >> 32) == 0);
+        const unsigned hi = pre_narrow ? pre_hi : (unsigned)(kand >> 32);
         const void *ik = tk, *iv = tv;
         for (int p = 0; p < np; p++) {
             const bool to_final = ((np - 1 - p) % 2) == 0;
             void *ok = to_final ? ix.keys : uk;
             void *ov = to_final ? ix.payload : uv;
             if (ok == ik) { ok = tk; ov = tv; }
-            const int kin = narrow && p > 0 ? 4 : kb, kout = narrow && p < np - 1 ? 4 : kb;
+            const int kin = pre_narrow || (narrow && p > 0) ? 4 : kb, kout = narrow && p < np - 1 ? 4 : kb;
             CUDA_TRY(c, ng::launch_radix_pass_x(kin, kout, vb, ik, ok, iv, ov, nsp, shifts[p], dbase + p * (1 << rb),
                                                 sscr, hi, c->stream, &c->launches, rb));
             ik = ok;
@@ -745,6 +771,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     }
     const int vb = value_agg ? dtype_width(ac->dtype) : 0;
     if ((P->agg == NG_SUM || P->agg == NG_AVG) && vb == 8) {
+        if (ac->caller_filled) ac->stats = false;   // recomputed: the caller may have rewritten it
         if ((s = column_stats(c, *ac))) return s;
         __int128 m = ac->mx > -(ac->mn) ? (__int128)ac->mx : -(__int128)ac->mn;
         if ((__int128)nS * m >= ((__int128)1 << 63))

@@ -259,9 +259,9 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
                 if (tp.n_key == 2)
                     key = (K)(((uint64_t)enc32((int)ld_col(sb, tp.key0, li)) << 32) |
                               enc32((int)ld_col(sb, tp.key1, li)));
-                else if constexpr (KB == 4)
+                else if (KB == 4 && tp.key0.w == 4)
                     key = (K)enc32((int)ld_col(sb, tp.key0, li));
-                else
+                else   // (KB == 4 with an 8-byte column: the low word of the 64-bit code, its high word constant)
                     key = (K)enc64(ld_col(sb, tp.key0, li));
                 if (out_keys) ((K *)out_keys)[pos] = key;
                 if (out_kvalid) out_kvalid[pos] = (kvalid >> j) & 1u;

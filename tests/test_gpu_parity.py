@@ -477,6 +477,8 @@ def _key_pattern(name, n, rng):
         return -(1 << 50) + rng.integers(0, 1 << 25, n) * (1 << 20), "int64"
     if name == "i64_full":            # all 64 bits vary
         return rng.integers(-2 ** 63, 2 ** 63 - 1, n, dtype=np.int64), "int64"
+    if name == "i64_all_equal":       # 64-bit, one value: no bit varies (the narrowed filter output still widens)
+        return np.full(n, (7 << 40) + 3, dtype=np.int64), "int64"
     if name == "i32_negative_dups":   # signed, heavy duplicates
         k = rng.integers(-1000, 1000, n)
         k[::5] = -7
@@ -485,7 +487,7 @@ def _key_pattern(name, n, rng):
 
 
 @pytest.mark.parametrize("pattern", ["mult32_lt2^26", "bits1_to_27", "i64_low_word", "i64_straddle",
-                                     "i64_full", "i32_negative_dups"])
+                                     "i64_full", "i64_all_equal", "i32_negative_dups"])
 @pytest.mark.parametrize("n", [1, 2, 4095, 4097, 1_000_003])
 @pytest.mark.parametrize("pay", ["int32", "int64", None])
 def test_index_sort_digit_windows(eng, pattern, n, pay):

@@ -26,6 +26,43 @@ sys.path.insert(0, ROOT)
 ALU_PAIRS_PER_CLK = {"min": 32.0, "max": 32.0, "count": 64.0, "sum": 32.0, "avg": 32.0}
 
 
+def ideal_stages(tabs, plan, st, use_index, survivors, hbm_gbps, alu_ms):
+    """Ideal time (ms) of each stage from the ALGORITHMIC work (SURVEY.md
+    §8(d)): HBM stages move their bytes at the measured copy bandwidth, the
+    nested loop runs at its integer-pipe bound.  Bytes per stage:
+      S' filter  n_S x (inner predicate + key + payload column widths) read
+                 + |S'| x (key + payload) written
+      sort       one read + one write of |S'| x (key + payload) (lower bound)
+      R' filter  n_R x (outer predicate + key column widths) read
+                 + |R'| x (4-byte id + key) written
+      probe      |R'| x key read + sum_k x payload read + |R'| x 16 B partials
+      finalize   |R'| x (16 B partials + id + compared column) read
+                 + survivors x 18 B written"""
+    R, S = tabs["R"], tabs["S"]
+
+    def w(t, c):
+        return t[c].dtype.itemsize
+
+    kb = 4 if (len(plan["inner_key"]) == 1 and w(S, plan["inner_key"][0]) == 4) else 8
+    vb = w(S, plan["agg_col"]) if plan.get("agg_col") else 0
+    n_r, n_s = len(next(iter(R.values()))), len(next(iter(S.values())))
+    in_cols = {p["col"] for p in plan["inner_preds"]} | {p["rhs"] for p in plan["inner_preds"] if p.get("rhs")}
+    in_w = sum(w(S, c) for c in in_cols | set(plan["inner_key"]) | ({plan["agg_col"]} if vb else set()))
+    out_cols = {p["col"] for p in plan["outer_preds"]} | {p["rhs"] for p in plan["outer_preds"] if p.get("rhs")}
+    out_w = sum(w(R, c) for c in out_cols | set(plan["outer_key"]))
+    xw = w(R, plan["outer_cmp_col"]) if plan.get("outer_cmp_col") else 0
+    b = {"inner_filter": n_s * in_w + st["n_sp"] * (kb + vb),
+         "outer_filter": n_r * out_w + st["n_rp"] * (4 + kb),
+         "finalize": st["n_rp"] * (16 + 4 + xw) + survivors * 18}
+    if use_index:
+        b["sort"] = 2 * st["n_sp"] * (kb + vb)
+        b["probe"] = st["n_rp"] * (kb + 16) + st["sum_k"] * vb
+    out = {k: v / (hbm_gbps * 1e9) * 1e3 for k, v in b.items()}
+    if not use_index:
+        out["nested_loop"] = alu_ms
+    return out, b
+
+
 def cases(skip_c5):
     from datagen import make_plan, query1, tpch
     out = []
@@ -149,6 +186,18 @@ def main():
             rec["pairs"] = pairs
             rec["pairs_per_s"] = pairs / (stages["subquery"] / 1e3)
             rec["nested_loop_alu_frac"] = ideal / stages["subquery"]
+        hbm = float(peaks.get("hbm_gbs", 6454.6))   # measured copy bandwidth (MEASURED_PEAKS.json)
+        alu_ms = None
+        if not use_index and plan["agg"] in ALU_PAIRS_PER_CLK:
+            alu_ms = st["n_rp"] * st["n_sp"] / (props.multi_processor_count * ALU_PAIRS_PER_CLK[plan["agg"]]
+                                                * sm_mhz * 1e6) * 1e3
+        if use_index or alu_ms is not None:
+            ideal, nbytes = ideal_stages(tabs, plan, st, use_index, res_n, hbm, alu_ms)
+            ideal_total = sum(ideal.values())
+            dev = stages["total"] + (sum(ix_prof[k] for k in ("inner_filter", "sort")) if ix_prof else 0.0)
+            rec["roofline"] = {"ideal_ms": {k: round(v, 5) for k, v in ideal.items()},
+                               "algorithmic_bytes": nbytes, "hbm_gbps": hbm,
+                               "query_frac": ideal_total / p50, "device_frac": ideal_total / dev if dev > 0 else None}
         print(json.dumps(rec), flush=True)
         if args.out:
             with open(args.out, "a") as f:
