@@ -98,8 +98,35 @@ __device__ __forceinline__ unsigned nonnull(const unsigned char *sb, const Col c
     return out;
 }
 
-template <int ITEMS, int OP>
-__device__ __forceinline__ unsigned cmp_items(const long long (&x)[ITEMS], const long long (&y)[ITEMS])
+// Encoded keys of a tile's items (column widths dispatched once):
+// composite (two int32-storage columns, reading R9), one int32 column, or
+// one int64 column (with KB == 4: the low word of its code -- the caller
+// knows the high word is constant).
+template <int KB, int ITEMS>
+__device__ __forceinline__ void load_keys(const unsigned char *sb, const TPlan &tp, int tid,
+                                          typename std::conditional<KB == 8, uint64_t, uint32_t>::type (&k)[ITEMS])
+{
+    using K = typename std::conditional<KB == 8, uint64_t, uint32_t>::type;
+    if (tp.n_key == 2) {
+        const int *a = reinterpret_cast<const int *>(sb + tp.key0.off);
+        const int *b = reinterpret_cast<const int *>(sb + tp.key1.off);
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++)
+            k[j] = (K)(((uint64_t)enc32(a[j * T_THREADS + tid]) << 32) | enc32(b[j * T_THREADS + tid]));
+    } else if (tp.key0.w == 4) {
+        const int *a = reinterpret_cast<const int *>(sb + tp.key0.off);
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++)
+            k[j] = KB == 4 ? (K)enc32(a[j * T_THREADS + tid]) : (K)enc64((long long)a[j * T_THREADS + tid]);
+    } else {
+        const long long *a = reinterpret_cast<const long long *>(sb + tp.key0.off);
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) k[j] = (K)enc64(a[j * T_THREADS + tid]);
+    }
+}
+
+template <int ITEMS, int OP, typename T>
+__device__ __forceinline__ unsigned cmp_items(const T (&x)[ITEMS], const T (&y)[ITEMS])
 {
     unsigned m = 0;
 #pragma unroll
@@ -181,22 +208,42 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
             const TPred p = tp.p[k];
             live = nonnull<ITEMS>(sb, p.xv, live, tid);
             live = nonnull<ITEMS>(sb, p.yv, live, tid);
-            long long x[ITEMS], y[ITEMS];
-            load_items<ITEMS>(sb, p.x, tid, x);
-            if (p.y.off >= 0) {
-                load_items<ITEMS>(sb, p.y, tid, y);
-            } else {
+#define NG_CMP_ALL(X, Y)                                                                              \
+            switch (p.op) {                                                                           \
+            case EQ: live &= cmp_items<ITEMS, EQ>(X, Y); break;                                       \
+            case NE: live &= cmp_items<ITEMS, NE>(X, Y); break;                                       \
+            case LT: live &= cmp_items<ITEMS, LT>(X, Y); break;                                       \
+            case LE: live &= cmp_items<ITEMS, LE>(X, Y); break;                                       \
+            case GT: live &= cmp_items<ITEMS, GT>(X, Y); break;                                       \
+            default: live &= cmp_items<ITEMS, GE>(X, Y); break;                                       \
+            }
+            if (p.x.w == 4 && (p.y.off >= 0 ? p.y.w == 4 : p.lit == (long long)(int)p.lit)) {
+                // int32 operands (the common case): 32-bit compares
+                int x[ITEMS], y[ITEMS];
+                const int *xa = reinterpret_cast<const int *>(sb + p.x.off);
 #pragma unroll
-                for (int j = 0; j < ITEMS; j++) y[j] = p.lit;
+                for (int j = 0; j < ITEMS; j++) x[j] = xa[j * T_THREADS + tid];
+                if (p.y.off >= 0) {
+                    const int *ya = reinterpret_cast<const int *>(sb + p.y.off);
+#pragma unroll
+                    for (int j = 0; j < ITEMS; j++) y[j] = ya[j * T_THREADS + tid];
+                } else {
+#pragma unroll
+                    for (int j = 0; j < ITEMS; j++) y[j] = (int)p.lit;
+                }
+                NG_CMP_ALL(x, y)
+            } else {
+                long long x[ITEMS], y[ITEMS];
+                load_items<ITEMS>(sb, p.x, tid, x);
+                if (p.y.off >= 0) {
+                    load_items<ITEMS>(sb, p.y, tid, y);
+                } else {
+#pragma unroll
+                    for (int j = 0; j < ITEMS; j++) y[j] = p.lit;
+                }
+                NG_CMP_ALL(x, y)
             }
-            switch (p.op) {
-            case EQ: live &= cmp_items<ITEMS, EQ>(x, y); break;
-            case NE: live &= cmp_items<ITEMS, NE>(x, y); break;
-            case LT: live &= cmp_items<ITEMS, LT>(x, y); break;
-            case LE: live &= cmp_items<ITEMS, LE>(x, y); break;
-            case GT: live &= cmp_items<ITEMS, GT>(x, y); break;
-            default: live &= cmp_items<ITEMS, GE>(x, y); break;
-            }
+#undef NG_CMP_ALL
         }
         unsigned kvalid = live;
         if constexpr (KB > 0) {
@@ -248,6 +295,17 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
             continue;
         }
         const unsigned long long tb = s_claim;
+        // keys and payloads of the tile's items, loaded with the column
+        // widths resolved ONCE per tile (uniform branches) -- per item only
+        // the stores and the optional reductions remain
+        K keys[ITEMS];
+        if constexpr (KB > 0) load_keys<KB, ITEMS>(sb, tp, tid, keys);
+        V vals[ITEMS];
+        if constexpr (VB > 0) {
+#pragma unroll
+            for (int j = 0; j < ITEMS; j++) vals[j] = reinterpret_cast<const V *>(sb + tp.val.off)[j * T_THREADS + tid];
+        }
+        const bool want_ext = extreme != nullptr, want_mask = keymask != nullptr;
 #pragma unroll
         for (int j = 0; j < ITEMS; j++) {
             if (!(live >> j & 1u)) continue;
@@ -255,26 +313,23 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
             const long long pos = (long long)tb + s_cnt[j][warp] + rank[j];
             if (out_ids) out_ids[pos] = (int)(base + li);
             if constexpr (KB > 0) {
-                K key;
-                if (tp.n_key == 2)
-                    key = (K)(((uint64_t)enc32((int)ld_col(sb, tp.key0, li)) << 32) |
-                              enc32((int)ld_col(sb, tp.key1, li)));
-                else if (KB == 4 && tp.key0.w == 4)
-                    key = (K)enc32((int)ld_col(sb, tp.key0, li));
-                else   // (KB == 4 with an 8-byte column: the low word of the 64-bit code, its high word constant)
-                    key = (K)enc64(ld_col(sb, tp.key0, li));
-                if (out_keys) ((K *)out_keys)[pos] = key;
+                if (out_keys) ((K *)out_keys)[pos] = keys[j];
                 if (out_kvalid) out_kvalid[pos] = (kvalid >> j) & 1u;
-                kand &= (unsigned long long)key;
-                kor |= (unsigned long long)key;
+                if (want_mask) {
+                    kand &= (unsigned long long)keys[j];
+                    kor |= (unsigned long long)keys[j];
+                }
             }
             if constexpr (VB > 0) {
-                const V v = (V)ld_col(sb, tp.val, li);
+                const V v = vals[j];
                 if (out_vals) ((V *)out_vals)[pos] = v;
-                ext_max |= v == (VB == 8 ? (V)LLONG_MAX : (V)INT_MAX);
-                ext_min |= v == (VB == 8 ? (V)LLONG_MIN : (V)INT_MIN);
-                const unsigned long long a = v < 0 ? 0ull - (unsigned long long)(long long)v : (unsigned long long)v;
-                vabs = a > vabs ? a : vabs;
+                if (want_ext) {
+                    ext_max |= v == (VB == 8 ? (V)LLONG_MAX : (V)INT_MAX);
+                    ext_min |= v == (VB == 8 ? (V)LLONG_MIN : (V)INT_MIN);
+                    const unsigned long long a = v < 0 ? 0ull - (unsigned long long)(long long)v
+                                                       : (unsigned long long)v;
+                    vabs = a > vabs ? a : vabs;
+                }
             }
         }
         __syncthreads();  // stage fully read before it is refilled; s_tile visible
