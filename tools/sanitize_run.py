@@ -2,7 +2,8 @@
 filter (ordered / unordered), sort + histogram, range (short, long, prefix
 aggregates), nested loop (all agg kinds, both R-block shapes), dedup (iota /
 group), finalize, gather, minmax, type-J collections + IN + materialise,
-cost-model calibration (fills)."""
+cost-model calibration (fills), and the radix-sort variants (pre-narrowed
+64-bit keys, 9-bit digit passes, keys without payload)."""
 import os
 import sys
 
@@ -47,6 +48,22 @@ ref = oracle.collect(t, plan)
 bad += not np.array_equal(np.diff(c["offsets"]), ref["lens"][ref["in_rp"].astype(bool)])
 eng.result_to_numpy(eng.collection_in(coll, R["col2"], emit_all=True))
 col = eng.column_from_device(coll.d_values, coll.n_values, "int32")
+# sort variants: 64-bit keys pre-narrowed to 32 bits by the filter, 18-bit
+# keys (9-bit digit passes), keys without payload (4-byte items), all vs numpy
+rng = np.random.default_rng(5)
+for keys, dt, pay in ((rng.integers(0, 1 << 29, 70001) + (7 << 40), "int64", True),
+                      (rng.integers(0, 1 << 18, 70001), "int32", True),
+                      (rng.integers(0, 1 << 26, 90001), "int32", False)):
+    cols = {"k": keys, "v": np.arange(len(keys))} if pay else {"k": keys}
+    T = eng.load_table(cols, dtypes={"k": dt, "v": "int32"} if pay else {"k": dt})
+    ix = eng.build_index(T, ["k"], "v" if pay else None)
+    info = eng.index_info(ix)
+    kb = info["key_bytes"]
+    import torch
+    got = eng.arena_view(info["d_keys"], len(keys) * kb).view(torch.int64 if kb == 8 else torch.int32).cpu().numpy()
+    enc = (keys.astype(np.int64).view(np.uint64) ^ np.uint64(1 << 63)) if kb == 8 else \
+        (keys.astype(np.int32).view(np.uint32) ^ np.uint32(1 << 31))
+    bad += not np.array_equal(got.view(enc.dtype), np.sort(enc))
 eng.cost_calibrate(1 << 16)
 print("sanitize workload done, mismatches:", bad)
 sys.exit(1 if bad else 0)
