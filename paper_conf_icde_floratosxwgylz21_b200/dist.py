@@ -1,21 +1,33 @@
 """Multi-GPU plumbing (one process per GPU, torch.distributed over NCCL).
 
 The paper runs on a single GPU (§IV).  The path shards
-naturally: outer tuples are independent (Fig. 2), so R is split
-into contiguous row blocks, one per rank; the inner relation is needed whole
-on every rank.  The one real exchange step is therefore
+naturally: outer tuples are evaluated independently (Fig. 2), so
+ONE R is split into contiguous row blocks, one per rank (strong scaling; the
+global row id of a shard's first row is passed to the engine as
+``row_id_base``); the inner relation is needed whole on every rank.  The
+exchange steps are therefore
 
   * a broadcast of the invariant inner side (S's columns, and the built index
     so only rank 0 sorts) from rank 0 -- over NVLink/NVSwitch via NCCL,
     directly into tensor views of each rank's engine arena;
-  * a gather of the variable-length survivor lists to rank 0 (NCCL has no
-    gatherv: counts are all-gathered first, payloads padded to the max).
+  * a gather of the variable-length survivor lists to rank 0 only: the
+    counts are exchanged (8 B per rank), then every rank sends its rows to
+    rank 0 with point-to-point sends (one grouped batch, so NCCL runs the
+    N-1 transfers concurrently) -- rank 0 receives each survivor once, no
+    padding and no copy on the other ranks.
 
 The helpers move tensors only; they work with NCCL (GPU box) and gloo (CPU
 tests, or several ranks sharing one GPU: gloo collectives that do not take
 CUDA tensors are staged through host memory).
+
+``launch_ranks`` starts the N-rank job (torchrun, 127.0.0.1 rendezvous) when
+a script is started without a torch.distributed environment.
 """
+import glob
 import os
+import socket
+import subprocess
+import sys
 
 import torch
 import torch.distributed as dist
@@ -37,12 +49,68 @@ def shard_range(n, rank, world):
     return lo, hi
 
 
+def free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def in_distributed_env():
+    return "WORLD_SIZE" in os.environ and "RANK" in os.environ
+
+
+def launch_ranks(script, argv, n, env=None, timeout=None):
+    """Run `script argv` as an n-rank job, one process per rank (torchrun
+    --standalone-style rendezvous on 127.0.0.1), inheriting stdout/stderr.
+    Returns the job's exit code.  Used by bench.py when it is started with
+    --gpus N > 1 outside torchrun."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", str(int(n)),
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()), script] + list(argv)
+    e = dict(os.environ if env is None else env)
+    e.setdefault("OMP_NUM_THREADS", "1")
+    return subprocess.call(cmd, env=e, timeout=timeout)
+
+
+def nccl_debug_setup(tag="nestgpu"):
+    """Ask NCCL (before the communicator exists) to log its INIT subsystem to
+    a per-process file, so the run can report what NCCL built (ranks,
+    transports, NVLS) without NCCL writing into stdout.  Returns the pattern."""
+    d = os.environ.get("TMPDIR", "/tmp")
+    pat = os.path.join(d, "%s_nccl.%d" % (tag, os.getpid()))
+    os.environ.setdefault("NCCL_DEBUG", "INFO")
+    os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT,NVLS")
+    os.environ.setdefault("NCCL_DEBUG_FILE", pat + ".%h.%p.log")
+    return pat
+
+
+def nccl_init_summary(pattern):
+    """The lines of this process's NCCL INIT log that show the communicator
+    (rank count, NVLS / channel setup, version)."""
+    out = []
+    for f in sorted(glob.glob(pattern + "*")):
+        try:
+            for ln in open(f, errors="replace"):
+                if ("Init COMPLETE" in ln or "NCCL version" in ln or "NVLS" in ln or "nRanks" in ln
+                        or "Connected all" in ln):
+                    out.append(ln.strip()[-240:])
+        except OSError:
+            pass
+    return out[:12]
+
+
 def broadcast_tensors(tensors, src=0, group=None):
     """Broadcast each tensor in place from `src` (tensor views of the arena on
     the receiving ranks, so the bytes land where the engine reads them)."""
     for t in tensors:
         if t.numel():
-            dist.broadcast(t, src=src, group=group)
+            if _is_gloo(group) and t.is_cuda:
+                h = t.cpu()
+                dist.broadcast(h, src=src, group=group)
+                t.copy_(h)
+            else:
+                dist.broadcast(t, src=src, group=group)
 
 
 def broadcast_ints(values, src=0, device="cpu", group=None):
@@ -56,27 +124,56 @@ def broadcast_int(value, src=0, device="cpu", group=None):
     return broadcast_ints([value], src=src, device=device, group=group)[0]
 
 
-def gather_rows(parts, dst=0, group=None):
-    """Gather variable-length 1-D tensors (same dtype per position in `parts`)
-    from every rank to `dst`.  Returns the per-field concatenation in rank
-    order on dst, None elsewhere.  Collective: every rank must call it."""
+def all_counts(n, device="cpu", group=None):
+    """Every rank's n (one int64 per rank, all-gathered)."""
     world = dist.get_world_size(group)
+    dev = "cpu" if _is_gloo(group) else device
+    t = torch.tensor([int(n)], dtype=torch.int64, device=dev)
+    bufs = [torch.zeros_like(t) for _ in range(world)]
+    dist.all_gather(bufs, t, group=group)
+    return [int(b.item()) for b in bufs]
+
+
+def gather_rows(parts, dst=0, group=None):
+    """Gather variable-length 1-D tensors (same length within a rank, same
+    dtype per position in `parts`) from every rank to `dst` only.  Returns the
+    per-field concatenation in rank order on dst, None elsewhere.
+    Collective: every rank must call it.
+
+    Counts first (8 B per rank), then one grouped batch of point-to-point
+    transfers into exactly-sized buffers on dst: dst receives sum(counts)
+    rows once per field; no rank pads or receives anything else."""
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
     dev = parts[0].device
-    stage = _is_gloo(group) and dev.type != "cpu"     # gloo all_gather takes CPU tensors
-    cdev = torch.device("cpu") if stage else dev
-    n = torch.tensor([parts[0].numel()], dtype=torch.int64, device=cdev)
-    counts = [torch.zeros_like(n) for _ in range(world)]
-    dist.all_gather(counts, n, group=group)
-    counts = [int(c.item()) for c in counts]
-    mx = max(counts) if counts else 0
+    gloo = _is_gloo(group)
+    cdev = torch.device("cpu") if (gloo and dev.type != "cpu") else dev
+    counts = all_counts(parts[0].numel(), device=dev, group=group)
+    if world == 1:
+        return list(parts)
+    ops, recv = [], {}
+    peer = (lambda r: dist.get_global_rank(group, r)) if group is not None else (lambda r: r)
+    if rank == dst:
+        for r in range(world):
+            if r == dst or counts[r] == 0:
+                continue
+            for i, p in enumerate(parts):
+                buf = torch.empty(counts[r], dtype=p.dtype, device=cdev)
+                recv[(r, i)] = buf
+                ops.append(dist.P2POp(dist.irecv, buf, peer(r), group))
+    elif counts[rank]:
+        for p in parts:
+            ops.append(dist.P2POp(dist.isend, p.contiguous().to(cdev), peer(dst), group))
+    if ops:
+        for w in dist.batch_isend_irecv(ops):
+            w.wait()
+    if rank != dst:
+        return None
     out = []
-    for p in parts:
-        pad = torch.zeros(mx, dtype=p.dtype, device=cdev)
-        pad[:p.numel()] = p.to(cdev)
-        bufs = [torch.zeros_like(pad) for _ in range(world)]
-        dist.all_gather(bufs, pad, group=group)
-        out.append(torch.cat([b[:c] for b, c in zip(bufs, counts)]).to(dev) if dist.get_rank(group) == dst else None)
-    return out if dist.get_rank(group) == dst else None
+    for i, p in enumerate(parts):
+        pieces = [p if r == dst else recv[(r, i)].to(dev) for r in range(world) if counts[r] and (r == dst or (r, i) in recv)]
+        out.append(torch.cat(pieces) if pieces else p[:0])
+    return out
 
 
 def max_over_ranks(x, device="cpu", group=None):
@@ -84,6 +181,14 @@ def max_over_ranks(x, device="cpu", group=None):
     t = torch.tensor([float(x)], dtype=torch.float64, device=dev)
     if dist.is_available() and dist.is_initialized():
         dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
+    return float(t.item())
+
+
+def sum_over_ranks(x, device="cpu", group=None):
+    dev = "cpu" if (dist.is_available() and dist.is_initialized() and _is_gloo(group)) else device
+    t = torch.tensor([float(x)], dtype=torch.float64, device=dev)
+    if dist.is_available() and dist.is_initialized():
+        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
     return float(t.item())
 
 
@@ -132,4 +237,4 @@ def gather_result(eng, res, group=None):
     """Gather one exec result's (row id, value, valid, passed) to rank 0 (row
     ids are global when the shard passed row_id_base)."""
     t = eng.result_tensors(res)
-    return gather_rows([t["row"].clone(), t["value"].clone(), t["valid"].clone(), t["passed"].clone()], group=group)
+    return gather_rows([t["row"], t["value"], t["valid"], t["passed"]], group=group)

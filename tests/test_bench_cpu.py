@@ -56,3 +56,21 @@ def test_bench_our_arm_c1_json_contract():
         assert k in d, k
     assert d["value"] > 0 and d["gpu_launches"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0
     assert d["roofline"]["bound"] == "alu" and 0 < d["roofline"]["frac"]
+
+
+@pytest.mark.gpu
+def test_bench_spawns_two_ranks_gloo():
+    """`bench.py --gpus 2` outside torchrun launches 2 ranks itself (here gloo,
+    both on the one B200); rank 0 reports n_gpus 2 and finds the gathered
+    survivors identical to the whole-R 1-GPU result."""
+    env = dict(os.environ, NESTGPU_DIST_BACKEND="gloo")
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--workload", "C1",
+                        "--steps", "3", "--warmup", "3", "--no-cpu-baseline"], capture_output=True, text=True,
+                       timeout=900, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["scaling"] == "strong"
+    assert d["whole_r_check"]["identical"] is True
+    assert d["multi_gpu_stages_ms_per_step"]["gather"] >= 0

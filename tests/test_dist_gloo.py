@@ -81,3 +81,19 @@ def test_gloo_world2_broadcast_shard_gather():
     status, ok, mx = q.get(timeout=10)
     assert status == "ok" and ok
     assert mx == 2.0
+
+
+def test_launch_ranks_world4(tmp_path):
+    """The spawn path of `bench.py --gpus N` outside torchrun
+    (dist.launch_ranks -> torchrun on 127.0.0.1) at world 4 with gloo: shard
+    one R, gather the survivors to rank 0 only (point-to-point, one rank with
+    an empty shard), compare with the whole-R result."""
+    out = tmp_path / "verdict.json"
+    env = dict(os.environ, NESTGPU_DIST_BACKEND="gloo")
+    rc = ngd.launch_ranks(os.path.join(os.path.dirname(__file__), "dist_worker.py"), [str(out)], 4, env=env,
+                          timeout=300)
+    assert rc == 0
+    import json
+    v = json.loads(out.read_text())
+    assert v["world"] == 4 and v["ok"] and v["plans"] == 4
+    assert v["counts_ok"] and v["max"] == 3.0 and v["sum"] == 4.0

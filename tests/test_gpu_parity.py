@@ -199,9 +199,12 @@ def test_c2_full_size(eng):
         g = run(eng, t, plan, mode, emit_all=True)
         ref = oracle.evaluate(t, plan, rows=rows)
         assert_parity(g, ref, plan, True, rows=rows, ctx=(corr_op, agg))
-        valid, value, _, _ = ind.closed_form(t["R"]["col1"], t["S"]["col1"], t["S"]["col2"], corr_op, agg)
+        valid, value, cnt, s_sum = ind.closed_form(t["R"]["col1"], t["S"]["col1"], t["S"]["col2"], corr_op, agg)
         assert np.array_equal(g["valid"].astype(bool), valid), (corr_op, agg)
         assert np.array_equal(g["value"], value), (corr_op, agg)
+        # the outer comparison on every row (not only the oracle's sample)
+        passed = ind.outer_passed(t["R"]["col2"], valid, value, cnt, s_sum, agg, "=")
+        assert np.array_equal(g["passed"].astype(bool), passed), (corr_op, agg)
         s = run(eng, t, plan, mode, emit_all=False)
         exp = np.nonzero(g["passed"])[0]
         assert np.array_equal(s["row"], exp)
@@ -450,18 +453,23 @@ def test_int64_keys_narrowed_sort(eng, base):
                 assert_parity(g, ref, plan, True, ctx=(base, corr_op, agg, dedup))
 
 
-def test_c5_full_size(eng):
-    """BASELINE configs[4] at its full size (|R| = |S| = 16M, '>' MIN on the
-    nested loop -- bench.py --workload C5's launch configuration): the closed
-    form on every one of the 16M rows, the oracle on 200 sampled rows."""
+@pytest.mark.parametrize("corr_op,agg", [(">", "min"), (">", "count"), ("!=", "min")])
+def test_c5_full_size(eng, corr_op, agg):
+    """BASELINE configs[4] at its full size (|R| = |S| = 16M, nested loop --
+    bench.py's headline launch configuration, '>' MIN, and its side plans
+    '>' COUNT and '!=' MIN, SURVEY §8(d) "Also run count and !="): the closed
+    form on every one of the 16M rows (value, valid and the outer comparison
+    'passed'), the oracle on 200 sampled rows."""
     t = query1.config("C5")
-    plan = make_plan(">", "min", "=")
+    plan = make_plan(corr_op, agg, "=")
     rows = np.unique(np.random.default_rng(9).integers(0, 16_000_000, 200))
     g = run(eng, t, plan, "bnl", emit_all=True)
-    valid, value, _, _ = ind.closed_form(t["R"]["col1"], t["S"]["col1"], t["S"]["col2"], ">", "min")
+    valid, value, cnt, s_sum = ind.closed_form(t["R"]["col1"], t["S"]["col1"], t["S"]["col2"], corr_op, agg)
     assert np.array_equal(g["value"], value)
     assert np.array_equal(g["valid"].astype(bool), valid)
-    assert_parity(g, oracle.evaluate(t, plan, rows=rows), plan, True, rows=rows, ctx="C5 full")
+    passed = ind.outer_passed(t["R"]["col2"], valid, value, cnt, s_sum, agg, "=")
+    assert np.array_equal(g["passed"].astype(bool), passed)
+    assert_parity(g, oracle.evaluate(t, plan, rows=rows), plan, True, rows=rows, ctx=("C5 full", corr_op, agg))
 
 
 def _key_pattern(name, n, rng):

@@ -345,3 +345,18 @@ def test_in_list_against_sqlite(oracle_lib, seed):
         plan = make_plan(corr_op, "min", "=", inner_preds=[{"col": "col3", "op": ">=", "lit": 1}])
         in_rp, passed = oracle.in_list(t, plan, "col2")
         assert np.nonzero(passed)[0].tolist() == ind.in_sqlite(t, plan, "col2", con), corr_op
+
+
+@pytest.mark.parametrize("outer_op", ["=", "!=", "<", "<=", ">", ">="])
+def test_closed_form_outer_passed(oracle_lib, outer_op):
+    """oracle/unnested.outer_passed (the full-size GPU tests' check of the
+    outer comparison on every row) against the oracle's `passed`, with
+    multipliers (reading R7) and every aggregate."""
+    t = query1.tables(n_r=2003, n_s=5003, key_hi=600, val_hi=30, seed=11)
+    for corr_op in ("=", "!=", ">"):
+        for agg in VALUE_AGGS + ("count", "exists", "not_exists"):
+            plan = make_plan(corr_op, agg, outer_op, lhs_mult=3, rhs_mult=2)
+            res = oracle.evaluate(t, plan)
+            valid, value, cnt, ssum = ind.closed_form(t["R"]["col1"], t["S"]["col1"], t["S"]["col2"], corr_op, agg)
+            got = ind.outer_passed(t["R"]["col2"], valid, value, cnt, ssum, agg, outer_op, 3, 2)
+            assert np.array_equal(res["passed"].astype(bool), got), (corr_op, agg, outer_op)
