@@ -12,12 +12,16 @@
 //   D2H of the survivor count.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <climits>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <map>
+#include <mutex>
 #include <string>
+#include <tuple>
 #include <utility>
 #include <vector>
 
@@ -53,10 +57,12 @@ struct IndexRec {
     std::vector<nestgpu_pred> inner;
     bool payload_nullable;
     // index-pruned evaluation (NEXT 3): prefix / suffix aggregates of the
-    // payload per kind (0 MIN, 1 MAX, 2 SUM), built on first use
-    long long *aux_pre[3];
-    long long *aux_suf[3];
-    size_t aux_off[3];
+    // payload per kind (0 MIN, 1 MAX, 2 SUM, 3 split SUM: pre = low halves,
+    // suf = high halves; 4 / 5: per-key group MIN / MAX for '='), built on
+    // first use
+    long long *aux_pre[6];
+    long long *aux_suf[6];
+    size_t aux_off[6];
 };
 
 constexpr int PIN_WORDS = 8 * 256 + 64;
@@ -321,6 +327,23 @@ nestgpu_status column_stats(nestgpu_ctx *c, Column &col)
 
 // Context accessors for the host-side modules (cost.cpp) -- internal.h.
 namespace ng {
+namespace {
+std::mutex g_launch_mu;
+std::map<std::tuple<const void *, long long, int>, int> g_launch_cache;
+}  // namespace
+bool launch_cache_get(const void *kernel, long long key, int dev, int *value)
+{
+    std::lock_guard<std::mutex> g(g_launch_mu);
+    auto it = g_launch_cache.find(std::make_tuple(kernel, key, dev));
+    if (it == g_launch_cache.end()) return false;
+    *value = it->second;
+    return true;
+}
+void launch_cache_put(const void *kernel, long long key, int dev, int value)
+{
+    std::lock_guard<std::mutex> g(g_launch_mu);
+    g_launch_cache[std::make_tuple(kernel, key, dev)] = value;
+}
 void *ctx_scratch_alloc(nestgpu_ctx *c, size_t bytes) { return salloc(c, bytes); }
 void ctx_scratch_reset(nestgpu_ctx *c) { scratch_reset(c); }
 cudaStream_t ctx_stream(nestgpu_ctx *c) { return c->stream; }
@@ -386,6 +409,18 @@ int64_t nestgpu_launch_count(const nestgpu_ctx *c) { return c ? c->launches : 0;
 nestgpu_status nestgpu_set_stream(nestgpu_ctx *c, void *s)
 {
     if (!c) return NESTGPU_ERR_INVALID;
+    cudaSetDevice(c->device);
+    // Work queued on the old stream (e.g. an index build's radix passes) may
+    // still write the arena: the new stream waits for it before anything
+    // enqueued after the switch (no host synchronisation).
+    if ((cudaStream_t)s != c->stream) {
+        cudaEvent_t ev;
+        CUDA_TRY(c, cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+        cudaError_t e = cudaEventRecord(ev, c->stream);
+        if (e == cudaSuccess) e = cudaStreamWaitEvent((cudaStream_t)s, ev, 0);
+        cudaEventDestroy(ev);
+        if (e != cudaSuccess) return fail(c, NESTGPU_ERR_CUDA, "set_stream: %s", cudaGetErrorString(e));
+    }
     c->stream = (cudaStream_t)s;
     return NESTGPU_OK;
 }
@@ -410,7 +445,7 @@ nestgpu_status nestgpu_release(nestgpu_ctx *c, uint64_t m)
         if (col.alive && col.off >= m) col.alive = false;
     for (auto &ix : c->idx) {
         if (ix.alive && ix.off >= m) ix.alive = false;
-        for (int k = 0; k < 3; k++)
+        for (int k = 0; k < 6; k++)
             if (ix.aux_pre[k] && ix.aux_off[k] >= m) ix.aux_pre[k] = ix.aux_suf[k] = nullptr;
     }
     return NESTGPU_OK;
@@ -679,6 +714,13 @@ nestgpu_status nestgpu_index_create_empty(nestgpu_ctx *c, int64_t n, int32_t key
     if (key_bytes(c, key_cols, n_key_cols) != key_bytes_)
         return fail(c, NESTGPU_ERR_TYPE, "index_create_empty: key width does not match the key columns");
     if (n_inner_preds < 0 || (n_inner_preds > 0 && !inner_preds)) return fail(c, NESTGPU_ERR_INVALID, "bad inner preds");
+    {
+        const Column *pcol = payload_col >= 0 ? col_get(c, payload_col) : nullptr;
+        if (payload_col >= 0 && !pcol) return fail(c, NESTGPU_ERR_INVALID, "index_create_empty: unknown payload column %d", payload_col);
+        if (payload_bytes != (pcol ? dtype_width(pcol->dtype) : 0))
+            return fail(c, NESTGPU_ERR_INVALID, "index_create_empty: payload_bytes must equal the payload column's width (0 without payload)");
+        if (pcol && pcol->n != ns) return fail(c, NESTGPU_ERR_INVALID, "index_create_empty: payload row count differs");
+    }
     cudaSetDevice(c->device);
     IndexRec ix{};
     ix.off = c->lo;
@@ -768,14 +810,22 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
             return fail(c, NESTGPU_ERR_INVALID, "exec: index %d dropped NULL-payload rows; COUNT/EXISTS need an index without payload", P->index);
         if (ix->kb != kb)
             return fail(c, NESTGPU_ERR_UNSUPPORTED, "exec: outer key is 64-bit but index %d has 32-bit keys", P->index);
+        if (value_agg && (ix->vb != dtype_width(ac->dtype) || (ix->n > 0 && !ix->payload)))
+            return fail(c, NESTGPU_ERR_INVALID, "exec: index %d carries %d-byte payloads, column %d has %d-byte values",
+                        P->index, ix->vb, P->agg_col, dtype_width(ac->dtype));
     }
     const int vb = value_agg ? dtype_width(ac->dtype) : 0;
+    // Exact SUM/AVG (reading R5): 32-bit payloads cannot overflow (|S| < 2^31);
+    // 64-bit payloads whose |S| * max|payload| could reach 2^63 are summed as
+    // split halves (low 32 bits unsigned, high 32 bits signed -- neither sum can
+    // overflow) and recombined in int128 by finalize, which reports
+    // NESTGPU_ERR_OVERFLOW only when an actual result leaves int64.
+    bool wide = false;
     if ((P->agg == NG_SUM || P->agg == NG_AVG) && vb == 8) {
         if (ac->caller_filled) ac->stats = false;   // recomputed: the caller may have rewritten it
         if ((s = column_stats(c, *ac))) return s;
-        __int128 m = ac->mx > -(ac->mn) ? (__int128)ac->mx : -(__int128)ac->mn;
-        if ((__int128)nS * m >= ((__int128)1 << 63))
-            return fail(c, NESTGPU_ERR_OVERFLOW, "exec: |S| * max|payload| may exceed int64 (reading R5)");
+        const __int128 m = std::max((__int128)ac->mx, -(__int128)ac->mn);
+        wide = (__int128)nS * m >= ((__int128)1 << 63);
     }
 
     // ------------------------------------------------------------ allocation
@@ -787,7 +837,8 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     uint8_t *rkvalid = ravalid ? (uint8_t *)salloc(c, (size_t)nR) : nullptr;
     long long *acc = (long long *)salloc(c, (size_t)nR * 8);
     long long *cnt = (long long *)salloc(c, (size_t)nR * 8);
-    long long *counts = (long long *)salloc(c, 64);  // [0] |R'| [1] |S'| [2] survivors; [4..5] extreme
+    long long *counts = (long long *)salloc(c, 128);  // [0] |R'| [1] |S'| [2] survivors; [4..5] extreme; [8] overflow
+    long long *acc_hi = wide ? (long long *)salloc(c, (size_t)nR * 8) : nullptr;
     size_t fsz = ng::filter_scratch_bytes(nR > nS ? nR : nS);
     void *fscr = salloc(c, fsz);
     void *kscr = salloc(c, ix ? ng::range_scratch_bytes(nR) : ng::bnl_scratch_bytes(nR));
@@ -803,10 +854,11 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         svals = vb ? salloc(c, (size_t)nS * vb) : nullptr;
     }
     if (!ids || !rkeys || (ravalid && !rkvalid) || !acc || !cnt || !counts || !fscr || !kscr || !o_ids || !o_vals ||
-        !o_valid || !o_pass || (P->agg == NG_AVG && (!o_sum || !o_cnt)) || (!ix && (!skeys || (vb && !svals))))
+        !o_valid || !o_pass || (P->agg == NG_AVG && (!o_sum || !o_cnt)) || (!ix && (!skeys || (vb && !svals))) ||
+        (wide && !acc_hi))
         return fail(c, NESTGPU_ERR_OOM, "arena exhausted executing a plan over |R|=%lld |S|=%lld", (long long)nR, (long long)nS);
     // counts: [0] |R'| [1] |S'| [2] survivors [3] distinct keys [4] extreme flags (2 x u32)
-    //         [6] AND / [7] OR of the R' keys (dedup sort planning)
+    //         [6] AND / [7] OR of the R' keys (dedup sort planning) [8] split-SUM overflow flag
     unsigned *extreme = (unsigned *)(counts + 4);
     long long *d_nrp = counts, *d_nsp = counts + 1, *d_out = counts + 2, *d_u = counts + 3;
     unsigned long long *rmask = (unsigned long long *)(counts + 6);
@@ -832,8 +884,9 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     prof_begin(c, 5);
     prof_begin(c, 0);
     ng::ValSrc none{nullptr, nullptr, 0};
-    CUDA_TRY(c, cudaMemsetAsync(counts, 0, 64, c->stream));
+    CUDA_TRY(c, cudaMemsetAsync(counts, 0, 128, c->stream));
     CUDA_TRY(c, cudaMemsetAsync(rmask, 0xff, 8, c->stream));   // AND identity
+    if (wide && nR > 0) CUDA_TRY(c, cudaMemsetAsync(acc_hi, 0, (size_t)nR * 8, c->stream));
     CUDA_TRY(c, ng::launch_filter(nR, ops, rks, kb, none, 0, 0, 0, ids, rkeys, rkvalid, nullptr,
                                   P->dedup ? rmask : nullptr, nullptr, fscr, d_nrp, c->stream, &c->launches));
     prof_end(c, 0);
@@ -885,29 +938,49 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         // index and aggregate kind, kept with the index.
         const long long *pre = nullptr, *suf = nullptr;
         if (value_agg && (P->corr_op != NG_EQ || P->agg == NG_SUM || P->agg == NG_AVG)) {
-            const int kind = P->agg == NG_MIN ? 0 : (P->agg == NG_MAX ? 1 : 2);
+            const int kind = P->agg == NG_MIN ? 0 : (P->agg == NG_MAX ? 1 : (wide ? 3 : 2));
             const int akind = kind == 0 ? ng::MIN : (kind == 1 ? ng::MAX : ng::SUM);
             if (!ix->aux_pre[kind]) {
                 const size_t off = c->lo;
                 long long *ap = (long long *)palloc(c, (size_t)(ix->n + 1) * 8);
-                long long *as = kind < 2 ? (long long *)palloc(c, (size_t)(ix->n + 1) * 8) : nullptr;
+                long long *as = kind != 2 ? (long long *)palloc(c, (size_t)(ix->n + 1) * 8) : nullptr;
                 void *ascr = salloc(c, ng::index_aux_scratch_bytes(ix->n));
-                if (!ap || (kind < 2 && !as) || !ascr) {
+                if (!ap || (kind != 2 && !as) || !ascr) {
                     c->lo = off;
                     return fail(c, NESTGPU_ERR_OOM, "arena exhausted (index prefix aggregates)");
                 }
-                CUDA_TRY(c, ng::launch_index_aux(akind, ix->vb, ix->payload, ix->n, ap, as, ascr, c->stream,
-                                                 &c->launches));
+                CUDA_TRY(c, ng::launch_index_aux(akind, ix->vb, ix->payload, ix->n, ap, kind == 3 ? nullptr : as, ascr,
+                                                 c->stream, &c->launches, kind == 3 ? as : nullptr));
                 ix->aux_pre[kind] = ap;
                 ix->aux_suf[kind] = as;
                 ix->aux_off[kind] = off;
             }
             pre = ix->aux_pre[kind];
             suf = ix->aux_suf[kind];
+        } else if (P->agg == NG_MIN || P->agg == NG_MAX) {
+            // '=' MIN/MAX: per-key group aggregates (segmented scan), so a hot
+            // key's run is folded once per index, not once per outer tuple
+            const int kind = P->agg == NG_MIN ? 4 : 5;
+            if (!ix->aux_pre[kind]) {
+                const size_t off = c->lo;
+                long long *gp = (long long *)palloc(c, (size_t)(ix->n + 1) * 8);
+                void *gscr2 = salloc(c, ng::index_aux_scratch_bytes(ix->n));
+                if (!gp || !gscr2) {
+                    c->lo = off;
+                    return fail(c, NESTGPU_ERR_OOM, "arena exhausted (index group aggregates)");
+                }
+                CUDA_TRY(c, ng::launch_index_group_agg(kind == 4 ? ng::MIN : ng::MAX, ix->kb, ix->vb, ix->keys,
+                                                       ix->payload, ix->n, gp, gscr2, c->stream, &c->launches));
+                ix->aux_pre[kind] = gp;
+                ix->aux_off[kind] = off;
+            }
+            pre = ix->aux_pre[kind];
         }
         prof_begin(c, 3);
+        const bool split = wide && pre && P->agg != NG_MIN && P->agg != NG_MAX;
         CUDA_TRY(c, ng::launch_range_agg(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, ix->keys, ix->payload,
-                                         ix->n, pre, suf, acc, cnt, kscr, c->stream, &c->launches));
+                                         ix->n, pre, split ? nullptr : suf, acc, cnt, kscr, c->stream, &c->launches,
+                                         split ? suf : nullptr, split ? acc_hi : nullptr));
         prof_end(c, 3);
     } else {
         prof_begin(c, 1);
@@ -920,7 +993,8 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         prof_end(c, 1);
         prof_begin(c, 3);
         CUDA_TRY(c, ng::launch_bnl(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, nS, d_nsp, skeys, svals,
-                                   extreme, acc, cnt, kscr, c->num_sms, c->bnl_shape, c->stream, &c->launches));
+                                   extreme, acc, cnt, kscr, c->num_sms, c->bnl_shape, c->stream, &c->launches,
+                                   wide ? acc_hi : nullptr));
         prof_end(c, 3);
     }
 
@@ -934,6 +1008,8 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     fa.kvalid = rkvalid;
     fa.acc = acc;
     fa.cnt = cnt;
+    fa.acc_hi = wide ? acc_hi : nullptr;
+    fa.overflow = (unsigned long long *)(counts + 8);
     fa.x_col = xc ? xc->d : nullptr;
     fa.x_valid = xc ? xc->valid : nullptr;
     fa.x_w = xc ? dtype_width(xc->dtype) : 4;
@@ -954,10 +1030,11 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     CUDA_TRY(c, ng::launch_finalize(fa, c->stream, &c->launches));
     prof_end(c, 4);
     prof_end(c, 5);
-    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, counts, 32, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, counts, 72, cudaMemcpyDeviceToHost, c->stream));
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
-    long long cnts[4];
-    memcpy(cnts, c->pinned, 32);
+    long long cnts[9];
+    memcpy(cnts, c->pinned, 72);
+    if (cnts[8]) return fail(c, NESTGPU_ERR_OVERFLOW, "exec: a SUM exceeds int64 (reading R5)");
     out->n_rows = cnts[2];
     out->n_evaluated = P->dedup ? n_distinct : cnts[0];
     out->d_row_ids = (const int64_t *)o_ids;

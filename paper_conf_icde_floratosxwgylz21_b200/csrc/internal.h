@@ -10,6 +10,29 @@ struct nestgpu_ctx;
 
 namespace ng {
 
+// Per-device launch setup cache (api.cpp).  The opt-in to more than 48 KB of
+// dynamic shared memory (cudaFuncSetAttribute) and the occupancy a launcher
+// sizes its persistent grid from are per DEVICE, so a process driving several
+// GPUs (one context per device) must not reuse the first device's setup.
+// Entries are keyed by (kernel, key, device) and guarded by a mutex.
+bool launch_cache_get(const void *kernel, long long key, int dev, int *value);
+void launch_cache_put(const void *kernel, long long key, int dev, int value);
+
+// *value = the cached setup of `kernel` for `key` on the current device, or
+// init(dev, value) once (cudaFuncSetAttribute + occupancy; it may run twice
+// when two threads race, which is harmless: both calls are idempotent).
+template <typename F>
+inline cudaError_t per_device_setup(const void *kernel, long long key, int *value, F init)
+{
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (launch_cache_get(kernel, key, dev, value)) return cudaSuccess;
+    if ((e = init(dev, value)) != cudaSuccess) return e;
+    launch_cache_put(kernel, key, dev, *value);
+    return cudaSuccess;
+}
+
 // Context accessors (api.cpp) for host-side modules such as cost.cpp.
 void *ctx_scratch_alloc(nestgpu_ctx *c, size_t bytes);   // nullptr when the arena is exhausted
 void ctx_scratch_reset(nestgpu_ctx *c);
@@ -80,16 +103,27 @@ cudaError_t launch_init_partials(long long n, const long long *d_n, int agg, lon
 size_t range_scratch_bytes(long long n_rp_max);
 //   pre / suf: optional prefix / suffix aggregates of the index payload
 //   (launch_index_aux); non-equality and SUM/AVG ranges are then O(1).
+//   pre_hi / acc_hi: exact SUM of 64-bit payloads (nullable): pre holds the
+//   prefix sums of the payloads' low 32-bit halves (unsigned) and pre_hi of
+//   their high halves (signed), neither of which can overflow; a range's two
+//   partial sums go to acc / acc_hi and finalize combines them in int128.
 cudaError_t launch_range_agg(int kb, int vb, int op, int agg, long long n_rp_max, const long long *d_nrp,
                              const void *rkeys, const void *skeys, const void *svals, long long ns,
                              const long long *pre, const long long *suf, long long *acc, long long *cnt,
-                             void *scratch, cudaStream_t st, long long *launches);
+                             void *scratch, cudaStream_t st, long long *launches,
+                             const long long *pre_hi = nullptr, long long *acc_hi = nullptr);
 
 // Index-pruned evaluation (NEXT 3): pre[0..n] / suf[0..n] aggregates (MIN,
 // MAX: both; SUM: pre only) of the co-sorted payload of an index.
 size_t index_aux_scratch_bytes(long long n);
+// '=' MIN/MAX: per-key group aggregates grp[p] = AGG(payload[run start .. p])
+// over the sorted index (segmented scan; runs of equal keys); n entries.
+cudaError_t launch_index_group_agg(int agg, int kb, int vb, const void *keys, const void *payload, long long n,
+                                   long long *grp, void *scratch, cudaStream_t st, long long *launches);
+//   pre_hi (SUM only, nullable): split prefix sums -- pre over the low 32-bit
+//   halves of the payload (unsigned), pre_hi over the high halves (signed).
 cudaError_t launch_index_aux(int agg, int vb, const void *payload, long long n, long long *pre, long long *suf,
-                             void *scratch, cudaStream_t st, long long *launches);
+                             void *scratch, cudaStream_t st, long long *launches, long long *pre_hi = nullptr);
 
 // a7: tiled block-nested-loop over R' x S'.  d_nrp / d_nsp: device counts.
 size_t bnl_scratch_bytes(long long n_rp_max);
@@ -97,7 +131,9 @@ cudaError_t launch_bnl(int kb, int vb, int op, int agg, long long n_rp_max, cons
                        const void *rkeys, long long ns_max, const long long *d_nsp, const void *skeys,
                        const void *svals, const unsigned *extreme, long long *acc, long long *cnt,
                        void *scratch, int num_sms, int shape /* 0 auto, 1 full, 2 warp-split */,
-                       cudaStream_t st, long long *launches);
+                       cudaStream_t st, long long *launches, long long *acc_hi = nullptr);
+//   acc_hi (SUM/AVG of 64-bit payloads, nullable, zeroed by the caller): exact
+//   split accumulation -- acc += low 32-bit halves, acc_hi += high halves.
 
 // Caching: R' positions 0..n-1; distinct keys of a sorted key run
 // and the map R' position -> distinct id.
@@ -114,6 +150,8 @@ struct FinalizeArgs {
     const int *map;          // R' position -> partial-aggregate slot (nullable = identity)
     const uint8_t *kvalid;   // R' key not NULL (nullable = all valid)
     const long long *acc, *cnt;
+    const long long *acc_hi;         // split SUM (nullable): sum = acc_hi * 2^32 + (u64)acc, exact in int128
+    unsigned long long *overflow;    // set when a split SUM leaves int64 (reading R5 -> NESTGPU_ERR_OVERFLOW)
     const void *x_col;       // outer comparison column (nullable for EXISTS)
     const uint8_t *x_valid;
     int x_w;

@@ -13,7 +13,7 @@
 //    in registers, so every S' element read from shared memory is reused
 //    2048 times per CTA (the cache-locality loop);
 //  * S' (key, payload) tiles of 16 KB stream global -> shared through a
-//    4-stage ring of cp.async.bulk copies (TMA bulk engine, UBLKCP) completed
+//    B_STAGES-deep ring (NG_B_STAGES, 3 by default) of cp.async.bulk copies (TMA bulk engine, UBLKCP) completed
 //    on mbarriers by one elected thread; consumers read them with 128-bit
 //    broadcast LDS;
 //  * per (r, s) pair the work is one compare (ISETP) and one predicated
@@ -62,6 +62,7 @@ struct BnlArgs {
     unsigned one;              // runtime 1 (keeps the IMAD multiplier opaque to ptxas)
     long long *acc;
     long long *cnt;
+    long long *acc_hi;         // SUM/AVG of 64-bit payloads, exact split accumulation (nullable)
     unsigned *unit_counter;
     unsigned *rb_done;         // EXISTS: per R block, set once every tuple of the block found a match
     long long target_units;    // work units to aim for (grid x 16)
@@ -189,7 +190,11 @@ __device__ __forceinline__ void sum32_if(const K rk, const K sk, const V v, V &s
 //   MIN/MAX: ISETP + predicated IMNMX (both ALU pipe); with TRACK also
 //            "found" (only when some payload equals the MIN/MAX identity).
 //   COUNT:   ISETP (ALU) + predicated IMAD (FMA).
-//   SUM/AVG: ISETP (ALU) + predicated IMAD + IMAD.WIDE (FMA).
+//   SUM/AVG: ISETP (ALU) + predicated IMAD + IMAD.WIDE (FMA).  With TRACK
+//            and 64-bit payloads ("wide": |S'| * max|payload| may reach
+//            2^63): the payload's low 32-bit half (unsigned) goes to sm and
+//            its high half (signed) to mm; neither sum can overflow int64
+//            (|S'| < 2^31), finalize recombines them exactly (reading R5).
 //   EXISTS:  predicate OR.
 template <int OP, int AGG, bool TRACK, typename K, typename V>
 __device__ __forceinline__ void pair_step(const K rk, const K sk, const V sv, V &mm, long long &sm, unsigned &c,
@@ -200,8 +205,17 @@ __device__ __forceinline__ void pair_step(const K rk, const K sk, const V sv, V 
         if (p) mm = (AGG == MIN) ? min(mm, sv) : max(mm, sv);
         if constexpr (TRACK) found |= p;
     } else if constexpr (AccKind<AGG>::sum) {
-        if constexpr (TRACK && sizeof(V) == 4) sum32_if<OP>(rk, sk, sv, mm, c, one);
-        else sum_if<OP>(rk, sk, sv, sm, c, one);
+        if constexpr (TRACK && sizeof(V) == 4) {
+            sum32_if<OP>(rk, sk, sv, mm, c, one);
+        } else if constexpr (TRACK) {
+            if (cmp_ct<OP>(rk, sk)) {
+                c += 1u;
+                sm += (long long)(unsigned long long)(unsigned)sv;
+                mm += sv >> 32;
+            }
+        } else {
+            sum_if<OP>(rk, sk, sv, sm, c, one);
+        }
     } else if constexpr (AccKind<AGG>::count) {
         count_if<OP>(rk, sk, c, one);
     } else {
@@ -305,7 +319,7 @@ __device__ __forceinline__ void bnl_body(const BnlArgs &A, unsigned char *smem, 
     constexpr V MM0 = AGG == MIN ? VMAX : (AGG == MAX ? VMIN : (V)0);
     constexpr long long RSTRIDE = SPLIT ? 32 : B_THREADS;   // tuple stride within a block
     constexpr long long RBLOCK = RSTRIDE * RPT;
-    static_assert(!SPLIT || RBLOCK * 20 <= (long long)B_STAGES * B_STAGE_BYTES, "split merge area");
+    static_assert(!SPLIT || RBLOCK * 28 <= (long long)B_STAGES * B_STAGE_BYTES, "split merge area");
     const int tid = threadIdx.x;
     const int rlane = SPLIT ? (tid & 31) : tid;
 
@@ -333,6 +347,7 @@ __device__ __forceinline__ void bnl_body(const BnlArgs &A, unsigned char *smem, 
     if constexpr (AccKind<AGG>::minmax) track = A.extreme[AGG == MIN ? 0 : 1] != 0;
     if constexpr (AccKind<AGG>::sum && VB == 4)
         track = *(const unsigned long long *)(A.extreme + 2) < (0x80000000ull / (unsigned long long)TILE);
+    if constexpr (AccKind<AGG>::sum && VB == 8) track = A.acc_hi != nullptr;   // exact split sums
     const unsigned mul = A.one;
     const K *rkeys = (const K *)A.rkeys;
     const K *skeys = (const K *)A.skeys;
@@ -439,10 +454,12 @@ __device__ __forceinline__ void bnl_body(const BnlArgs &A, unsigned char *smem, 
             long long *s_acc = (long long *)smem;
             unsigned long long *s_cnt = (unsigned long long *)(smem + RBLOCK * 8);
             int *s_found = (int *)(smem + RBLOCK * 16);
+            long long *s_hi = (long long *)(smem + RBLOCK * 20);   // split SUM high halves
             for (int t = tid; t < RBLOCK; t += B_THREADS) {
                 s_acc[t] = AccKind<AGG>::minmax ? (long long)MM0 : 0;
                 s_cnt[t] = 0;
                 s_found[t] = 0;
+                s_hi[t] = 0;
             }
             __syncthreads();
 #pragma unroll
@@ -459,6 +476,7 @@ __device__ __forceinline__ void bnl_body(const BnlArgs &A, unsigned char *smem, 
                     if (c[i]) {
                         atomicAdd((unsigned long long *)&s_acc[t], (unsigned long long)sm[i]);
                         atomicAdd(&s_cnt[t], (unsigned long long)c[i]);
+                        if (VB == 8 && track) atomicAdd((unsigned long long *)&s_hi[t], (unsigned long long)mm[i]);
                     }
                 } else if constexpr (AccKind<AGG>::count) {
                     if (c[i]) atomicAdd(&s_cnt[t], (unsigned long long)c[i]);
@@ -480,6 +498,7 @@ __device__ __forceinline__ void bnl_body(const BnlArgs &A, unsigned char *smem, 
                     if (s_cnt[t]) {
                         atomicAdd((unsigned long long *)&A.acc[r], (unsigned long long)s_acc[t]);
                         atomicAdd((unsigned long long *)&A.cnt[r], s_cnt[t]);
+                        if (VB == 8 && track) atomicAdd((unsigned long long *)&A.acc_hi[r], (unsigned long long)s_hi[t]);
                     }
                 } else if constexpr (AccKind<AGG>::count) {
                     if (s_cnt[t]) atomicAdd((unsigned long long *)&A.cnt[r], s_cnt[t]);
@@ -504,6 +523,7 @@ __device__ __forceinline__ void bnl_body(const BnlArgs &A, unsigned char *smem, 
                     if (c[i]) {
                         atomicAdd((unsigned long long *)&A.acc[r], (unsigned long long)sm[i]);
                         atomicAdd((unsigned long long *)&A.cnt[r], (unsigned long long)c[i]);
+                        if (VB == 8 && track) atomicAdd((unsigned long long *)&A.acc_hi[r], (unsigned long long)mm[i]);
                     }
                 } else if constexpr (AccKind<AGG>::count) {
                     if (c[i]) atomicAdd((unsigned long long *)&A.cnt[r], (unsigned long long)c[i]);

@@ -444,14 +444,13 @@ cudaError_t launch_t(long long n, const SrcCols &sc, const TPlan &tp, const Filt
 {
     auto kern = filter_tma_kernel<KB, VB, ITEMS>;
     const int smem = 2 * sc.stage_bytes;
-    static int occ_for = -1, occ = 0;
-    if (occ_for != smem) {
+    int occ = 0;
+    cudaError_t e0 = per_device_setup((const void *)kern, smem, &occ, [&](int, int *v) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * STAGE_MAX);
         if (e != cudaSuccess) return e;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, T_THREADS, smem);
-        if (e != cudaSuccess) return e;
-        occ_for = smem;
-    }
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(v, kern, T_THREADS, smem);
+    });
+    if (e0 != cudaSuccess) return e0;
     const long long tiles = (n + T_THREADS * ITEMS - 1) / (T_THREADS * ITEMS);
     long long grid = (long long)num_sms * (occ > 0 ? occ : 1);
     if (grid > tiles) grid = tiles;

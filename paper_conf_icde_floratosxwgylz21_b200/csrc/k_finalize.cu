@@ -93,8 +93,17 @@ __global__ void __launch_bounds__(F_THREADS) finalize_kernel(FinalizeArgs A, uns
                 const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
                 const long long g = A.map ? (long long)A.map[i] : i;  // cached result slot
                 const long long c = kval ? A.cnt[g] : 0;     // NULL key: empty subquery (R2)
-                const long long acc = A.acc[g];
+                long long acc = A.acc[g];
                 bool vv = true;
+                if (A.acc_hi && c > 0) {   // split SUM: hi * 2^32 + lo, exact (reading R5)
+                    const __int128 t = (__int128)A.acc_hi[g] * 4294967296ll + (__int128)(unsigned long long)acc;
+                    if (t > (__int128)LLONG_MAX || t < (__int128)LLONG_MIN) {
+                        atomicOr(A.overflow, 1ull);
+                        acc = 0;
+                    } else {
+                        acc = (long long)t;
+                    }
+                }
                 long long v = 0;
                 switch (A.agg) {
                 case MIN: case MAX: case SUM: vv = c > 0; v = acc; break;
@@ -145,7 +154,10 @@ __global__ void __launch_bounds__(F_THREADS) finalize_kernel(FinalizeArgs A, uns
             if (A.out_sum) {
                 const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
                 const long long g = A.map ? (long long)A.map[i] : i;
-                A.out_sum[pos] = kval ? A.acc[g] : 0;
+                long long sum = kval ? A.acc[g] : 0;
+                if (A.acc_hi && kval)
+                    sum = (long long)((__int128)A.acc_hi[g] * 4294967296ll + (__int128)(unsigned long long)sum);
+                A.out_sum[pos] = sum;
                 A.out_cnt[pos] = kval ? A.cnt[g] : 0;
             }
         }
@@ -160,13 +172,14 @@ cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *l
     e = cudaMemsetAsync(a.scratch, 0, finalize_scratch_bytes(a.n_rp_max), st);
     if (e != cudaSuccess) return e;
     long long tiles = (a.n_rp_max + F_TILE - 1) / F_TILE;
-    static int cap = 0;
-    if (!cap) {
-        int dev = 0, sms = 148;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        cap = sms * 4;
-    }
+    int cap = 0;
+    e = per_device_setup((const void *)finalize_kernel, 0, &cap, [](int dev, int *v) {
+        int sms = 0;
+        cudaError_t e2 = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        *v = sms * 4;
+        return e2;
+    });
+    if (e != cudaSuccess) return e;
     if (tiles > cap) tiles = cap;
     finalize_kernel<<<(unsigned)tiles, F_THREADS, 0, st>>>(a, (unsigned long long *)((char *)a.scratch + 256),
                                                          (unsigned *)a.scratch);

@@ -21,6 +21,10 @@
 // and any SUM/AVG range is answered in O(1) from them instead of scanned:
 //   pre[p] = AGG(payload[0..p)),  suf[p] = AGG(payload[p..N)),  pre[0] =
 //   suf[N] = identity;  SUM uses pre only (sum[a,b) = pre[b] - pre[a]).
+// '=' MIN/MAX (skew, P:331's hot keys): per-key group aggregates grp[p] =
+// AGG(payload[start of p's key run .. p]) (a segmented scan, built once per
+// index), passed in `pre`: the group [lb, ub) folds to grp[ub - 1] in O(1),
+// so a hot key costs one load per outer tuple instead of its whole run.
 #include <type_traits>
 
 #include "internal.h"
@@ -140,7 +144,8 @@ __global__ void __launch_bounds__(R_THREADS)
 range_short_kernel(const long long *__restrict__ d_nrp, const K *__restrict__ rkeys, const K *__restrict__ skeys,
                    const void *__restrict__ svals_, int N, const K *__restrict__ samp, int M, int stride,
                    const long long *__restrict__ pre, const long long *__restrict__ suf, long long *__restrict__ acc,
-                   long long *__restrict__ cnt, LongItem *__restrict__ list, unsigned *__restrict__ list_n)
+                   long long *__restrict__ cnt, LongItem *__restrict__ list, unsigned *__restrict__ list_n,
+                   const long long *__restrict__ pre_hi, long long *__restrict__ acc_hi)
 {
     using V = typename std::conditional<VB == 8, long long, int>::type;
     const V *svals = (const V *)svals_;
@@ -166,10 +171,18 @@ range_short_kernel(const long long *__restrict__ d_nrp, const K *__restrict__ rk
         if constexpr (AGG == COUNT || AGG == EXISTS || AGG == NOT_EXISTS) {
             cnt[i] = L;
         } else {
+            if constexpr (OP == EQ && (AGG == MIN || AGG == MAX)) {
+                if (pre) {   // '=' MIN/MAX: O(1) from the per-key group aggregates (pre = grp)
+                    acc[i] = L ? pre[ub - 1] : (AGG == MIN ? LLONG_MAX : LLONG_MIN);
+                    cnt[i] = L;
+                    continue;
+                }
+            }
             if (pre && (AGG == SUM || OP != EQ)) {   // O(1) from the prefix / suffix aggregates
                 long long a;
                 if constexpr (AGG == SUM) {
                     a = (pre[b0] - pre[a0]) + (pre[b1] - pre[a1]);
+                    if (pre_hi) acc_hi[i] = (pre_hi[b0] - pre_hi[a0]) + (pre_hi[b1] - pre_hi[a1]);
                 } else if constexpr (OP == NE) {
                     a = AGG == MIN ? min(pre[lb], suf[ub]) : max(pre[lb], suf[ub]);
                 } else if constexpr (OP == GT || OP == GE) {
@@ -234,7 +247,8 @@ range_long_kernel(const void *__restrict__ svals_, int N, const LongItem *__rest
 template <typename K, int VB, int OP, int AGG>
 static void launch_range_t(long long n_rp_max, const long long *d_nrp, const void *rkeys, const void *skeys,
                            const void *svals, long long ns, const long long *pre, const long long *suf,
-                           long long *acc, long long *cnt, void *scratch, cudaStream_t st, long long *launches)
+                           long long *acc, long long *cnt, void *scratch, cudaStream_t st, long long *launches,
+                           const long long *pre_hi, long long *acc_hi)
 {
     unsigned *list_n = (unsigned *)scratch;
     LongItem *list = (LongItem *)((char *)scratch + 256);
@@ -247,17 +261,18 @@ static void launch_range_t(long long n_rp_max, const long long *d_nrp, const voi
         sample_kernel<K><<<(M + 255) / 256, 256, 0, st>>>((const K *)skeys, stride, M, samp);
         ++*launches;
     }
-    static int max_blocks = 0;   // persistent-ish grid: the samples are staged once per CTA
-    if (!max_blocks) {
-        int dev = 0, sms = 148;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        max_blocks = sms * 8;
-    }
+    int max_blocks = 148 * 8;   // persistent-ish grid: the samples are staged once per CTA
+    per_device_setup((const void *)range_short_kernel<K, VB, OP, AGG>, 0, &max_blocks, [](int dev, int *v) {
+        int sms = 0;
+        cudaError_t e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        *v = sms * 8;
+        return e;
+    });
     long long blocks = (n_rp_max + R_THREADS - 1) / R_THREADS;
     if (blocks > max_blocks) blocks = max_blocks;
     range_short_kernel<K, VB, OP, AGG><<<(unsigned)blocks, R_THREADS, 0, st>>>(
-        d_nrp, (const K *)rkeys, (const K *)skeys, svals, N, samp, M, stride, pre, suf, acc, cnt, list, list_n);
+        d_nrp, (const K *)rkeys, (const K *)skeys, svals, N, samp, M, stride, pre, suf, acc, cnt, list, list_n,
+        pre_hi, acc_hi);
     ++*launches;
     if constexpr (AGG != COUNT && AGG != EXISTS && AGG != NOT_EXISTS) {
         range_long_kernel<VB, OP, AGG><<<148 * 8, R_THREADS, 0, st>>>(svals, (int)ns, list, list_n, acc, cnt);
@@ -268,10 +283,11 @@ static void launch_range_t(long long n_rp_max, const long long *d_nrp, const voi
 template <typename K, int VB, int OP>
 static void dispatch_agg(int agg, long long n_rp_max, const long long *d_nrp, const void *rkeys, const void *skeys,
                          const void *svals, long long ns, const long long *pre, const long long *suf, long long *acc,
-                         long long *cnt, void *scratch, cudaStream_t st, long long *launches)
+                         long long *cnt, void *scratch, cudaStream_t st, long long *launches, const long long *pre_hi,
+                         long long *acc_hi)
 {
 #define NG_R(A) launch_range_t<K, VB, OP, A>(n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, \
-                                             launches)
+                                             launches, pre_hi, acc_hi)
     switch (agg) {
     case MIN: NG_R(MIN); break;
     case MAX: NG_R(MAX); break;
@@ -286,10 +302,11 @@ static void dispatch_agg(int agg, long long n_rp_max, const long long *d_nrp, co
 template <typename K, int VB>
 static void dispatch_op(int op, int agg, long long n_rp_max, const long long *d_nrp, const void *rkeys,
                         const void *skeys, const void *svals, long long ns, const long long *pre, const long long *suf,
-                        long long *acc, long long *cnt, void *scratch, cudaStream_t st, long long *launches)
+                        long long *acc, long long *cnt, void *scratch, cudaStream_t st, long long *launches,
+                        const long long *pre_hi, long long *acc_hi)
 {
 #define NG_O(O) dispatch_agg<K, VB, O>(agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, \
-                                       launches)
+                                       launches, pre_hi, acc_hi)
     switch (op) {
     case EQ: NG_O(EQ); break;
     case NE: NG_O(NE); break;
@@ -304,18 +321,21 @@ static void dispatch_op(int op, int agg, long long n_rp_max, const long long *d_
 cudaError_t launch_range_agg(int kb, int vb, int op, int agg, long long n_rp_max, const long long *d_nrp,
                              const void *rkeys, const void *skeys, const void *svals, long long ns,
                              const long long *pre, const long long *suf, long long *acc, long long *cnt,
-                             void *scratch, cudaStream_t st, long long *launches)
+                             void *scratch, cudaStream_t st, long long *launches, const long long *pre_hi,
+                             long long *acc_hi)
 {
     if (n_rp_max <= 0) return cudaSuccess;
+    if (agg != SUM && agg != AVG) pre_hi = nullptr, acc_hi = nullptr;
+    if (!pre_hi || !acc_hi) pre_hi = nullptr, acc_hi = nullptr;
     cudaError_t e = cudaMemsetAsync(scratch, 0, 256, st);
     if (e != cudaSuccess) return e;
     const bool noval = agg == COUNT || agg == EXISTS || agg == NOT_EXISTS;
     if (kb == 4) {
-        if (noval || vb == 4) dispatch_op<uint32_t, 4>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, launches);
-        else dispatch_op<uint32_t, 8>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, launches);
+        if (noval || vb == 4) dispatch_op<uint32_t, 4>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, launches, pre_hi, acc_hi);
+        else dispatch_op<uint32_t, 8>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, launches, pre_hi, acc_hi);
     } else {
-        if (noval || vb == 4) dispatch_op<uint64_t, 4>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, launches);
-        else dispatch_op<uint64_t, 8>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, launches);
+        if (noval || vb == 4) dispatch_op<uint64_t, 4>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, launches, pre_hi, acc_hi);
+        else dispatch_op<uint64_t, 8>(op, agg, n_rp_max, d_nrp, rkeys, skeys, svals, ns, pre, suf, acc, cnt, scratch, st, launches, pre_hi, acc_hi);
     }
     return cudaGetLastError();
 }
@@ -338,14 +358,19 @@ __device__ __forceinline__ long long comb(long long a, long long b)
 template <int AGG>
 constexpr long long ident() { return AGG == MIN ? LLONG_MAX : (AGG == MAX ? LLONG_MIN : 0); }
 
-// element e of the direction's sequence: forward v[e], backward v[N-1-e]
-template <typename V, bool BACK>
+// element e of the direction's sequence: forward v[e], backward v[N-1-e];
+// PART 1 / 2: the low 32-bit half (unsigned) / high half (signed) of the
+// value, for the split prefix sums of 64-bit payloads (exact SUM)
+template <typename V, bool BACK, int PART = 0>
 __device__ __forceinline__ long long elem(const V *v, long long N, long long e)
 {
-    return (long long)v[BACK ? N - 1 - e : e];
+    const long long x = (long long)v[BACK ? N - 1 - e : e];
+    if constexpr (PART == 1) return (long long)(unsigned long long)(unsigned)x;
+    else if constexpr (PART == 2) return x >> 32;
+    else return x;
 }
 
-template <typename V, int AGG, bool BACK>
+template <typename V, int AGG, bool BACK, int PART>
 __global__ void __launch_bounds__(P_THREADS) block_agg_kernel(const V *__restrict__ v, long long N,
                                                               long long *__restrict__ bagg)
 {
@@ -354,7 +379,7 @@ __global__ void __launch_bounds__(P_THREADS) block_agg_kernel(const V *__restric
     long long a = ident<AGG>();
     for (int j = 0; j < P_ITEMS; j++) {
         const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
-        if (e < N) a = comb<AGG>(a, elem<V, BACK>(v, N, e));
+        if (e < N) a = comb<AGG>(a, elem<V, BACK, PART>(v, N, e));
     }
     for (int o = 16; o > 0; o >>= 1) a = comb<AGG>(a, __shfl_xor_sync(FULL, a, o));
     if ((threadIdx.x & 31) == 0) s_w[threadIdx.x >> 5] = a;
@@ -397,7 +422,7 @@ __global__ void __launch_bounds__(1024) block_scan_kernel(long long *__restrict_
     }
 }
 
-template <typename V, int AGG, bool BACK>
+template <typename V, int AGG, bool BACK, int PART>
 __global__ void __launch_bounds__(P_THREADS) block_prefix_kernel(const V *__restrict__ v, long long N,
                                                                  const long long *__restrict__ bpre,
                                                                  long long *__restrict__ out)
@@ -413,7 +438,7 @@ __global__ void __launch_bounds__(P_THREADS) block_prefix_kernel(const V *__rest
     __syncthreads();
     for (int j = 0; j < P_ITEMS; j++) {   // rows of the block in order, 256 at a time
         const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
-        long long incl = e < N ? elem<V, BACK>(v, N, e) : ident<AGG>();
+        long long incl = e < N ? elem<V, BACK, PART>(v, N, e) : ident<AGG>();
         for (int o = 1; o < 32; o <<= 1) {
             const long long y = __shfl_up_sync(FULL, incl, o);
             if (lane >= o) incl = comb<AGG>(incl, y);
@@ -431,29 +456,141 @@ __global__ void __launch_bounds__(P_THREADS) block_prefix_kernel(const V *__rest
     }
 }
 
-template <typename V, int AGG, bool BACK>
+template <typename V, int AGG, bool BACK, int PART = 0>
 static void scan_dir(const void *v, long long N, long long *out, long long *bagg, cudaStream_t st, long long *launches)
 {
     const long long nb = (N + P_BLOCK - 1) / P_BLOCK;
-    block_agg_kernel<V, AGG, BACK><<<(unsigned)nb, P_THREADS, 0, st>>>((const V *)v, N, bagg);
+    block_agg_kernel<V, AGG, BACK, PART><<<(unsigned)nb, P_THREADS, 0, st>>>((const V *)v, N, bagg);
     block_scan_kernel<AGG><<<1, 1024, 0, st>>>(bagg, nb);
-    block_prefix_kernel<V, AGG, BACK><<<(unsigned)nb, P_THREADS, 0, st>>>((const V *)v, N, bagg, out);
+    block_prefix_kernel<V, AGG, BACK, PART><<<(unsigned)nb, P_THREADS, 0, st>>>((const V *)v, N, bagg, out);
     *launches += 3;
 }
 
-size_t index_aux_scratch_bytes(long long n) { return (size_t)((n + P_BLOCK - 1) / P_BLOCK + 1) * 8; }
+size_t index_aux_scratch_bytes(long long n) { return (size_t)((n + P_BLOCK - 1) / P_BLOCK + 1) * 16; }
+
+// ---- per-key group aggregates: segmented inclusive scan over the sorted
+// index, segments = runs of equal keys.  Pairs (f, v): f = a run starts in
+// the span, v = AGG since the span's last run start; combine(earlier, later)
+// = (f_e | f_l, f_l ? v_l : AGG(v_e, v_l)) -- associative, applied in order.
+template <int AGG>
+struct SegPair {
+    long long v;
+    int f;
+};
+template <int AGG>
+__device__ __forceinline__ SegPair<AGG> seg_comb(SegPair<AGG> e, SegPair<AGG> l)
+{
+    return SegPair<AGG>{l.f ? l.v : comb<AGG>(e.v, l.v), e.f | l.f};
+}
+template <int AGG>
+__device__ __forceinline__ SegPair<AGG> warp_seg_scan(SegPair<AGG> x, int lane)
+{
+    for (int o = 1; o < 32; o <<= 1) {
+        SegPair<AGG> y{__shfl_up_sync(FULL, x.v, o), __shfl_up_sync(FULL, x.f, o)};
+        if (lane >= o) x = seg_comb<AGG>(y, x);
+    }
+    return x;
+}
+
+// One block of P_BLOCK sorted (key, payload) rows scanned in order, 256 at a
+// time; WRITE: write grp[e], else only the block's total pair (bagg).
+template <typename K, typename V, int AGG, bool WRITE>
+__global__ void __launch_bounds__(P_THREADS) seg_block_kernel(const K *__restrict__ keys, const V *__restrict__ v,
+                                                              long long N, long long *__restrict__ bv,
+                                                              int *__restrict__ bf, long long *__restrict__ grp)
+{
+    __shared__ long long s_wv[P_THREADS / 32];
+    __shared__ int s_wf[P_THREADS / 32];
+    __shared__ SegPair<AGG> s_carry;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const long long b0 = blockIdx.x * (long long)P_BLOCK;
+    if (threadIdx.x == 0) s_carry = WRITE ? SegPair<AGG>{bv[blockIdx.x], 0} : SegPair<AGG>{ident<AGG>(), 0};
+    __syncthreads();
+    for (int j = 0; j < P_ITEMS; j++) {
+        const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
+        SegPair<AGG> x{ident<AGG>(), 0};
+        if (e < N) x = SegPair<AGG>{(long long)v[e], (e == 0 || keys[e] != keys[e - 1]) ? 1 : 0};
+        const SegPair<AGG> incl = warp_seg_scan<AGG>(x, lane);
+        if (lane == 31) {
+            s_wv[warp] = incl.v;
+            s_wf[warp] = incl.f;
+        }
+        __syncthreads();
+        SegPair<AGG> wpre{ident<AGG>(), 0};
+        for (int w = 0; w < warp; w++) wpre = seg_comb<AGG>(wpre, SegPair<AGG>{s_wv[w], s_wf[w]});
+        const SegPair<AGG> val = seg_comb<AGG>(s_carry, seg_comb<AGG>(wpre, incl));
+        if (WRITE && e < N) grp[e] = val.v;
+        __syncthreads();
+        if (threadIdx.x == P_THREADS - 1) s_carry = val;
+        __syncthreads();
+    }
+    if (!WRITE && threadIdx.x == 0) {
+        bv[blockIdx.x] = s_carry.v;
+        bf[blockIdx.x] = s_carry.f;
+    }
+}
+
+// exclusive scan of the block pairs (one CTA, sequentially: blocks are few)
+template <int AGG>
+__global__ void seg_block_scan_kernel(long long *__restrict__ bv, const int *__restrict__ bf, long long nb)
+{
+    if (threadIdx.x != 0) return;
+    SegPair<AGG> run{ident<AGG>(), 0};
+    for (long long b = 0; b < nb; b++) {
+        const SegPair<AGG> x{bv[b], bf[b]};
+        bv[b] = run.v;
+        run = seg_comb<AGG>(run, x);
+    }
+}
+
+template <typename K, typename V, int AGG>
+static void seg_scan(const void *keys, const void *v, long long N, long long *grp, void *scratch, cudaStream_t st,
+                     long long *launches)
+{
+    const long long nb = (N + P_BLOCK - 1) / P_BLOCK;
+    long long *bv = (long long *)scratch;
+    int *bf = (int *)(bv + nb + 1);
+    seg_block_kernel<K, V, AGG, false><<<(unsigned)nb, P_THREADS, 0, st>>>((const K *)keys, (const V *)v, N, bv, bf,
+                                                                           nullptr);
+    seg_block_scan_kernel<AGG><<<1, 32, 0, st>>>(bv, bf, nb);
+    seg_block_kernel<K, V, AGG, true><<<(unsigned)nb, P_THREADS, 0, st>>>((const K *)keys, (const V *)v, N, bv, bf,
+                                                                          grp);
+    *launches += 3;
+}
+
+cudaError_t launch_index_group_agg(int agg, int kb, int vb, const void *keys, const void *payload, long long n,
+                                   long long *grp, void *scratch, cudaStream_t st, long long *launches)
+{
+    if (n <= 0) return cudaSuccess;
+#define NG_SEG(K_, V_)                                                                             \
+    if (agg == MIN) seg_scan<K_, V_, MIN>(keys, payload, n, grp, scratch, st, launches);           \
+    else seg_scan<K_, V_, MAX>(keys, payload, n, grp, scratch, st, launches);
+    if (kb == 4) {
+        if (vb == 8) { NG_SEG(uint32_t, long long) } else { NG_SEG(uint32_t, int) }
+    } else {
+        if (vb == 8) { NG_SEG(uint64_t, long long) } else { NG_SEG(uint64_t, int) }
+    }
+#undef NG_SEG
+    return cudaGetLastError();
+}
 
 cudaError_t launch_index_aux(int agg, int vb, const void *payload, long long n, long long *pre, long long *suf,
-                             void *scratch, cudaStream_t st, long long *launches)
+                             void *scratch, cudaStream_t st, long long *launches, long long *pre_hi)
 {
     if (n <= 0) {
         const long long id = agg == MIN ? LLONG_MAX : (agg == MAX ? LLONG_MIN : 0);
         cudaError_t e = cudaMemcpyAsync(pre, &id, 8, cudaMemcpyHostToDevice, st);
         if (e == cudaSuccess && suf) e = cudaMemcpyAsync(suf, &id, 8, cudaMemcpyHostToDevice, st);
+        if (e == cudaSuccess && pre_hi) e = cudaMemcpyAsync(pre_hi, &id, 8, cudaMemcpyHostToDevice, st);
         if (e == cudaSuccess) e = cudaStreamSynchronize(st);   // &id is a host stack value
         return e;
     }
     long long *bagg = (long long *)scratch;
+    if (agg == SUM && pre_hi && vb == 8) {   // exact split prefix sums (no int64 wrap anywhere)
+        scan_dir<long long, SUM, false, 1>(payload, n, pre, bagg, st, launches);
+        scan_dir<long long, SUM, false, 2>(payload, n, pre_hi, bagg, st, launches);
+        return cudaGetLastError();
+    }
 #define NG_SCAN(V_)                                                                               \
     if (agg == MIN) {                                                                             \
         scan_dir<V_, MIN, false>(payload, n, pre, bagg, st, launches);                            \

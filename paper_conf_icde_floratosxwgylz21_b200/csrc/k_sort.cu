@@ -426,21 +426,23 @@ static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *
 {
     using Cfg = PassCfg<K, VB, RB>;
     const long long tiles = (n + Cfg::TILE - 1) / Cfg::TILE;
-    static int grid_max = 0;   // resident CTAs (persistent grid), per instantiation
-    if (!grid_max) {
-        cudaError_t e = cudaFuncSetAttribute(onesweep_p_kernel<K, VB, KO, RB>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Cfg::SMEM);
-        if (e != cudaSuccess) return e;
-        int dev = 0, sms = 0, occ = 0;
-        if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
-        if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
-        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, onesweep_p_kernel<K, VB, KO, RB>, S_THREADS,
-                                                               Cfg::SMEM)) != cudaSuccess)
-            return e;
+    int grid_max = 0;   // resident CTAs (persistent grid), per instantiation and device
+    cudaError_t e = per_device_setup((const void *)onesweep_p_kernel<K, VB, KO, RB>, 0, &grid_max,
+                                     [](int dev, int *v) {
+        cudaError_t e1 = cudaFuncSetAttribute(onesweep_p_kernel<K, VB, KO, RB>,
+                                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Cfg::SMEM);
+        if (e1 != cudaSuccess) return e1;
+        int sms = 0, occ = 0;
+        if ((e1 = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e1;
+        if ((e1 = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, onesweep_p_kernel<K, VB, KO, RB>, S_THREADS,
+                                                                Cfg::SMEM)) != cudaSuccess)
+            return e1;
         if (occ < 1) return cudaErrorInvalidConfiguration;
-        grid_max = sms * occ;
-    }
-    cudaError_t e = cudaMemsetAsync(scratch, 0, (size_t)tiles * (1 << RB) * 4 + 256, st);
+        *v = sms * occ;
+        return cudaSuccess;
+    });
+    if (e != cudaSuccess) return e;
+    e = cudaMemsetAsync(scratch, 0, (size_t)tiles * (1 << RB) * 4 + 256, st);
     if (e != cudaSuccess) return e;
     const unsigned grid = (unsigned)(tiles < grid_max ? tiles : grid_max);
     onesweep_p_kernel<K, VB, KO, RB><<<grid, S_THREADS, Cfg::SMEM, st>>>(

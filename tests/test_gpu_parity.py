@@ -306,7 +306,7 @@ def test_error_paths(eng):
         R2 = eng.load_table({"k": np.zeros(2, np.int64), "x": np.zeros(2, np.int64)})
         with pytest.raises(NestGPUError) as ei:
             eng.exec(make_plan("=", "sum", "=", outer_key=["k"], inner_key=["k"], agg_col="v", outer_cmp_col="x"), R2, S2)
-        assert ei.value.code == -5  # OVERFLOW pre-check
+        assert ei.value.code == -5  # OVERFLOW: the group's exact sum (2^64) leaves int64
     finally:
         eng.release(m)
     small = Engine(0, arena_bytes=1 << 20)
@@ -610,3 +610,71 @@ def test_avg_large_int64_payloads(eng, mode):
             ref = oracle.evaluate(t, plan)
             g = run(eng, t, plan, mode, emit_all=True, dtypes=dt)
             assert_parity(g, ref, plan, True, ctx=(mode, corr_op, outer))
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_exact_int64_sums_not_refused(eng, mode):
+    """SUM/AVG over 64-bit payloads where |S| * max|payload| >= 2^63 but every
+    qualifying set's sum fits int64 (pairs (A + x, -A + y) share a key, so
+    every '=' group and every key prefix / suffix holds whole pairs): the
+    engine must return the oracle's exact values, not NESTGPU_ERR_OVERFLOW
+    (reading R5: only a sum that actually leaves int64 is an error).  S rows
+    are shuffled, so unit / tile partial sums of the nested loop are random
+    walks of +-A that a plain int64 accumulator would wrap."""
+    rng = np.random.default_rng(77)
+    pairs = 6007
+    A = (1 << 62) + (1 << 61)
+    keys = np.repeat(np.arange(pairs, dtype=np.int64) * 3, 2)
+    vals = np.empty(2 * pairs, np.int64)
+    vals[0::2] = A + rng.integers(-1000, 1000, pairs)
+    vals[1::2] = -A + rng.integers(-1000, 1000, pairs)
+    perm = rng.permutation(2 * pairs)
+    n_r = 4001
+    t = {"R": {"col1": rng.integers(-5, 3 * pairs + 5, n_r).astype(np.int64),
+               "col2": rng.integers(-3000, 3000, n_r).astype(np.int64)},
+         "S": {"col1": keys[perm], "col2": vals[perm]}}
+    dt = {"R": {"col1": "int64", "col2": "int64"}, "S": {"col1": "int64", "col2": "decimal"}}
+    for corr_op in PLAN_OPS:
+        for agg, outer in (("sum", "<"), ("avg", ">=")):
+            plan = make_plan(corr_op, agg, outer)
+            ref = oracle.evaluate(t, plan)
+            assert_parity(run(eng, t, plan, mode, emit_all=True, dtypes=dt), ref, plan, True,
+                          ctx=("wide", mode, corr_op, agg))
+    # a real overflow (a qualifying set whose sum leaves int64) is still an
+    # error, on both paths, like the oracle's
+    t2 = {"R": {"col1": np.array([10], np.int64), "col2": np.zeros(1, np.int64)},
+          "S": {"col1": np.arange(4, dtype=np.int64), "col2": np.full(4, A, np.int64)}}
+    plan = make_plan(">", "sum", "=")
+    with pytest.raises(oracle.OracleOverflow):
+        oracle.evaluate(t2, plan)
+    with pytest.raises(NestGPUError) as ei:
+        run(eng, t2, plan, mode, emit_all=True, dtypes=dt)
+    assert ei.value.code == -5
+
+
+def test_c2_zipf_full_size_index_no_cache(eng):
+    """C2's Zipf(1.0) variant at full size WITHOUT caching, every aggregate on
+    the index path: '=' MIN/MAX read the per-key group aggregates (O(1) per
+    outer tuple, no hot-key blow-up), the other operators the prefix /
+    suffix aggregates.  Closed form + outer comparison on every row, oracle
+    on sampled rows; the '=' MIN kernel must stay far below the per-tuple
+    fold of the hot keys' runs (sum over keys of |R_k| x |S_k|, ~1e10
+    element visits)."""
+    import time
+    t = query1.config("C2z")
+    rng = np.random.default_rng(4)
+    rows = np.unique(rng.integers(0, 1_000_000, 300))
+    for corr_op in ("=", "!=", ">"):
+        for agg in ("min", "max", "sum", "count"):
+            plan = make_plan(corr_op, agg, "=")
+            t0 = time.perf_counter()
+            g = run(eng, t, plan, "index", emit_all=True)
+            dt = time.perf_counter() - t0
+            valid, value, cnt, s_sum = ind.closed_form(t["R"]["col1"], t["S"]["col1"], t["S"]["col2"], corr_op, agg)
+            assert np.array_equal(g["valid"].astype(bool), valid), (corr_op, agg)
+            assert np.array_equal(g["value"], value), (corr_op, agg)
+            passed = ind.outer_passed(t["R"]["col2"], valid, value, cnt, s_sum, agg, "=")
+            assert np.array_equal(g["passed"].astype(bool), passed), (corr_op, agg)
+            ref = oracle.evaluate(t, plan, rows=rows)
+            assert_parity(g, ref, plan, True, rows=rows, ctx=("zipf nocache", corr_op, agg))
+            assert dt < 5.0, (corr_op, agg, dt)   # load + index + exec + copy-out
