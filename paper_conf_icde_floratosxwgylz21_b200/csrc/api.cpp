@@ -66,6 +66,10 @@ struct IndexRec {
 };
 
 constexpr int PIN_WORDS = 8 * 256 + 64;
+// Pinned staging for small results: exec copies the first rows of every
+// result field into it before its one synchronisation, so a result of at
+// most that many rows reaches the host with no further GPU operation.
+constexpr size_t STAGE_BYTES = 256 << 10;
 constexpr size_t ALIGN = 256;
 
 }  // namespace
@@ -84,6 +88,13 @@ struct nestgpu_ctx {
     std::vector<Column> cols;
     std::vector<IndexRec> idx;
     unsigned *pinned;  // host pinned words for small D2H / H2D
+    char *stage;       // STAGE_BYTES of pinned host memory (results staged by exec)
+    struct {
+        bool ok;
+        const void *ids;        // d_row_ids of the staged result
+        long long rows;         // rows staged per field
+        size_t w8;              // 8-byte fields in the block (2, or 4 with AVG)
+    } staged;
     bool profiling;
     // Ablation knob (NESTGPU_OPT_MALLOC_SCRATCH): scratch comes from
     // cudaMalloc per allocation, freed at the next scratch reset -- the
@@ -165,6 +176,7 @@ size_t align_up(size_t x) { return (x + ALIGN - 1) / ALIGN * ALIGN; }
 void scratch_reset(nestgpu_ctx *c)
 {
     c->hi = c->size;
+    c->staged.ok = false;
     if (!c->mallocs.empty()) {
         cudaStreamSynchronize(c->stream);
         for (void *p : c->mallocs) cudaFree(p);
@@ -374,8 +386,15 @@ nestgpu_status nestgpu_create(int device, void *d_arena, size_t arena_bytes, voi
     c->profiling = false;
     c->malloc_scratch = false;
     c->bnl_shape = 0;
+    c->stage = nullptr;
+    c->staged.ok = false;
     if (cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess ||
         cudaMallocHost((void **)&c->pinned, PIN_WORDS * sizeof(unsigned)) != cudaSuccess) {
+        delete c;
+        return NESTGPU_ERR_CUDA;
+    }
+    if (cudaMallocHost((void **)&c->stage, STAGE_BYTES) != cudaSuccess) {
+        cudaFreeHost(c->pinned);
         delete c;
         return NESTGPU_ERR_CUDA;
     }
@@ -399,6 +418,7 @@ nestgpu_status nestgpu_destroy(nestgpu_ctx *c)
         cudaEventDestroy(c->ev[s][1]);
     }
     cudaFreeHost(c->pinned);
+    cudaFreeHost(c->stage);
     delete c;
     return NESTGPU_OK;
 }
@@ -593,19 +613,24 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     void *tk = salloc(c, (size_t)n * kb), *tv = vb ? salloc(c, (size_t)n * vb) : nullptr;
     void *uk = salloc(c, (size_t)n * kb), *uv = vb ? salloc(c, (size_t)n * vb) : nullptr;
     void *fscr = salloc(c, ng::filter_scratch_bytes(n));
-    void *sscr = salloc(c, ng::sort_scratch_bytes(n));
     unsigned *hist = (unsigned *)salloc(c, 8 * 512 * 4);
     unsigned *dbase = (unsigned *)salloc(c, 8 * 512 * 4);
     long long *dsmall = (long long *)salloc(c, 64);   // [0] |S'|, [2] key AND, [3] key OR
-    if (!tk || !uk || !fscr || !sscr || !hist || !dbase || !dsmall || (vb && (!tv || !uv)))
+    if (!tk || !uk || !fscr || !hist || !dbase || !dsmall || (vb && (!tv || !uv)))
         return fail(c, NESTGPU_ERR_OOM, "arena exhausted building an index over %lld rows", (long long)n);
     long long *d_count = dsmall;
     unsigned long long *keymask = (unsigned long long *)(dsmall + 2);
-    CUDA_TRY(c, cudaMemsetAsync(dsmall, 0, 64, c->stream));
-    CUDA_TRY(c, cudaMemsetAsync(keymask, 0xff, 8, c->stream));   // AND identity
+    {   // one fill kernel instead of a memset per scratch region
+        ng::FillList fl;
+        fl.add(dsmall, 16);
+        fl.add(keymask, 8, 0xff);   // AND identity
+        fl.add(dsmall + 3, 40);
+        fl.add(fscr, ng::filter_zero_bytes(n, false));
+        CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
+    }
     prof_begin(c, 1);
     CUDA_TRY(c, ng::launch_filter(n, ps, ks, fkb, vs, vb, 1, pc ? 1 : 0, nullptr, tk, nullptr, tv, keymask, nullptr,
-                                  fscr, d_count, c->stream, &c->launches));
+                                  fscr, d_count, c->stream, &c->launches, true));
     prof_end(c, 1);
     CUDA_TRY(c, cudaMemcpyAsync(c->pinned, dsmall, 32, cudaMemcpyDeviceToHost, c->stream));
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
@@ -620,9 +645,29 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
         np = 1;
         shifts[0] = 0;
     }
+    // 64-bit keys whose high words all agree (AND == OR there, e.g. Q4's
+    // order keys) travel as 32-bit keys between the first and the last
+    // pass: the first pass drops the high word, the last re-attaches it.
+    const bool narrow = pre_narrow || (kb == 8 && np >= 2 && ((kand ^ kor) >> 32) == 0);
+    const unsigned hi = pre_narrow ? pre_hi : (unsigned)(kand >> 32);
+    // one scratch region per pass, all zeroed with the digit histograms by
+    // one fill kernel
+    void *pscr[8] = {};
+    {
+        ng::FillList fl;
+        fl.add(hist, (size_t)(np > 0 ? np : 1) * (1u << rb) * 4);
+        for (int p = 0; p < np; p++) {
+            const int kin = pre_narrow || (narrow && p > 0) ? 4 : kb;
+            const size_t zb = ng::sort_pass_zero_bytes(nsp, kin, vb, rb);
+            pscr[p] = salloc(c, zb);
+            if (!pscr[p]) return fail(c, NESTGPU_ERR_OOM, "arena exhausted (sort scratch)");
+            fl.add(pscr[p], zb);
+        }
+        CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
+    }
     prof_begin(c, 2);
     CUDA_TRY(c, ng::launch_digit_hist(fkb, tk, nsp, shifts, np, hist, dbase, c->num_sms, c->stream, &c->launches,
-                                      rb));
+                                      rb, true));
 
     IndexRec ix{};
     ix.off = c->lo;
@@ -646,11 +691,6 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
         }
     } else {
         // T -> ... -> P with ping-pong so that the last pass writes P.
-        // 64-bit keys whose high words all agree (AND == OR there, e.g. Q4's
-        // order keys) travel as 32-bit keys between the first and the last
-        // pass: the first pass drops the high word, the last re-attaches it.
-        const bool narrow = pre_narrow || (kb == 8 && np >= 2 && ((kand ^ kor) >> 32) == 0);
-        const unsigned hi = pre_narrow ? pre_hi : (unsigned)(kand >> 32);
         const void *ik = tk, *iv = tv;
         for (int p = 0; p < np; p++) {
             const bool to_final = ((np - 1 - p) % 2) == 0;
@@ -659,7 +699,7 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
             if (ok == ik) { ok = tk; ov = tv; }
             const int kin = pre_narrow || (narrow && p > 0) ? 4 : kb, kout = narrow && p < np - 1 ? 4 : kb;
             CUDA_TRY(c, ng::launch_radix_pass_x(kin, kout, vb, ik, ok, iv, ov, nsp, shifts[p], dbase + p * (1 << rb),
-                                                sscr, hi, c->stream, &c->launches, rb));
+                                                pscr[p], hi, c->stream, &c->launches, rb, true));
             ik = ok;
             iv = ov;
         }
@@ -839,23 +879,29 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     long long *cnt = (long long *)salloc(c, (size_t)nR * 8);
     long long *counts = (long long *)salloc(c, 128);  // [0] |R'| [1] |S'| [2] survivors; [4..5] extreme; [8] overflow
     long long *acc_hi = wide ? (long long *)salloc(c, (size_t)nR * 8) : nullptr;
-    size_t fsz = ng::filter_scratch_bytes(nR > nS ? nR : nS);
-    void *fscr = salloc(c, fsz);
+    // one scratch per filter / finalize (all zeroed up front by one fill kernel)
+    void *fscr = salloc(c, ng::filter_scratch_bytes(nR));
+    void *fscr_s = ix ? nullptr : salloc(c, ng::filter_scratch_bytes(nS));
+    void *fscr_f = salloc(c, ng::finalize_scratch_bytes(nR));
     void *kscr = salloc(c, ix ? ng::range_scratch_bytes(nR) : ng::bnl_scratch_bytes(nR));
-    long long *o_ids = (long long *)salloc(c, (size_t)nR * 8);
-    long long *o_vals = (long long *)salloc(c, (size_t)nR * 8);
-    uint8_t *o_valid = (uint8_t *)salloc(c, (size_t)nR);
-    uint8_t *o_pass = (uint8_t *)salloc(c, (size_t)nR);
-    long long *o_sum = P->agg == NG_AVG ? (long long *)salloc(c, (size_t)nR * 8) : nullptr;
-    long long *o_cnt = P->agg == NG_AVG ? (long long *)salloc(c, (size_t)nR * 8) : nullptr;
+    // result block: ids | values | [AVG sum | AVG nn] | valid | passed, one
+    // allocation so its first rows reach the host in two copies (staging)
+    const bool is_avg = P->agg == NG_AVG;
+    const size_t w8 = is_avg ? 4 : 2;
+    char *rblk = (char *)salloc(c, (size_t)nR * (8 * w8 + 2));
+    long long *o_ids = rblk ? (long long *)rblk : nullptr;
+    long long *o_vals = rblk ? (long long *)(rblk + (size_t)nR * 8) : nullptr;
+    long long *o_sum = rblk && is_avg ? (long long *)(rblk + (size_t)nR * 16) : nullptr;
+    long long *o_cnt = rblk && is_avg ? (long long *)(rblk + (size_t)nR * 24) : nullptr;
+    uint8_t *o_valid = rblk ? (uint8_t *)(rblk + (size_t)nR * 8 * w8) : nullptr;
+    uint8_t *o_pass = rblk ? o_valid + nR : nullptr;
     void *skeys = nullptr, *svals = nullptr;
     if (!ix) {
         skeys = salloc(c, (size_t)nS * kb);
         svals = vb ? salloc(c, (size_t)nS * vb) : nullptr;
     }
-    if (!ids || !rkeys || (ravalid && !rkvalid) || !acc || !cnt || !counts || !fscr || !kscr || !o_ids || !o_vals ||
-        !o_valid || !o_pass || (P->agg == NG_AVG && (!o_sum || !o_cnt)) || (!ix && (!skeys || (vb && !svals))) ||
-        (wide && !acc_hi))
+    if (!ids || !rkeys || (ravalid && !rkvalid) || !acc || !cnt || !counts || !fscr || !fscr_f || !kscr || !rblk ||
+        (!ix && (!fscr_s || !skeys || (vb && !svals))) || (wide && !acc_hi))
         return fail(c, NESTGPU_ERR_OOM, "arena exhausted executing a plan over |R|=%lld |S|=%lld", (long long)nR, (long long)nS);
     // counts: [0] |R'| [1] |S'| [2] survivors [3] distinct keys [4] extreme flags (2 x u32)
     //         [6] AND / [7] OR of the R' keys (dedup sort planning) [8] split-SUM overflow flag
@@ -884,11 +930,27 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     prof_begin(c, 5);
     prof_begin(c, 0);
     ng::ValSrc none{nullptr, nullptr, 0};
-    CUDA_TRY(c, cudaMemsetAsync(counts, 0, 128, c->stream));
-    CUDA_TRY(c, cudaMemsetAsync(rmask, 0xff, 8, c->stream));   // AND identity
-    if (wide && nR > 0) CUDA_TRY(c, cudaMemsetAsync(acc_hi, 0, (size_t)nR * 8, c->stream));
+    {   // every small scratch region of this exec zeroed by ONE kernel
+        ng::FillList fl;
+        fl.add(counts, 48);
+        fl.add(rmask, 8, 0xff);    // [6] AND identity
+        fl.add(counts + 7, 8);     // [7] OR
+        fl.add(counts + 8, 64);
+        fl.add(fscr, ng::filter_zero_bytes(nR, true));
+        if (fscr_s) fl.add(fscr_s, ng::filter_zero_bytes(nS, false));
+        fl.add(fscr_f, ng::finalize_scratch_bytes(nR));
+        fl.add(kscr, ix ? 256 : ng::bnl_scratch_bytes(nR));
+        if (wide) fl.add(acc_hi, (size_t)nR * 8);
+        // the staged rows (copied to the host even when fewer survive):
+        // defined contents for compute-sanitizer's initcheck
+        const long long kr = std::min<long long>(nR, (long long)(STAGE_BYTES / (8 * w8 + 2)));
+        for (size_t f = 0; f < w8; f++) fl.add(rblk + (size_t)nR * 8 * f, (size_t)kr * 8);
+        fl.add(o_valid, (size_t)kr);
+        fl.add(o_pass, (size_t)kr);
+        CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
+    }
     CUDA_TRY(c, ng::launch_filter(nR, ops, rks, kb, none, 0, 0, 0, ids, rkeys, rkvalid, nullptr,
-                                  P->dedup ? rmask : nullptr, nullptr, fscr, d_nrp, c->stream, &c->launches));
+                                  P->dedup ? rmask : nullptr, nullptr, fscr, d_nrp, c->stream, &c->launches, true));
     prof_end(c, 0);
 
     // The keys the subquery kernels evaluate: every R' key, or (dedup) each
@@ -980,21 +1042,21 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         const bool split = wide && pre && P->agg != NG_MIN && P->agg != NG_MAX;
         CUDA_TRY(c, ng::launch_range_agg(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, ix->keys, ix->payload,
                                          ix->n, pre, split ? nullptr : suf, acc, cnt, kscr, c->stream, &c->launches,
-                                         split ? suf : nullptr, split ? acc_hi : nullptr));
+                                         split ? suf : nullptr, split ? acc_hi : nullptr, true));
         prof_end(c, 3);
     } else {
         prof_begin(c, 1);
         ng::ValSrc vs{nullptr, nullptr, 0};
         if (value_agg) { vs.c = ac->d; vs.v = ac->valid; vs.w = vb; }
         CUDA_TRY(c, ng::launch_filter(nS, ips, sks, kb, vs, vb, 1, value_agg ? 1 : 0, nullptr, skeys, nullptr, svals,
-                                      nullptr, value_agg ? extreme : nullptr, fscr, d_nsp, c->stream,
-                                      &c->launches));
+                                      nullptr, value_agg ? extreme : nullptr, fscr_s, d_nsp, c->stream,
+                                      &c->launches, true));
         CUDA_TRY(c, ng::launch_init_partials(n_eval, d_neval, P->agg, acc, cnt, c->stream, &c->launches));
         prof_end(c, 1);
         prof_begin(c, 3);
         CUDA_TRY(c, ng::launch_bnl(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, nS, d_nsp, skeys, svals,
                                    extreme, acc, cnt, kscr, c->num_sms, c->bnl_shape, c->stream, &c->launches,
-                                   wide ? acc_hi : nullptr));
+                                   wide ? acc_hi : nullptr, true));
         prof_end(c, 3);
     }
 
@@ -1026,15 +1088,28 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     fa.out_valid = o_valid;
     fa.out_passed = o_pass;
     fa.out_count = d_out;
-    fa.scratch = fscr;
-    CUDA_TRY(c, ng::launch_finalize(fa, c->stream, &c->launches));
+    fa.scratch = fscr_f;
+    CUDA_TRY(c, ng::launch_finalize(fa, c->stream, &c->launches, true));
     prof_end(c, 4);
     prof_end(c, 5);
     CUDA_TRY(c, cudaMemcpyAsync(c->pinned, counts, 72, cudaMemcpyDeviceToHost, c->stream));
+    // the first rows of every result field, staged on the host before the
+    // one synchronisation (8-byte fields, then the two byte fields)
+    const long long krows = std::min<long long>(nR, (long long)(STAGE_BYTES / (8 * w8 + 2)));
+    if (krows > 0) {
+        CUDA_TRY(c, cudaMemcpy2DAsync(c->stage, (size_t)krows * 8, rblk, (size_t)nR * 8, (size_t)krows * 8, w8,
+                                      cudaMemcpyDeviceToHost, c->stream));
+        CUDA_TRY(c, cudaMemcpy2DAsync(c->stage + (size_t)krows * 8 * w8, (size_t)krows, o_valid, (size_t)nR,
+                                      (size_t)krows, 2, cudaMemcpyDeviceToHost, c->stream));
+    }
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
     long long cnts[9];
     memcpy(cnts, c->pinned, 72);
     if (cnts[8]) return fail(c, NESTGPU_ERR_OVERFLOW, "exec: a SUM exceeds int64 (reading R5)");
+    c->staged.ok = krows > 0;
+    c->staged.ids = o_ids;
+    c->staged.rows = krows;
+    c->staged.w8 = w8;
     out->n_rows = cnts[2];
     out->n_evaluated = P->dedup ? n_distinct : cnts[0];
     out->d_row_ids = (const int64_t *)o_ids;
@@ -1053,6 +1128,20 @@ nestgpu_status nestgpu_result_to_host(nestgpu_ctx *c, const nestgpu_result *r, i
     if (cap < r->n_rows) return fail(c, NESTGPU_ERR_BUFFER, "result_to_host: %lld rows, buffer holds %lld", (long long)r->n_rows, (long long)cap);
     cudaSetDevice(c->device);
     const size_t n = (size_t)r->n_rows;
+    if (c->staged.ok && r->d_row_ids == c->staged.ids && r->n_rows <= c->staged.rows) {
+        // staged by exec: host copies only, no GPU operation
+        const size_t k = (size_t)c->staged.rows;
+        const char *s = c->stage;
+        if (n) {
+            if (row_ids) memcpy(row_ids, s, n * 8);
+            if (values) memcpy(values, s + k * 8, n * 8);
+            if (avg_sum && r->d_avg_sum) memcpy(avg_sum, s + k * 16, n * 8);
+            if (avg_cnt && r->d_avg_cnt) memcpy(avg_cnt, s + k * 24, n * 8);
+            if (valid) memcpy(valid, s + k * 8 * c->staged.w8, n);
+            if (passed) memcpy(passed, s + k * 8 * c->staged.w8 + k, n);
+        }
+        return NESTGPU_OK;
+    }
     if (n) {
         if (row_ids) CUDA_TRY(c, cudaMemcpyAsync(row_ids, r->d_row_ids, n * 8, cudaMemcpyDeviceToHost, c->stream));
         if (values) CUDA_TRY(c, cudaMemcpyAsync(values, r->d_values, n * 8, cudaMemcpyDeviceToHost, c->stream));

@@ -52,6 +52,33 @@ cudaError_t launch_fill_runs(void *out, int w, long long n, long long div, long 
 
 // Every launcher returns the cudaError_t of its launch(es) and bumps *launches
 // by the number of kernels it launched.
+//
+// Small scratch regions (counters, look-back status words, tile offsets) of
+// one public call are zeroed by ONE fill kernel before its first launch
+// instead of one cudaMemsetAsync per launcher (each a separate GPU operation
+// on the latency path of small queries); launchers given prezeroed = true
+// skip their own memsets -- the caller has put every region they need
+// (see the *_zero_bytes helpers) on the fill list.
+struct FillList {
+    int n = 0;
+    void *p[24];
+    unsigned long long bytes[24];
+    unsigned char val[24];
+    bool add(void *ptr, size_t b, unsigned char v = 0)
+    {
+        if (!ptr || !b) return true;
+        if (n >= 24) return false;
+        p[n] = ptr;
+        bytes[n] = b;
+        val[n] = v;
+        n++;
+        return true;
+    }
+};
+cudaError_t launch_fill(const FillList &f, cudaStream_t st, long long *launches);
+// scratch bytes a prezeroed launcher expects zero (regions start at scratch)
+size_t filter_zero_bytes(long long n, bool ordered);
+size_t finalize_scratch_bytes(long long n);
 
 // a2 / a3: filter rows [0, n) by `preds`, compact survivors in row order.
 //   out_ids    : int32 row ids of survivors (nullable)
@@ -71,13 +98,14 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
                           const ValSrc &val, int vb, int drop_null_key, int drop_null_val,
                           int *out_ids, void *out_keys, uint8_t *out_kvalid, void *out_vals,
                           unsigned long long *keymask, unsigned *extreme, void *scratch,
-                          long long *out_count, cudaStream_t st, long long *launches);
+                          long long *out_count, cudaStream_t st, long long *launches, bool prezeroed = false);
 
 // a4: histograms of the digits at `shifts` (np of them) over n encoded keys,
 // and their exclusive scans into digit_base[np][256].
 //   rb: digit bits (8 or 9); hist / digit_base hold np * 2^rb words
 cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *shifts, int np, unsigned *hist,
-                              unsigned *digit_base, int num_sms, cudaStream_t st, long long *launches, int rb = 8);
+                              unsigned *digit_base, int num_sms, cudaStream_t st, long long *launches, int rb = 8,
+                              bool prezeroed = false);
 
 // a4: one stable LSD radix pass on the rb-bit digit (rb = 8 or 9) at bit
 // `shift` of the encoded keys.
@@ -90,7 +118,10 @@ cudaError_t launch_radix_pass(int kb, int vb, const void *kin, void *kout, const
 // (all keys must share it), 4 -> 8 re-attaches `hi` as the high word.
 cudaError_t launch_radix_pass_x(int kb_in, int kb_out, int vb, const void *kin, void *kout, const void *vin,
                                 void *vout, long long n, int shift, const unsigned *digit_base, void *scratch,
-                                unsigned hi, cudaStream_t st, long long *launches, int rb = 8);
+                                unsigned hi, cudaStream_t st, long long *launches, int rb = 8,
+                                bool prezeroed = false);
+// scratch bytes of one radix pass that must be zero (per-tile digit counts + counter)
+size_t sort_pass_zero_bytes(long long n, int kb, int vb, int rb);
 
 // Partial aggregates per R' tuple: acc (int64) + cnt (int64); identity init.
 // n: host upper bound (grid size); d_n: the actual count (device)
@@ -111,7 +142,7 @@ cudaError_t launch_range_agg(int kb, int vb, int op, int agg, long long n_rp_max
                              const void *rkeys, const void *skeys, const void *svals, long long ns,
                              const long long *pre, const long long *suf, long long *acc, long long *cnt,
                              void *scratch, cudaStream_t st, long long *launches,
-                             const long long *pre_hi = nullptr, long long *acc_hi = nullptr);
+                             const long long *pre_hi = nullptr, long long *acc_hi = nullptr, bool prezeroed = false);
 
 // Index-pruned evaluation (NEXT 3): pre[0..n] / suf[0..n] aggregates (MIN,
 // MAX: both; SUM: pre only) of the co-sorted payload of an index.
@@ -131,7 +162,7 @@ cudaError_t launch_bnl(int kb, int vb, int op, int agg, long long n_rp_max, cons
                        const void *rkeys, long long ns_max, const long long *d_nsp, const void *skeys,
                        const void *svals, const unsigned *extreme, long long *acc, long long *cnt,
                        void *scratch, int num_sms, int shape /* 0 auto, 1 full, 2 warp-split */,
-                       cudaStream_t st, long long *launches, long long *acc_hi = nullptr);
+                       cudaStream_t st, long long *launches, long long *acc_hi = nullptr, bool prezeroed = false);
 //   acc_hi (SUM/AVG of 64-bit payloads, nullable, zeroed by the caller): exact
 //   split accumulation -- acc += low 32-bit halves, acc_hi += high halves.
 
@@ -164,7 +195,7 @@ struct FinalizeArgs {
     long long *out_count;
     void *scratch;           // filter_scratch_bytes(n_rp_max)
 };
-cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *launches);
+cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *launches, bool prezeroed = false);
 
 // out[i] = src[ids[i] - base] (w = 4 or 8 bytes per value).
 cudaError_t launch_gather(int w, const void *src, const long long *ids, long long n, long long base, void *out,

@@ -9,7 +9,7 @@ size_t bnl_scratch_bytes(long long n_rp_max) { return 256 + (size_t)((n_rp_max +
 cudaError_t launch_bnl(int kb, int vb, int op, int agg, long long n_rp_max, const long long *d_nrp, const void *rkeys,
                        long long ns_max, const long long *d_nsp, const void *skeys, const void *svals,
                        const unsigned *extreme, long long *acc, long long *cnt, void *scratch, int num_sms,
-                       int shape, cudaStream_t st, long long *launches, long long *acc_hi)
+                       int shape, cudaStream_t st, long long *launches, long long *acc_hi, bool prezeroed)
 {
     if (n_rp_max <= 0 || ns_max <= 0) return cudaSuccess;
     BnlArgs a{};
@@ -21,6 +21,7 @@ cudaError_t launch_bnl(int kb, int vb, int op, int agg, long long n_rp_max, cons
     a.extreme = extreme;
     a.one = 1u;
     a.shape = shape;
+    a.prezeroed = prezeroed;
     a.acc = acc;
     a.cnt = cnt;
     a.acc_hi = (agg == SUM || agg == AVG) && vb == 8 ? acc_hi : nullptr;

@@ -67,6 +67,7 @@ struct BnlArgs {
     unsigned *rb_done;         // EXISTS: per R block, set once every tuple of the block found a match
     long long target_units;    // work units to aim for (grid x 16)
     int shape;                 // R-block shape: 0 automatic, 1 full, 2 warp-split (test knob)
+    bool prezeroed;            // scratch already zeroed by the caller's fill list (host side only)
 };
 
 template <typename K, int VB>

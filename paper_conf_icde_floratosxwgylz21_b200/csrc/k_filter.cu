@@ -23,10 +23,12 @@
 // which all keys agree need no sort pass) and flags payloads equal to the
 // MIN/MAX identity.
 #include <climits>
+#include <cstdlib>
 #include <cstring>
 #include <type_traits>
 
 #include "internal.h"
+#include "scan.cuh"
 
 namespace ng {
 
@@ -361,6 +363,157 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
     }
 }
 
+// ------------------------------------------------------------------ ordered R'
+// One pass (P:235's scan -> 0-1 vector -> prefix sum -> materialize fused):
+// a tile stages ONLY its predicate columns (cp.async.bulk, single buffer:
+// occupancy supplies the overlap, and no tile id is taken before its data is
+// processed, so no successor waits on a prefetched tile), evaluates them,
+// gets its output offset from the CTA-wide decoupled look-back (scan.cuh),
+// then loads the key (+ validity) of its SURVIVORS straight from global
+// memory and writes ids / encoded keys / key-valid in row order.  A
+// selective outer predicate (SF10 Q4: 3.8 %) thus reads the key column only
+// where rows survive, instead of staging it for every row.
+template <int KB, int ITEMS>
+__global__ void __launch_bounds__(T_THREADS)
+filter_rp_kernel(long long n, SrcCols sc, TPlan tp, KeySrc ks, int *__restrict__ out_ids, void *__restrict__ out_keys,
+                 uint8_t *__restrict__ out_kvalid, unsigned long long *__restrict__ keymask,
+                 unsigned long long *__restrict__ status, unsigned *__restrict__ counter,
+                 long long *__restrict__ out_count)
+{
+    using K = typename std::conditional<KB == 8, uint64_t, uint32_t>::type;
+    constexpr int TILE = T_THREADS * ITEMS;
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ __align__(8) unsigned long long bar;
+    __shared__ unsigned s_cnt[ITEMS][T_WARPS];
+    __shared__ long long s_tile;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const long long num_tiles = (n + TILE - 1) / TILE;
+    if (tid == 0) {
+        mbar_init(&bar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    unsigned phase = 0u;
+    unsigned long long kand = ~0ull, kor = 0ull;
+    for (;;) {
+        if (tid == 0) {
+            const long long t = atomicAdd(counter, 1u);
+            s_tile = t;
+            if (t < num_tiles && sc.n > 0) {
+                const long long rows = min((long long)TILE, n - t * TILE);
+                unsigned total = 0;
+                for (int c = 0; c < sc.n; c++) total += ((unsigned)rows * sc.w[c] + 15u) & ~15u;
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_expect_tx(&bar, total);
+                for (int c = 0; c < sc.n; c++)
+                    bulk_g2s(smem + sc.off[c], (const char *)sc.ptr[c] + t * TILE * sc.w[c],
+                             ((unsigned)rows * sc.w[c] + 15u) & ~15u, &bar);
+            }
+        }
+        __syncthreads();
+        const long long tile = s_tile;
+        if (tile >= num_tiles) break;
+        if (sc.n > 0) {
+            mbar_wait(&bar, phase);
+            phase ^= 1u;
+        }
+        const long long base = tile * TILE;
+        const long long rows = min((long long)TILE, n - base);
+        unsigned live = 0;
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++)
+            if (j * T_THREADS + tid < rows) live |= 1u << j;
+        for (int k = 0; k < tp.n_preds; k++) {   // local predicates, NULL is not TRUE (R2)
+            const TPred p = tp.p[k];
+            live = nonnull<ITEMS>(smem, p.xv, live, tid);
+            live = nonnull<ITEMS>(smem, p.yv, live, tid);
+#define NG_CMP_ALL(X, Y)                                                                              \
+            switch (p.op) {                                                                           \
+            case EQ: live &= cmp_items<ITEMS, EQ>(X, Y); break;                                       \
+            case NE: live &= cmp_items<ITEMS, NE>(X, Y); break;                                       \
+            case LT: live &= cmp_items<ITEMS, LT>(X, Y); break;                                       \
+            case LE: live &= cmp_items<ITEMS, LE>(X, Y); break;                                       \
+            case GT: live &= cmp_items<ITEMS, GT>(X, Y); break;                                       \
+            default: live &= cmp_items<ITEMS, GE>(X, Y); break;                                       \
+            }
+            if (p.x.w == 4 && (p.y.off >= 0 ? p.y.w == 4 : p.lit == (long long)(int)p.lit)) {
+                int x[ITEMS], y[ITEMS];
+                const int *xa = reinterpret_cast<const int *>(smem + p.x.off);
+#pragma unroll
+                for (int j = 0; j < ITEMS; j++) x[j] = xa[j * T_THREADS + tid];
+                if (p.y.off >= 0) {
+                    const int *ya = reinterpret_cast<const int *>(smem + p.y.off);
+#pragma unroll
+                    for (int j = 0; j < ITEMS; j++) y[j] = ya[j * T_THREADS + tid];
+                } else {
+#pragma unroll
+                    for (int j = 0; j < ITEMS; j++) y[j] = (int)p.lit;
+                }
+                NG_CMP_ALL(x, y)
+            } else {
+                long long x[ITEMS], y[ITEMS];
+                load_items<ITEMS>(smem, p.x, tid, x);
+                if (p.y.off >= 0) {
+                    load_items<ITEMS>(smem, p.y, tid, y);
+                } else {
+#pragma unroll
+                    for (int j = 0; j < ITEMS; j++) y[j] = p.lit;
+                }
+                NG_CMP_ALL(x, y)
+            }
+#undef NG_CMP_ALL
+        }
+        unsigned rank[ITEMS];
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            const unsigned m = __ballot_sync(FULL, live >> j & 1u);
+            if (lane == 0) s_cnt[j][warp] = __popc(m);
+            rank[j] = __popc(m & lanemask_lt());
+        }
+        // survivors' keys from global memory (issued before the look-back
+        // so their latency overlaps it)
+        K key[ITEMS];
+        unsigned kv = live;
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            key[j] = 0;
+            if (!(live >> j & 1u)) continue;
+            const long long row = base + j * T_THREADS + tid;
+            if (ks.n_key == 2) {
+                key[j] = (K)(((uint64_t)enc32(__ldg((const int *)ks.c0 + row)) << 32) |
+                             enc32(__ldg((const int *)ks.c1 + row)));
+            } else if (ks.w0 == 4) {
+                const int x = __ldg((const int *)ks.c0 + row);
+                key[j] = KB == 4 ? (K)enc32(x) : (K)enc64((long long)x);
+            } else {
+                key[j] = (K)enc64(__ldg((const long long *)ks.c0 + row));
+            }
+            if ((ks.v0 && !__ldg(ks.v0 + row)) || (ks.v1 && !__ldg(ks.v1 + row))) kv &= ~(1u << j);
+        }
+        const unsigned long long tb = tile_offsets<ITEMS, T_THREADS>(s_cnt, status, tile, num_tiles, out_count);
+#pragma unroll
+        for (int j = 0; j < ITEMS; j++) {
+            if (!(live >> j & 1u)) continue;
+            const long long pos = (long long)tb + s_cnt[j][warp] + rank[j];
+            out_ids[pos] = (int)(base + j * T_THREADS + tid);
+            if (out_keys) ((K *)out_keys)[pos] = key[j];
+            if (out_kvalid) out_kvalid[pos] = (kv >> j) & 1u;
+            kand &= (unsigned long long)key[j];
+            kor |= (unsigned long long)key[j];
+        }
+        __syncthreads();   // the stage and s_cnt are reused by the next tile
+    }
+    if (keymask) {   // bits shared by every survivor key (dedup sort planning)
+        const unsigned alo = __reduce_and_sync(FULL, (unsigned)kand);
+        const unsigned ahi = __reduce_and_sync(FULL, (unsigned)(kand >> 32));
+        const unsigned olo = __reduce_or_sync(FULL, (unsigned)kor);
+        const unsigned ohi = __reduce_or_sync(FULL, (unsigned)(kor >> 32));
+        if (lane == 0) {
+            atomicAnd(&keymask[0], ((unsigned long long)ahi << 32) | alo);
+            atomicOr(&keymask[1], ((unsigned long long)ohi << 32) | olo);
+        }
+    }
+}
+
 // ------------------------------------------------------------------ host side
 // Exclusive scan of the per-tile counts (ordered mode): one CTA, chunks of 1024.
 __global__ void __launch_bounds__(1024) tile_scan_kernel(const unsigned *__restrict__ cnt, long long tiles,
@@ -488,6 +641,103 @@ cudaError_t dispatch(int k, int v, int items, long long n, const SrcCols &sc, co
 
 size_t filter_scratch_bytes(long long n) { return 1024 + 256 + (size_t)(n / T_THREADS + 2) * 12; }
 
+// counter words + (ordered one-pass) the look-back status of every tile --
+// tiles of at least T_THREADS rows, so n / T_THREADS + 1 words bound it
+size_t filter_zero_bytes(long long n, bool ordered)
+{
+    return 1024 + (ordered ? (size_t)(n / T_THREADS + 1) * 8 : 0);
+}
+
+// ---- one kernel filling a list of small regions (FillList)
+__global__ void fill_list_kernel(FillList f)
+{
+    for (int r = 0; r < f.n; r++) {
+        unsigned char *p = (unsigned char *)f.p[r];
+        const unsigned long long b = f.bytes[r];
+        const unsigned v = f.val[r] * 0x01010101u;
+        // aligned 16-B body, byte head / tail
+        const unsigned long long head = (16 - ((unsigned long long)p & 15)) & 15;
+        const unsigned long long h = head < b ? head : b;
+        const unsigned long long body = (b - h) / 16;
+        const long long t = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+        const long long nt = (long long)gridDim.x * blockDim.x;
+        for (long long i = t; i < (long long)h; i += nt) p[i] = (unsigned char)v;
+        uint4 *q = (uint4 *)(p + h);
+        for (long long i = t; i < (long long)body; i += nt) q[i] = make_uint4(v, v, v, v);
+        for (long long i = (long long)(h + body * 16) + t; i < (long long)b; i += nt) p[i] = (unsigned char)v;
+    }
+}
+
+cudaError_t launch_fill(const FillList &f, cudaStream_t st, long long *launches)
+{
+    if (f.n == 0) return cudaSuccess;
+    unsigned long long mx = 0;
+    for (int r = 0; r < f.n; r++) mx = f.bytes[r] > mx ? f.bytes[r] : mx;
+    long long blocks = (long long)((mx / 16 + 255) / 256);
+    if (blocks < 1) blocks = 1;
+    if (blocks > 148 * 4) blocks = 148 * 4;
+    fill_list_kernel<<<(unsigned)blocks, 256, 0, st>>>(f);
+    ++*launches;
+    return cudaGetLastError();
+}
+
+namespace {
+// NESTGPU_FILTER_TWO_PASS=1: the round-1 count + scan + write R' filter
+// (kept for side-by-side measurement)
+bool getenv_two_pass()
+{
+    static const bool v = [] {
+        const char *s = getenv("NESTGPU_FILTER_TWO_PASS");
+        return s && s[0] == '1';
+    }();
+    return v;
+}
+
+template <int KB, int ITEMS>
+cudaError_t launch_rp_t(long long n, const SrcCols &sc, const TPlan &tp, const KeySrc &ks, int *ids, void *keys,
+                        uint8_t *kvalid, unsigned long long *keymask, unsigned long long *status, unsigned *counter,
+                        long long *count, int num_sms, cudaStream_t st)
+{
+    auto kern = filter_rp_kernel<KB, ITEMS>;
+    const int smem = sc.n > 0 ? sc.stage_bytes : 0;
+    int occ = 0;
+    cudaError_t e0 = per_device_setup((const void *)kern, smem, &occ, [&](int, int *v) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, STAGE_MAX);
+        if (e != cudaSuccess) return e;
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(v, kern, T_THREADS, smem);
+    });
+    if (e0 != cudaSuccess) return e0;
+    const long long tiles = (n + T_THREADS * ITEMS - 1) / (T_THREADS * ITEMS);
+    long long grid = (long long)num_sms * (occ > 0 ? occ : 1);
+    if (grid > tiles) grid = tiles;
+    kern<<<(unsigned)grid, T_THREADS, smem, st>>>(n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count);
+    return cudaGetLastError();
+}
+
+template <int KB>
+cudaError_t launch_rp_items(int items, long long n, const SrcCols &sc, const TPlan &tp, const KeySrc &ks, int *ids,
+                            void *keys, uint8_t *kvalid, unsigned long long *keymask, unsigned long long *status,
+                            unsigned *counter, long long *count, int num_sms, cudaStream_t st)
+{
+    switch (items) {
+    case 16: return launch_rp_t<KB, 16>(n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
+    case 8: return launch_rp_t<KB, 8>(n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
+    case 4: return launch_rp_t<KB, 4>(n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
+    case 2: return launch_rp_t<KB, 2>(n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
+    default: return launch_rp_t<KB, 1>(n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
+    }
+}
+
+cudaError_t launch_rp(int kb, int items, long long n, const SrcCols &sc, const TPlan &tp, const KeySrc &ks, int *ids,
+                      void *keys, uint8_t *kvalid, unsigned long long *keymask, unsigned long long *status,
+                      unsigned *counter, long long *count, int num_sms, cudaStream_t st)
+{
+    if (kb == 8)
+        return launch_rp_items<8>(items, n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
+    return launch_rp_items<4>(items, n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
+}
+}  // namespace
+
 // Source indices of a plan (host side), resolved into stage offsets by
 // resolve() once the tile size / stage layout is known.
 struct SrcPlan {
@@ -519,9 +769,9 @@ static void resolve(const SrcCols &sc, const SrcPlan &sp, TPlan &tp)
 cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, int kb, const ValSrc &val, int vb,
                           int drop_null_key, int drop_null_val, int *out_ids, void *out_keys, uint8_t *out_kvalid,
                           void *out_vals, unsigned long long *keymask, unsigned *extreme, void *scratch,
-                          long long *out_count, cudaStream_t st, long long *launches)
+                          long long *out_count, cudaStream_t st, long long *launches, bool prezeroed)
 {
-    cudaError_t e = cudaMemsetAsync(out_count, 0, sizeof(long long), st);
+    cudaError_t e = prezeroed ? cudaSuccess : cudaMemsetAsync(out_count, 0, sizeof(long long), st);
     if (e != cudaSuccess || n <= 0) return e;
     // the column segments a tile needs, deduplicated
     SrcCols sc;
@@ -561,13 +811,39 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
     const int items = layout(sc, 16);
     if (!items) return cudaErrorInvalidValue;
     resolve(sc, sp, tp);
-    e = cudaMemsetAsync(scratch, 0, 1024, st);
-    if (e != cudaSuccess) return e;
+    const bool one_pass = out_ids && !out_vals && !extreme && !drop_null_key && !drop_null_val && k &&
+                          !getenv_two_pass();
+    if (!prezeroed || (out_ids && !one_pass)) {
+        e = cudaMemsetAsync(scratch, 0, 1024, st);
+        if (e != cudaSuccess) return e;
+    }
     int dev = 0, num_sms = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&num_sms, cudaDevAttrMultiProcessorCount, dev);
     FilterOut o{out_ids, out_keys, out_kvalid, out_vals, keymask, extreme, nullptr, nullptr,
                 (unsigned *)scratch, out_count};
+    if (one_pass) {
+        // ordered R': one pass with the decoupled look-back (predicate
+        // columns staged; survivors' keys gathered)
+        SrcCols sc1 = sc;
+        sc1.n = n_pred_src;   // predicate columns come first in the source list
+        const int it1 = layout(sc1, 16);
+        if (!it1) return cudaErrorInvalidValue;
+        SrcPlan sp1 = sp;
+        sp1.key0 = sp1.key0v = sp1.key1 = sp1.key1v = sp1.val = sp1.valv = -1;
+        TPlan tp1 = tp;
+        resolve(sc1, sp1, tp1);
+        const long long tiles = (n + T_THREADS * it1 - 1) / (T_THREADS * it1);
+        unsigned long long *status = (unsigned long long *)((char *)scratch + 1024);
+        if (!prezeroed) {
+            e = cudaMemsetAsync((char *)scratch + 1024, 0, (size_t)tiles * 8, st);
+            if (e != cudaSuccess) return e;
+        }
+        e = launch_rp(k, it1, n, sc1, tp1, key, out_ids, out_keys, out_kvalid, keymask, status, (unsigned *)scratch,
+                      out_count, num_sms, st);
+        ++*launches;
+        return e;
+    }
     if (out_ids) {
         // Ordered (R'): pass 1 counts survivors per tile reading only the
         // predicate columns (same tile size as pass 2), then an exclusive scan.

@@ -165,12 +165,14 @@ __global__ void __launch_bounds__(F_THREADS) finalize_kernel(FinalizeArgs A, uns
     }
 }
 
-cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *launches)
+cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *launches, bool prezeroed)
 {
-    cudaError_t e = cudaMemsetAsync(a.out_count, 0, sizeof(long long), st);
+    cudaError_t e = prezeroed ? cudaSuccess : cudaMemsetAsync(a.out_count, 0, sizeof(long long), st);
     if (e != cudaSuccess || a.n_rp_max <= 0) return e;
-    e = cudaMemsetAsync(a.scratch, 0, finalize_scratch_bytes(a.n_rp_max), st);
-    if (e != cudaSuccess) return e;
+    if (!prezeroed) {
+        e = cudaMemsetAsync(a.scratch, 0, finalize_scratch_bytes(a.n_rp_max), st);
+        if (e != cudaSuccess) return e;
+    }
     long long tiles = (a.n_rp_max + F_TILE - 1) / F_TILE;
     int cap = 0;
     e = per_device_setup((const void *)finalize_kernel, 0, &cap, [](int dev, int *v) {

@@ -322,12 +322,12 @@ cudaError_t launch_range_agg(int kb, int vb, int op, int agg, long long n_rp_max
                              const void *rkeys, const void *skeys, const void *svals, long long ns,
                              const long long *pre, const long long *suf, long long *acc, long long *cnt,
                              void *scratch, cudaStream_t st, long long *launches, const long long *pre_hi,
-                             long long *acc_hi)
+                             long long *acc_hi, bool prezeroed)
 {
     if (n_rp_max <= 0) return cudaSuccess;
     if (agg != SUM && agg != AVG) pre_hi = nullptr, acc_hi = nullptr;
     if (!pre_hi || !acc_hi) pre_hi = nullptr, acc_hi = nullptr;
-    cudaError_t e = cudaMemsetAsync(scratch, 0, 256, st);
+    cudaError_t e = prezeroed ? cudaSuccess : cudaMemsetAsync(scratch, 0, 256, st);
     if (e != cudaSuccess) return e;
     const bool noval = agg == COUNT || agg == EXISTS || agg == NOT_EXISTS;
     if (kb == 4) {

@@ -123,6 +123,23 @@ struct PassCfg {
     static constexpr size_t SMEM = NG_S_NBUF * (size_t)BUF;
 };
 
+template <typename K, int VB, int RB>
+static size_t pass_zero_t(long long n)
+{
+    using Cfg = PassCfg<K, VB, RB>;
+    const long long tiles = (n + Cfg::TILE - 1) / Cfg::TILE;
+    return (size_t)tiles * (1 << RB) * 4 + 256;
+}
+
+// kb: the key width the pass READS (the tile size follows the items read)
+size_t sort_pass_zero_bytes(long long n, int kb, int vb, int rb)
+{
+#define NG_PZ(K_, RB_) (vb == 0 ? pass_zero_t<K_, 0, RB_>(n) : (vb == 4 ? pass_zero_t<K_, 4, RB_>(n) : pass_zero_t<K_, 8, RB_>(n)))
+    if (kb == 4) return rb == 8 ? NG_PZ(uint32_t, 8) : NG_PZ(uint32_t, 9);
+    return rb == 8 ? NG_PZ(uint64_t, 8) : NG_PZ(uint64_t, 9);
+#undef NG_PZ
+}
+
 template <typename K, int VB, typename KO, int RB>
 __global__ void __launch_bounds__(S_THREADS, NG_S_PMINB)
 onesweep_p_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *__restrict__ vin_,
@@ -396,11 +413,12 @@ __global__ void __launch_bounds__(512) digit_scan_kernel(const unsigned *__restr
 }
 
 cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *shifts, int np, unsigned *hist,
-                              unsigned *digit_base, int num_sms, cudaStream_t st, long long *launches, int rb)
+                              unsigned *digit_base, int num_sms, cudaStream_t st, long long *launches, int rb,
+                              bool prezeroed)
 {
     if (np <= 0) return cudaSuccess;
     const int nb = 1 << rb;
-    cudaError_t e = cudaMemsetAsync(hist, 0, (size_t)np * nb * 4, st);
+    cudaError_t e = prezeroed ? cudaSuccess : cudaMemsetAsync(hist, 0, (size_t)np * nb * 4, st);
     if (e != cudaSuccess) return e;
     DigitList dl{};
     dl.n = np;
@@ -422,7 +440,7 @@ cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *
 
 template <typename K, int VB, typename KO, int RB>
 static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *vout, long long n, int shift,
-                            const unsigned *digit_base, void *scratch, unsigned hi, cudaStream_t st)
+                            const unsigned *digit_base, void *scratch, unsigned hi, cudaStream_t st, bool prezeroed)
 {
     using Cfg = PassCfg<K, VB, RB>;
     const long long tiles = (n + Cfg::TILE - 1) / Cfg::TILE;
@@ -442,8 +460,10 @@ static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *
         return cudaSuccess;
     });
     if (e != cudaSuccess) return e;
-    e = cudaMemsetAsync(scratch, 0, (size_t)tiles * (1 << RB) * 4 + 256, st);
-    if (e != cudaSuccess) return e;
+    if (!prezeroed) {
+        e = cudaMemsetAsync(scratch, 0, (size_t)tiles * (1 << RB) * 4 + 256, st);
+        if (e != cudaSuccess) return e;
+    }
     const unsigned grid = (unsigned)(tiles < grid_max ? tiles : grid_max);
     onesweep_p_kernel<K, VB, KO, RB><<<grid, S_THREADS, Cfg::SMEM, st>>>(
         (const K *)kin, (KO *)kout, vin, vout, n, shift, digit_base, (unsigned *)((char *)scratch + 256),
@@ -453,38 +473,38 @@ static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *
 
 template <typename K, typename KO, int RB>
 static cudaError_t run_pass_v(int vb, const void *kin, void *kout, const void *vin, void *vout, long long n, int shift,
-                              const unsigned *digit_base, void *scratch, unsigned hi, cudaStream_t st)
+                              const unsigned *digit_base, void *scratch, unsigned hi, cudaStream_t st, bool pz)
 {
-    if (vb == 0) return run_pass<K, 0, KO, RB>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
-    if (vb == 4) return run_pass<K, 4, KO, RB>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
-    return run_pass<K, 8, KO, RB>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
+    if (vb == 0) return run_pass<K, 0, KO, RB>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
+    if (vb == 4) return run_pass<K, 4, KO, RB>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
+    return run_pass<K, 8, KO, RB>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
 }
 
 template <int RB>
 static cudaError_t run_pass_kk(int kb_in, int kb_out, int vb, const void *kin, void *kout, const void *vin,
                                void *vout, long long n, int shift, const unsigned *digit_base, void *scratch,
-                               unsigned hi, cudaStream_t st)
+                               unsigned hi, cudaStream_t st, bool pz)
 {
     if (kb_in == 4 && kb_out == 4)
-        return run_pass_v<uint32_t, uint32_t, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
+        return run_pass_v<uint32_t, uint32_t, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
     if (kb_in == 8 && kb_out == 8)
-        return run_pass_v<uint64_t, uint64_t, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
+        return run_pass_v<uint64_t, uint64_t, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
     if (kb_in == 8)
-        return run_pass_v<uint64_t, uint32_t, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
-    return run_pass_v<uint32_t, uint64_t, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st);
+        return run_pass_v<uint64_t, uint32_t, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
+    return run_pass_v<uint32_t, uint64_t, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
 }
 
 cudaError_t launch_radix_pass_x(int kb_in, int kb_out, int vb, const void *kin, void *kout, const void *vin,
                                 void *vout, long long n, int shift, const unsigned *digit_base, void *scratch,
-                                unsigned hi, cudaStream_t st, long long *launches, int rb)
+                                unsigned hi, cudaStream_t st, long long *launches, int rb, bool prezeroed)
 {
     if (n <= 0) return cudaSuccess;
     if (n >= (1ll << 30)) return cudaErrorInvalidValue;
     if (rb != 8 && rb != 9) return cudaErrorInvalidValue;
     const cudaError_t e = rb == 8 ? run_pass_kk<8>(kb_in, kb_out, vb, kin, kout, vin, vout, n, shift, digit_base,
-                                                   scratch, hi, st)
+                                                   scratch, hi, st, prezeroed)
                                   : run_pass_kk<9>(kb_in, kb_out, vb, kin, kout, vin, vout, n, shift, digit_base,
-                                                   scratch, hi, st);
+                                                   scratch, hi, st, prezeroed);
     ++*launches;
     return e;
 }

@@ -642,6 +642,7 @@ def test_exact_int64_sums_not_refused(eng, mode):
                           ctx=("wide", mode, corr_op, agg))
     # a real overflow (a qualifying set whose sum leaves int64) is still an
     # error, on both paths, like the oracle's
+    from paper_conf_icde_floratosxwgylz21_b200 import NestGPUError
     t2 = {"R": {"col1": np.array([10], np.int64), "col2": np.zeros(1, np.int64)},
           "S": {"col1": np.arange(4, dtype=np.int64), "col2": np.full(4, A, np.int64)}}
     plan = make_plan(">", "sum", "=")
