@@ -67,6 +67,11 @@ def parse_args(argv=None):
     ap.add_argument("--e2e-steps", type=int, default=2, help="e2e steps (at most --steps)")
     ap.add_argument("--no-side", action="store_true", help="skip the side keys (other plans, C2, index path)")
     ap.add_argument("--no-check", action="store_true", help="skip rank 0's whole-R result check")
+    ap.add_argument("--gather", choices=("peer", "nccl"), default="peer",
+                    help="N > 1: survivors to rank 0 by peer stores into an IPC window (default) or NCCL send/recv")
+    ap.add_argument("--index-mode", choices=("local", "broadcast"), default="local",
+                    help="N > 1: every rank builds the index from its resident S (default), or rank 0 builds "
+                         "and broadcasts it")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="CPU oracle sample budget")
     ap.add_argument("--out", default=None, help="also append the JSON line to this file")
@@ -313,9 +318,10 @@ class Rank:
     """One rank's engine state for one workload: its R shard (resident), S
     (broadcast from rank 0 at N > 1, resident) and the step function."""
 
-    def __init__(self, eng, dev, stream, name, rank, world, R, S, plans):
+    def __init__(self, eng, dev, stream, name, rank, world, R, S, plans, gather="peer", index_mode="local"):
         from paper_conf_icde_floratosxwgylz21_b200 import dist as ngd
         self.ngd = ngd
+        self.gather_mode, self.index_mode = gather, index_mode
         self.eng, self.dev, self.stream = eng, dev, stream
         self.name, self.rank, self.world = name, rank, world
         self.R_full, self.S_host, self.plans = R, S, plans
@@ -328,6 +334,9 @@ class Rank:
         else:
             self.Sc = eng.load_table(S)
         self.launches = 0
+        self.pg = None
+        if world > 1 and gather == "peer":
+            self.pg = ngd.PeerGather(eng, self.n_r, device=dev)
 
     def step(self, plans=None, profs=None, stages=None, keep=None):
         """One pass of the hot path over the batch (every plan).  At N > 1 the
@@ -347,7 +356,8 @@ class Rank:
                 payload = "col2" if plan["agg"] in ("min", "max", "sum", "avg") else None
                 if payload not in idx:
                     idx[payload] = (ngd.share_index(eng, self.Sc, ["col1"], payload, device=self.dev)
-                                    if self.world > 1 else eng.build_index(self.Sc, ["col1"], payload))
+                                    if self.world > 1 and self.index_mode == "broadcast"
+                                    else eng.build_index(self.Sc, ["col1"], payload))
         if ev:
             ev[1].record(self.stream)
         out = []
@@ -361,8 +371,11 @@ class Rank:
                 profs.append((plan, mode, eng.last_profile(), res.n_evaluated))
             out.append(res.n_rows)
             if self.world > 1:
-                t = eng.result_tensors(res)
-                g = ngd.gather_rows([t["row"], t["value"]])
+                if self.pg is not None:
+                    g = self.pg.gather(res)
+                else:
+                    t = eng.result_tensors(res)
+                    g = ngd.gather_rows([t["row"], t["value"]])
                 if keep is not None and self.rank == 0:
                     keep.append((g[0].clone(), g[1].clone()))
             elif keep is not None:
@@ -464,7 +477,7 @@ def main(argv=None):
     arena = max(1 << 30, (n_r + n_s) * 8 * 24 + (512 << 20))
     eng = Engine(dev_idx, arena_bytes=arena, stream=stream)
     eng.set_profiling(True)
-    rk = Rank(eng, dev, stream, args.workload, rank, world, R, S_host, plans)
+    rk = Rank(eng, dev, stream, args.workload, rank, world, R, S_host, plans, args.gather, args.index_mode)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 
     def barrier():
@@ -540,7 +553,7 @@ def main(argv=None):
             # C2's 12-plan step (BASELINE configs[1]) as an extra key
             R2, S2, plans2, _ = workload("C2")
             m0 = eng.mark()
-            rk2 = Rank(eng, dev, stream, "C2", rank, world, R2, S2, plans2)
+            rk2 = Rank(eng, dev, stream, "C2", rank, world, R2, S2, plans2, args.gather, args.index_mode)
             for _ in range(2):
                 rk2.step()
             barrier()
@@ -552,6 +565,8 @@ def main(argv=None):
             side["C2 12-plan step"] = {"value": len(plans2) * len(R2["col1"]) / (t / 1000.0), "ms_per_step": t,
                                        "steps": k2, "workload": DESC["C2"],
                                        "roofline_frac": rf2["frac"] if rf2 else None}
+            if rk2.pg is not None:
+                rk2.pg.close()
             del rk2
             eng.release(m0)
             barrier()
@@ -615,8 +630,11 @@ def main(argv=None):
         for plan, mode, prof, _ in profs:
             key = "%s %s (%s)" % (plan["corr_op"], plan["agg"], mode)
             latency.setdefault(key, []).append(prof["total"])
-        par = "1 GPU" if world == 1 else ("R sharded x%d (contiguous row blocks, one R), S broadcast once, "
-                                          "survivors gathered to rank 0 each step (%s)" % (world, backend))
+        par = "1 GPU" if world == 1 else (
+            "R sharded x%d (contiguous row blocks, one R), S broadcast once (%s), index %s, survivors gathered "
+            "to rank 0 each step by %s" % (
+                world, backend, "built on every rank" if args.index_mode == "local" else "built on rank 0 + broadcast",
+                "peer stores into an IPC window on rank 0" if args.gather == "peer" else "NCCL send/recv"))
         line = {
             "metric": "outer tuples/s", "value": value, "unit": "outer tuples/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
@@ -644,6 +662,8 @@ def main(argv=None):
         if nccl_pat:
             line["nccl_init"] = ngd.nccl_init_summary(nccl_pat)
         emit(line, args)
+    if rk.pg is not None:
+        rk.pg.close()
     eng.close()
     if world > 1:
         dist.destroy_process_group()

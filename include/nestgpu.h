@@ -56,7 +56,7 @@ enum {
     NESTGPU_ERR_OOM = -2,          /* the caller's arena is exhausted */
     NESTGPU_ERR_TYPE = -3,         /* dtype mismatch */
     NESTGPU_ERR_UNSUPPORTED = -4,  /* valid SQL outside this engine's template */
-    NESTGPU_ERR_OVERFLOW = -5,     /* |S'| * max|payload| may exceed int64 (reading R5) */
+    NESTGPU_ERR_OVERFLOW = -5,     /* an exact SUM leaves int64 (reading R5) */
     NESTGPU_ERR_CUDA = -6,         /* a CUDA runtime call or launch failed */
     NESTGPU_ERR_BUFFER = -7        /* caller's host buffer too small */
 };
@@ -108,13 +108,20 @@ nestgpu_status nestgpu_destroy(nestgpu_ctx *ctx);
 const char *nestgpu_last_error(const nestgpu_ctx *ctx);
 /* Number of kernels this context has launched since creation. */
 int64_t nestgpu_launch_count(const nestgpu_ctx *ctx);
-/* Switch the stream subsequent calls enqueue on. */
+/* Switch the stream subsequent calls enqueue on.  Work already queued on the
+ * old stream is ordered before anything enqueued afterwards (the new stream
+ * waits on an event recorded on the old one; no host synchronisation).
+ * Errors: INVALID, CUDA. */
 nestgpu_status nestgpu_set_stream(nestgpu_ctx *ctx, void *cuda_stream);
 
 /* Memory pool (Fig. 7: "record where to free", then move the
  * tail back).  nestgpu_mark returns the current tail of the persistent side of
  * the arena; nestgpu_release drops every column, index and result created
- * after that mark.  Errors: INVALID. */
+ * after that mark.  Column and index ids are slots: the id of a dropped /
+ * released object is handed to the next object created, so a
+ * load -> build -> exec -> release loop keeps reusing the same ids (a plan
+ * struct built once stays valid) and the host tables stay bounded; an id
+ * kept past its object's release may name a newer object.  Errors: INVALID. */
 nestgpu_status nestgpu_mark(nestgpu_ctx *ctx, uint64_t *out_mark);
 nestgpu_status nestgpu_release(nestgpu_ctx *ctx, uint64_t mark);
 /* Bytes in use (persistent + scratch) and the high-water mark. */
@@ -242,13 +249,21 @@ typedef struct {
  * S is filtered here and the tiled block-nested-loop kernel runs.  Work is
  * enqueued on the context stream; the call synchronises once at the end to
  * read the survivor count (dedup adds two synchronisations: to plan the sort
- * of R' keys and to size the evaluation of the distinct keys).  Errors: INVALID, TYPE, UNSUPPORTED, OVERFLOW,
+ * of R' keys and to size the evaluation of the distinct keys); before that
+ * sync the first rows of every result field (256 KB worth) are copied to
+ * pinned host memory, so nestgpu_result_to_host of a result that small is a
+ * host copy.  SUM / AVG are exact (reading R5): 64-bit payloads whose
+ * |S| * max|payload| could reach 2^63 are accumulated as split 32-bit halves
+ * and combined in int128; OVERFLOW only when some R' tuple's sum leaves
+ * int64 (as the oracle).  Errors: INVALID, TYPE, UNSUPPORTED, OVERFLOW,
  * OOM, CUDA.  Nothing is launched when validation fails. */
 nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *ctx, const nestgpu_plan *plan,
                                        nestgpu_result *out);
 
 /* Copy up to cap rows of a result to host buffers (each pointer may be NULL
- * to skip that field).  BUFFER if cap < n_rows (nothing copied).  Synchronous. */
+ * to skip that field).  BUFFER if cap < n_rows (nothing copied).  Synchronous;
+ * a result staged by its exec (see above) is served from pinned host memory
+ * without any GPU operation. */
 nestgpu_status nestgpu_result_to_host(nestgpu_ctx *ctx, const nestgpu_result *res,
                                       int64_t *row_ids, int64_t *values, uint8_t *valid,
                                       uint8_t *passed, int64_t *avg_sum, int64_t *avg_cnt,
@@ -402,6 +417,42 @@ nestgpu_status nestgpu_cost_calibrate(nestgpu_ctx *ctx, int64_t n_rows, nestgpu_
  * work, no context).  Errors: INVALID (negative sizes, bad widths / enums). */
 nestgpu_status nestgpu_cost_estimate_plan(const nestgpu_cost_params *params, const nestgpu_cost_input *in,
                                           nestgpu_cost_estimate *out);
+
+/* ---------------------------------------------------------------- multi-GPU
+ * Peer-memory survivor gather (north_star: "results are gathered"; the paper
+ * is single-GPU).  Outer tuples are independent (Fig. 2),
+ * so each rank's survivors are a contiguous block of the global result in
+ * rank order.  Rank 0 creates a WINDOW -- device memory other processes map
+ * through a CUDA IPC handle (NVLink / NVSwitch peer memory on a multi-GPU
+ * box; plain device memory for ranks sharing one GPU) -- and every rank
+ * stores its survivors straight into it at its row offset with
+ * nestgpu_result_put: the bulk data moves by peer stores from the rank's own
+ * kernel, no NCCL on the data path.  The caller exchanges the survivor counts
+ * (8 B per rank) to get the offsets and orders the puts before rank 0 reads
+ * the window (a barrier).
+ *
+ * Window layout (cap rows): int64 row ids [cap], then int64 values [cap].
+ * The window is allocated with cudaMalloc at creation (setup time, never on
+ * the exec path) and owned by the context until nestgpu_window_free. */
+typedef struct {
+    unsigned char bytes[64];   /* cudaIpcMemHandle_t */
+} nestgpu_ipc_handle;
+/* Create a window of cap rows; *d_window = its device address on this
+ * context's device, *out its IPC handle.  Errors: INVALID, CUDA. */
+nestgpu_status nestgpu_window_create(nestgpu_ctx *ctx, int64_t cap, void **d_window, nestgpu_ipc_handle *out);
+/* Map a window created by another process; *d_peer is valid in this
+ * context until nestgpu_window_close.  Errors: INVALID, CUDA (IPC not
+ * available between the two devices). */
+nestgpu_status nestgpu_window_open(nestgpu_ctx *ctx, const nestgpu_ipc_handle *handle, void **d_peer);
+nestgpu_status nestgpu_window_close(nestgpu_ctx *ctx, void *d_peer);
+nestgpu_status nestgpu_window_free(nestgpu_ctx *ctx, void *d_window);
+/* Store a result's rows (ids, values) into window rows [offset, offset +
+ * n_rows) of a window of cap rows (own or peer).  Synchronous: on return the
+ * stores are complete and visible system-wide (__threadfence_system + stream
+ * sync), so a host barrier then orders them before the owner's reads.
+ * Errors: INVALID (offset + n_rows > cap), CUDA. */
+nestgpu_status nestgpu_result_put(nestgpu_ctx *ctx, const nestgpu_result *res, void *d_window, int64_t cap,
+                                  int64_t offset);
 
 /* Ablation knobs -- NOT for production use; they exist to measure the
  * paper's design claims against their baselines (tools/ablations.py).

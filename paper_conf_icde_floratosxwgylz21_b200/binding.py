@@ -32,7 +32,9 @@ SYMBOLS = ("nestgpu_create", "nestgpu_destroy", "nestgpu_last_error", "nestgpu_l
            "nestgpu_index_create_empty", "nestgpu_exec_correlated", "nestgpu_result_to_host",
            "nestgpu_exec_collect", "nestgpu_collection_in", "nestgpu_column_from_device",
            "nestgpu_set_option", "nestgpu_set_profiling", "nestgpu_last_profile",
-           "nestgpu_cost_calibrate", "nestgpu_cost_estimate_plan")
+           "nestgpu_cost_calibrate", "nestgpu_cost_estimate_plan",
+           "nestgpu_window_create", "nestgpu_window_open", "nestgpu_window_close", "nestgpu_window_free",
+           "nestgpu_result_put")
 STRATEGIES = ("nested_loop", "index", "nested_loop_cached", "index_cached")
 OPT_MALLOC_SCRATCH = 1
 OPT_BNL_SHAPE = 2
@@ -84,6 +86,10 @@ class Collection(ctypes.Structure):
                 ("d_values", ctypes.c_void_p), ("d_owner", ctypes.c_void_p)]
 
 
+class IpcHandle(ctypes.Structure):
+    _fields_ = [("bytes", ctypes.c_ubyte * 64)]
+
+
 class CostParams(ctypes.Structure):
     _fields_ = [("launch_ms", ctypes.c_double), ("filter_ms_per_row", ctypes.c_double),
                 ("hist_ms_per_key_digit", ctypes.c_double), ("sort_ms_per_key", ctypes.c_double),
@@ -112,6 +118,16 @@ class CostInput(ctypes.Structure):
 class CostEstimate(ctypes.Structure):
     _fields_ = [("ms", ctypes.c_double * 4), ("index_build_ms", ctypes.c_double), ("outer_ms", ctypes.c_double),
                 ("nested_ms", ctypes.c_double * 4), ("best", ctypes.c_int32)]
+
+
+class Prepared:
+    """A plan marshalled once (Engine.prepare): the C struct and the
+    predicate arrays it points to, kept alive together."""
+
+    def __init__(self, plan_struct, keep):
+        self.plan = plan_struct
+        self._keep = keep
+        self.ref = ctypes.byref(plan_struct)
 
 
 _lib = None
@@ -186,6 +202,11 @@ def load_library(path=LIB_PATH):
         "nestgpu_cost_calibrate": (i32, [vp, i64, P(CostParams)]),
         "nestgpu_cost_estimate_plan": (i32, [P(CostParams), P(CostInput), P(CostEstimate)]),
         "nestgpu_set_profiling": (i32, [vp, i32]),
+        "nestgpu_window_create": (i32, [vp, i64, P(vp), P(IpcHandle)]),
+        "nestgpu_window_open": (i32, [vp, P(IpcHandle), P(vp)]),
+        "nestgpu_window_close": (i32, [vp, vp]),
+        "nestgpu_window_free": (i32, [vp, vp]),
+        "nestgpu_result_put": (i32, [vp, P(Result), vp, i64, i64]),
         "nestgpu_last_profile": (i32, [vp, P(ctypes.c_float), i32]),
     }
     for name, (res, args) in sig.items():
@@ -194,6 +215,19 @@ def load_library(path=LIB_PATH):
         f.argtypes = args
     _lib = lib
     return lib
+
+
+def _device_view(ptr, n, device):
+    """int64 torch tensor aliasing n values of device memory at ptr (memory
+    the library owns, e.g. a window; no copy).  Built on a __cuda_array_interface__
+    shim, so torch keeps no ownership."""
+    import torch
+
+    class _Shim:
+        __cuda_array_interface__ = {"shape": (int(n),), "typestr": "<i8", "data": (int(ptr), False), "version": 2,
+                                    "strides": None}
+
+    return torch.as_tensor(_Shim(), device=device)
 
 
 def _np_ptr(a):
@@ -415,9 +449,21 @@ class Engine:
         self._keep = (opa, ipa)
         return p
 
-    def exec(self, plan, R, S, index=-1, emit_all=False, row_id_base=0, dedup=False):
-        """Run one plan (datagen.plans dict).  R / S map column names to ids.
-        dedup: evaluate each distinct correlated value once (P:331 caching)."""
+    def prepare(self, plan, R, S, index=-1, emit_all=False, row_id_base=0, dedup=False):
+        """Marshal a plan into its C struct once (Prepared); exec(prepared)
+        then skips the per-call Python marshalling -- the repeated-query
+        path of small, latency-bound queries."""
+        p = self._plan(plan, R, S, index, emit_all, row_id_base, dedup)
+        return Prepared(p, self._keep)
+
+    def exec(self, plan, R=None, S=None, index=-1, emit_all=False, row_id_base=0, dedup=False):
+        """Run one plan (datagen.plans dict, or a Prepared from prepare()).
+        R / S map column names to ids.  dedup: evaluate each distinct
+        correlated value once (P:331 caching)."""
+        if isinstance(plan, Prepared):
+            res = Result()
+            self._check(self.lib.nestgpu_exec_correlated(self.ctx, plan.ref, ctypes.byref(res)))
+            return res
         p = self._plan(plan, R, S, index, emit_all, row_id_base, dedup)
         res = Result()
         self._check(self.lib.nestgpu_exec_correlated(self.ctx, ctypes.byref(p), ctypes.byref(res)))
@@ -483,6 +529,40 @@ class Engine:
                                                     _np_ptr(out["value"]), _np_ptr(out["valid"]),
                                                     _np_ptr(out["passed"]), _np_ptr(s), _np_ptr(c), n))
         return out
+
+    # ------------------------------------------------------------ peer windows (multi-GPU gather)
+    def window_create(self, cap):
+        """A device window of cap (row id, value) rows other processes can map;
+        returns (device pointer, 64 IPC handle bytes)."""
+        p, h = ctypes.c_void_p(), IpcHandle()
+        self._check(self.lib.nestgpu_window_create(self.ctx, int(cap), ctypes.byref(p), ctypes.byref(h)))
+        return p.value, bytes(h.bytes)
+
+    def window_open(self, handle_bytes):
+        h = IpcHandle()
+        ctypes.memmove(h.bytes, bytes(handle_bytes), 64)
+        p = ctypes.c_void_p()
+        self._check(self.lib.nestgpu_window_open(self.ctx, ctypes.byref(h), ctypes.byref(p)))
+        return p.value
+
+    def window_close(self, ptr):
+        self._check(self.lib.nestgpu_window_close(self.ctx, ctypes.c_void_p(ptr)))
+
+    def window_free(self, ptr):
+        self._check(self.lib.nestgpu_window_free(self.ctx, ctypes.c_void_p(ptr)))
+
+    def result_put(self, res, window_ptr, cap, offset):
+        """Store res's (row id, value) rows into window rows [offset, offset+n)."""
+        self._check(self.lib.nestgpu_result_put(self.ctx, ctypes.byref(res), ctypes.c_void_p(window_ptr), int(cap),
+                                                int(offset)))
+
+    def window_tensors(self, ptr, cap, n):
+        """torch views (row ids, values) of the first n rows of an OWN window."""
+        torch = self._torch
+        if n == 0:
+            e = torch.empty(0, dtype=torch.int64, device=self.device)
+            return e, e
+        return (_device_view(ptr, n, self.device), _device_view(ptr + 8 * int(cap), n, self.device))
 
     def result_tensors(self, res):
         """torch views of the device result (valid until the next exec)."""

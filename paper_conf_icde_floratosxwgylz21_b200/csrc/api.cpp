@@ -172,6 +172,21 @@ static int plan_sort_passes(int kb, unsigned long long kand, unsigned long long 
 
 size_t align_up(size_t x) { return (x + ALIGN - 1) / ALIGN * ALIGN; }
 
+// Column / index ids are slots that are reused once their object died
+// (release / drop): a loop of load -> query -> release keeps the id set and
+// the host tables bounded, and a re-built object gets its old id back.
+template <typename T>
+int32_t put_slot(std::vector<T> &v, const T &x)
+{
+    for (size_t i = 0; i < v.size(); i++)
+        if (!v[i].alive) {
+            v[i] = x;
+            return (int32_t)i;
+        }
+    v.push_back(x);
+    return (int32_t)v.size() - 1;
+}
+
 // Start a new scratch generation: everything salloc'd before dies here.
 void scratch_reset(nestgpu_ctx *c)
 {
@@ -500,8 +515,7 @@ static nestgpu_status new_column(nestgpu_ctx *c, nestgpu_dtype dtype, int32_t sc
         }
     }
     col.alive = true;
-    c->cols.push_back(col);
-    *out = (int32_t)c->cols.size() - 1;
+    *out = put_slot(c->cols, col);
     return NESTGPU_OK;
 }
 
@@ -712,8 +726,7 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     ix.inner.assign(inner_preds, inner_preds + n_inner_preds);
     ix.payload_nullable = pc && pc->valid;
     ix.alive = true;
-    c->idx.push_back(ix);
-    *out_index = (int32_t)c->idx.size() - 1;
+    *out_index = put_slot(c->idx, ix);
     CUDA_TRY(c, cudaGetLastError());
     return NESTGPU_OK;
 }
@@ -786,8 +799,7 @@ nestgpu_status nestgpu_index_create_empty(nestgpu_ctx *c, int64_t n, int32_t key
     const Column *pc = payload_col >= 0 ? col_get(c, payload_col) : nullptr;
     ix.payload_nullable = pc && pc->valid;
     ix.alive = true;
-    c->idx.push_back(ix);
-    *out_index = (int32_t)c->idx.size() - 1;
+    *out_index = put_slot(c->idx, ix);
     out->n = n;
     out->key_bytes = key_bytes_;
     out->payload_bytes = payload_bytes;
@@ -1311,7 +1323,7 @@ nestgpu_status nestgpu_column_from_device(nestgpu_ctx *c, nestgpu_dtype dtype, i
     if (w == 4) {
         bad = (unsigned long long *)salloc(c, 8);
         if (!bad) {
-            c->cols.pop_back();
+            c->cols[id].alive = false;
             c->lo = off;
             return fail(c, NESTGPU_ERR_OOM, "arena exhausted (column_from_device)");
         }
@@ -1326,12 +1338,77 @@ nestgpu_status nestgpu_column_from_device(nestgpu_ctx *c, nestgpu_dtype dtype, i
         unsigned long long nb;
         memcpy(&nb, c->pinned, 8);
         if (nb) {
-            c->cols.pop_back();
+            c->cols[id].alive = false;
             c->lo = off;
             return fail(c, NESTGPU_ERR_OVERFLOW, "column_from_device: %llu values do not fit a 4-byte column", nb);
         }
     }
     *out_col = id;
+    return NESTGPU_OK;
+}
+
+// ---------------------------------------------------------------- peer windows
+static_assert(sizeof(nestgpu_ipc_handle) == sizeof(cudaIpcMemHandle_t), "IPC handle size");
+
+nestgpu_status nestgpu_window_create(nestgpu_ctx *c, int64_t cap, void **d_window, nestgpu_ipc_handle *out)
+{
+    if (!c || !d_window || !out || cap < 0) return fail(c, NESTGPU_ERR_INVALID, "window_create: bad argument");
+    cudaSetDevice(c->device);
+    void *p = nullptr;
+    CUDA_TRY(c, cudaMalloc(&p, (size_t)(cap > 0 ? cap : 1) * 16));
+    cudaIpcMemHandle_t h;
+    cudaError_t e = cudaIpcGetMemHandle(&h, p);
+    if (e != cudaSuccess) {
+        cudaFree(p);
+        return fail(c, NESTGPU_ERR_CUDA, "window_create: cudaIpcGetMemHandle: %s", cudaGetErrorString(e));
+    }
+    memcpy(out->bytes, &h, sizeof h);
+    *d_window = p;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_window_open(nestgpu_ctx *c, const nestgpu_ipc_handle *handle, void **d_peer)
+{
+    if (!c || !handle || !d_peer) return fail(c, NESTGPU_ERR_INVALID, "window_open: null argument");
+    cudaSetDevice(c->device);
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle->bytes, sizeof h);
+    void *p = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) return fail(c, NESTGPU_ERR_CUDA, "window_open: cudaIpcOpenMemHandle: %s", cudaGetErrorString(e));
+    *d_peer = p;
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_window_close(nestgpu_ctx *c, void *d_peer)
+{
+    if (!c || !d_peer) return NESTGPU_ERR_INVALID;
+    cudaSetDevice(c->device);
+    CUDA_TRY(c, cudaIpcCloseMemHandle(d_peer));
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_window_free(nestgpu_ctx *c, void *d_window)
+{
+    if (!c || !d_window) return NESTGPU_ERR_INVALID;
+    cudaSetDevice(c->device);
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    CUDA_TRY(c, cudaFree(d_window));
+    return NESTGPU_OK;
+}
+
+nestgpu_status nestgpu_result_put(nestgpu_ctx *c, const nestgpu_result *r, void *d_window, int64_t cap, int64_t offset)
+{
+    if (!c || !r || !d_window || cap < 0 || offset < 0) return fail(c, NESTGPU_ERR_INVALID, "result_put: bad argument");
+    if (offset + r->n_rows > cap)
+        return fail(c, NESTGPU_ERR_INVALID, "result_put: rows [%lld, %lld) outside the window's %lld", (long long)offset,
+                    (long long)(offset + r->n_rows), (long long)cap);
+    cudaSetDevice(c->device);
+    long long *wi = (long long *)d_window + offset;
+    long long *wv = (long long *)d_window + cap + offset;
+    CUDA_TRY(c, ng::launch_put_rows((const long long *)r->d_row_ids, (const long long *)r->d_values, r->n_rows, wi,
+                                    wv, c->stream, &c->launches));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
     return NESTGPU_OK;
 }
 

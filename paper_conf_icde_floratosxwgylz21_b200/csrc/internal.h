@@ -197,6 +197,11 @@ struct FinalizeArgs {
 };
 cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *launches, bool prezeroed = false);
 
+// Survivor rows into a (peer) window: win_ids[off + i] = ids[i],
+// win_vals[off + i] = vals[i], i < n; ends with __threadfence_system.
+cudaError_t launch_put_rows(const long long *ids, const long long *vals, long long n, long long *win_ids,
+                            long long *win_vals, cudaStream_t st, long long *launches);
+
 // out[i] = src[ids[i] - base] (w = 4 or 8 bytes per value).
 cudaError_t launch_gather(int w, const void *src, const long long *ids, long long n, long long base, void *out,
                           cudaStream_t st, long long *launches);

@@ -269,6 +269,48 @@ __global__ void gather_kernel(const T *__restrict__ src, const long long *__rest
         out[i] = src[ids[i] - base];
 }
 
+// ------------------------------------------------------------------ peer put
+// Rank r's survivors -> rank 0's window (multi-GPU gather by peer stores):
+// 16-byte vector loads / stores where both sides are 16-B aligned, the
+// stores go over NVLink when the window is a peer device's memory.
+__global__ void put_rows_kernel(const long long *__restrict__ ids, const long long *__restrict__ vals, long long n,
+                                long long *__restrict__ wi, long long *__restrict__ wv)
+{
+    const long long t = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    const long long nt = (long long)gridDim.x * blockDim.x;
+    const bool vec = ((((unsigned long long)ids | (unsigned long long)vals | (unsigned long long)wi |
+                        (unsigned long long)wv) & 15) == 0);
+    if (vec) {
+        const long long n2 = n / 2;
+        for (long long i = t; i < n2; i += nt) {
+            reinterpret_cast<longlong2 *>(wi)[i] = reinterpret_cast<const longlong2 *>(ids)[i];
+            reinterpret_cast<longlong2 *>(wv)[i] = reinterpret_cast<const longlong2 *>(vals)[i];
+        }
+        if (t == 0 && (n & 1)) {
+            wi[n - 1] = ids[n - 1];
+            wv[n - 1] = vals[n - 1];
+        }
+    } else {
+        for (long long i = t; i < n; i += nt) {
+            wi[i] = ids[i];
+            wv[i] = vals[i];
+        }
+    }
+    __threadfence_system();
+}
+
+cudaError_t launch_put_rows(const long long *ids, const long long *vals, long long n, long long *win_ids,
+                            long long *win_vals, cudaStream_t st, long long *launches)
+{
+    if (n <= 0) return cudaSuccess;
+    long long blocks = (n / 2 + 255) / 256;
+    if (blocks < 1) blocks = 1;
+    if (blocks > 148 * 8) blocks = 148 * 8;
+    put_rows_kernel<<<(unsigned)blocks, 256, 0, st>>>(ids, vals, n, win_ids, win_vals);
+    ++*launches;
+    return cudaGetLastError();
+}
+
 cudaError_t launch_gather(int w, const void *src, const long long *ids, long long n, long long base, void *out,
                           cudaStream_t st, long long *launches)
 {

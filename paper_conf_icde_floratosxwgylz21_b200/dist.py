@@ -11,10 +11,12 @@ exchange steps are therefore
     so only rank 0 sorts) from rank 0 -- over NVLink/NVSwitch via NCCL,
     directly into tensor views of each rank's engine arena;
   * a gather of the variable-length survivor lists to rank 0 only: the
-    counts are exchanged (8 B per rank), then every rank sends its rows to
-    rank 0 with point-to-point sends (one grouped batch, so NCCL runs the
-    N-1 transfers concurrently) -- rank 0 receives each survivor once, no
-    padding and no copy on the other ranks.
+    counts are exchanged (8 B per rank), then either every rank STORES its
+    rows into a window on rank 0 from its own kernel (PeerGather: CUDA IPC
+    peer memory, over NVLink/NVSwitch between GPUs -- the default of
+    bench.py) or sends them with point-to-point NCCL sends (gather_rows: one
+    grouped batch) -- rank 0 receives each survivor once, no padding and no
+    copy on the other ranks.
 
 The helpers move tensors only; they work with NCCL (GPU box) and gloo (CPU
 tests, or several ranks sharing one GPU: gloo collectives that do not take
@@ -231,6 +233,57 @@ def share_index(eng, S, key, payload, inner_preds=(), device=None, group=None):
         views.append(eng.arena_view(info["d_payload"], n * vb))
     broadcast_tensors(views, group=group)
     return idx
+
+
+class PeerGather:
+    """Survivor gather by peer stores (nestgpu_window_* / nestgpu_result_put):
+    rank 0 owns a window of `cap` rows; every rank maps it once (CUDA IPC: an
+    NVLink/NVSwitch peer mapping across GPUs, the same memory for ranks that
+    share a device) and, per gather, stores its survivors into it at its row
+    offset from its own kernel.  The control path is two tiny host
+    collectives -- the survivor counts (8 B per rank) and a barrier that
+    orders the puts before rank 0 reads; no NCCL send/recv carries rows.
+    Collective: every rank constructs it and calls gather()."""
+
+    def __init__(self, eng, cap, device=None, group=None):
+        self.eng, self.cap, self.group = eng, int(cap), group
+        self.device = device if device is not None else eng.device
+        self.rank = dist.get_rank(group)
+        self.own = None
+        if self.rank == 0:
+            self.own, handle = eng.window_create(self.cap)
+            h = torch.tensor(list(handle), dtype=torch.uint8)
+        else:
+            h = torch.zeros(64, dtype=torch.uint8)
+        hd = h if _is_gloo(group) else h.to(self.device)
+        dist.broadcast(hd, src=0, group=group)
+        self.handle = bytes(hd.cpu().tolist())
+        self.peer = self.own if self.rank == 0 else eng.window_open(self.handle)
+
+    def gather(self, res):
+        """Rank 0: (row ids, values) torch views of the gathered rows in rank
+        order (valid until the next gather); other ranks: None."""
+        counts = all_counts(res.n_rows, device=self.device, group=self.group)
+        off = sum(counts[:self.rank])
+        if sum(counts) > self.cap:
+            raise ValueError("PeerGather: %d rows exceed the window's %d" % (sum(counts), self.cap))
+        self.eng.result_put(res, self.peer, self.cap, off)   # synchronous: stores complete + visible
+        dist.barrier(group=self.group)
+        if self.rank != 0:
+            return None
+        return self.eng.window_tensors(self.own, self.cap, sum(counts))
+
+    def close(self):
+        if self.rank == 0:
+            dist.barrier(group=self.group)   # every peer has unmapped
+            if self.own:
+                self.eng.window_free(self.own)
+                self.own = None
+        else:
+            if self.peer:
+                self.eng.window_close(self.peer)
+                self.peer = None
+            dist.barrier(group=self.group)
 
 
 def gather_result(eng, res, group=None):
