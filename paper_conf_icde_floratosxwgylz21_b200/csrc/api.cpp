@@ -22,6 +22,8 @@
 #include <mutex>
 #include <string>
 #include <tuple>
+#include <chrono>
+#include <cstdlib>
 #include <utility>
 #include <vector>
 
@@ -70,6 +72,10 @@ constexpr int PIN_WORDS = 8 * 256 + 64;
 // result field into it before its one synchronisation, so a result of at
 // most that many rows reaches the host with no further GPU operation.
 constexpr size_t STAGE_BYTES = 256 << 10;
+// Inputs this small take the latency-oriented shortcuts (fewer launches):
+// partial-aggregate init folded into the exec's fill kernel, the whole
+// index-build scratch zeroed by one fill before the S' filter.
+constexpr long long SMALL_ROWS = 1 << 16;
 constexpr size_t ALIGN = 256;
 
 }  // namespace
@@ -103,6 +109,11 @@ struct nestgpu_ctx {
     std::vector<void *> mallocs;
     int bnl_shape;   // NESTGPU_OPT_BNL_SHAPE (test knob): 0 automatic, 1 full, 2 warp-split
     cudaEvent_t ev[NESTGPU_N_STAGES][2];
+    // NESTGPU_TRACE=1 (diagnostics): host time of each step of an exec,
+    // printed to stderr when the exec returns
+    bool trace;
+    std::chrono::steady_clock::time_point t0, tl;
+    std::string tlog;
     bool ran[NESTGPU_N_STAGES];
 };
 
@@ -313,6 +324,29 @@ int key_bytes(const nestgpu_ctx *c, const int32_t *cols, int32_t nk)
     return (nk == 1 && dtype_width(c->cols[cols[0]].dtype) == 4) ? 4 : 8;
 }
 
+void htrace(nestgpu_ctx *c, const char *what)
+{
+    if (!c->trace) return;
+    const auto now = std::chrono::steady_clock::now();
+    char buf[64];
+    snprintf(buf, sizeof buf, " %s=%.1f", what, std::chrono::duration<double, std::micro>(now - c->tl).count());
+    c->tlog += buf;
+    c->tl = now;
+}
+void htrace_begin(nestgpu_ctx *c)
+{
+    if (!c->trace) return;
+    c->t0 = c->tl = std::chrono::steady_clock::now();
+    c->tlog.clear();
+}
+void htrace_end(nestgpu_ctx *c, const char *call)
+{
+    if (!c->trace) return;
+    htrace(c, "tail");
+    fprintf(stderr, "[nestgpu trace] %s total=%.1f us:%s\n", call,
+            std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - c->t0).count(), c->tlog.c_str());
+}
+
 void prof_begin(nestgpu_ctx *c, int s)
 {
     if (c->profiling) {
@@ -401,6 +435,10 @@ nestgpu_status nestgpu_create(int device, void *d_arena, size_t arena_bytes, voi
     c->profiling = false;
     c->malloc_scratch = false;
     c->bnl_shape = 0;
+    {
+        const char *tr = getenv("NESTGPU_TRACE");
+        c->trace = tr && tr[0] == '1';
+    }
     c->stage = nullptr;
     c->staged.ok = false;
     if (cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess ||
@@ -585,6 +623,7 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
 {
     if (!c || !key_cols || !out_index) return fail(c, NESTGPU_ERR_INVALID, "build_index: null argument");
     cudaSetDevice(c->device);
+    htrace_begin(c);
     ng::KeySrc ks;
     int64_t n;
     nestgpu_status s = make_key(c, key_cols, n_key_cols, n, ks, "build_index");
@@ -627,27 +666,43 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     void *tk = salloc(c, (size_t)n * kb), *tv = vb ? salloc(c, (size_t)n * vb) : nullptr;
     void *uk = salloc(c, (size_t)n * kb), *uv = vb ? salloc(c, (size_t)n * vb) : nullptr;
     void *fscr = salloc(c, ng::filter_scratch_bytes(n));
-    unsigned *hist = (unsigned *)salloc(c, 8 * 512 * 4);
+    unsigned *hist = (unsigned *)salloc(c, ng::hist_bytes());
     unsigned *dbase = (unsigned *)salloc(c, 8 * 512 * 4);
     long long *dsmall = (long long *)salloc(c, 64);   // [0] |S'|, [2] key AND, [3] key OR
     if (!tk || !uk || !fscr || !hist || !dbase || !dsmall || (vb && (!tv || !uv)))
         return fail(c, NESTGPU_ERR_OOM, "arena exhausted building an index over %lld rows", (long long)n);
     long long *d_count = dsmall;
     unsigned long long *keymask = (unsigned long long *)(dsmall + 2);
+    // small S: the scratch of the histogram and of every possible pass is
+    // allocated now and zeroed by the same fill (no second fill after the sync)
+    const bool small = n <= SMALL_ROWS;
+    void *pscr[8] = {};
+    if (small)
+        for (int p = 0; p < kb; p++)
+            if (!(pscr[p] = salloc(c, ng::sort_scratch_bytes(n))))
+                return fail(c, NESTGPU_ERR_OOM, "arena exhausted (sort scratch)");
     {   // one fill kernel instead of a memset per scratch region
         ng::FillList fl;
         fl.add(dsmall, 16);
         fl.add(keymask, 8, 0xff);   // AND identity
         fl.add(dsmall + 3, 40);
         fl.add(fscr, ng::filter_zero_bytes(n, false));
+        if (small) {
+            fl.add(hist, ng::hist_bytes());
+            for (int p = 0; p < kb; p++) fl.add(pscr[p], ng::sort_scratch_bytes(n));
+        }
+        htrace(c, "setup");
         CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
+        htrace(c, "fill");
     }
     prof_begin(c, 1);
     CUDA_TRY(c, ng::launch_filter(n, ps, ks, fkb, vs, vb, 1, pc ? 1 : 0, nullptr, tk, nullptr, tv, keymask, nullptr,
                                   fscr, d_count, c->stream, &c->launches, true));
     prof_end(c, 1);
+    htrace(c, "filter");
     CUDA_TRY(c, cudaMemcpyAsync(c->pinned, dsmall, 32, cudaMemcpyDeviceToHost, c->stream));
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    htrace(c, "sync");
     long long nsp;
     unsigned long long kand, kor;
     memcpy(&nsp, c->pinned, 8);
@@ -666,10 +721,9 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     const unsigned hi = pre_narrow ? pre_hi : (unsigned)(kand >> 32);
     // one scratch region per pass, all zeroed with the digit histograms by
     // one fill kernel
-    void *pscr[8] = {};
-    {
+    if (!small) {
         ng::FillList fl;
-        fl.add(hist, (size_t)(np > 0 ? np : 1) * (1u << rb) * 4);
+        fl.add(hist, ng::hist_bytes());
         for (int p = 0; p < np; p++) {
             const int kin = pre_narrow || (narrow && p > 0) ? 4 : kb;
             const size_t zb = ng::sort_pass_zero_bytes(nsp, kin, vb, rb);
@@ -680,8 +734,10 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
         CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
     }
     prof_begin(c, 2);
+    htrace(c, "fill2");
     CUDA_TRY(c, ng::launch_digit_hist(fkb, tk, nsp, shifts, np, hist, dbase, c->num_sms, c->stream, &c->launches,
                                       rb, true));
+    htrace(c, "hist");
 
     IndexRec ix{};
     ix.off = c->lo;
@@ -719,6 +775,7 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
         }
     }
     prof_end(c, 2);
+    htrace(c, "passes");
     ix.key_cols[0] = key_cols[0];
     ix.key_cols[1] = n_key_cols == 2 ? key_cols[1] : -1;
     ix.n_key = n_key_cols;
@@ -728,6 +785,7 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     ix.alive = true;
     *out_index = put_slot(c->idx, ix);
     CUDA_TRY(c, cudaGetLastError());
+    htrace_end(c, "build_index");
     return NESTGPU_OK;
 }
 
@@ -812,6 +870,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
 {
     if (!c || !P || !out) return fail(c, NESTGPU_ERR_INVALID, "exec: null argument");
     cudaSetDevice(c->device);
+    htrace_begin(c);
     memset(out, 0, sizeof *out);
     // ------------------------------------------------------------ validation
     if (P->agg < NG_MIN || P->agg > NG_NOT_EXISTS) return fail(c, NESTGPU_ERR_INVALID, "exec: bad aggregate");
@@ -880,6 +939,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         wide = (__int128)nS * m >= ((__int128)1 << 63);
     }
 
+    htrace(c, "validate");
     // ------------------------------------------------------------ allocation
     scratch_reset(c);  // previous results die here
     for (int st = 0; st < NESTGPU_N_STAGES; st++) c->ran[st] = false;
@@ -932,7 +992,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         ukeys = salloc(c, (size_t)nR * kb);
         sscr = salloc(c, ng::sort_scratch_bytes(nR));
         gscr = salloc(c, ng::group_scratch_bytes(nR));
-        hist = (unsigned *)salloc(c, 8 * 512 * 4);
+        hist = (unsigned *)salloc(c, ng::hist_bytes());
         dbase = (unsigned *)salloc(c, 8 * 512 * 4);
         if (!pos || !tpos || !map || !tkeys || !ukeys || !sscr || !gscr || !hist || !dbase)
             return fail(c, NESTGPU_ERR_OOM, "arena exhausted (dedup buffers for |R|=%lld)", (long long)nR);
@@ -953,16 +1013,24 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         fl.add(fscr_f, ng::finalize_scratch_bytes(nR));
         fl.add(kscr, ix ? 256 : ng::bnl_scratch_bytes(nR));
         if (wide) fl.add(acc_hi, (size_t)nR * 8);
+        if (!ix && nR <= SMALL_ROWS) {   // small R: the partials' identity init rides on the fill
+            const long long acc0 = P->agg == NG_MIN ? LLONG_MAX : (P->agg == NG_MAX ? LLONG_MIN : 0);
+            fl.add_words(acc, (size_t)nR * 8, (unsigned long long)acc0);
+            fl.add(cnt, (size_t)nR * 8);
+        }
         // the staged rows (copied to the host even when fewer survive):
         // defined contents for compute-sanitizer's initcheck
         const long long kr = std::min<long long>(nR, (long long)(STAGE_BYTES / (8 * w8 + 2)));
         for (size_t f = 0; f < w8; f++) fl.add(rblk + (size_t)nR * 8 * f, (size_t)kr * 8);
         fl.add(o_valid, (size_t)kr);
         fl.add(o_pass, (size_t)kr);
+        htrace(c, "alloc");
         CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
+        htrace(c, "fill");
     }
     CUDA_TRY(c, ng::launch_filter(nR, ops, rks, kb, none, 0, 0, 0, ids, rkeys, rkvalid, nullptr,
                                   P->dedup ? rmask : nullptr, nullptr, fscr, d_nrp, c->stream, &c->launches, true));
+    htrace(c, "rfilter");
     prof_end(c, 0);
 
     // The keys the subquery kernels evaluate: every R' key, or (dedup) each
@@ -1031,7 +1099,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
             }
             pre = ix->aux_pre[kind];
             suf = ix->aux_suf[kind];
-        } else if (P->agg == NG_MIN || P->agg == NG_MAX) {
+        } else if ((P->agg == NG_MIN || P->agg == NG_MAX) && ix->n > ng::RANGE_INLINE_MAX) {
             // '=' MIN/MAX: per-key group aggregates (segmented scan), so a hot
             // key's run is folded once per index, not once per outer tuple
             const int kind = P->agg == NG_MIN ? 4 : 5;
@@ -1055,6 +1123,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         CUDA_TRY(c, ng::launch_range_agg(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, ix->keys, ix->payload,
                                          ix->n, pre, split ? nullptr : suf, acc, cnt, kscr, c->stream, &c->launches,
                                          split ? suf : nullptr, split ? acc_hi : nullptr, true));
+        htrace(c, "range");
         prof_end(c, 3);
     } else {
         prof_begin(c, 1);
@@ -1063,12 +1132,16 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         CUDA_TRY(c, ng::launch_filter(nS, ips, sks, kb, vs, vb, 1, value_agg ? 1 : 0, nullptr, skeys, nullptr, svals,
                                       nullptr, value_agg ? extreme : nullptr, fscr_s, d_nsp, c->stream,
                                       &c->launches, true));
-        CUDA_TRY(c, ng::launch_init_partials(n_eval, d_neval, P->agg, acc, cnt, c->stream, &c->launches));
+        htrace(c, "sfilter");
+        if (nR > SMALL_ROWS)
+            CUDA_TRY(c, ng::launch_init_partials(n_eval, d_neval, P->agg, acc, cnt, c->stream, &c->launches));
+        htrace(c, "init");
         prof_end(c, 1);
         prof_begin(c, 3);
         CUDA_TRY(c, ng::launch_bnl(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, nS, d_nsp, skeys, svals,
                                    extreme, acc, cnt, kscr, c->num_sms, c->bnl_shape, c->stream, &c->launches,
                                    wide ? acc_hi : nullptr, true));
+        htrace(c, "bnl");
         prof_end(c, 3);
     }
 
@@ -1102,19 +1175,24 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     fa.out_count = d_out;
     fa.scratch = fscr_f;
     CUDA_TRY(c, ng::launch_finalize(fa, c->stream, &c->launches, true));
+    htrace(c, "finalize");
     prof_end(c, 4);
     prof_end(c, 5);
     CUDA_TRY(c, cudaMemcpyAsync(c->pinned, counts, 72, cudaMemcpyDeviceToHost, c->stream));
     // the first rows of every result field, staged on the host before the
     // one synchronisation (8-byte fields, then the two byte fields)
     const long long krows = std::min<long long>(nR, (long long)(STAGE_BYTES / (8 * w8 + 2)));
-    if (krows > 0) {
+    if (krows == nR && krows > 0) {   // the whole result block fits: one copy, same layout
+        CUDA_TRY(c, cudaMemcpyAsync(c->stage, rblk, (size_t)nR * (8 * w8 + 2), cudaMemcpyDeviceToHost, c->stream));
+    } else if (krows > 0) {
         CUDA_TRY(c, cudaMemcpy2DAsync(c->stage, (size_t)krows * 8, rblk, (size_t)nR * 8, (size_t)krows * 8, w8,
                                       cudaMemcpyDeviceToHost, c->stream));
         CUDA_TRY(c, cudaMemcpy2DAsync(c->stage + (size_t)krows * 8 * w8, (size_t)krows, o_valid, (size_t)nR,
                                       (size_t)krows, 2, cudaMemcpyDeviceToHost, c->stream));
     }
+    htrace(c, "copies");
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    htrace(c, "sync");
     long long cnts[9];
     memcpy(cnts, c->pinned, 72);
     if (cnts[8]) return fail(c, NESTGPU_ERR_OVERFLOW, "exec: a SUM exceeds int64 (reading R5)");
@@ -1130,6 +1208,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     out->d_passed = o_pass;
     out->d_avg_sum = (const int64_t *)o_sum;
     out->d_avg_cnt = (const int64_t *)o_cnt;
+    htrace_end(c, "exec");
     return NESTGPU_OK;
 }
 

@@ -86,7 +86,7 @@ nestgpu_status nestgpu_cost_calibrate(nestgpu_ctx *c, int64_t n_rows, nestgpu_co
         kraw = A(n * 4); vraw = A(n * 4); ids = A(n * 4); k1 = A(n * 4); v1 = A(n * 4); k2 = A(n * 4);
         v2 = A(n * 4); acc = A(n * 8); cnt = A(n * 8); oid = A(n * 8); oval = A(n * 8); oflag = A(n * 2);
         fscr = A(ng::filter_scratch_bytes(n)); sscr = A(ng::sort_scratch_bytes(n)); small = A(256);
-        hist = A(8 * 256 * 4); dbase = A(8 * 256 * 4); pre = A((n + 1) * 8); suf = A((n + 1) * 8);
+        hist = A(ng::hist_bytes()); dbase = A(8 * 256 * 4); pre = A((n + 1) * 8); suf = A((n + 1) * 8);
         rscr = A(ng::range_scratch_bytes(n)); bscr = A(ng::bnl_scratch_bytes(n)); gscr = A(ng::group_scratch_bytes(n));
         uk = A(n * 4); map = A(n * 4);
         if (kraw && vraw && ids && k1 && v1 && k2 && v2 && acc && cnt && oid && oval && oflag && fscr && sscr &&
@@ -369,11 +369,13 @@ nestgpu_status nestgpu_cost_estimate_plan(const nestgpu_cost_params *p, const ne
     const bool sumavg = in->agg == NG_SUM || in->agg == NG_AVG;
     const bool value_agg = minmax || sumavg;
     const int cls = minmax ? 0 : (in->agg == NG_COUNT ? 1 : (sumavg ? 2 : 3));
-    auto selection = [&](double rows) { return 3 * C + p->filter_ms_per_row * rows; };   // Eq. (1)
+    // launch counts follow api.cpp: one fill kernel per exec / index build
+    // zeroes every scratch region, a filter is one launch
+    auto selection = [&](double rows) { return C + p->filter_ms_per_row * rows; };   // Eq. (1)
 
     // U, Eq. (8): outer selection, then finalize + compaction (M * D_r * sum Rs)
     const double rs = 18.0 + (in->agg == NG_AVG ? 16.0 : 0.0);   // id + value + valid + passed (+ sum, nn)
-    const double U = selection(nR) + C + p->final_ms_per_row * nRp +
+    const double U = selection(nR) + 2 * C + p->final_ms_per_row * nRp +
                      p->materialize_ms_per_byte * (double)in->survivors * rs + p->sync_ms + p->exec_overhead_ms;
     out->outer_ms = U;
 
@@ -395,9 +397,9 @@ nestgpu_status nestgpu_cost_estimate_plan(const nestgpu_cost_params *p, const ne
     // index build (invariant, once): S' selection + histogram + radix passes;
     // plus the payload prefix aggregates when the plan reads them (NEXT 3)
     const double sp = in->sort_passes;
-    double build = selection(nS) + p->sync_ms + p->build_overhead_ms +
+    double build = C + selection(nS) + p->sync_ms + p->build_overhead_ms +
                    (sp > 0 ? 2 * C + p->hist_ms_per_key_digit * nSp * sp : 0) +
-                   sp * (2 * C + p->sort_ms_per_key * nSp) + p->sort_ms_per_byte * nSp * pass_bytes(sp);
+                   sp * (C + p->sort_ms_per_key * nSp) + p->sort_ms_per_byte * nSp * pass_bytes(sp);
     if (value_agg && (in->corr_op != NG_EQ || sumavg)) build += (minmax ? 6 : 3) * C + p->aux_ms_per_elem * nSp;
     out->index_build_ms = build;
 
@@ -411,7 +413,7 @@ nestgpu_status nestgpu_cost_estimate_plan(const nestgpu_cost_params *p, const ne
     };
     // nested loop: S' selection (invariant) + init + |evaluations| x |S'| pairs
     auto nested_loop = [&](double ev) {
-        return selection(nS) + C + 2 * C + p->bnl_ms_per_pair[in->key_bytes == 8][cls] * ev * nSp;
+        return selection(nS) + 2 * C + p->bnl_ms_per_pair[in->key_bytes == 8][cls] * ev * nSp;
     };
     const double nd = (double)in->n_distinct;
     out->nested_ms[NESTGPU_STRATEGY_NESTED_LOOP] = nested_loop(nRp);

@@ -63,14 +63,27 @@ struct FillList {
     int n = 0;
     void *p[24];
     unsigned long long bytes[24];
-    unsigned char val[24];
+    unsigned long long pat[24];   // byte value replicated, or (word) a 64-bit pattern
+    unsigned char word[24];       // 1: 8-byte pattern (8-B aligned region, bytes % 8 == 0)
     bool add(void *ptr, size_t b, unsigned char v = 0)
     {
         if (!ptr || !b) return true;
         if (n >= 24) return false;
         p[n] = ptr;
         bytes[n] = b;
-        val[n] = v;
+        pat[n] = 0x0101010101010101ull * v;
+        word[n] = 0;
+        n++;
+        return true;
+    }
+    bool add_words(void *ptr, size_t b, unsigned long long v)
+    {
+        if (!ptr || !b) return true;
+        if (n >= 24) return false;
+        p[n] = ptr;
+        bytes[n] = b;
+        pat[n] = v;
+        word[n] = 1;
         n++;
         return true;
     }
@@ -103,6 +116,9 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
 // a4: histograms of the digits at `shifts` (np of them) over n encoded keys,
 // and their exclusive scans into digit_base[np][256].
 //   rb: digit bits (8 or 9); hist / digit_base hold np * 2^rb words
+// hist: hist_bytes() of scratch (8 x 512 bins + a CTA-done counter); the
+// kernel's last CTA scans the bins into digit_base (one launch).
+size_t hist_bytes();
 cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *shifts, int np, unsigned *hist,
                               unsigned *digit_base, int num_sms, cudaStream_t st, long long *launches, int rb = 8,
                               bool prezeroed = false);
@@ -132,6 +148,11 @@ cudaError_t launch_init_partials(long long n, const long long *d_n, int agg, lon
 // qualifying range(s).  d_nrp: device count of R'.  Long ranges go to a
 // warp-per-range second kernel.
 size_t range_scratch_bytes(long long n_rp_max);
+// Indexes of at most this many entries: every range is folded inline by its
+// thread (no long-range kernel) and the keys themselves serve as the search
+// samples (no sample kernel) -- fewer launches for small, latency-bound
+// queries.
+constexpr long long RANGE_INLINE_MAX = 4096;
 //   pre / suf: optional prefix / suffix aggregates of the index payload
 //   (launch_index_aux); non-equality and SUM/AVG ranges are then O(1).
 //   pre_hi / acc_hi: exact SUM of 64-bit payloads (nullable): pre holds the

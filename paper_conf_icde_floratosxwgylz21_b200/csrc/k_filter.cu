@@ -654,7 +654,14 @@ __global__ void fill_list_kernel(FillList f)
     for (int r = 0; r < f.n; r++) {
         unsigned char *p = (unsigned char *)f.p[r];
         const unsigned long long b = f.bytes[r];
-        const unsigned v = f.val[r] * 0x01010101u;
+        if (f.word[r]) {   // 64-bit pattern (e.g. the MIN/MAX identity of the partials)
+            unsigned long long *w = (unsigned long long *)p;
+            for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < (long long)(b / 8);
+                 i += (long long)gridDim.x * blockDim.x)
+                w[i] = f.pat[r];
+            continue;
+        }
+        const unsigned v = (unsigned)f.pat[r];
         // aligned 16-B body, byte head / tail
         const unsigned long long head = (16 - ((unsigned long long)p & 15)) & 15;
         const unsigned long long h = head < b ? head : b;

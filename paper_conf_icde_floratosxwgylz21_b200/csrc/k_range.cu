@@ -192,7 +192,7 @@ range_short_kernel(const long long *__restrict__ d_nrp, const K *__restrict__ rk
                 }
                 acc[i] = a;
                 cnt[i] = L;
-            } else if (L <= R_SHORT) {
+            } else if (L <= R_SHORT || N <= (int)RANGE_INLINE_MAX) {
                 long long a = AGG == MIN ? LLONG_MAX : (AGG == MAX ? LLONG_MIN : 0);
                 for (int s = a0; s < b0; s++) fold<AGG>(a, svals[s]);
                 for (int s = a1; s < b1; s++) fold<AGG>(a, svals[s]);
@@ -257,7 +257,9 @@ static void launch_range_t(long long n_rp_max, const long long *d_nrp, const voi
     const int N = (int)ns;
     const int stride = N > SMAX ? (N + SMAX - 1) / SMAX : 1;
     const int M = N > 0 ? (N + stride - 1) / stride : 0;
-    if (M > 0) {
+    if (stride == 1) {
+        samp = (K *)skeys;   // every key fits the shared-memory sample buffer: the keys are the samples
+    } else if (M > 0) {
         sample_kernel<K><<<(M + 255) / 256, 256, 0, st>>>((const K *)skeys, stride, M, samp);
         ++*launches;
     }
@@ -274,9 +276,13 @@ static void launch_range_t(long long n_rp_max, const long long *d_nrp, const voi
         d_nrp, (const K *)rkeys, (const K *)skeys, svals, N, samp, M, stride, pre, suf, acc, cnt, list, list_n,
         pre_hi, acc_hi);
     ++*launches;
+    // long ranges exist only when no range is answered in O(1) (prefix /
+    // suffix / group aggregates) and the index is too large to fold inline
     if constexpr (AGG != COUNT && AGG != EXISTS && AGG != NOT_EXISTS) {
-        range_long_kernel<VB, OP, AGG><<<148 * 8, R_THREADS, 0, st>>>(svals, (int)ns, list, list_n, acc, cnt);
-        ++*launches;
+        if (!pre && ns > RANGE_INLINE_MAX) {
+            range_long_kernel<VB, OP, AGG><<<148 * 8, R_THREADS, 0, st>>>(svals, (int)ns, list, list_n, acc, cnt);
+            ++*launches;
+        }
     }
 }
 

@@ -373,9 +373,13 @@ struct DigitList {
 
 template <typename K, int NB>
 __global__ void __launch_bounds__(256) digit_hist_kernel(const K *__restrict__ keys, long long n, DigitList dl,
-                                                         unsigned *__restrict__ hist)
+                                                         unsigned *__restrict__ hist,
+                                                         unsigned *__restrict__ done,
+                                                         unsigned *__restrict__ digit_base)
 {
     __shared__ unsigned s_hist[8 * NB];
+    __shared__ bool s_last;
+    __shared__ unsigned s_w[8];
     for (int i = threadIdx.x; i < dl.n * NB; i += 256) s_hist[i] = 0;
     __syncthreads();
     const long long stride = (long long)gridDim.x * 256;
@@ -388,29 +392,43 @@ __global__ void __launch_bounds__(256) digit_hist_kernel(const K *__restrict__ k
     __syncthreads();
     for (int i = threadIdx.x; i < dl.n * NB; i += 256)
         if (s_hist[i]) atomicAdd(&hist[i], s_hist[i]);
+    // the last CTA to finish scans every pass's bins into the digit bases
+    // (replaces a separate scan launch)
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) s_last = atomicAdd(done, 1u) == gridDim.x - 1;
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    constexpr int PER = NB / 256;   // bins per thread (consecutive)
+    for (int p = 0; p < dl.n; p++) {
+        unsigned c[PER], s = 0;
+#pragma unroll
+        for (int q = 0; q < PER; q++) {
+            c[q] = __ldcg(hist + p * NB + threadIdx.x * PER + q);
+            s += c[q];
+        }
+        unsigned incl = s;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned v = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl += v;
+        }
+        if (lane == 31) s_w[warp] = incl;
+        __syncthreads();
+        unsigned run = incl - s;
+        for (int w = 0; w < warp; w++) run += s_w[w];
+#pragma unroll
+        for (int q = 0; q < PER; q++) {
+            digit_base[p * NB + threadIdx.x * PER + q] = run;
+            run += c[q];
+        }
+        __syncthreads();
+    }
 }
 
-// Exclusive scan of each pass's NB bins -> global digit base offsets
-// (one CTA of NB threads per pass).
-__global__ void __launch_bounds__(512) digit_scan_kernel(const unsigned *__restrict__ hist, unsigned *__restrict__ base)
-{
-    __shared__ unsigned s_w[16];
-    const int nb = blockDim.x;
-    const unsigned *h = hist + blockIdx.x * nb;
-    const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
-    const unsigned c = h[t];
-    unsigned incl = c;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        unsigned v = __shfl_up_sync(FULL, incl, o);
-        if (lane >= o) incl += v;
-    }
-    if (lane == 31) s_w[warp] = incl;
-    __syncthreads();
-    unsigned pre = 0;
-    for (int w = 0; w < warp; w++) pre += s_w[w];
-    base[blockIdx.x * nb + t] = pre + incl - c;
-}
+size_t hist_bytes() { return 8 * 512 * 4 + 256; }
 
 cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *shifts, int np, unsigned *hist,
                               unsigned *digit_base, int num_sms, cudaStream_t st, long long *launches, int rb,
@@ -418,7 +436,9 @@ cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *
 {
     if (np <= 0) return cudaSuccess;
     const int nb = 1 << rb;
-    cudaError_t e = prezeroed ? cudaSuccess : cudaMemsetAsync(hist, 0, (size_t)np * nb * 4, st);
+    // hist holds 8 * 512 bins + the CTA-done counter at hist[8 * 512]
+    unsigned *done = hist + 8 * 512;
+    cudaError_t e = prezeroed ? cudaSuccess : cudaMemsetAsync(hist, 0, hist_bytes(), st);
     if (e != cudaSuccess) return e;
     DigitList dl{};
     dl.n = np;
@@ -427,14 +447,13 @@ cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *
     if (blocks > (long long)num_sms * 8) blocks = (long long)num_sms * 8;
     if (blocks < 1) blocks = 1;
     if (rb == 8) {
-        if (kb == 4) digit_hist_kernel<uint32_t, 256><<<(unsigned)blocks, 256, 0, st>>>((const uint32_t *)keys, n, dl, hist);
-        else digit_hist_kernel<uint64_t, 256><<<(unsigned)blocks, 256, 0, st>>>((const uint64_t *)keys, n, dl, hist);
+        if (kb == 4) digit_hist_kernel<uint32_t, 256><<<(unsigned)blocks, 256, 0, st>>>((const uint32_t *)keys, n, dl, hist, done, digit_base);
+        else digit_hist_kernel<uint64_t, 256><<<(unsigned)blocks, 256, 0, st>>>((const uint64_t *)keys, n, dl, hist, done, digit_base);
     } else {
-        if (kb == 4) digit_hist_kernel<uint32_t, 512><<<(unsigned)blocks, 256, 0, st>>>((const uint32_t *)keys, n, dl, hist);
-        else digit_hist_kernel<uint64_t, 512><<<(unsigned)blocks, 256, 0, st>>>((const uint64_t *)keys, n, dl, hist);
+        if (kb == 4) digit_hist_kernel<uint32_t, 512><<<(unsigned)blocks, 256, 0, st>>>((const uint32_t *)keys, n, dl, hist, done, digit_base);
+        else digit_hist_kernel<uint64_t, 512><<<(unsigned)blocks, 256, 0, st>>>((const uint64_t *)keys, n, dl, hist, done, digit_base);
     }
-    digit_scan_kernel<<<np, nb, 0, st>>>(hist, digit_base);
-    *launches += 2;
+    *launches += 1;
     return cudaGetLastError();
 }
 

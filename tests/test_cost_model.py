@@ -44,7 +44,8 @@ def test_nested_part_scales_with_evaluations():
     """Eq. (6): N = (S - Ch) * per-evaluation cost + invariant parts."""
     a = cost_estimate(P, **shape(corr_op="<", n_rp=400_000, n_distinct=100_000, survivors=0))
     b = cost_estimate(P, **shape(corr_op="<", n_rp=800_000, n_distinct=100_000, survivors=0))
-    inv = 3 * P["launch_ms"] + P["filter_ms_per_row"] * 1_000_000 + 3 * P["launch_ms"]   # S' selection + launches
+    # S' selection (one filter launch) + init + nested-loop launches
+    inv = P["launch_ms"] + P["filter_ms_per_row"] * 1_000_000 + 2 * P["launch_ms"]
     na, nb = a["nested"]["nested_loop"] - inv, b["nested"]["nested_loop"] - inv
     assert nb == pytest.approx(2 * na, rel=1e-9)
     # caching evaluates each distinct value once: the pair term drops to n_distinct / n_rp of it
