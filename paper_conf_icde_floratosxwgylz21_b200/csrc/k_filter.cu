@@ -32,7 +32,18 @@
 
 namespace ng {
 
+#ifndef NG_RP_BATCH
+#define NG_RP_BATCH 4   // ordered R' filter, phase 2: rounds of key loads in flight per warp
+#endif
+constexpr int RP_BATCH = NG_RP_BATCH;
+#ifndef NG_RP_ITEMS
+#define NG_RP_ITEMS 8   // ordered R' filter: rows per thread per staged tile
+#endif
 constexpr int T_THREADS = 256;
+// scratch of the ordered one-launch R' filter: [0, 1024) the barrier word
+// (zeroed), then the per-chunk counts, then the ballot words (n / 8 bytes)
+constexpr size_t RP_COUNTS_OFF = 1024;
+constexpr size_t RP_BITS_OFF = 1024 + 16384;
 constexpr int T_WARPS = T_THREADS / 32;
 constexpr int MAX_SRC = 40;
 constexpr int STAGE_MAX = 49152;  // bytes per stage (2 stages per CTA)
@@ -364,143 +375,249 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
 }
 
 // ------------------------------------------------------------------ ordered R'
-// One pass (P:235's scan -> 0-1 vector -> prefix sum -> materialize fused):
-// a tile stages ONLY its predicate columns (cp.async.bulk, single buffer:
-// occupancy supplies the overlap, and no tile id is taken before its data is
-// processed, so no successor waits on a prefetched tile), evaluates them,
-// gets its output offset from the CTA-wide decoupled look-back (scan.cuh),
-// then loads the key (+ validity) of its SURVIVORS straight from global
-// memory and writes ids / encoded keys / key-valid in row order.  A
-// selective outer predicate (SF10 Q4: 3.8 %) thus reads the key column only
-// where rows survive, instead of staging it for every row.
+// One launch, no chained look-back (P:235's scan -> 0-1 vector -> prefix sum
+// -> materialize): a persistent cooperative grid, CTA c owns a contiguous
+// chunk of rows.
+//  phase 1: the chunk's predicate columns stream through a double-buffered
+//           cp.async.bulk stage; the 0-1 vector is written as one 32-bit
+//           ballot word per 32 consecutive rows (n / 8 bytes, L2-resident)
+//           and the chunk's survivor count is published;
+//  barrier: one grid-wide barrier (every CTA is resident: cooperative
+//           launch), then each CTA sums the counts of the chunks before it;
+//  phase 2: warps read 32 ballot words at a time, rank survivors with popc
+//           and a warp scan, load the survivors' keys (+ validity) straight
+//           from global memory and write ids / encoded keys / key-valid in
+//           row order.
+// The predicate columns are read once and the key column only where rows
+// survive (a selective date window reads a fraction of it); with no outer
+// predicate phase 1 and the barrier are skipped (every row survives, the
+// chunk offset is its first row).  The round-1 count pass + scan + write
+// pass read the predicate columns twice and staged every key; a decoupled
+// look-back chain over the tiles measured slower than both.
+#ifndef NG_RP_MINB
+#define NG_RP_MINB 2   // ordered R' filter: CTAs per SM the register budget must allow (latency hiding)
+#endif
 template <int KB, int ITEMS>
-__global__ void __launch_bounds__(T_THREADS)
-filter_rp_kernel(long long n, SrcCols sc, TPlan tp, KeySrc ks, int *__restrict__ out_ids, void *__restrict__ out_keys,
-                 uint8_t *__restrict__ out_kvalid, unsigned long long *__restrict__ keymask,
-                 unsigned long long *__restrict__ status, unsigned *__restrict__ counter,
+__global__ void __launch_bounds__(T_THREADS, NG_RP_MINB)
+filter_rp_kernel(long long n, long long chunk, SrcCols sc, TPlan tp, KeySrc ks, int *__restrict__ out_ids,
+                 void *__restrict__ out_keys, uint8_t *__restrict__ out_kvalid,
+                 unsigned long long *__restrict__ keymask, unsigned *__restrict__ bits,
+                 unsigned long long *__restrict__ counts, unsigned *__restrict__ barrier,
                  long long *__restrict__ out_count)
 {
     using K = typename std::conditional<KB == 8, uint64_t, uint32_t>::type;
     constexpr int TILE = T_THREADS * ITEMS;
     extern __shared__ __align__(128) unsigned char smem[];
-    __shared__ __align__(8) unsigned long long bar;
-    __shared__ unsigned s_cnt[ITEMS][T_WARPS];
-    __shared__ long long s_tile;
+    __shared__ __align__(8) unsigned long long bar[2];
+    __shared__ unsigned long long s_red[T_WARPS];
+    __shared__ unsigned s_wtot[T_WARPS];
+    __shared__ unsigned long long s_base;
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const long long num_tiles = (n + TILE - 1) / TILE;
-    if (tid == 0) {
-        mbar_init(&bar, 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    unsigned phase = 0u;
-    unsigned long long kand = ~0ull, kor = 0ull;
-    for (;;) {
+    const long long c0 = blockIdx.x * chunk;
+    const long long c1 = min(n, c0 + chunk);
+    const bool preds = sc.n > 0;
+    unsigned long long mycount = 0;
+
+    if (preds) {
+        // ---- phase 1: predicates -> ballot words, chunk count
+        const long long ntile = c1 > c0 ? (c1 - c0 + TILE - 1) / TILE : 0;
+        auto issue = [&](long long t, int stage) {
+            const long long r0 = c0 + t * TILE;
+            const long long rows = min((long long)TILE, c1 - r0);
+            unsigned total = 0;
+            for (int c = 0; c < sc.n; c++) total += ((unsigned)rows * sc.w[c] + 15u) & ~15u;
+            unsigned char *dst = smem + stage * sc.stage_bytes;
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_expect_tx(&bar[stage], total);
+            for (int c = 0; c < sc.n; c++)
+                bulk_g2s(dst + sc.off[c], (const char *)sc.ptr[c] + r0 * sc.w[c], ((unsigned)rows * sc.w[c] + 15u) & ~15u,
+                         &bar[stage]);
+        };
         if (tid == 0) {
-            const long long t = atomicAdd(counter, 1u);
-            s_tile = t;
-            if (t < num_tiles && sc.n > 0) {
-                const long long rows = min((long long)TILE, n - t * TILE);
-                unsigned total = 0;
-                for (int c = 0; c < sc.n; c++) total += ((unsigned)rows * sc.w[c] + 15u) & ~15u;
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                mbar_expect_tx(&bar, total);
-                for (int c = 0; c < sc.n; c++)
-                    bulk_g2s(smem + sc.off[c], (const char *)sc.ptr[c] + t * TILE * sc.w[c],
-                             ((unsigned)rows * sc.w[c] + 15u) & ~15u, &bar);
+            mbar_init(&bar[0], 1);
+            mbar_init(&bar[1], 1);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+            if (ntile > 0) issue(0, 0);
+        }
+        __syncthreads();
+        for (long long t = 0; t < ntile; t++) {
+            const int stage = (int)(t & 1);
+            if (tid == 0 && t + 1 < ntile) issue(t + 1, stage ^ 1);   // the next tile streams in meanwhile
+            mbar_wait(&bar[stage], (unsigned)((t >> 1) & 1));
+            const unsigned char *sb = smem + stage * sc.stage_bytes;
+            const long long r0 = c0 + t * TILE;
+            const long long rows = min((long long)TILE, c1 - r0);
+            unsigned live = 0;
+#pragma unroll
+            for (int j = 0; j < ITEMS; j++)
+                if (j * T_THREADS + tid < rows) live |= 1u << j;
+            for (int k = 0; k < tp.n_preds; k++) {   // local predicates, NULL is not TRUE (R2)
+                const TPred p = tp.p[k];
+                live = nonnull<ITEMS>(sb, p.xv, live, tid);
+                live = nonnull<ITEMS>(sb, p.yv, live, tid);
+#define NG_CMP_ALL(X, Y)                                                                              \
+                switch (p.op) {                                                                       \
+                case EQ: live &= cmp_items<ITEMS, EQ>(X, Y); break;                                   \
+                case NE: live &= cmp_items<ITEMS, NE>(X, Y); break;                                   \
+                case LT: live &= cmp_items<ITEMS, LT>(X, Y); break;                                   \
+                case LE: live &= cmp_items<ITEMS, LE>(X, Y); break;                                   \
+                case GT: live &= cmp_items<ITEMS, GT>(X, Y); break;                                   \
+                default: live &= cmp_items<ITEMS, GE>(X, Y); break;                                   \
+                }
+                if (p.x.w == 4 && (p.y.off >= 0 ? p.y.w == 4 : p.lit == (long long)(int)p.lit)) {
+                    int x[ITEMS], y[ITEMS];
+                    const int *xa = reinterpret_cast<const int *>(sb + p.x.off);
+#pragma unroll
+                    for (int j = 0; j < ITEMS; j++) x[j] = xa[j * T_THREADS + tid];
+                    if (p.y.off >= 0) {
+                        const int *ya = reinterpret_cast<const int *>(sb + p.y.off);
+#pragma unroll
+                        for (int j = 0; j < ITEMS; j++) y[j] = ya[j * T_THREADS + tid];
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < ITEMS; j++) y[j] = (int)p.lit;
+                    }
+                    NG_CMP_ALL(x, y)
+                } else {
+                    long long x[ITEMS], y[ITEMS];
+                    load_items<ITEMS>(sb, p.x, tid, x);
+                    if (p.y.off >= 0) {
+                        load_items<ITEMS>(sb, p.y, tid, y);
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < ITEMS; j++) y[j] = p.lit;
+                    }
+                    NG_CMP_ALL(x, y)
+                }
+#undef NG_CMP_ALL
+            }
+            // row r0 + j*256 + warp*32 + lane -> bit lane of word (r0 + j*256)/32 + warp
+#pragma unroll
+            for (int j = 0; j < ITEMS; j++) {
+                const unsigned m = __ballot_sync(FULL, live >> j & 1u);
+                if (j * T_THREADS + warp * 32 < rows && lane == 0) {
+                    bits[(r0 + j * T_THREADS) / 32 + warp] = m;
+                    mycount += __popc(m);
+                }
+            }
+            __syncthreads();   // the stage is refilled two tiles later
+        }
+        // chunk count -> counts[block]; grid barrier; this chunk's offset
+        if (lane == 0) s_red[warp] = mycount;
+        __syncthreads();
+        if (tid == 0) {
+            unsigned long long t = 0;
+            for (int w = 0; w < T_WARPS; w++) t += s_red[w];
+            st_relaxed_u64(counts + blockIdx.x, t);
+            __threadfence();
+            atomicAdd(barrier, 1u);
+            while (ld_relaxed_u32(barrier) < gridDim.x) __nanosleep(64);
+            __threadfence();
+        }
+        __syncthreads();
+        unsigned long long pre = 0;
+        for (int b = tid; b < (int)blockIdx.x; b += T_THREADS) pre += ld_relaxed_u64(counts + b);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) pre += __shfl_xor_sync(FULL, pre, o);
+        if (lane == 0) s_red[warp] = pre;
+        __syncthreads();
+        if (tid == 0) {
+            unsigned long long t = 0;
+            for (int w = 0; w < T_WARPS; w++) t += s_red[w];
+            s_base = t;
+            if (blockIdx.x == gridDim.x - 1) {   // the grand total
+                unsigned long long mine = ld_relaxed_u64(counts + blockIdx.x);
+                *out_count = (long long)(t + mine);
             }
         }
         __syncthreads();
-        const long long tile = s_tile;
-        if (tile >= num_tiles) break;
-        if (sc.n > 0) {
-            mbar_wait(&bar, phase);
-            phase ^= 1u;
+    } else {
+        if (tid == 0) {
+            s_base = (unsigned long long)min(c0, n);   // every row before the chunk survives
+            if (blockIdx.x == gridDim.x - 1) *out_count = n;
         }
-        const long long base = tile * TILE;
-        const long long rows = min((long long)TILE, n - base);
-        unsigned live = 0;
-#pragma unroll
-        for (int j = 0; j < ITEMS; j++)
-            if (j * T_THREADS + tid < rows) live |= 1u << j;
-        for (int k = 0; k < tp.n_preds; k++) {   // local predicates, NULL is not TRUE (R2)
-            const TPred p = tp.p[k];
-            live = nonnull<ITEMS>(smem, p.xv, live, tid);
-            live = nonnull<ITEMS>(smem, p.yv, live, tid);
-#define NG_CMP_ALL(X, Y)                                                                              \
-            switch (p.op) {                                                                           \
-            case EQ: live &= cmp_items<ITEMS, EQ>(X, Y); break;                                       \
-            case NE: live &= cmp_items<ITEMS, NE>(X, Y); break;                                       \
-            case LT: live &= cmp_items<ITEMS, LT>(X, Y); break;                                       \
-            case LE: live &= cmp_items<ITEMS, LE>(X, Y); break;                                       \
-            case GT: live &= cmp_items<ITEMS, GT>(X, Y); break;                                       \
-            default: live &= cmp_items<ITEMS, GE>(X, Y); break;                                       \
-            }
-            if (p.x.w == 4 && (p.y.off >= 0 ? p.y.w == 4 : p.lit == (long long)(int)p.lit)) {
-                int x[ITEMS], y[ITEMS];
-                const int *xa = reinterpret_cast<const int *>(smem + p.x.off);
-#pragma unroll
-                for (int j = 0; j < ITEMS; j++) x[j] = xa[j * T_THREADS + tid];
-                if (p.y.off >= 0) {
-                    const int *ya = reinterpret_cast<const int *>(smem + p.y.off);
-#pragma unroll
-                    for (int j = 0; j < ITEMS; j++) y[j] = ya[j * T_THREADS + tid];
-                } else {
-#pragma unroll
-                    for (int j = 0; j < ITEMS; j++) y[j] = (int)p.lit;
-                }
-                NG_CMP_ALL(x, y)
+        __syncthreads();
+    }
+
+    // ---- phase 2: ballot words -> ordered ids / keys / key-valid
+    unsigned long long run = s_base;
+    unsigned long long kand = ~0ull, kor = 0ull;
+    const unsigned lt = lanemask_lt();
+    const long long w0 = c0 / 32, w1 = (c1 + 31) / 32;
+    for (long long g = w0; g < w1; g += 32 * T_WARPS) {
+        const long long wi = g + warp * 32 + lane;
+        unsigned word = 0;
+        if (wi < w1) {
+            if (preds) {
+                word = __ldcg(bits + wi);
             } else {
-                long long x[ITEMS], y[ITEMS];
-                load_items<ITEMS>(smem, p.x, tid, x);
-                if (p.y.off >= 0) {
-                    load_items<ITEMS>(smem, p.y, tid, y);
-                } else {
+                const long long r = wi * 32;
+                word = (c1 - r >= 32) ? FULL : ((1u << (unsigned)(c1 - r)) - 1u);
+            }
+        }
+        const unsigned c = __popc(word);
+        unsigned incl = c;
 #pragma unroll
-                    for (int j = 0; j < ITEMS; j++) y[j] = p.lit;
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned t = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl += t;
+        }
+        if (lane == 31) s_wtot[warp] = incl;
+        __syncthreads();
+        unsigned woff = 0, btot = 0;
+#pragma unroll
+        for (int w = 0; w < T_WARPS; w++) {
+            const unsigned t = s_wtot[w];
+            woff += w < warp ? t : 0;
+            btot += t;
+        }
+        const unsigned excl = incl - c;
+        // 32 rounds of 32 consecutive rows, RP_BATCH rounds' key loads in
+        // flight at once (a load -> store chain per round would leave the
+        // warp latency-bound)
+        for (int i0 = 0; i0 < 32; i0 += RP_BATCH) {
+            unsigned wv[RP_BATCH];
+            uint64_t raw[RP_BATCH];
+            bool kvl[RP_BATCH];
+#pragma unroll
+            for (int q = 0; q < RP_BATCH; q++) {
+                wv[q] = __shfl_sync(FULL, word, i0 + q);
+                raw[q] = 0;
+                kvl[q] = true;
+                if ((wv[q] >> lane) & 1u) {
+                    const long long row = (g + warp * 32 + i0 + q) * 32 + lane;
+                    if (ks.n_key == 2)
+                        raw[q] = ((uint64_t)(uint32_t)__ldg((const int *)ks.c0 + row) << 32) |
+                                 (uint32_t)__ldg((const int *)ks.c1 + row);
+                    else if (ks.w0 == 4)
+                        raw[q] = (uint32_t)__ldg((const int *)ks.c0 + row);
+                    else
+                        raw[q] = (uint64_t)__ldg((const long long *)ks.c0 + row);
+                    kvl[q] = !((ks.v0 && !__ldg(ks.v0 + row)) || (ks.v1 && !__ldg(ks.v1 + row)));
                 }
-                NG_CMP_ALL(x, y)
             }
-#undef NG_CMP_ALL
-        }
-        unsigned rank[ITEMS];
 #pragma unroll
-        for (int j = 0; j < ITEMS; j++) {
-            const unsigned m = __ballot_sync(FULL, live >> j & 1u);
-            if (lane == 0) s_cnt[j][warp] = __popc(m);
-            rank[j] = __popc(m & lanemask_lt());
-        }
-        // survivors' keys from global memory (issued before the look-back
-        // so their latency overlaps it)
-        K key[ITEMS];
-        unsigned kv = live;
-#pragma unroll
-        for (int j = 0; j < ITEMS; j++) {
-            key[j] = 0;
-            if (!(live >> j & 1u)) continue;
-            const long long row = base + j * T_THREADS + tid;
-            if (ks.n_key == 2) {
-                key[j] = (K)(((uint64_t)enc32(__ldg((const int *)ks.c0 + row)) << 32) |
-                             enc32(__ldg((const int *)ks.c1 + row)));
-            } else if (ks.w0 == 4) {
-                const int x = __ldg((const int *)ks.c0 + row);
-                key[j] = KB == 4 ? (K)enc32(x) : (K)enc64((long long)x);
-            } else {
-                key[j] = (K)enc64(__ldg((const long long *)ks.c0 + row));
+            for (int q = 0; q < RP_BATCH; q++) {
+                const unsigned ov = __shfl_sync(FULL, excl, i0 + q);
+                if (!((wv[q] >> lane) & 1u)) continue;
+                const long long row = (g + warp * 32 + i0 + q) * 32 + lane;
+                const long long pos = (long long)run + woff + ov + __popc(wv[q] & lt);
+                K key;
+                if (ks.n_key == 2)
+                    key = (K)(((uint64_t)enc32((int)(uint32_t)(raw[q] >> 32)) << 32) | enc32((int)(uint32_t)raw[q]));
+                else if (ks.w0 == 4)
+                    key = KB == 4 ? (K)enc32((int)(uint32_t)raw[q]) : (K)enc64((long long)(int)(uint32_t)raw[q]);
+                else
+                    key = (K)enc64((long long)raw[q]);
+                out_ids[pos] = (int)row;
+                if (out_keys) ((K *)out_keys)[pos] = key;
+                if (out_kvalid) out_kvalid[pos] = kvl[q] ? 1 : 0;
+                kand &= (unsigned long long)key;
+                kor |= (unsigned long long)key;
             }
-            if ((ks.v0 && !__ldg(ks.v0 + row)) || (ks.v1 && !__ldg(ks.v1 + row))) kv &= ~(1u << j);
         }
-        const unsigned long long tb = tile_offsets<ITEMS, T_THREADS>(s_cnt, status, tile, num_tiles, out_count);
-#pragma unroll
-        for (int j = 0; j < ITEMS; j++) {
-            if (!(live >> j & 1u)) continue;
-            const long long pos = (long long)tb + s_cnt[j][warp] + rank[j];
-            out_ids[pos] = (int)(base + j * T_THREADS + tid);
-            if (out_keys) ((K *)out_keys)[pos] = key[j];
-            if (out_kvalid) out_kvalid[pos] = (kv >> j) & 1u;
-            kand &= (unsigned long long)key[j];
-            kor |= (unsigned long long)key[j];
-        }
-        __syncthreads();   // the stage and s_cnt are reused by the next tile
+        run += btot;
+        __syncthreads();   // s_wtot is rewritten next round
     }
     if (keymask) {   // bits shared by every survivor key (dedup sort planning)
         const unsigned alo = __reduce_and_sync(FULL, (unsigned)kand);
@@ -639,14 +756,17 @@ cudaError_t dispatch(int k, int v, int items, long long n, const SrcCols &sc, co
 
 }  // namespace
 
-size_t filter_scratch_bytes(long long n) { return 1024 + 256 + (size_t)(n / T_THREADS + 2) * 12; }
-
-// counter words + (ordered one-pass) the look-back status of every tile --
-// tiles of at least T_THREADS rows, so n / T_THREADS + 1 words bound it
-size_t filter_zero_bytes(long long n, bool ordered)
+size_t filter_scratch_bytes(long long n)
 {
-    return 1024 + (ordered ? (size_t)(n / T_THREADS + 1) * 8 : 0);
+    // counters + per-tile counts / offsets (two-pass mode), or the ordered
+    // filter's chunk counts + ballot words
+    const size_t two_pass = 1024 + 256 + (size_t)(n / T_THREADS + 2) * 12;
+    const size_t one_launch = RP_BITS_OFF + (size_t)(n / 32 + 2) * 4 + 256;
+    return two_pass > one_launch ? two_pass : one_launch;
 }
+
+// the counter words (the ordered filter's grid barrier among them)
+size_t filter_zero_bytes(long long, bool) { return 1024; }
 
 // ---- one kernel filling a list of small regions (FillList)
 __global__ void fill_list_kernel(FillList f)
@@ -702,46 +822,63 @@ bool getenv_two_pass()
 
 template <int KB, int ITEMS>
 cudaError_t launch_rp_t(long long n, const SrcCols &sc, const TPlan &tp, const KeySrc &ks, int *ids, void *keys,
-                        uint8_t *kvalid, unsigned long long *keymask, unsigned long long *status, unsigned *counter,
-                        long long *count, int num_sms, cudaStream_t st)
+                        uint8_t *kvalid, unsigned long long *keymask, void *scratch, long long *count, int num_sms,
+                        cudaStream_t st)
 {
     auto kern = filter_rp_kernel<KB, ITEMS>;
-    const int smem = sc.n > 0 ? sc.stage_bytes : 0;
+    const bool preds = sc.n > 0;
+    const int smem = preds ? 2 * sc.stage_bytes : 0;
     int occ = 0;
     cudaError_t e0 = per_device_setup((const void *)kern, smem, &occ, [&](int, int *v) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, STAGE_MAX);
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * STAGE_MAX);
         if (e != cudaSuccess) return e;
         return cudaOccupancyMaxActiveBlocksPerMultiprocessor(v, kern, T_THREADS, smem);
     });
     if (e0 != cudaSuccess) return e0;
-    const long long tiles = (n + T_THREADS * ITEMS - 1) / (T_THREADS * ITEMS);
-    long long grid = (long long)num_sms * (occ > 0 ? occ : 1);
-    if (grid > tiles) grid = tiles;
-    kern<<<(unsigned)grid, T_THREADS, smem, st>>>(n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count);
-    return cudaGetLastError();
+    if (occ < 1) return cudaErrorInvalidConfiguration;
+    // every CTA resident (the grid barrier): SMs x occupancy, chunks of whole
+    // 256-row groups (ballot words never straddle two chunks)
+    long long grid = (long long)num_sms * occ;
+    if (grid > 2048) grid = 2048;   // counts area: 16 KB
+    long long chunk = (n + grid - 1) / grid;
+    chunk = (chunk + T_THREADS - 1) / T_THREADS * T_THREADS;
+    const long long used = (n + chunk - 1) / chunk;
+    if (!preds) grid = used;   // no barrier: only CTAs with rows
+    unsigned *barrier = (unsigned *)scratch;
+    unsigned long long *counts = (unsigned long long *)((char *)scratch + RP_COUNTS_OFF);
+    unsigned *bits = (unsigned *)((char *)scratch + RP_BITS_OFF);
+    if (!preds) {
+        kern<<<(unsigned)grid, T_THREADS, 0, st>>>(n, chunk, sc, tp, ks, ids, keys, kvalid, keymask, bits, counts,
+                                                 barrier, count);
+        return cudaGetLastError();
+    }
+    void *args[] = {(void *)&n, (void *)&chunk, (void *)&sc, (void *)&tp, (void *)&ks, (void *)&ids, (void *)&keys,
+                    (void *)&kvalid, (void *)&keymask, (void *)&bits, (void *)&counts, (void *)&barrier,
+                    (void *)&count};
+    return cudaLaunchCooperativeKernel((const void *)kern, dim3((unsigned)grid), dim3(T_THREADS), args, (size_t)smem, st);
 }
 
 template <int KB>
 cudaError_t launch_rp_items(int items, long long n, const SrcCols &sc, const TPlan &tp, const KeySrc &ks, int *ids,
-                            void *keys, uint8_t *kvalid, unsigned long long *keymask, unsigned long long *status,
-                            unsigned *counter, long long *count, int num_sms, cudaStream_t st)
+                            void *keys, uint8_t *kvalid, unsigned long long *keymask, void *scratch, long long *count,
+                            int num_sms, cudaStream_t st)
 {
     switch (items) {
-    case 16: return launch_rp_t<KB, 16>(n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
-    case 8: return launch_rp_t<KB, 8>(n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
-    case 4: return launch_rp_t<KB, 4>(n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
-    case 2: return launch_rp_t<KB, 2>(n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
-    default: return launch_rp_t<KB, 1>(n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
+    case 32: return launch_rp_t<KB, 32>(n, sc, tp, ks, ids, keys, kvalid, keymask, scratch, count, num_sms, st);
+    case 16: return launch_rp_t<KB, 16>(n, sc, tp, ks, ids, keys, kvalid, keymask, scratch, count, num_sms, st);
+    case 8: return launch_rp_t<KB, 8>(n, sc, tp, ks, ids, keys, kvalid, keymask, scratch, count, num_sms, st);
+    case 4: return launch_rp_t<KB, 4>(n, sc, tp, ks, ids, keys, kvalid, keymask, scratch, count, num_sms, st);
+    case 2: return launch_rp_t<KB, 2>(n, sc, tp, ks, ids, keys, kvalid, keymask, scratch, count, num_sms, st);
+    default: return launch_rp_t<KB, 1>(n, sc, tp, ks, ids, keys, kvalid, keymask, scratch, count, num_sms, st);
     }
 }
 
 cudaError_t launch_rp(int kb, int items, long long n, const SrcCols &sc, const TPlan &tp, const KeySrc &ks, int *ids,
-                      void *keys, uint8_t *kvalid, unsigned long long *keymask, unsigned long long *status,
-                      unsigned *counter, long long *count, int num_sms, cudaStream_t st)
+                      void *keys, uint8_t *kvalid, unsigned long long *keymask, void *scratch, long long *count,
+                      int num_sms, cudaStream_t st)
 {
-    if (kb == 8)
-        return launch_rp_items<8>(items, n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
-    return launch_rp_items<4>(items, n, sc, tp, ks, ids, keys, kvalid, keymask, status, counter, count, num_sms, st);
+    if (kb == 8) return launch_rp_items<8>(items, n, sc, tp, ks, ids, keys, kvalid, keymask, scratch, count, num_sms, st);
+    return launch_rp_items<4>(items, n, sc, tp, ks, ids, keys, kvalid, keymask, scratch, count, num_sms, st);
 }
 }  // namespace
 
@@ -830,24 +967,18 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
     FilterOut o{out_ids, out_keys, out_kvalid, out_vals, keymask, extreme, nullptr, nullptr,
                 (unsigned *)scratch, out_count};
     if (one_pass) {
-        // ordered R': one pass with the decoupled look-back (predicate
-        // columns staged; survivors' keys gathered)
+        // ordered R': one launch, predicate columns read once, survivors'
+        // keys gathered (filter_rp_kernel)
         SrcCols sc1 = sc;
         sc1.n = n_pred_src;   // predicate columns come first in the source list
-        const int it1 = layout(sc1, 16);
+        const int it1 = layout(sc1, NG_RP_ITEMS);
         if (!it1) return cudaErrorInvalidValue;
         SrcPlan sp1 = sp;
         sp1.key0 = sp1.key0v = sp1.key1 = sp1.key1v = sp1.val = sp1.valv = -1;
         TPlan tp1 = tp;
         resolve(sc1, sp1, tp1);
-        const long long tiles = (n + T_THREADS * it1 - 1) / (T_THREADS * it1);
-        unsigned long long *status = (unsigned long long *)((char *)scratch + 1024);
-        if (!prezeroed) {
-            e = cudaMemsetAsync((char *)scratch + 1024, 0, (size_t)tiles * 8, st);
-            if (e != cudaSuccess) return e;
-        }
-        e = launch_rp(k, it1, n, sc1, tp1, key, out_ids, out_keys, out_kvalid, keymask, status, (unsigned *)scratch,
-                      out_count, num_sms, st);
+        e = launch_rp(k, it1, n, sc1, tp1, key, out_ids, out_keys, out_kvalid, keymask, scratch, out_count, num_sms,
+                      st);
         ++*launches;
         return e;
     }

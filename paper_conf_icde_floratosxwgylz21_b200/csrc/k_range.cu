@@ -472,7 +472,7 @@ static void scan_dir(const void *v, long long N, long long *out, long long *bagg
     *launches += 3;
 }
 
-size_t index_aux_scratch_bytes(long long n) { return (size_t)((n + P_BLOCK - 1) / P_BLOCK + 1) * 16; }
+size_t index_aux_scratch_bytes(long long n) { return (size_t)((n + 1024 - 1) / 1024 + 1) * 16; }
 
 // ---- per-key group aggregates: segmented inclusive scan over the sorted
 // index, segments = runs of equal keys.  Pairs (f, v): f = a run starts in
@@ -498,8 +498,11 @@ __device__ __forceinline__ SegPair<AGG> warp_seg_scan(SegPair<AGG> x, int lane)
     return x;
 }
 
-// One block of P_BLOCK sorted (key, payload) rows scanned in order, 256 at a
-// time; WRITE: write grp[e], else only the block's total pair (bagg).
+// One block of G_BLOCK sorted (key, payload) rows scanned in order, 256 at a
+// time; WRITE: write grp[e], else only the block's total pair (bv, bf).
+// Small blocks (4 rows of 256): the scan is latency-bound, so many CTAs.
+constexpr int G_ITEMS = 4;
+constexpr int G_BLOCK = P_THREADS * G_ITEMS;
 template <typename K, typename V, int AGG, bool WRITE>
 __global__ void __launch_bounds__(P_THREADS) seg_block_kernel(const K *__restrict__ keys, const V *__restrict__ v,
                                                               long long N, long long *__restrict__ bv,
@@ -509,10 +512,10 @@ __global__ void __launch_bounds__(P_THREADS) seg_block_kernel(const K *__restric
     __shared__ int s_wf[P_THREADS / 32];
     __shared__ SegPair<AGG> s_carry;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const long long b0 = blockIdx.x * (long long)P_BLOCK;
+    const long long b0 = blockIdx.x * (long long)G_BLOCK;
     if (threadIdx.x == 0) s_carry = WRITE ? SegPair<AGG>{bv[blockIdx.x], 0} : SegPair<AGG>{ident<AGG>(), 0};
     __syncthreads();
-    for (int j = 0; j < P_ITEMS; j++) {
+    for (int j = 0; j < G_ITEMS; j++) {
         const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
         SegPair<AGG> x{ident<AGG>(), 0};
         if (e < N) x = SegPair<AGG>{(long long)v[e], (e == 0 || keys[e] != keys[e - 1]) ? 1 : 0};
@@ -536,16 +539,38 @@ __global__ void __launch_bounds__(P_THREADS) seg_block_kernel(const K *__restric
     }
 }
 
-// exclusive scan of the block pairs (one CTA, sequentially: blocks are few)
+// exclusive scan of the block pairs: one CTA of 1024 threads, chunks of
+// 1024 pairs in order (segmented warp scans + a scan of the warp totals)
 template <int AGG>
-__global__ void seg_block_scan_kernel(long long *__restrict__ bv, const int *__restrict__ bf, long long nb)
+__global__ void __launch_bounds__(1024) seg_block_scan_kernel(long long *__restrict__ bv, const int *__restrict__ bf,
+                                                              long long nb)
 {
-    if (threadIdx.x != 0) return;
-    SegPair<AGG> run{ident<AGG>(), 0};
-    for (long long b = 0; b < nb; b++) {
-        const SegPair<AGG> x{bv[b], bf[b]};
-        bv[b] = run.v;
-        run = seg_comb<AGG>(run, x);
+    __shared__ long long s_wv[32];
+    __shared__ int s_wf[32];
+    __shared__ SegPair<AGG> s_carry;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (threadIdx.x == 0) s_carry = SegPair<AGG>{ident<AGG>(), 0};
+    __syncthreads();
+    for (long long b0 = 0; b0 < nb; b0 += 1024) {
+        const long long b = b0 + threadIdx.x;
+        const SegPair<AGG> x = b < nb ? SegPair<AGG>{bv[b], bf[b]} : SegPair<AGG>{ident<AGG>(), 0};
+        const SegPair<AGG> incl = warp_seg_scan<AGG>(x, lane);
+        if (lane == 31) {
+            s_wv[warp] = incl.v;
+            s_wf[warp] = incl.f;
+        }
+        __syncthreads();
+        SegPair<AGG> wpre{ident<AGG>(), 0};
+        for (int w = 0; w < warp; w++) wpre = seg_comb<AGG>(wpre, SegPair<AGG>{s_wv[w], s_wf[w]});
+        const SegPair<AGG> carry = s_carry;
+        // exclusive: everything before b = carry (+) warps before (+) lanes before
+        SegPair<AGG> up{__shfl_up_sync(FULL, incl.v, 1), __shfl_up_sync(FULL, incl.f, 1)};
+        if (lane == 0) up = SegPair<AGG>{ident<AGG>(), 0};
+        const SegPair<AGG> ex = seg_comb<AGG>(carry, seg_comb<AGG>(wpre, up));
+        __syncthreads();
+        if (b < nb) bv[b] = ex.v;
+        if (threadIdx.x == 1023) s_carry = seg_comb<AGG>(carry, seg_comb<AGG>(wpre, incl));
+        __syncthreads();
     }
 }
 
@@ -553,12 +578,12 @@ template <typename K, typename V, int AGG>
 static void seg_scan(const void *keys, const void *v, long long N, long long *grp, void *scratch, cudaStream_t st,
                      long long *launches)
 {
-    const long long nb = (N + P_BLOCK - 1) / P_BLOCK;
+    const long long nb = (N + G_BLOCK - 1) / G_BLOCK;
     long long *bv = (long long *)scratch;
     int *bf = (int *)(bv + nb + 1);
     seg_block_kernel<K, V, AGG, false><<<(unsigned)nb, P_THREADS, 0, st>>>((const K *)keys, (const V *)v, N, bv, bf,
                                                                            nullptr);
-    seg_block_scan_kernel<AGG><<<1, 32, 0, st>>>(bv, bf, nb);
+    seg_block_scan_kernel<AGG><<<1, 1024, 0, st>>>(bv, bf, nb);
     seg_block_kernel<K, V, AGG, true><<<(unsigned)nb, P_THREADS, 0, st>>>((const K *)keys, (const V *)v, N, bv, bf,
                                                                           grp);
     *launches += 3;

@@ -443,7 +443,9 @@ cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *
     DigitList dl{};
     dl.n = np;
     for (int p = 0; p < np; p++) dl.shift[p] = shifts[p];
-    long long blocks = (n + 255) / 256;
+    // >= 4096 keys per CTA: the shared bins' init / merge and the last CTA's
+    // scan stay small next to the counting
+    long long blocks = (n + 4095) / 4096;
     if (blocks > (long long)num_sms * 8) blocks = (long long)num_sms * 8;
     if (blocks < 1) blocks = 1;
     if (rb == 8) {

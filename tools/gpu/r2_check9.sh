@@ -1,0 +1,6 @@
+set -x
+python -c "import __graft_entry__ as g; g.build()"
+python tools/time_filter.py
+NESTGPU_LIB=vlib/rp16.so python tools/time_filter.py
+NESTGPU_FILTER_TWO_PASS=1 python tools/time_filter.py
+timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_tpch.py tests/test_gpu_typej.py -x -q > gpurun_out/pytest9.log 2>&1; echo rc=$?; tail -3 gpurun_out/pytest9.log
