@@ -1,0 +1,5 @@
+python -c "import __graft_entry__ as g; g.build()"
+for tool in memcheck racecheck synccheck initcheck; do
+  echo "== compute-sanitizer --tool $tool python tools/sanitize_run.py"
+  timeout 1500 compute-sanitizer --tool $tool python tools/sanitize_run.py 2>&1 | tail -3
+done

@@ -2,8 +2,10 @@
 filter (ordered / unordered), sort + histogram, range (short, long, prefix
 aggregates), nested loop (all agg kinds, both R-block shapes), dedup (iota /
 group), finalize, gather, minmax, type-J collections + IN + materialise,
-cost-model calibration (fills), and the radix-sort variants (pre-narrowed
-64-bit keys, 9-bit digit passes, keys without payload)."""
+cost-model calibration (fills), the radix-sort variants (pre-narrowed
+64-bit keys, 9-bit digit passes, keys without payload), and (round 2) the
+exact split SUM/AVG, the one-launch ordered R' filter with and without
+predicates, group aggregates, staged small results and a window put."""
 import os
 import sys
 
@@ -64,6 +66,36 @@ for keys, dt, pay in ((rng.integers(0, 1 << 29, 70001) + (7 << 40), "int64", Tru
     enc = (keys.astype(np.int64).view(np.uint64) ^ np.uint64(1 << 63)) if kb == 8 else \
         (keys.astype(np.int32).view(np.uint32) ^ np.uint32(1 << 31))
     bad += not np.array_equal(got.view(enc.dtype), np.sort(enc))
+# round 2: exact split SUM/AVG of 64-bit payloads (both kernels), the
+# ordered R' filter without predicates, '=' MIN over a large index (group
+# aggregates), a result stored into a peer-gather window
+A = (1 << 62) + (1 << 61)
+keys = np.repeat(np.arange(3001, dtype=np.int64) * 3, 2)
+vals = np.empty(6002, np.int64)
+vals[0::2], vals[1::2] = A + rng.integers(-9, 9, 3001), -A + rng.integers(-9, 9, 3001)
+perm = rng.permutation(6002)
+tw = {"R": {"col1": rng.integers(-3, 9010, 5003).astype(np.int64), "col2": rng.integers(-99, 99, 5003).astype(np.int64)},
+      "S": {"col1": keys[perm], "col2": vals[perm]}}
+Rw = eng.load_table(tw["R"], dtypes={"col1": "int64", "col2": "int64"})
+Sw = eng.load_table(tw["S"], dtypes={"col1": "int64", "col2": "decimal"})
+for op in ("=", ">", "!="):
+    for agg in ("sum", "avg"):
+        plan = make_plan(op, agg, "<")
+        for mode in ("bnl", "index"):
+            idx = eng.index_for_plan(plan, Sw) if mode == "index" else -1
+            g = eng.result_to_numpy(eng.exec(plan, Rw, Sw, index=idx, emit_all=True))
+            ref = oracle.evaluate(tw, plan)
+            bad += not np.array_equal(g["value"], ref["value"][ref["in_rp"].astype(bool)])
+tn = query1.tables(n_r=70001, n_s=90001, key_hi=5000, val_hi=50, seed=9)
+Rn, Sn = eng.load_table(tn["R"]), eng.load_table(tn["S"])
+plan = make_plan("=", "min", "=")
+res = eng.exec(plan, Rn, Sn, index=eng.index_for_plan(plan, Sn))
+win, _ = eng.window_create(res.n_rows + 5)
+eng.result_put(res, win, res.n_rows + 5, 0)
+er, ev = oracle.survivors(oracle.evaluate(tn, plan))
+wi, wv = eng.window_tensors(win, res.n_rows + 5, res.n_rows)
+bad += not (np.array_equal(wi.cpu().numpy(), er) and np.array_equal(wv.cpu().numpy(), ev))
+eng.window_free(win)
 eng.cost_calibrate(1 << 16)
 print("sanitize workload done, mismatches:", bad)
 sys.exit(1 if bad else 0)
