@@ -464,8 +464,14 @@ nestgpu_status nestgpu_result_put(nestgpu_ctx *ctx, const nestgpu_result *res, v
  *   NESTGPU_OPT_BNL_SHAPE (value 0/1/2): the nested-loop kernel's R-block
  *     shape -- 0 automatic (from |R'|, |S'|), 1 full blocks, 2 warp-split.
  *     Results are identical; tests use it to cover both shapes on one input.
+ *   NESTGPU_OPT_GRAPHS (value 0/1, default 1; env NESTGPU_GRAPHS=0 at
+ *     create): exec's launch sequence is captured into a CUDA graph the first
+ *     time a (plan, columns, index, arena state) combination is seen and
+ *     replayed afterwards (one graph launch instead of one launch per
+ *     kernel; not with dedup, profiling or the malloc ablation).  Results
+ *     are identical either way.
  * Errors: INVALID (unknown option). */
-enum { NESTGPU_OPT_MALLOC_SCRATCH = 1, NESTGPU_OPT_BNL_SHAPE = 2 };
+enum { NESTGPU_OPT_MALLOC_SCRATCH = 1, NESTGPU_OPT_BNL_SHAPE = 2, NESTGPU_OPT_GRAPHS = 3 };
 nestgpu_status nestgpu_set_option(nestgpu_ctx *ctx, int32_t option, int64_t value);
 
 /* Per-stage device times (ms, CUDA events on the context stream) of the last

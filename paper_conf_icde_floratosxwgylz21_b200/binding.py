@@ -38,6 +38,7 @@ SYMBOLS = ("nestgpu_create", "nestgpu_destroy", "nestgpu_last_error", "nestgpu_l
 STRATEGIES = ("nested_loop", "index", "nested_loop_cached", "index_cached")
 OPT_MALLOC_SCRATCH = 1
 OPT_BNL_SHAPE = 2
+OPT_GRAPHS = 3
 
 
 class NestGPUError(RuntimeError):

@@ -22,6 +22,7 @@
 #include <mutex>
 #include <string>
 #include <tuple>
+#include <unordered_map>
 #include <chrono>
 #include <cstdlib>
 #include <utility>
@@ -109,6 +110,17 @@ struct nestgpu_ctx {
     std::vector<void *> mallocs;
     int bnl_shape;   // NESTGPU_OPT_BNL_SHAPE (test knob): 0 automatic, 1 full, 2 warp-split
     cudaEvent_t ev[NESTGPU_N_STAGES][2];
+    // CUDA graphs of exec launch sequences (NESTGPU_OPT_GRAPHS, default on):
+    // key = every argument that determines the sequence (plan, column /
+    // index addresses and sizes, arena state); kernels = launches per replay
+    // (-1: the sequence could not be captured, run it directly)
+    struct GraphEntry {
+        cudaGraphExec_t exec;
+        long long kernels;
+    };
+    bool graphs_on;
+    std::unordered_map<std::string, GraphEntry> graphs;
+    cudaStream_t cap_stream;   // private stream the sequences are captured on
     // NESTGPU_TRACE=1 (diagnostics): host time of each step of an exec,
     // printed to stderr when the exec returns
     bool trace;
@@ -435,6 +447,11 @@ nestgpu_status nestgpu_create(int device, void *d_arena, size_t arena_bytes, voi
     c->profiling = false;
     c->malloc_scratch = false;
     c->bnl_shape = 0;
+    c->cap_stream = nullptr;
+    {
+        const char *gr = getenv("NESTGPU_GRAPHS");
+        c->graphs_on = !(gr && gr[0] == '0');
+    }
     {
         const char *tr = getenv("NESTGPU_TRACE");
         c->trace = tr && tr[0] == '1';
@@ -472,6 +489,9 @@ nestgpu_status nestgpu_destroy(nestgpu_ctx *c)
     }
     cudaFreeHost(c->pinned);
     cudaFreeHost(c->stage);
+    for (auto &kv : c->graphs)
+        if (kv.second.exec) cudaGraphExecDestroy(kv.second.exec);
+    if (c->cap_stream) cudaStreamDestroy(c->cap_stream);
     delete c;
     return NESTGPU_OK;
 }
@@ -866,6 +886,142 @@ nestgpu_status nestgpu_index_create_empty(nestgpu_ctx *c, int64_t n, int32_t key
     return NESTGPU_OK;
 }
 
+// ---------------------------------------------------------------- exec graphs
+}  // extern "C"
+namespace {
+template <typename T>
+void kput(std::string &k, const T &v)
+{
+    k.append((const char *)&v, sizeof v);
+}
+
+bool graph_ok(const nestgpu_ctx *c, const nestgpu_plan *P, const IndexRec *)
+{
+    // dedup synchronises mid-sequence; profiling / tracing record host-side
+    // state per call; the malloc ablation allocates per call
+    return c->graphs_on && !P->dedup && !c->profiling && !c->malloc_scratch;
+}
+
+// Everything the exec's launch sequence depends on: the plan (predicates by
+// value), every referenced column's address / validity / rows / type, the
+// index record (arrays, size, widths, aux arrays), the arena state (scratch
+// addresses follow from it) and the knobs.  Equal keys => identical launches.
+std::string exec_graph_key(const nestgpu_ctx *c, const nestgpu_plan *P, const IndexRec *ix, bool wide)
+{
+    std::string k;
+    k.reserve(512);
+    nestgpu_plan q = *P;
+    q.outer_preds = nullptr;
+    q.inner_preds = nullptr;
+    kput(k, q);
+    for (int i = 0; i < P->n_outer_preds; i++) kput(k, P->outer_preds[i]);
+    for (int i = 0; i < P->n_inner_preds; i++) kput(k, P->inner_preds[i]);
+    auto col = [&](int32_t id) {
+        kput(k, id);
+        if (id < 0 || id >= (int32_t)c->cols.size() || !c->cols[id].alive) return;
+        const Column &x = c->cols[id];
+        kput(k, x.d);
+        kput(k, x.valid);
+        kput(k, x.n);
+        kput(k, x.dtype);
+    };
+    for (int i = 0; i < P->n_key_cols; i++) {
+        col(P->outer_key_cols[i]);
+        col(P->inner_key_cols[i]);
+    }
+    col(P->outer_cmp_col);
+    col(P->agg_col);
+    for (int i = 0; i < P->n_outer_preds; i++) {
+        col(P->outer_preds[i].col);
+        col(P->outer_preds[i].rhs_col);
+    }
+    for (int i = 0; i < P->n_inner_preds; i++) {
+        col(P->inner_preds[i].col);
+        col(P->inner_preds[i].rhs_col);
+    }
+    if (ix) {
+        kput(k, ix->keys);
+        kput(k, ix->payload);
+        kput(k, ix->n);
+        kput(k, ix->kb);
+        kput(k, ix->vb);
+        for (int i = 0; i < 6; i++) {
+            kput(k, ix->aux_pre[i]);
+            kput(k, ix->aux_suf[i]);
+        }
+    }
+    kput(k, c->lo);
+    kput(k, c->size);
+    kput(k, c->base);
+    kput(k, c->bnl_shape);
+    kput(k, wide);
+    return k;
+}
+
+// Replay the captured launch sequence for `key`, capturing it first (and
+// running it once) when it is new.  A sequence that cannot be captured
+// (e.g. a launch kind the graph API refuses) is remembered and run directly.
+template <typename F>
+nestgpu_status run_graph(nestgpu_ctx *c, const std::string &key, F &enqueue)
+{
+    auto it = c->graphs.find(key);
+    if (it == c->graphs.end()) {
+        const long long l0 = c->launches;
+        const std::string err0 = c->err;
+        // capture on the context's private stream (the caller's may be the
+        // legacy default stream, which cannot be captured); the graph is
+        // then launched on the caller's stream
+        if (!c->cap_stream && cudaStreamCreateWithFlags(&c->cap_stream, cudaStreamNonBlocking) != cudaSuccess) {
+            cudaGetLastError();
+            c->cap_stream = nullptr;
+            c->graphs_on = false;
+            return enqueue();
+        }
+        cudaStream_t user = c->stream;
+        c->stream = c->cap_stream;
+        if (cudaStreamBeginCapture(c->stream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+            cudaGetLastError();
+            c->stream = user;
+            c->graphs.emplace(key, nestgpu_ctx::GraphEntry{nullptr, -1});
+            return enqueue();
+        }
+        const nestgpu_status st = enqueue();
+        cudaGraph_t g = nullptr;
+        cudaError_t e = cudaStreamEndCapture(c->stream, &g);
+        c->stream = user;
+        cudaGraphExec_t ge = nullptr;
+        if (st == NESTGPU_OK && e == cudaSuccess && g) e = cudaGraphInstantiate(&ge, g, 0);
+        if (g) cudaGraphDestroy(g);
+        const long long kernels = c->launches - l0;
+        c->launches = l0;
+        if (c->graphs.size() >= 64) {
+            for (auto &kv : c->graphs)
+                if (kv.second.exec) cudaGraphExecDestroy(kv.second.exec);
+            c->graphs.clear();
+        }
+        if (st != NESTGPU_OK || e != cudaSuccess || !ge) {
+            if (c->trace)
+                fprintf(stderr, "[nestgpu trace] graph capture failed: status %d, %s, %s\n", (int)st,
+                        cudaGetErrorString(e), c->err.c_str());
+            cudaGetLastError();   // clear the capture error; run this sequence directly from now on
+            c->err = err0;
+            c->graphs.emplace(key, nestgpu_ctx::GraphEntry{nullptr, -1});
+            return enqueue();
+        }
+        it = c->graphs.emplace(key, nestgpu_ctx::GraphEntry{ge, kernels}).first;
+    }
+    if (!it->second.exec) {
+        htrace(c, "graph:direct");
+        return enqueue();
+    }
+    htrace(c, "graph:replay");
+    CUDA_TRY(c, cudaGraphLaunch(it->second.exec, c->stream));
+    c->launches += it->second.kernels;
+    return NESTGPU_OK;
+}
+}  // namespace
+extern "C" {
+
 nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, nestgpu_result *out)
 {
     if (!c || !P || !out) return fail(c, NESTGPU_ERR_INVALID, "exec: null argument");
@@ -998,87 +1154,15 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
             return fail(c, NESTGPU_ERR_OOM, "arena exhausted (dedup buffers for |R|=%lld)", (long long)nR);
     }
 
-    // ------------------------------------------------------------ a2: R'
-    prof_begin(c, 5);
-    prof_begin(c, 0);
-    ng::ValSrc none{nullptr, nullptr, 0};
-    {   // every small scratch region of this exec zeroed by ONE kernel
-        ng::FillList fl;
-        fl.add(counts, 48);
-        fl.add(rmask, 8, 0xff);    // [6] AND identity
-        fl.add(counts + 7, 8);     // [7] OR
-        fl.add(counts + 8, 64);
-        fl.add(fscr, ng::filter_zero_bytes(nR, true));
-        if (fscr_s) fl.add(fscr_s, ng::filter_zero_bytes(nS, false));
-        fl.add(fscr_f, ng::finalize_scratch_bytes(nR));
-        fl.add(kscr, ix ? 256 : ng::bnl_scratch_bytes(nR));
-        if (wide) fl.add(acc_hi, (size_t)nR * 8);
-        if (!ix && nR <= SMALL_ROWS) {   // small R: the partials' identity init rides on the fill
-            const long long acc0 = P->agg == NG_MIN ? LLONG_MAX : (P->agg == NG_MAX ? LLONG_MIN : 0);
-            fl.add_words(acc, (size_t)nR * 8, (unsigned long long)acc0);
-            fl.add(cnt, (size_t)nR * 8);
-        }
-        // the staged rows (copied to the host even when fewer survive):
-        // defined contents for compute-sanitizer's initcheck
-        const long long kr = std::min<long long>(nR, (long long)(STAGE_BYTES / (8 * w8 + 2)));
-        for (size_t f = 0; f < w8; f++) fl.add(rblk + (size_t)nR * 8 * f, (size_t)kr * 8);
-        fl.add(o_valid, (size_t)kr);
-        fl.add(o_pass, (size_t)kr);
-        htrace(c, "alloc");
-        CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
-        htrace(c, "fill");
-    }
-    CUDA_TRY(c, ng::launch_filter(nR, ops, rks, kb, none, 0, 0, 0, ids, rkeys, rkvalid, nullptr,
-                                  P->dedup ? rmask : nullptr, nullptr, fscr, d_nrp, c->stream, &c->launches, true));
-    htrace(c, "rfilter");
-    prof_end(c, 0);
-
-    // The keys the subquery kernels evaluate: every R' key, or (dedup) each
-    // distinct R' key once -- P:331's cache keyed by the passed-in parameter.
-    const void *eval_keys = rkeys;
-    const long long *d_neval = d_nrp;
-    long long n_eval = nR;
-    long long n_distinct = -1;
-    if (P->dedup) {
-        prof_begin(c, 2);
-        CUDA_TRY(c, cudaMemcpyAsync(c->pinned, counts, 64, cudaMemcpyDeviceToHost, c->stream));
-        CUDA_TRY(c, cudaStreamSynchronize(c->stream));
-        long long nrp;
-        unsigned long long kand, kor;
-        memcpy(&nrp, c->pinned, 8);
-        memcpy(&kand, c->pinned + 12, 8);
-        memcpy(&kor, c->pinned + 14, 8);
-        int shifts[8], rb = 8;
-        const int np = plan_sort_passes(kb, kand, kor, nrp, shifts, &rb);
-        CUDA_TRY(c, ng::launch_iota(pos, nrp, c->stream, &c->launches));
-        CUDA_TRY(c, ng::launch_digit_hist(kb, rkeys, nrp, shifts, np, hist, dbase, c->num_sms, c->stream,
-                                          &c->launches, rb));
-        void *ck = rkeys, *ok = tkeys;
-        int *cv = pos, *ov = tpos;
-        const bool narrow = kb == 8 && np >= 2 && ((kand ^ kor) >> 32) == 0;   // as in build_index
-        for (int p = 0; p < np; p++) {
-            const int kin = narrow && p > 0 ? 4 : kb, kout = narrow && p < np - 1 ? 4 : kb;
-            CUDA_TRY(c, ng::launch_radix_pass_x(kin, kout, 4, ck, ok, cv, ov, nrp, shifts[p], dbase + p * (1 << rb),
-                                                sscr, (unsigned)(kand >> 32), c->stream, &c->launches, rb));
-            std::swap(ck, ok);
-            std::swap(cv, ov);
-        }
-        CUDA_TRY(c, ng::launch_group(kb, ck, cv, nrp, ukeys, map, d_u, gscr, c->stream, &c->launches));
-        CUDA_TRY(c, cudaMemcpyAsync(c->pinned, d_u, 8, cudaMemcpyDeviceToHost, c->stream));
-        CUDA_TRY(c, cudaStreamSynchronize(c->stream));
-        memcpy(&n_distinct, c->pinned, 8);
-        eval_keys = ukeys;
-        d_neval = d_u;
-        n_eval = n_distinct;
-        prof_end(c, 2);
-    }
-
-    // ------------------------------------------------------------ a3 / a5-a7
+    // Index aux arrays (built on first use and kept with the index) are
+    // built here, outside the per-exec launch sequence: that sequence may be
+    // a replayed CUDA graph, and a build changes host state (arena tail,
+    // the index record) that a replay would not.
+    const long long *pre = nullptr, *suf = nullptr;
     if (ix) {
         // Index-pruned evaluation (NEXT 3): prefix / suffix aggregates of the
         // payload make non-equality and SUM/AVG ranges O(1); built once per
         // index and aggregate kind, kept with the index.
-        const long long *pre = nullptr, *suf = nullptr;
         if (value_agg && (P->corr_op != NG_EQ || P->agg == NG_SUM || P->agg == NG_AVG)) {
             const int kind = P->agg == NG_MIN ? 0 : (P->agg == NG_MAX ? 1 : (wide ? 3 : 2));
             const int akind = kind == 0 ? ng::MIN : (kind == 1 ? ng::MAX : ng::SUM);
@@ -1118,77 +1202,169 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
             }
             pre = ix->aux_pre[kind];
         }
-        prof_begin(c, 3);
-        const bool split = wide && pre && P->agg != NG_MIN && P->agg != NG_MAX;
-        CUDA_TRY(c, ng::launch_range_agg(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, ix->keys, ix->payload,
-                                         ix->n, pre, split ? nullptr : suf, acc, cnt, kscr, c->stream, &c->launches,
-                                         split ? suf : nullptr, split ? acc_hi : nullptr, true));
-        htrace(c, "range");
-        prof_end(c, 3);
-    } else {
-        prof_begin(c, 1);
-        ng::ValSrc vs{nullptr, nullptr, 0};
-        if (value_agg) { vs.c = ac->d; vs.v = ac->valid; vs.w = vb; }
-        CUDA_TRY(c, ng::launch_filter(nS, ips, sks, kb, vs, vb, 1, value_agg ? 1 : 0, nullptr, skeys, nullptr, svals,
-                                      nullptr, value_agg ? extreme : nullptr, fscr_s, d_nsp, c->stream,
-                                      &c->launches, true));
-        htrace(c, "sfilter");
-        if (nR > SMALL_ROWS)
-            CUDA_TRY(c, ng::launch_init_partials(n_eval, d_neval, P->agg, acc, cnt, c->stream, &c->launches));
-        htrace(c, "init");
-        prof_end(c, 1);
-        prof_begin(c, 3);
-        CUDA_TRY(c, ng::launch_bnl(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, nS, d_nsp, skeys, svals,
-                                   extreme, acc, cnt, kscr, c->num_sms, c->bnl_shape, c->stream, &c->launches,
-                                   wide ? acc_hi : nullptr, true));
-        htrace(c, "bnl");
-        prof_end(c, 3);
     }
 
-    // ------------------------------------------------------------ a8 + a9
-    prof_begin(c, 4);
-    ng::FinalizeArgs fa{};
-    fa.n_rp_max = nR;
-    fa.d_nrp = d_nrp;
-    fa.ids = ids;
-    fa.map = map;
-    fa.kvalid = rkvalid;
-    fa.acc = acc;
-    fa.cnt = cnt;
-    fa.acc_hi = wide ? acc_hi : nullptr;
-    fa.overflow = (unsigned long long *)(counts + 8);
-    fa.x_col = xc ? xc->d : nullptr;
-    fa.x_valid = xc ? xc->valid : nullptr;
-    fa.x_w = xc ? dtype_width(xc->dtype) : 4;
-    fa.agg = P->agg;
-    fa.outer_op = P->outer_op;
-    fa.a = P->lhs_mult;
-    fa.b = P->rhs_mult;
-    fa.row_id_base = P->row_id_base;
-    fa.emit_all = P->emit_all;
-    fa.out_ids = o_ids;
-    fa.out_vals = o_vals;
-    fa.out_sum = o_sum;
-    fa.out_cnt = o_cnt;
-    fa.out_valid = o_valid;
-    fa.out_passed = o_pass;
-    fa.out_count = d_out;
-    fa.scratch = fscr_f;
-    CUDA_TRY(c, ng::launch_finalize(fa, c->stream, &c->launches, true));
-    htrace(c, "finalize");
-    prof_end(c, 4);
-    prof_end(c, 5);
-    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, counts, 72, cudaMemcpyDeviceToHost, c->stream));
-    // the first rows of every result field, staged on the host before the
-    // one synchronisation (8-byte fields, then the two byte fields)
     const long long krows = std::min<long long>(nR, (long long)(STAGE_BYTES / (8 * w8 + 2)));
-    if (krows == nR && krows > 0) {   // the whole result block fits: one copy, same layout
-        CUDA_TRY(c, cudaMemcpyAsync(c->stage, rblk, (size_t)nR * (8 * w8 + 2), cudaMemcpyDeviceToHost, c->stream));
-    } else if (krows > 0) {
-        CUDA_TRY(c, cudaMemcpy2DAsync(c->stage, (size_t)krows * 8, rblk, (size_t)nR * 8, (size_t)krows * 8, w8,
-                                      cudaMemcpyDeviceToHost, c->stream));
-        CUDA_TRY(c, cudaMemcpy2DAsync(c->stage + (size_t)krows * 8 * w8, (size_t)krows, o_valid, (size_t)nR,
-                                      (size_t)krows, 2, cudaMemcpyDeviceToHost, c->stream));
+    long long n_distinct = -1;
+    // Everything enqueued from here to the result copies: run directly, or
+    // captured once into a CUDA graph and replayed (§17) -- a repeated small
+    // query then costs one graph launch instead of one launch per kernel.
+    auto enqueue = [&]() -> nestgpu_status {
+        // ------------------------------------------------------------ a2: R'
+        prof_begin(c, 5);
+        prof_begin(c, 0);
+        ng::ValSrc none{nullptr, nullptr, 0};
+        {   // every small scratch region of this exec zeroed by ONE kernel
+            ng::FillList fl;
+            fl.add(counts, 48);
+            fl.add(rmask, 8, 0xff);    // [6] AND identity
+            fl.add(counts + 7, 8);     // [7] OR
+            fl.add(counts + 8, 64);
+            fl.add(fscr, ng::filter_zero_bytes(nR, true));
+            if (fscr_s) fl.add(fscr_s, ng::filter_zero_bytes(nS, false));
+            fl.add(fscr_f, ng::finalize_scratch_bytes(nR));
+            fl.add(kscr, ix ? 256 : ng::bnl_scratch_bytes(nR));
+            if (wide) fl.add(acc_hi, (size_t)nR * 8);
+            if (!ix && nR <= SMALL_ROWS) {   // small R: the partials' identity init rides on the fill
+                const long long acc0 = P->agg == NG_MIN ? LLONG_MAX : (P->agg == NG_MAX ? LLONG_MIN : 0);
+                fl.add_words(acc, (size_t)nR * 8, (unsigned long long)acc0);
+                fl.add(cnt, (size_t)nR * 8);
+            }
+            // the staged rows (copied to the host even when fewer survive):
+            // defined contents for compute-sanitizer's initcheck
+            const long long kr = std::min<long long>(nR, (long long)(STAGE_BYTES / (8 * w8 + 2)));
+            for (size_t f = 0; f < w8; f++) fl.add(rblk + (size_t)nR * 8 * f, (size_t)kr * 8);
+            fl.add(o_valid, (size_t)kr);
+            fl.add(o_pass, (size_t)kr);
+            htrace(c, "alloc");
+            CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
+            htrace(c, "fill");
+        }
+        CUDA_TRY(c, ng::launch_filter(nR, ops, rks, kb, none, 0, 0, 0, ids, rkeys, rkvalid, nullptr,
+                                      P->dedup ? rmask : nullptr, nullptr, fscr, d_nrp, c->stream, &c->launches, true));
+        htrace(c, "rfilter");
+        prof_end(c, 0);
+
+        // The keys the subquery kernels evaluate: every R' key, or (dedup) each
+        // distinct R' key once -- P:331's cache keyed by the passed-in parameter.
+        const void *eval_keys = rkeys;
+        const long long *d_neval = d_nrp;
+        long long n_eval = nR;
+        if (P->dedup) {
+            prof_begin(c, 2);
+            CUDA_TRY(c, cudaMemcpyAsync(c->pinned, counts, 64, cudaMemcpyDeviceToHost, c->stream));
+            CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+            long long nrp;
+            unsigned long long kand, kor;
+            memcpy(&nrp, c->pinned, 8);
+            memcpy(&kand, c->pinned + 12, 8);
+            memcpy(&kor, c->pinned + 14, 8);
+            int shifts[8], rb = 8;
+            const int np = plan_sort_passes(kb, kand, kor, nrp, shifts, &rb);
+            CUDA_TRY(c, ng::launch_iota(pos, nrp, c->stream, &c->launches));
+            CUDA_TRY(c, ng::launch_digit_hist(kb, rkeys, nrp, shifts, np, hist, dbase, c->num_sms, c->stream,
+                                              &c->launches, rb));
+            void *ck = rkeys, *ok = tkeys;
+            int *cv = pos, *ov = tpos;
+            const bool narrow = kb == 8 && np >= 2 && ((kand ^ kor) >> 32) == 0;   // as in build_index
+            for (int p = 0; p < np; p++) {
+                const int kin = narrow && p > 0 ? 4 : kb, kout = narrow && p < np - 1 ? 4 : kb;
+                CUDA_TRY(c, ng::launch_radix_pass_x(kin, kout, 4, ck, ok, cv, ov, nrp, shifts[p], dbase + p * (1 << rb),
+                                                    sscr, (unsigned)(kand >> 32), c->stream, &c->launches, rb));
+                std::swap(ck, ok);
+                std::swap(cv, ov);
+            }
+            CUDA_TRY(c, ng::launch_group(kb, ck, cv, nrp, ukeys, map, d_u, gscr, c->stream, &c->launches));
+            CUDA_TRY(c, cudaMemcpyAsync(c->pinned, d_u, 8, cudaMemcpyDeviceToHost, c->stream));
+            CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+            memcpy(&n_distinct, c->pinned, 8);
+            eval_keys = ukeys;
+            d_neval = d_u;
+            n_eval = n_distinct;
+            prof_end(c, 2);
+        }
+
+        // ------------------------------------------------------------ a3 / a5-a7
+        if (ix) {
+            prof_begin(c, 3);
+            const bool split = wide && pre && P->agg != NG_MIN && P->agg != NG_MAX;
+            CUDA_TRY(c, ng::launch_range_agg(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, ix->keys, ix->payload,
+                                             ix->n, pre, split ? nullptr : suf, acc, cnt, kscr, c->stream, &c->launches,
+                                             split ? suf : nullptr, split ? acc_hi : nullptr, true));
+            htrace(c, "range");
+            prof_end(c, 3);
+        } else {
+            prof_begin(c, 1);
+            ng::ValSrc vs{nullptr, nullptr, 0};
+            if (value_agg) { vs.c = ac->d; vs.v = ac->valid; vs.w = vb; }
+            CUDA_TRY(c, ng::launch_filter(nS, ips, sks, kb, vs, vb, 1, value_agg ? 1 : 0, nullptr, skeys, nullptr, svals,
+                                          nullptr, value_agg ? extreme : nullptr, fscr_s, d_nsp, c->stream,
+                                          &c->launches, true));
+            htrace(c, "sfilter");
+            if (nR > SMALL_ROWS)
+                CUDA_TRY(c, ng::launch_init_partials(n_eval, d_neval, P->agg, acc, cnt, c->stream, &c->launches));
+            htrace(c, "init");
+            prof_end(c, 1);
+            prof_begin(c, 3);
+            CUDA_TRY(c, ng::launch_bnl(kb, vb, P->corr_op, P->agg, n_eval, d_neval, eval_keys, nS, d_nsp, skeys, svals,
+                                       extreme, acc, cnt, kscr, c->num_sms, c->bnl_shape, c->stream, &c->launches,
+                                       wide ? acc_hi : nullptr, true));
+            htrace(c, "bnl");
+            prof_end(c, 3);
+        }
+
+        // ------------------------------------------------------------ a8 + a9
+        prof_begin(c, 4);
+        ng::FinalizeArgs fa{};
+        fa.n_rp_max = nR;
+        fa.d_nrp = d_nrp;
+        fa.ids = ids;
+        fa.map = map;
+        fa.kvalid = rkvalid;
+        fa.acc = acc;
+        fa.cnt = cnt;
+        fa.acc_hi = wide ? acc_hi : nullptr;
+        fa.overflow = (unsigned long long *)(counts + 8);
+        fa.x_col = xc ? xc->d : nullptr;
+        fa.x_valid = xc ? xc->valid : nullptr;
+        fa.x_w = xc ? dtype_width(xc->dtype) : 4;
+        fa.agg = P->agg;
+        fa.outer_op = P->outer_op;
+        fa.a = P->lhs_mult;
+        fa.b = P->rhs_mult;
+        fa.row_id_base = P->row_id_base;
+        fa.emit_all = P->emit_all;
+        fa.out_ids = o_ids;
+        fa.out_vals = o_vals;
+        fa.out_sum = o_sum;
+        fa.out_cnt = o_cnt;
+        fa.out_valid = o_valid;
+        fa.out_passed = o_pass;
+        fa.out_count = d_out;
+        fa.scratch = fscr_f;
+        CUDA_TRY(c, ng::launch_finalize(fa, c->stream, &c->launches, true));
+        htrace(c, "finalize");
+        prof_end(c, 4);
+        prof_end(c, 5);
+        CUDA_TRY(c, cudaMemcpyAsync(c->pinned, counts, 72, cudaMemcpyDeviceToHost, c->stream));
+        // the first rows of every result field, staged on the host before the
+        // one synchronisation (8-byte fields, then the two byte fields)
+        if (krows == nR && krows > 0) {   // the whole result block fits: one copy, same layout
+            CUDA_TRY(c, cudaMemcpyAsync(c->stage, rblk, (size_t)nR * (8 * w8 + 2), cudaMemcpyDeviceToHost, c->stream));
+        } else if (krows > 0) {
+            CUDA_TRY(c, cudaMemcpy2DAsync(c->stage, (size_t)krows * 8, rblk, (size_t)nR * 8, (size_t)krows * 8, w8,
+                                          cudaMemcpyDeviceToHost, c->stream));
+            CUDA_TRY(c, cudaMemcpy2DAsync(c->stage + (size_t)krows * 8 * w8, (size_t)krows, o_valid, (size_t)nR,
+                                          (size_t)krows, 2, cudaMemcpyDeviceToHost, c->stream));
+        }
+        return NESTGPU_OK;
+    };
+    if (graph_ok(c, P, ix)) {
+        nestgpu_status gs = run_graph(c, exec_graph_key(c, P, ix, wide), enqueue);
+        if (gs) return gs;
+    } else {
+        nestgpu_status es = enqueue();
+        if (es) return es;
     }
     htrace(c, "copies");
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
@@ -1503,6 +1679,9 @@ nestgpu_status nestgpu_set_option(nestgpu_ctx *c, int32_t option, int64_t value)
     case NESTGPU_OPT_BNL_SHAPE:
         if (value < 0 || value > 2) return fail(c, NESTGPU_ERR_INVALID, "set_option: BNL shape 0, 1 or 2");
         c->bnl_shape = (int)value;
+        return NESTGPU_OK;
+    case NESTGPU_OPT_GRAPHS:
+        c->graphs_on = value != 0;
         return NESTGPU_OK;
     }
     return fail(c, NESTGPU_ERR_INVALID, "set_option: unknown option %d", option);

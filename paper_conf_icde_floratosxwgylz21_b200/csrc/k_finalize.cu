@@ -83,6 +83,37 @@ __global__ void __launch_bounds__(F_THREADS) finalize_kernel(FinalizeArgs A, uns
         if (tile >= num_tiles) return;
         const long long base = tile * F_TILE;
 
+        // the rows' inputs are loaded for all F_ITEMS rows first (independent
+        // loads in flight together; the rolled evaluation below would
+        // otherwise wait one memory round trip per row)
+        long long r_acc[F_ITEMS], r_cnt[F_ITEMS], r_x[F_ITEMS];
+        int r_row[F_ITEMS];
+        bool r_kval[F_ITEMS], r_xv[F_ITEMS];
+#pragma unroll
+        for (int j = 0; j < F_ITEMS; j++) {
+            const long long i = base + (long long)j * F_THREADS + tid;
+            r_acc[j] = r_cnt[j] = r_x[j] = 0;
+            r_row[j] = 0;
+            r_kval[j] = false;
+            r_xv[j] = false;
+            if (i < n) {
+                r_kval[j] = A.kvalid ? A.kvalid[i] != 0 : true;
+                const long long g = A.map ? (long long)A.map[i] : i;  // cached result slot (P:331)
+                r_cnt[j] = A.cnt[g];
+                r_acc[j] = A.acc[g];
+                r_row[j] = A.ids[i];
+            }
+        }
+        if (A.agg != EXISTS && A.agg != NOT_EXISTS) {
+#pragma unroll
+            for (int j = 0; j < F_ITEMS; j++) {
+                const long long i = base + (long long)j * F_THREADS + tid;
+                if (i < n) {
+                    r_xv[j] = !(A.x_valid && !A.x_valid[r_row[j]]);
+                    r_x[j] = load_w(A.x_col, A.x_w, r_row[j]);
+                }
+            }
+        }
 #pragma unroll 1
         for (int j = 0; j < F_ITEMS; j++) {
             const long long i = base + (long long)j * F_THREADS + tid;
@@ -90,10 +121,10 @@ __global__ void __launch_bounds__(F_THREADS) finalize_kernel(FinalizeArgs A, uns
             long long value = 0;
             uint8_t vp = 0;
             if (in) {
-                const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
-                const long long g = A.map ? (long long)A.map[i] : i;  // cached result slot (P:331)
-                const long long c = kval ? A.cnt[g] : 0;     // NULL key: empty subquery (R2)
-                long long acc = A.acc[g];
+                const bool kval = r_kval[j];
+                const long long g = A.map ? (long long)A.map[i] : i;
+                const long long c = kval ? r_cnt[j] : 0;     // NULL key: empty subquery (R2)
+                long long acc = r_acc[j];
                 bool vv = true;
                 if (A.acc_hi && c > 0) {   // split SUM: hi * 2^32 + lo, exact (reading R5)
                     const __int128 t = (__int128)A.acc_hi[g] * 4294967296ll + (__int128)(unsigned long long)acc;
@@ -116,11 +147,10 @@ __global__ void __launch_bounds__(F_THREADS) finalize_kernel(FinalizeArgs A, uns
                 if (A.agg == EXISTS || A.agg == NOT_EXISTS) {
                     p = v != 0;
                 } else {
-                    const int row = A.ids[i];
-                    const bool xv = !(A.x_valid && !A.x_valid[row]);
+                    const bool xv = r_xv[j];
                     p = false;
                     if (vv && xv) {
-                        const __int128 x = load_w(A.x_col, A.x_w, row);
+                        const __int128 x = r_x[j];
                         if (A.agg == AVG)
                             p = cmp_rt<__int128>((__int128)A.a * x * c, A.outer_op, (__int128)A.b * acc);
                         else

@@ -679,3 +679,42 @@ def test_c2_zipf_full_size_index_no_cache(eng):
             ref = oracle.evaluate(t, plan, rows=rows)
             assert_parity(g, ref, plan, True, rows=rows, ctx=("zipf nocache", corr_op, agg))
             assert dt < 5.0, (corr_op, agg, dt)   # load + index + exec + copy-out
+
+
+def test_exec_graph_replay_matches(eng):
+    """NESTGPU_OPT_GRAPHS: the exec launch sequence is captured into a CUDA
+    graph on first use and replayed afterwards.  Replays give the oracle's
+    result on every call, identical to running with graphs off, including
+    after the column contents change in place (a graph references addresses,
+    not data) and for the split-SUM path."""
+    import torch
+    from paper_conf_icde_floratosxwgylz21_b200.binding import OPT_GRAPHS
+    t = query1.random_small(7, n_r=3001, n_s=4001, key_hi=50, val_lo=-9, val_hi=9, null_frac=0.1)
+    plans = [(make_plan(op, agg, "<", outer_preds=[{"col": "col3", "op": "<=", "lit": 1}]), mode)
+             for op, agg, mode in (("=", "min", "index"), (">", "count", "bnl"), ("!=", "sum", "bnl"),
+                                   ("<", "avg", "index"), ("=", "exists", "bnl"))]
+    m = eng.mark()
+    try:
+        R = eng.load_table(t["R"], t.get("R_valid"))
+        S = eng.load_table(t["S"], t.get("S_valid"))
+        for graphs in (1, 0, 1):
+            eng.set_option(OPT_GRAPHS, graphs)
+            for plan, mode in plans:
+                ref = oracle.evaluate(t, plan)
+                idx = eng.index_for_plan(plan, S) if mode == "index" else -1
+                for rep in range(3):
+                    g = eng.result_to_numpy(eng.exec(plan, R, S, index=idx, emit_all=True))
+                    assert_parity(g, ref, plan, True, ctx=("graphs", graphs, plan["corr_op"], plan["agg"], rep))
+        # in-place change of R.col2 (the compared column): replays read the new values
+        eng.set_option(OPT_GRAPHS, 1)
+        plan, mode = plans[1]
+        eng.result_to_numpy(eng.exec(plan, R, S, emit_all=True))
+        info = eng.column_info(R["col2"])
+        new = (t["R"]["col2"].astype(np.int32) * 3 + 1).astype(np.int32)
+        eng.arena_view(info["d_values"], 4 * len(new)).copy_(torch.from_numpy(new.view(np.uint8)))
+        t2 = {"R": dict(t["R"], col2=new), "S": t["S"], "R_valid": t["R_valid"], "S_valid": t["S_valid"]}
+        g = eng.result_to_numpy(eng.exec(plan, R, S, emit_all=True))
+        assert_parity(g, oracle.evaluate(t2, plan), plan, True, ctx="in-place change")
+    finally:
+        eng.set_option(OPT_GRAPHS, 1)
+        eng.release(m)
