@@ -40,6 +40,9 @@ namespace ng {
 #ifndef NG_S_PITEMS4
 #define NG_S_PITEMS4 48   // ... for 4-byte items (32-bit keys, no payload)
 #endif
+#ifndef NG_S_PREAGG
+#define NG_S_PREAGG 0   // 1: a tile-histogram kernel publishes every tile's digit counts before the pass
+#endif
 #ifndef NG_S_PMINB
 #define NG_S_PMINB 3  // persistent pass: CTAs per SM the register budget must allow
 #endif
@@ -237,7 +240,7 @@ onesweep_p_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *
             }
             cnt[q] = c;
             loc += c;
-            st_relaxed_u32(status + tile * NB + d, (tile == 0 ? D_INC : D_AGG) | c);
+            if (!NG_S_PREAGG) st_relaxed_u32(status + tile * NB + d, (tile == 0 ? D_INC : D_AGG) | c);
         }
         unsigned sv[DPT][LBB];
 #pragma unroll
@@ -459,6 +462,28 @@ cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *
     return cudaGetLastError();
 }
 
+// NG_S_PREAGG: every tile's per-digit counts published (as look-back AGG
+// statuses, tile 0 as INC) by one extra pass over the keys before the
+// radix pass, so the pass's look-back never waits for a predecessor to load
+// and count its tile -- it only sums published counts back to the nearest
+// inclusive prefix.  Also zeroes the tile counter.
+template <typename K, int NB, int TILE>
+__global__ void __launch_bounds__(256) tile_agg_kernel(const K *__restrict__ keys, long long n, int shift,
+                                                       unsigned *__restrict__ status, unsigned *__restrict__ counter)
+{
+    __shared__ unsigned h[NB];
+    for (int d = threadIdx.x; d < NB; d += 256) h[d] = 0;
+    __syncthreads();
+    const long long t = blockIdx.x;
+    const long long b0 = t * TILE;
+    const long long b1 = min(n, b0 + TILE);
+    for (long long i = b0 + threadIdx.x; i < b1; i += 256)
+        atomicAdd(&h[(unsigned)(__ldg(keys + i) >> shift) & (NB - 1)], 1u);
+    __syncthreads();
+    for (int d = threadIdx.x; d < NB; d += 256) status[t * NB + d] = (t == 0 ? D_INC : D_AGG) | h[d];
+    if (t == 0 && threadIdx.x == 0) *counter = 0;
+}
+
 template <typename K, int VB, typename KO, int RB>
 static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *vout, long long n, int shift,
                             const unsigned *digit_base, void *scratch, unsigned hi, cudaStream_t st, bool prezeroed)
@@ -481,7 +506,10 @@ static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *
         return cudaSuccess;
     });
     if (e != cudaSuccess) return e;
-    if (!prezeroed) {
+    if (NG_S_PREAGG) {
+        tile_agg_kernel<K, (1 << RB), Cfg::TILE><<<(unsigned)tiles, 256, 0, st>>>(
+            (const K *)kin, n, shift, (unsigned *)((char *)scratch + 256), (unsigned *)scratch);
+    } else if (!prezeroed) {
         e = cudaMemsetAsync(scratch, 0, (size_t)tiles * (1 << RB) * 4 + 256, st);
         if (e != cudaSuccess) return e;
     }
