@@ -578,7 +578,7 @@ def main(argv=None):
         pin_s = {k: torch.from_numpy(np.ascontiguousarray(v)).pin_memory() for k, v in S_host.items()}
         h2d = sum(v.numel() * v.element_size() for v in pin.values()) + sum(
             v.numel() * v.element_size() for v in pin_s.values())
-        nloc = rk.hi - rk.lo
+        nloc = rk.hi - rk.lo if world == 1 or rank != 0 else n_r   # rank 0 receives every rank's survivors
         res_pin = {k: torch.empty(max(1, nloc), dtype=dt, pin_memory=True).numpy()
                    for k, dt in (("row", torch.int64), ("value", torch.int64), ("valid", torch.uint8),
                                  ("passed", torch.uint8))}
@@ -595,8 +595,20 @@ def main(argv=None):
                 if mode == "index" and payload not in idx:
                     idx[payload] = eng.build_index(Sx, ["col1"], payload)
                 res = eng.exec(plan, Rx, Sx, index=idx[payload] if mode == "index" else -1, row_id_base=rk.lo)
-                out = eng.result_to_numpy(res, out=res_pin)
-                nb += sum(a.nbytes for a in out.values())
+                if world > 1:   # the survivors reach rank 0 (window / NCCL), then rank 0's host
+                    if rk.pg is not None:
+                        g = rk.pg.gather(res)
+                    else:
+                        t = eng.result_tensors(res)
+                        g = ngd.gather_rows([t["row"], t["value"]])
+                    if rank == 0:
+                        n_g = int(g[0].numel())
+                        res_pin["row"][:n_g] = g[0].cpu().numpy()
+                        res_pin["value"][:n_g] = g[1].cpu().numpy()
+                        nb += 16 * n_g
+                else:
+                    out = eng.result_to_numpy(res, out=res_pin)
+                    nb += sum(a.nbytes for a in out.values())
             eng.release(m)
             d2h[0] = nb
 
@@ -618,8 +630,10 @@ def main(argv=None):
                "steps": ke,
                "h2d_bytes_per_step": int(ngd.sum_over_ranks(h2d, device=dev) if world > 1 else h2d),
                "d2h_bytes_per_step": int(ngd.sum_over_ranks(d2h[0], device=dev) if world > 1 else d2h[0]),
-               "path": "nestgpu_load_column (pinned host) -> [build_index] -> exec x%d -> "
-                       "nestgpu_result_to_host (pinned host), per rank" % len(plans)}
+               "path": ("nestgpu_load_column (pinned host) -> [build_index] -> exec x%d -> "
+                        "nestgpu_result_to_host (pinned host)" % len(plans)) if world == 1 else
+                       ("per rank: nestgpu_load_column (pinned host) -> [build_index] -> exec x%d -> survivors "
+                        "gathered to rank 0 (%s) -> rank 0 host" % (len(plans), args.gather))}
 
     if rank == 0:
         cpu = None
