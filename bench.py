@@ -547,8 +547,8 @@ def main(argv=None):
         t = ngd.max_over_ranks(sum(ms), device=dev) / len(ms)
         side["index_pruned (all plans on the index path)"] = {
             "value": outer_per_step / (t / 1000.0), "ms_per_step": t, "steps": len(ms),
-            "note": "sorted index (built + broadcast every step) + binary search; non-equality ranges "
-                    "from prefix/suffix aggregates"}
+            "note": "sorted index built every step (on every rank; broadcast from rank 0 with "
+                    "--index-mode broadcast) + binary search; non-equality ranges from prefix/suffix aggregates"}
         if args.workload == "C5":
             # C2's 12-plan step (BASELINE configs[1]) as an extra key
             R2, S2, plans2, _ = workload("C2")

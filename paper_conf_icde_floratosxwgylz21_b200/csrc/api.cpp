@@ -113,7 +113,8 @@ struct nestgpu_ctx {
     // CUDA graphs of exec launch sequences (NESTGPU_OPT_GRAPHS, default on):
     // key = every argument that determines the sequence (plan, column /
     // index addresses and sizes, arena state); kernels = launches per replay
-    // (-1: the sequence could not be captured, run it directly)
+    // (0 with no exec: seen once, captured when it repeats; -1: the sequence
+    // could not be captured, run it directly)
     struct GraphEntry {
         cudaGraphExec_t exec;
         long long kernels;
@@ -958,14 +959,28 @@ std::string exec_graph_key(const nestgpu_ctx *c, const nestgpu_plan *P, const In
     return k;
 }
 
-// Replay the captured launch sequence for `key`, capturing it first (and
-// running it once) when it is new.  A sequence that cannot be captured
+// Replay the captured launch sequence for `key`: the first sighting of a key
+// runs directly, the second captures the sequence (and runs it once through
+// the graph), later ones replay it.  A sequence that cannot be captured
 // (e.g. a launch kind the graph API refuses) is remembered and run directly.
 template <typename F>
 nestgpu_status run_graph(nestgpu_ctx *c, const std::string &key, F &enqueue)
 {
     auto it = c->graphs.find(key);
     if (it == c->graphs.end()) {
+        // first sighting: run directly and remember the key -- a sequence is
+        // captured only when it repeats, so one-off execs (fresh tables, a
+        // per-tuple drive program) never pay for a capture
+        if (c->graphs.size() >= 256) {
+            for (auto &kv : c->graphs)
+                if (kv.second.exec) cudaGraphExecDestroy(kv.second.exec);
+            c->graphs.clear();
+        }
+        c->graphs.emplace(key, nestgpu_ctx::GraphEntry{nullptr, 0});
+        htrace(c, "graph:first");
+        return enqueue();
+    }
+    if (!it->second.exec && it->second.kernels == 0) {
         const long long l0 = c->launches;
         const std::string err0 = c->err;
         // capture on the context's private stream (the caller's may be the
@@ -982,7 +997,7 @@ nestgpu_status run_graph(nestgpu_ctx *c, const std::string &key, F &enqueue)
         if (cudaStreamBeginCapture(c->stream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
             cudaGetLastError();
             c->stream = user;
-            c->graphs.emplace(key, nestgpu_ctx::GraphEntry{nullptr, -1});
+            it->second = nestgpu_ctx::GraphEntry{nullptr, -1};
             return enqueue();
         }
         const nestgpu_status st = enqueue();
@@ -994,21 +1009,16 @@ nestgpu_status run_graph(nestgpu_ctx *c, const std::string &key, F &enqueue)
         if (g) cudaGraphDestroy(g);
         const long long kernels = c->launches - l0;
         c->launches = l0;
-        if (c->graphs.size() >= 64) {
-            for (auto &kv : c->graphs)
-                if (kv.second.exec) cudaGraphExecDestroy(kv.second.exec);
-            c->graphs.clear();
-        }
         if (st != NESTGPU_OK || e != cudaSuccess || !ge) {
             if (c->trace)
                 fprintf(stderr, "[nestgpu trace] graph capture failed: status %d, %s, %s\n", (int)st,
                         cudaGetErrorString(e), c->err.c_str());
             cudaGetLastError();   // clear the capture error; run this sequence directly from now on
             c->err = err0;
-            c->graphs.emplace(key, nestgpu_ctx::GraphEntry{nullptr, -1});
+            it->second = nestgpu_ctx::GraphEntry{nullptr, -1};
             return enqueue();
         }
-        it = c->graphs.emplace(key, nestgpu_ctx::GraphEntry{ge, kernels}).first;
+        it->second = nestgpu_ctx::GraphEntry{ge, kernels};
     }
     if (!it->second.exec) {
         htrace(c, "graph:direct");
