@@ -113,11 +113,12 @@ struct nestgpu_ctx {
     // CUDA graphs of exec launch sequences (NESTGPU_OPT_GRAPHS, default on):
     // key = every argument that determines the sequence (plan, column /
     // index addresses and sizes, arena state); kernels = launches per replay
-    // (0 with no exec: seen once, captured when it repeats; -1: the sequence
-    // could not be captured, run it directly)
+    // (0 with no exec: seen `seen` times, captured once it keeps repeating;
+    // -1: the sequence could not be captured, run it directly)
     struct GraphEntry {
         cudaGraphExec_t exec;
         long long kernels;
+        int seen;   // direct runs so far
     };
     bool graphs_on;
     std::unordered_map<std::string, GraphEntry> graphs;
@@ -959,10 +960,12 @@ std::string exec_graph_key(const nestgpu_ctx *c, const nestgpu_plan *P, const In
     return k;
 }
 
-// Replay the captured launch sequence for `key`: the first sighting of a key
-// runs directly, the second captures the sequence (and runs it once through
-// the graph), later ones replay it.  A sequence that cannot be captured
-// (e.g. a launch kind the graph API refuses) is remembered and run directly.
+// Replay the captured launch sequence for `key`: the first GRAPH_AFTER
+// sightings of a key run directly, the next captures the sequence (and runs
+// it once through the graph), later ones replay it.  A sequence that cannot
+// be captured (e.g. a launch kind the graph API refuses) is remembered and
+// run directly.
+constexpr int GRAPH_AFTER = 8;
 template <typename F>
 nestgpu_status run_graph(nestgpu_ctx *c, const std::string &key, F &enqueue)
 {
@@ -976,8 +979,15 @@ nestgpu_status run_graph(nestgpu_ctx *c, const std::string &key, F &enqueue)
                 if (kv.second.exec) cudaGraphExecDestroy(kv.second.exec);
             c->graphs.clear();
         }
-        c->graphs.emplace(key, nestgpu_ctx::GraphEntry{nullptr, 0});
+        c->graphs.emplace(key, nestgpu_ctx::GraphEntry{nullptr, 0, 1});
         htrace(c, "graph:first");
+        return enqueue();
+    }
+    if (!it->second.exec && it->second.kernels == 0 && it->second.seen < GRAPH_AFTER) {
+        // capturing + instantiating costs ~1-3 ms: only sequences that keep
+        // repeating are worth it
+        it->second.seen++;
+        htrace(c, "graph:direct");
         return enqueue();
     }
     if (!it->second.exec && it->second.kernels == 0) {
@@ -997,7 +1007,7 @@ nestgpu_status run_graph(nestgpu_ctx *c, const std::string &key, F &enqueue)
         if (cudaStreamBeginCapture(c->stream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
             cudaGetLastError();
             c->stream = user;
-            it->second = nestgpu_ctx::GraphEntry{nullptr, -1};
+            it->second = nestgpu_ctx::GraphEntry{nullptr, -1, 0};
             return enqueue();
         }
         const nestgpu_status st = enqueue();
@@ -1015,10 +1025,10 @@ nestgpu_status run_graph(nestgpu_ctx *c, const std::string &key, F &enqueue)
                         cudaGetErrorString(e), c->err.c_str());
             cudaGetLastError();   // clear the capture error; run this sequence directly from now on
             c->err = err0;
-            it->second = nestgpu_ctx::GraphEntry{nullptr, -1};
+            it->second = nestgpu_ctx::GraphEntry{nullptr, -1, 0};
             return enqueue();
         }
-        it->second = nestgpu_ctx::GraphEntry{ge, kernels};
+        it->second = nestgpu_ctx::GraphEntry{ge, kernels, 0};
     }
     if (!it->second.exec) {
         htrace(c, "graph:direct");

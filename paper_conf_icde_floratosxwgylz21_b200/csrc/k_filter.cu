@@ -542,7 +542,6 @@ filter_rp_kernel(long long n, long long chunk, SrcCols sc, TPlan tp, KeySrc ks, 
     // ---- phase 2: ballot words -> ordered ids / keys / key-valid
     unsigned long long run = s_base;
     unsigned long long kand = ~0ull, kor = 0ull;
-    const unsigned lt = lanemask_lt();
     const long long w0 = c0 / 32, w1 = (c1 + 31) / 32;
     for (long long g = w0; g < w1; g += 32 * T_WARPS) {
         const long long wi = g + warp * 32 + lane;
@@ -572,36 +571,48 @@ filter_rp_kernel(long long n, long long chunk, SrcCols sc, TPlan tp, KeySrc ks, 
             btot += t;
         }
         const unsigned excl = incl - c;
-        // 32 rounds of 32 consecutive rows, RP_BATCH rounds' key loads in
-        // flight at once (a load -> store chain per round would leave the
-        // warp latency-bound)
-        for (int i0 = 0; i0 < 32; i0 += RP_BATCH) {
-            unsigned wv[RP_BATCH];
+        // survivors of the warp's 1024 rows, 32 at a time: lane j takes the
+        // survivor of warp-local rank r = b + j, finds its word by a binary
+        // search over the lanes' exclusive counts (shuffles) and its row by
+        // the rank within the word (__fns) -- every lane loads a key whatever
+        // the selectivity, RP_BATCH batches of loads in flight per warp
+        const unsigned wtotal = __shfl_sync(FULL, incl, 31);
+        for (unsigned b = 0; b < wtotal; b += 32 * RP_BATCH) {
+            long long row[RP_BATCH];
             uint64_t raw[RP_BATCH];
             bool kvl[RP_BATCH];
 #pragma unroll
             for (int q = 0; q < RP_BATCH; q++) {
-                wv[q] = __shfl_sync(FULL, word, i0 + q);
+                const unsigned r = b + q * 32 + lane;
+                int w = 0;   // the last lane whose exclusive count is <= r
+#pragma unroll
+                for (int step = 16; step > 0; step >>= 1) {
+                    const unsigned e = __shfl_sync(FULL, excl, w + step);
+                    if (e <= r) w += step;
+                }
+                const unsigned ew = __shfl_sync(FULL, excl, w);
+                const unsigned wv = __shfl_sync(FULL, word, w);
+                row[q] = -1;
                 raw[q] = 0;
                 kvl[q] = true;
-                if ((wv[q] >> lane) & 1u) {
-                    const long long row = (g + warp * 32 + i0 + q) * 32 + lane;
+                if (r < wtotal) {
+                    const int bit = (int)__fns(wv, 0, (int)(r - ew) + 1);
+                    const long long rw = (g + warp * 32 + w) * 32 + bit;
+                    row[q] = rw;
                     if (ks.n_key == 2)
-                        raw[q] = ((uint64_t)(uint32_t)__ldg((const int *)ks.c0 + row) << 32) |
-                                 (uint32_t)__ldg((const int *)ks.c1 + row);
+                        raw[q] = ((uint64_t)(uint32_t)__ldg((const int *)ks.c0 + rw) << 32) |
+                                 (uint32_t)__ldg((const int *)ks.c1 + rw);
                     else if (ks.w0 == 4)
-                        raw[q] = (uint32_t)__ldg((const int *)ks.c0 + row);
+                        raw[q] = (uint32_t)__ldg((const int *)ks.c0 + rw);
                     else
-                        raw[q] = (uint64_t)__ldg((const long long *)ks.c0 + row);
-                    kvl[q] = !((ks.v0 && !__ldg(ks.v0 + row)) || (ks.v1 && !__ldg(ks.v1 + row)));
+                        raw[q] = (uint64_t)__ldg((const long long *)ks.c0 + rw);
+                    kvl[q] = !((ks.v0 && !__ldg(ks.v0 + rw)) || (ks.v1 && !__ldg(ks.v1 + rw)));
                 }
             }
 #pragma unroll
             for (int q = 0; q < RP_BATCH; q++) {
-                const unsigned ov = __shfl_sync(FULL, excl, i0 + q);
-                if (!((wv[q] >> lane) & 1u)) continue;
-                const long long row = (g + warp * 32 + i0 + q) * 32 + lane;
-                const long long pos = (long long)run + woff + ov + __popc(wv[q] & lt);
+                if (row[q] < 0) continue;
+                const long long pos = (long long)run + woff + b + q * 32 + lane;
                 K key;
                 if (ks.n_key == 2)
                     key = (K)(((uint64_t)enc32((int)(uint32_t)(raw[q] >> 32)) << 32) | enc32((int)(uint32_t)raw[q]));
@@ -609,7 +620,7 @@ filter_rp_kernel(long long n, long long chunk, SrcCols sc, TPlan tp, KeySrc ks, 
                     key = KB == 4 ? (K)enc32((int)(uint32_t)raw[q]) : (K)enc64((long long)(int)(uint32_t)raw[q]);
                 else
                     key = (K)enc64((long long)raw[q]);
-                out_ids[pos] = (int)row;
+                out_ids[pos] = (int)row[q];
                 if (out_keys) ((K *)out_keys)[pos] = key;
                 if (out_kvalid) out_kvalid[pos] = kvl[q] ? 1 : 0;
                 kand &= (unsigned long long)key;
@@ -629,6 +640,85 @@ filter_rp_kernel(long long n, long long chunk, SrcCols sc, TPlan tp, KeySrc ks, 
             atomicOr(&keymask[1], ((unsigned long long)ohi << 32) | olo);
         }
     }
+}
+
+// R' without outer predicates (every row survives, in order): a pure
+// transform ids[i] = i, keys[i] = enc(key[i]), kvalid[i] -- 4 rows per thread
+// with 16-byte loads / stores (a 4-byte access per lane keeps too few bytes
+// in flight per SM to approach HBM bandwidth).
+template <int KB>
+__global__ void __launch_bounds__(256) rp_dense_kernel(long long n, KeySrc ks, int *__restrict__ out_ids,
+                                                       void *__restrict__ out_keys, uint8_t *__restrict__ out_kvalid,
+                                                       unsigned long long *__restrict__ keymask,
+                                                       long long *__restrict__ out_count)
+{
+    using K = typename std::conditional<KB == 8, uint64_t, uint32_t>::type;
+    unsigned long long kand = ~0ull, kor = 0ull;
+    const long long n4 = n / 4;
+    const long long t0 = blockIdx.x * 256LL + threadIdx.x, nt = (long long)gridDim.x * 256;
+    for (long long q = t0; q <= n4; q += nt) {   // q == n4: the ragged tail (n % 4 rows)
+        const long long r0 = q * 4;
+        const int m = (int)min(4LL, n - r0);
+        if (m <= 0) break;
+        K k[4];
+        if (m == 4 && ks.n_key == 1 && ks.w0 == 4) {
+            const int4 v = __ldg(reinterpret_cast<const int4 *>((const int *)ks.c0 + r0));
+            const int x[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+            for (int j = 0; j < 4; j++) k[j] = KB == 4 ? (K)enc32(x[j]) : (K)enc64((long long)x[j]);
+        } else {
+#pragma unroll
+            for (int j = 0; j < 4; j++) {
+                k[j] = 0;
+                if (j >= m) continue;
+                const long long row = r0 + j;
+                if (ks.n_key == 2)
+                    k[j] = (K)(((uint64_t)enc32(__ldg((const int *)ks.c0 + row)) << 32) |
+                               enc32(__ldg((const int *)ks.c1 + row)));
+                else if (ks.w0 == 4)
+                    k[j] = KB == 4 ? (K)enc32(__ldg((const int *)ks.c0 + row))
+                                   : (K)enc64((long long)__ldg((const int *)ks.c0 + row));
+                else
+                    k[j] = (K)enc64(__ldg((const long long *)ks.c0 + row));
+            }
+        }
+        if (m == 4) {
+            reinterpret_cast<int4 *>(out_ids)[q] = make_int4((int)r0, (int)r0 + 1, (int)r0 + 2, (int)r0 + 3);
+            if (out_keys) {
+                if constexpr (KB == 4) {
+                    reinterpret_cast<uint4 *>(out_keys)[q] = make_uint4(k[0], k[1], k[2], k[3]);
+                } else {
+                    reinterpret_cast<ulonglong2 *>(out_keys)[2 * q] = make_ulonglong2(k[0], k[1]);
+                    reinterpret_cast<ulonglong2 *>(out_keys)[2 * q + 1] = make_ulonglong2(k[2], k[3]);
+                }
+            }
+        } else {
+            for (int j = 0; j < m; j++) {
+                out_ids[r0 + j] = (int)(r0 + j);
+                if (out_keys) ((K *)out_keys)[r0 + j] = k[j];
+            }
+        }
+        if (out_kvalid)
+            for (int j = 0; j < m; j++) {
+                const long long row = r0 + j;
+                out_kvalid[row] = ((ks.v0 && !__ldg(ks.v0 + row)) || (ks.v1 && !__ldg(ks.v1 + row))) ? 0 : 1;
+            }
+        for (int j = 0; j < m; j++) {
+            kand &= (unsigned long long)k[j];
+            kor |= (unsigned long long)k[j];
+        }
+    }
+    if (keymask) {
+        const unsigned alo = __reduce_and_sync(FULL, (unsigned)kand);
+        const unsigned ahi = __reduce_and_sync(FULL, (unsigned)(kand >> 32));
+        const unsigned olo = __reduce_or_sync(FULL, (unsigned)kor);
+        const unsigned ohi = __reduce_or_sync(FULL, (unsigned)(kor >> 32));
+        if ((threadIdx.x & 31) == 0) {
+            atomicAnd(&keymask[0], ((unsigned long long)ahi << 32) | alo);
+            atomicOr(&keymask[1], ((unsigned long long)ohi << 32) | olo);
+        }
+    }
+    if (t0 == 0) *out_count = n;
 }
 
 // ------------------------------------------------------------------ host side
@@ -847,9 +937,10 @@ cudaError_t launch_rp_t(long long n, const SrcCols &sc, const TPlan &tp, const K
     unsigned *barrier = (unsigned *)scratch;
     unsigned long long *counts = (unsigned long long *)((char *)scratch + RP_COUNTS_OFF);
     unsigned *bits = (unsigned *)((char *)scratch + RP_BITS_OFF);
-    if (!preds) {
-        kern<<<(unsigned)grid, T_THREADS, 0, st>>>(n, chunk, sc, tp, ks, ids, keys, kvalid, keymask, bits, counts,
-                                                 barrier, count);
+    if (!preds) {   // every row survives: the vectorised transform
+        long long blocks = (n / 4 + 1 + 255) / 256;
+        if (blocks > (long long)num_sms * 16) blocks = (long long)num_sms * 16;
+        rp_dense_kernel<KB><<<(unsigned)blocks, 256, 0, st>>>(n, ks, ids, keys, kvalid, keymask, count);
         return cudaGetLastError();
     }
     void *args[] = {(void *)&n, (void *)&chunk, (void *)&sc, (void *)&tp, (void *)&ks, (void *)&ids, (void *)&keys,

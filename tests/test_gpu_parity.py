@@ -702,13 +702,14 @@ def test_exec_graph_replay_matches(eng):
             for plan, mode in plans:
                 ref = oracle.evaluate(t, plan)
                 idx = eng.index_for_plan(plan, S) if mode == "index" else -1
-                for rep in range(3):
+                for rep in range(11):   # 8 direct runs, the capture, replays
                     g = eng.result_to_numpy(eng.exec(plan, R, S, index=idx, emit_all=True))
                     assert_parity(g, ref, plan, True, ctx=("graphs", graphs, plan["corr_op"], plan["agg"], rep))
         # in-place change of R.col2 (the compared column): replays read the new values
         eng.set_option(OPT_GRAPHS, 1)
         plan, mode = plans[1]
-        eng.result_to_numpy(eng.exec(plan, R, S, emit_all=True))
+        for _ in range(10):
+            eng.result_to_numpy(eng.exec(plan, R, S, emit_all=True))
         info = eng.column_info(R["col2"])
         new = (t["R"]["col2"].astype(np.int32) * 3 + 1).astype(np.int32)
         eng.arena_view(info["d_values"], 4 * len(new)).copy_(torch.from_numpy(new.view(np.uint8)))
