@@ -335,8 +335,12 @@ class Rank:
             self.Sc = eng.load_table(S)
         self.launches = 0
         self.pg = None
+        self.gather_note = None
         if world > 1 and gather == "peer":
             self.pg = ngd.PeerGather(eng, self.n_r, device=dev)
+            if not self.pg.ok:   # some rank cannot map rank 0's window: NCCL send/recv instead
+                self.gather_note = "peer window unavailable (%s); NCCL send/recv used" % self.pg.error
+                self.pg = None
 
     def step(self, plans=None, profs=None, stages=None, keep=None):
         """One pass of the hot path over the batch (every plan).  At N > 1 the
@@ -675,6 +679,8 @@ def main(argv=None):
         }
         if nccl_pat:
             line["nccl_init"] = ngd.nccl_init_summary(nccl_pat)
+        if rk.gather_note:
+            line["gather_note"] = rk.gather_note
         emit(line, args)
     if rk.pg is not None:
         rk.pg.close()

@@ -258,7 +258,19 @@ class PeerGather:
         hd = h if _is_gloo(group) else h.to(self.device)
         dist.broadcast(hd, src=0, group=group)
         self.handle = bytes(hd.cpu().tolist())
-        self.peer = self.own if self.rank == 0 else eng.window_open(self.handle)
+        self.peer, self.error = self.own, None
+        if self.rank != 0:
+            try:
+                self.peer = eng.window_open(self.handle)
+            except Exception as e:   # no peer access between these devices
+                self.peer, self.error = None, str(e)
+        # every rank must agree: if any rank cannot map the window, nobody uses it
+        ok = torch.tensor([0.0 if self.error else 1.0], dtype=torch.float64,
+                          device="cpu" if _is_gloo(group) else self.device)
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN, group=group)
+        self.ok = bool(ok.item() > 0.5)
+        if not self.ok:
+            self.close()
 
     def gather(self, res):
         """Rank 0: (row ids, values) torch views of the gathered rows in rank
@@ -274,6 +286,9 @@ class PeerGather:
         return self.eng.window_tensors(self.own, self.cap, sum(counts))
 
     def close(self):
+        if getattr(self, "_closed", False):
+            return
+        self._closed = True
         if self.rank == 0:
             dist.barrier(group=self.group)   # every peer has unmapped
             if self.own:

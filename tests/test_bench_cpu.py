@@ -74,3 +74,21 @@ def test_bench_spawns_two_ranks_gloo():
     assert d["n_gpus"] == 2 and d["scaling"] == "strong"
     assert d["whole_r_check"]["identical"] is True
     assert d["multi_gpu_stages_ms_per_step"]["gather"] >= 0
+
+
+def test_bench_defaults_to_c5_headline():
+    """The driver's `bench.py --gpus 1 --steps 20 --warmup 5` measures C5
+    (BASELINE configs[4], the largest single-GPU config) -- VERDICT r1 item 1."""
+    a = bench.parse_args(["--gpus", "1", "--steps", "20", "--warmup", "5"])
+    assert a.workload == "C5" and a.gather == "peer" and a.index_mode == "local"
+    assert bench.DESC["C5"].startswith("C5: non-equality Query 1 '>' MIN, |R|=|S|=16M")
+
+
+def test_cpu_baselines_report_model_and_closed_form():
+    """cpu_baseline fields: the oracle sample with the CPU model, and the
+    timed closed-form checker over the whole (here C1) workload."""
+    R, S, plans, _ = bench.workload("C1")
+    cb = bench.time_oracle({"R": R, "S": S}, plans, 0.2)
+    assert cb["kind"] == "oracle" and cb["cores"] >= 1 and cb["cpu_model"] and cb["value"] > 0
+    cf = bench.time_closed_form(R, S, plans)
+    assert cf["value"] > 0 and cf["sample"].startswith("full workload: 2000 outer tuples")
