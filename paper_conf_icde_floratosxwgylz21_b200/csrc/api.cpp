@@ -1242,7 +1242,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
             fl.add(counts + 8, 64);
             fl.add(fscr, ng::filter_zero_bytes(nR, true));
             if (fscr_s) fl.add(fscr_s, ng::filter_zero_bytes(nS, false));
-            fl.add(fscr_f, ng::finalize_scratch_bytes(nR));
+            fl.add(fscr_f, ng::finalize_zero_bytes());
             fl.add(kscr, ix ? 256 : ng::bnl_scratch_bytes(nR));
             if (wide) fl.add(acc_hi, (size_t)nR * 8);
             if (!ix && nR <= SMALL_ROWS) {   // small R: the partials' identity init rides on the fill

@@ -92,6 +92,7 @@ cudaError_t launch_fill(const FillList &f, cudaStream_t st, long long *launches)
 // scratch bytes a prezeroed launcher expects zero (regions start at scratch)
 size_t filter_zero_bytes(long long n, bool ordered);
 size_t finalize_scratch_bytes(long long n);
+size_t finalize_zero_bytes();   // the part of the finalize scratch that must be zero
 
 // a2 / a3: filter rows [0, n) by `preds`, compact survivors in row order.
 //   out_ids    : int32 row ids of survivors (nullable)

@@ -25,8 +25,8 @@ constexpr int F_TILE = F_THREADS * F_ITEMS;
 
 size_t finalize_scratch_bytes(long long n)
 {
-    long long tiles = (n + F_TILE - 1) / F_TILE;
-    return (size_t)(tiles + 1) * 8 + 256;
+    // barrier word, per-CTA counts (<= 2048), ballot words (n / 8 bytes)
+    return 1024 + 16384 + (size_t)(n / 32 + 2) * 4 + 256;
 }
 
 // ------------------------------------------------------------------ a8 + a9
@@ -56,167 +56,285 @@ __device__ __forceinline__ long long avg_scaled(long long acc, long long c)
     return div_round_half_away((__int128)acc * 1000000, c);
 }
 
-// The per-row evaluation (int128 compares, the rare int128 division) is
-// large; unrolled over the tile's 16 rows per thread it made a ~175 KB kernel
-// whose instruction-cache misses dominated small R' (SF1 Q17: 69 us for 6.3k
-// rows).  Rows are therefore evaluated in a rolled loop and staged in shared
-// memory (value, valid|passed bits, one ballot per (row group, warp)).
-__global__ void __launch_bounds__(F_THREADS) finalize_kernel(FinalizeArgs A, unsigned long long *__restrict__ status,
-                                                             unsigned *__restrict__ counter)
-{
-    __shared__ unsigned s_tile;
-    __shared__ unsigned s_cnt[F_ITEMS][F_WARPS];
-    __shared__ unsigned s_bal[F_ITEMS][F_WARPS];
-    __shared__ long long s_val[F_ITEMS][F_THREADS];
-    __shared__ uint8_t s_vp[F_ITEMS][F_THREADS];   // bit 0 valid, bit 1 passed
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const unsigned lt = lanemask_lt();
-    const long long n = *A.d_nrp;
-    const long long num_tiles = (n + F_TILE - 1) / F_TILE;
-    // persistent: the grid is sized for the host's upper bound of |R'| but
-    // capped; CTAs take tiles of the ACTUAL |R'| until none are left
-    for (;;) {
-        if (tid == 0) s_tile = atomicAdd(counter, 1u);
-        __syncthreads();
-        const long long tile = s_tile;
-        __syncthreads();
-        if (tile >= num_tiles) return;
-        const long long base = tile * F_TILE;
+// ---- one R' row: inputs, then Res[i] + the outer comparison (R1, R2, R6, R7)
+struct FinIn {
+    long long acc, cnt, x, g;
+    int row;
+    bool kval, xv;
+};
 
-        // the rows' inputs are loaded for all F_ITEMS rows first (independent
-        // loads in flight together; the rolled evaluation below would
-        // otherwise wait one memory round trip per row)
-        long long r_acc[F_ITEMS], r_cnt[F_ITEMS], r_x[F_ITEMS];
-        int r_row[F_ITEMS];
-        bool r_kval[F_ITEMS], r_xv[F_ITEMS];
-#pragma unroll
-        for (int j = 0; j < F_ITEMS; j++) {
-            const long long i = base + (long long)j * F_THREADS + tid;
-            r_acc[j] = r_cnt[j] = r_x[j] = 0;
-            r_row[j] = 0;
-            r_kval[j] = false;
-            r_xv[j] = false;
-            if (i < n) {
-                r_kval[j] = A.kvalid ? A.kvalid[i] != 0 : true;
-                const long long g = A.map ? (long long)A.map[i] : i;  // cached result slot
-                r_cnt[j] = A.cnt[g];
-                r_acc[j] = A.acc[g];
-                r_row[j] = A.ids[i];
-            }
-        }
-        if (A.agg != EXISTS && A.agg != NOT_EXISTS) {
-#pragma unroll
-            for (int j = 0; j < F_ITEMS; j++) {
-                const long long i = base + (long long)j * F_THREADS + tid;
-                if (i < n) {
-                    r_xv[j] = !(A.x_valid && !A.x_valid[r_row[j]]);
-                    r_x[j] = load_w(A.x_col, A.x_w, r_row[j]);
-                }
-            }
-        }
-#pragma unroll 1
-        for (int j = 0; j < F_ITEMS; j++) {
-            const long long i = base + (long long)j * F_THREADS + tid;
-            bool in = i < n;
-            long long value = 0;
-            uint8_t vp = 0;
-            if (in) {
-                const bool kval = r_kval[j];
-                const long long g = A.map ? (long long)A.map[i] : i;
-                const long long c = kval ? r_cnt[j] : 0;     // NULL key: empty subquery (R2)
-                long long acc = r_acc[j];
-                bool vv = true;
-                if (A.acc_hi && c > 0) {   // split SUM: hi * 2^32 + lo, exact (reading R5)
-                    const __int128 t = (__int128)A.acc_hi[g] * 4294967296ll + (__int128)(unsigned long long)acc;
-                    if (t > (__int128)LLONG_MAX || t < (__int128)LLONG_MIN) {
-                        atomicOr(A.overflow, 1ull);
-                        acc = 0;
-                    } else {
-                        acc = (long long)t;
-                    }
-                }
-                long long v = 0;
-                switch (A.agg) {
-                case MIN: case MAX: case SUM: vv = c > 0; v = acc; break;
-                case COUNT: v = c; break;
-                case AVG: vv = c > 0; if (vv) v = avg_scaled(acc, c); break;
-                case EXISTS: v = c > 0; break;
-                default: v = c == 0; break;
-                }
-                bool p;
-                if (A.agg == EXISTS || A.agg == NOT_EXISTS) {
-                    p = v != 0;
-                } else {
-                    const bool xv = r_xv[j];
-                    p = false;
-                    if (vv && xv) {
-                        const __int128 x = r_x[j];
-                        if (A.agg == AVG)
-                            p = cmp_rt<__int128>((__int128)A.a * x * c, A.outer_op, (__int128)A.b * acc);
-                        else
-                            p = cmp_rt<__int128>((__int128)A.a * x, A.outer_op, (__int128)A.b * v);
-                    }
-                }
-                value = vv ? v : 0;
-                vp = (uint8_t)((vv ? 1 : 0) | (p ? 2 : 0));
-                in = A.emit_all ? true : p;
-            }
-            s_val[j][tid] = value;
-            s_vp[j][tid] = vp;
-            const unsigned m = __ballot_sync(FULL, in);
-            if (lane == 0) {
-                s_cnt[j][warp] = __popc(m);
-                s_bal[j][warp] = m;
-            }
-        }
-        const unsigned long long tb = tile_offsets<F_ITEMS, F_THREADS>(s_cnt, status, tile, num_tiles, A.out_count);
-#pragma unroll 1
-        for (int j = 0; j < F_ITEMS; j++) {
-            const unsigned m = s_bal[j][warp];
-            if (!((m >> lane) & 1u)) continue;
-            const long long i = base + (long long)j * F_THREADS + tid;
-            const long long pos = (long long)tb + s_cnt[j][warp] + __popc(m & lt);
-            const uint8_t vp = s_vp[j][tid];
-            A.out_ids[pos] = A.row_id_base + A.ids[i];
-            A.out_vals[pos] = s_val[j][tid];
-            A.out_valid[pos] = vp & 1;
-            A.out_passed[pos] = (vp >> 1) & 1;
-            if (A.out_sum) {
-                const bool kval = A.kvalid ? A.kvalid[i] != 0 : true;
-                const long long g = A.map ? (long long)A.map[i] : i;
-                long long sum = kval ? A.acc[g] : 0;
-                if (A.acc_hi && kval)
-                    sum = (long long)((__int128)A.acc_hi[g] * 4294967296ll + (__int128)(unsigned long long)sum);
-                A.out_sum[pos] = sum;
-                A.out_cnt[pos] = kval ? A.cnt[g] : 0;
-            }
-        }
-        __syncthreads();   // shared staging is rewritten by the next tile
+__device__ __forceinline__ void fin_load(const FinalizeArgs &A, long long i, FinIn &r)
+{
+    r.kval = A.kvalid ? A.kvalid[i] != 0 : true;
+    r.g = A.map ? (long long)A.map[i] : i;   // cached result slot
+    r.cnt = A.cnt[r.g];
+    r.acc = A.acc[r.g];
+    r.row = A.ids[i];
+    r.x = 0;
+    r.xv = false;
+}
+
+__device__ __forceinline__ void fin_load_x(const FinalizeArgs &A, FinIn &r)
+{
+    if (A.agg != EXISTS && A.agg != NOT_EXISTS) {
+        r.xv = !(A.x_valid && !A.x_valid[r.row]);
+        r.x = load_w(A.x_col, A.x_w, r.row);
     }
 }
+
+// value (0 when NULL), valid, passed.  Not inlined: the int128 compares and
+// the rare int128 division are large, and the callers loop over rows
+// (round 1: an unrolled evaluation made a ~175 KB kernel whose instruction-
+// cache misses dominated small R').
+__device__ __noinline__ void fin_eval(const FinalizeArgs &A, const FinIn &r, long long &value, bool &valid,
+                                      bool &passed)
+{
+    const long long c = r.kval ? r.cnt : 0;   // NULL key: empty subquery (R2)
+    long long acc = r.acc;
+    bool vv = true;
+    if (A.acc_hi && c > 0) {   // split SUM: hi * 2^32 + lo, exact (reading R5)
+        const __int128 t = (__int128)A.acc_hi[r.g] * 4294967296ll + (__int128)(unsigned long long)acc;
+        if (t > (__int128)LLONG_MAX || t < (__int128)LLONG_MIN) {
+            atomicOr(A.overflow, 1ull);
+            acc = 0;
+        } else {
+            acc = (long long)t;
+        }
+    }
+    long long v = 0;
+    switch (A.agg) {
+    case MIN: case MAX: case SUM: vv = c > 0; v = acc; break;
+    case COUNT: v = c; break;
+    case AVG: vv = c > 0; if (vv) v = avg_scaled(acc, c); break;
+    case EXISTS: v = c > 0; break;
+    default: v = c == 0; break;
+    }
+    bool p;
+    if (A.agg == EXISTS || A.agg == NOT_EXISTS) {
+        p = v != 0;
+    } else {
+        p = false;
+        if (vv && r.xv) {
+            const __int128 x = r.x;
+            if (A.agg == AVG)
+                p = cmp_rt<__int128>((__int128)A.a * x * c, A.outer_op, (__int128)A.b * acc);
+            else
+                p = cmp_rt<__int128>((__int128)A.a * x, A.outer_op, (__int128)A.b * v);
+        }
+    }
+    value = vv ? v : 0;
+    valid = vv;
+    passed = p;
+}
+
+__device__ __forceinline__ void fin_write(const FinalizeArgs &A, const FinIn &r, long long pos, long long value,
+                                          bool valid, bool passed)
+{
+    A.out_ids[pos] = A.row_id_base + r.row;
+    A.out_vals[pos] = value;
+    A.out_valid[pos] = valid ? 1 : 0;
+    A.out_passed[pos] = passed ? 1 : 0;
+    if (A.out_sum) {
+        long long sum = r.kval ? r.acc : 0;
+        if (A.acc_hi && r.kval)
+            sum = (long long)((__int128)A.acc_hi[r.g] * 4294967296ll + (__int128)(unsigned long long)sum);
+        A.out_sum[pos] = sum;
+        A.out_cnt[pos] = r.kval ? r.cnt : 0;
+    }
+}
+
+// emit_all: every R' tuple at its own position (no compaction, no scan)
+__global__ void __launch_bounds__(F_THREADS) finalize_all_kernel(FinalizeArgs A)
+{
+    const long long n = *A.d_nrp;
+    const long long t0 = blockIdx.x * (long long)F_THREADS + threadIdx.x, nt = (long long)gridDim.x * F_THREADS;
+    for (long long b = t0; b < n; b += nt * F_ITEMS) {
+        FinIn r[F_ITEMS];
+#pragma unroll
+        for (int j = 0; j < F_ITEMS; j++)
+            if (b + j * nt < n) fin_load(A, b + j * nt, r[j]);
+#pragma unroll
+        for (int j = 0; j < F_ITEMS; j++)
+            if (b + j * nt < n) fin_load_x(A, r[j]);
+#pragma unroll 1
+        for (int j = 0; j < F_ITEMS; j++) {
+            if (b + j * nt >= n) break;
+            long long v;
+            bool vv, p;
+            fin_eval(A, r[j], v, vv, p);
+            fin_write(A, r[j], b + j * nt, v, vv, p);
+        }
+    }
+    if (t0 == 0) *A.out_count = n;
+}
+
+// Survivors only: the ordered compaction as one cooperative launch (P:235's
+// 0-1 vector -> prefix sum -> materialize, like the R' filter, §8): a chunk
+// per CTA; phase 1 evaluates every row of the chunk into ballot words (the
+// 0-1 vector, n / 8 bytes) + the chunk count; one grid barrier; phase 2 walks
+// the survivors 32 at a time and re-evaluates each from its inputs to write
+// it (the round-1 kernel's decoupled look-back over ~16k tiles serialised on
+// L2 round trips: 0.44 ms for C5's 16M R').
+__global__ void __launch_bounds__(F_THREADS, 2)
+finalize_compact_kernel(FinalizeArgs A, long long chunk, unsigned *__restrict__ bits,
+                        unsigned long long *__restrict__ counts, unsigned *__restrict__ barrier)
+{
+    __shared__ unsigned long long s_red[F_WARPS];
+    __shared__ unsigned s_wtot[F_WARPS];
+    __shared__ unsigned long long s_base;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const long long n = *A.d_nrp;
+    const long long c0 = blockIdx.x * chunk;
+    const long long c1 = min(n, c0 + chunk);
+    // ---- phase 1: passed bits of every row of the chunk
+    unsigned long long mycount = 0;
+    const long long w0 = c0 / 32, w1 = c1 > c0 ? (c1 + 31) / 32 : w0;
+    for (long long wb = w0 + warp; wb < w1; wb += F_WARPS * F_ITEMS) {
+        FinIn r[F_ITEMS];
+        bool live[F_ITEMS];
+#pragma unroll
+        for (int j = 0; j < F_ITEMS; j++) {
+            const long long row = (wb + (long long)j * F_WARPS) * 32 + lane;
+            live[j] = wb + (long long)j * F_WARPS < w1 && row < c1;
+            if (live[j]) fin_load(A, row, r[j]);
+        }
+#pragma unroll
+        for (int j = 0; j < F_ITEMS; j++)
+            if (live[j]) fin_load_x(A, r[j]);
+#pragma unroll 1
+        for (int j = 0; j < F_ITEMS; j++) {
+            bool p = false;
+            if (live[j]) {
+                long long v;
+                bool vv;
+                fin_eval(A, r[j], v, vv, p);
+            }
+            const unsigned m = __ballot_sync(FULL, p);
+            if (wb + (long long)j * F_WARPS < w1 && lane == 0) {
+                bits[wb + (long long)j * F_WARPS] = m;
+                mycount += __popc(m);
+            }
+        }
+    }
+    if (lane == 0) s_red[warp] = mycount;
+    __syncthreads();
+    if (tid == 0) {
+        unsigned long long t = 0;
+        for (int w = 0; w < F_WARPS; w++) t += s_red[w];
+        st_relaxed_u64(counts + blockIdx.x, t);
+        __threadfence();
+        atomicAdd(barrier, 1u);
+        while (ld_relaxed_u32(barrier) < gridDim.x) __nanosleep(64);
+        __threadfence();
+    }
+    __syncthreads();
+    unsigned long long pre = 0;
+    for (int b = tid; b < (int)blockIdx.x; b += F_THREADS) pre += ld_relaxed_u64(counts + b);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) pre += __shfl_xor_sync(FULL, pre, o);
+    if (lane == 0) s_red[warp] = pre;
+    __syncthreads();
+    if (tid == 0) {
+        unsigned long long t = 0;
+        for (int w = 0; w < F_WARPS; w++) t += s_red[w];
+        s_base = t;
+        if (blockIdx.x == gridDim.x - 1) *A.out_count = (long long)(t + ld_relaxed_u64(counts + blockIdx.x));
+    }
+    __syncthreads();
+    // ---- phase 2: survivors, 32 at a time per warp (cf. filter_rp_kernel)
+    unsigned long long run = s_base;
+    for (long long g = w0; g < w1; g += 32 * F_WARPS) {
+        const long long wi = g + warp * 32 + lane;
+        const unsigned word = wi < w1 ? __ldcg(bits + wi) : 0u;
+        const unsigned c = __popc(word);
+        unsigned incl = c;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned t = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl += t;
+        }
+        if (lane == 31) s_wtot[warp] = incl;
+        __syncthreads();
+        unsigned woff = 0, btot = 0;
+#pragma unroll
+        for (int w = 0; w < F_WARPS; w++) {
+            const unsigned t = s_wtot[w];
+            woff += w < warp ? t : 0;
+            btot += t;
+        }
+        const unsigned excl = incl - c;
+        const unsigned wtotal = __shfl_sync(FULL, incl, 31);
+        for (unsigned b = 0; b < wtotal; b += 32) {
+            const unsigned rk = b + lane;
+            int w = 0;
+#pragma unroll
+            for (int step = 16; step > 0; step >>= 1) {
+                const unsigned e = __shfl_sync(FULL, excl, w + step);
+                if (e <= rk) w += step;
+            }
+            const unsigned ew = __shfl_sync(FULL, excl, w);
+            const unsigned wv = __shfl_sync(FULL, word, w);
+            if (rk < wtotal) {
+                const long long row = (g + warp * 32 + w) * 32 + (int)__fns(wv, 0, (int)(rk - ew) + 1);
+                FinIn r;
+                fin_load(A, row, r);
+                fin_load_x(A, r);
+                long long v;
+                bool vv, p;
+                fin_eval(A, r, v, vv, p);
+                fin_write(A, r, (long long)run + woff + rk, v, vv, p);
+            }
+        }
+        run += btot;
+        __syncthreads();
+    }
+}
+
+size_t finalize_zero_bytes() { return 1024; }
 
 cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *launches, bool prezeroed)
 {
     cudaError_t e = prezeroed ? cudaSuccess : cudaMemsetAsync(a.out_count, 0, sizeof(long long), st);
     if (e != cudaSuccess || a.n_rp_max <= 0) return e;
-    if (!prezeroed) {
-        e = cudaMemsetAsync(a.scratch, 0, finalize_scratch_bytes(a.n_rp_max), st);
-        if (e != cudaSuccess) return e;
-    }
-    long long tiles = (a.n_rp_max + F_TILE - 1) / F_TILE;
-    int cap = 0;
-    e = per_device_setup((const void *)finalize_kernel, 0, &cap, [](int dev, int *v) {
-        int sms = 0;
-        cudaError_t e2 = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        *v = sms * 4;
-        return e2;
+    int sms = 0;
+    e = per_device_setup((const void *)finalize_all_kernel, 0, &sms, [](int dev, int *v) {
+        return cudaDeviceGetAttribute(v, cudaDevAttrMultiProcessorCount, dev);
     });
     if (e != cudaSuccess) return e;
-    if (tiles > cap) tiles = cap;
-    finalize_kernel<<<(unsigned)tiles, F_THREADS, 0, st>>>(a, (unsigned long long *)((char *)a.scratch + 256),
-                                                         (unsigned *)a.scratch);
+    if (a.emit_all) {
+        long long blocks = (a.n_rp_max + F_THREADS * F_ITEMS - 1) / (F_THREADS * F_ITEMS);
+        if (blocks > (long long)sms * 8) blocks = (long long)sms * 8;
+        finalize_all_kernel<<<(unsigned)blocks, F_THREADS, 0, st>>>(a);
+        ++*launches;
+        return cudaGetLastError();
+    }
+    if (!prezeroed) {
+        e = cudaMemsetAsync(a.scratch, 0, finalize_zero_bytes(), st);
+        if (e != cudaSuccess) return e;
+    }
+    int occ = 0;
+    e = per_device_setup((const void *)finalize_compact_kernel, 0, &occ, [](int, int *v) {
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(v, finalize_compact_kernel, F_THREADS, 0);
+    });
+    if (e != cudaSuccess) return e;
+    if (occ < 1) return cudaErrorInvalidConfiguration;
+    // resident grid (the barrier), chunks of whole 32-row words; no more CTAs
+    // than chunks of >= 1024 rows
+    long long grid = (long long)sms * occ;
+    if (grid > 2048) grid = 2048;
+    const long long need = (a.n_rp_max + 1023) / 1024;
+    if (grid > need) grid = need < 1 ? 1 : need;
+    long long chunk = (a.n_rp_max + grid - 1) / grid;
+    chunk = (chunk + 31) / 32 * 32;
+    unsigned *barrier = (unsigned *)a.scratch;
+    unsigned long long *counts = (unsigned long long *)((char *)a.scratch + 1024);
+    unsigned *bits = (unsigned *)((char *)a.scratch + 1024 + 16384);
+    FinalizeArgs aa = a;
+    void *args[] = {(void *)&aa, (void *)&chunk, (void *)&bits, (void *)&counts, (void *)&barrier};
+    e = cudaLaunchCooperativeKernel((const void *)finalize_compact_kernel, dim3((unsigned)grid), dim3(F_THREADS),
+                                    args, 0, st);
     ++*launches;
-    return cudaGetLastError();
+    return e;
 }
 
 // ------------------------------------------------------------------ partials
