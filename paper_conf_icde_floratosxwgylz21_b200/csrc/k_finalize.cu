@@ -18,10 +18,11 @@ namespace ng {
 constexpr int F_THREADS = 256;
 constexpr int F_WARPS = F_THREADS / 32;
 #ifndef NG_F_ITEMS
-#define NG_F_ITEMS 4   // rows per thread per tile (rolled loop: also the serial memory-latency chain)
+#define NG_F_ITEMS 2   // rows per thread per batch (loads of all of them in flight, then evaluated)
 #endif
 constexpr int F_ITEMS = NG_F_ITEMS;
 constexpr int F_TILE = F_THREADS * F_ITEMS;
+constexpr int F_STAGE_ROWS = 8192;   // compaction: rows per chunk kept in shared memory (9 B each)
 
 size_t finalize_scratch_bytes(long long n)
 {
@@ -82,11 +83,11 @@ __device__ __forceinline__ void fin_load_x(const FinalizeArgs &A, FinIn &r)
     }
 }
 
-// value (0 when NULL), valid, passed.  Not inlined: the int128 compares and
-// the rare int128 division are large, and the callers loop over rows
-// (round 1: an unrolled evaluation made a ~175 KB kernel whose instruction-
-// cache misses dominated small R').
-__device__ __noinline__ void fin_eval(const FinalizeArgs &A, const FinIn &r, long long &value, bool &valid,
+// value (0 when NULL), valid, passed.  Inlined (a call would put the kernel
+// parameters and the row in local memory); callers unroll over at most
+// F_EVAL rows (round 1: 16 unrolled rows made a ~175 KB kernel whose
+// instruction-cache misses dominated small R').
+__device__ __forceinline__ void fin_eval(const FinalizeArgs &A, const FinIn &r, long long &value, bool &valid,
                                       bool &passed)
 {
     const long long c = r.kval ? r.cnt : 0;   // NULL key: empty subquery (R2)
@@ -115,11 +116,15 @@ __device__ __noinline__ void fin_eval(const FinalizeArgs &A, const FinIn &r, lon
     } else {
         p = false;
         if (vv && r.xv) {
-            const __int128 x = r.x;
-            if (A.agg == AVG)
-                p = cmp_rt<__int128>((__int128)A.a * x * c, A.outer_op, (__int128)A.b * acc);
-            else
-                p = cmp_rt<__int128>((__int128)A.a * x, A.outer_op, (__int128)A.b * v);
+            if (A.a == 1 && A.b == 1 && A.agg != AVG) {   // no scaling: a plain 64-bit compare (uniform branch)
+                p = cmp_rt<long long>(r.x, A.outer_op, v);
+            } else {
+                const __int128 x = r.x;
+                if (A.agg == AVG)
+                    p = cmp_rt<__int128>((__int128)A.a * x * c, A.outer_op, (__int128)A.b * acc);
+                else
+                    p = cmp_rt<__int128>((__int128)A.a * x, A.outer_op, (__int128)A.b * v);
+            }
         }
     }
     value = vv ? v : 0;
@@ -156,13 +161,14 @@ __global__ void __launch_bounds__(F_THREADS) finalize_all_kernel(FinalizeArgs A)
 #pragma unroll
         for (int j = 0; j < F_ITEMS; j++)
             if (b + j * nt < n) fin_load_x(A, r[j]);
-#pragma unroll 1
+#pragma unroll
         for (int j = 0; j < F_ITEMS; j++) {
-            if (b + j * nt >= n) break;
-            long long v;
-            bool vv, p;
-            fin_eval(A, r[j], v, vv, p);
-            fin_write(A, r[j], b + j * nt, v, vv, p);
+            if (b + j * nt < n) {
+                long long v;
+                bool vv, p;
+                fin_eval(A, r[j], v, vv, p);
+                fin_write(A, r[j], b + j * nt, v, vv, p);
+            }
         }
     }
     if (t0 == 0) *A.out_count = n;
@@ -179,13 +185,24 @@ __global__ void __launch_bounds__(F_THREADS, 2)
 finalize_compact_kernel(FinalizeArgs A, long long chunk, unsigned *__restrict__ bits,
                         unsigned long long *__restrict__ counts, unsigned *__restrict__ barrier)
 {
+    extern __shared__ __align__(16) unsigned char f_smem[];
     __shared__ unsigned long long s_red[F_WARPS];
     __shared__ unsigned s_wtot[F_WARPS];
     __shared__ unsigned long long s_base;
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const long long n = *A.d_nrp;
-    const long long c0 = blockIdx.x * chunk;
-    const long long c1 = min(n, c0 + chunk);
+    // chunks from the ACTUAL |R'| (the host sized the grid by its upper
+    // bound): whole 32-row words, every CTA a share
+    (void)chunk;
+    const long long chunk_d = ((n + gridDim.x - 1) / gridDim.x + 31) / 32 * 32;
+    const long long c0 = min(n, blockIdx.x * chunk_d);
+    const long long c1 = min(n, c0 + chunk_d);
+    // chunks that fit shared memory keep every row's (value, valid|passed)
+    // from phase 1, so phase 2 writes survivors without re-evaluating them
+    // (dense survivors, e.g. SF10 Q4's 92 %); larger chunks re-evaluate
+    const bool staged = chunk_d <= F_STAGE_ROWS && !A.out_sum;
+    long long *s_v = (long long *)f_smem;
+    uint8_t *s_f = f_smem + F_STAGE_ROWS * 8;
     // ---- phase 1: passed bits of every row of the chunk
     unsigned long long mycount = 0;
     const long long w0 = c0 / 32, w1 = c1 > c0 ? (c1 + 31) / 32 : w0;
@@ -201,13 +218,18 @@ finalize_compact_kernel(FinalizeArgs A, long long chunk, unsigned *__restrict__ 
 #pragma unroll
         for (int j = 0; j < F_ITEMS; j++)
             if (live[j]) fin_load_x(A, r[j]);
-#pragma unroll 1
+#pragma unroll
         for (int j = 0; j < F_ITEMS; j++) {
             bool p = false;
             if (live[j]) {
                 long long v;
                 bool vv;
                 fin_eval(A, r[j], v, vv, p);
+                if (staged) {
+                    const long long lr = (wb + (long long)j * F_WARPS) * 32 + lane - c0;
+                    s_v[lr] = v;
+                    s_f[lr] = (uint8_t)((vv ? 1 : 0) | (p ? 2 : 0));
+                }
             }
             const unsigned m = __ballot_sync(FULL, p);
             if (wb + (long long)j * F_WARPS < w1 && lane == 0) {
@@ -276,13 +298,22 @@ finalize_compact_kernel(FinalizeArgs A, long long chunk, unsigned *__restrict__ 
             const unsigned wv = __shfl_sync(FULL, word, w);
             if (rk < wtotal) {
                 const long long row = (g + warp * 32 + w) * 32 + (int)__fns(wv, 0, (int)(rk - ew) + 1);
-                FinIn r;
-                fin_load(A, row, r);
-                fin_load_x(A, r);
-                long long v;
-                bool vv, p;
-                fin_eval(A, r, v, vv, p);
-                fin_write(A, r, (long long)run + woff + rk, v, vv, p);
+                const long long pos = (long long)run + woff + rk;
+                if (staged) {
+                    const uint8_t f = s_f[row - c0];
+                    A.out_ids[pos] = A.row_id_base + A.ids[row];
+                    A.out_vals[pos] = s_v[row - c0];
+                    A.out_valid[pos] = f & 1;
+                    A.out_passed[pos] = (f >> 1) & 1;
+                } else {
+                    FinIn r;
+                    fin_load(A, row, r);
+                    fin_load_x(A, r);
+                    long long v;
+                    bool vv, p;
+                    fin_eval(A, r, v, vv, p);
+                    fin_write(A, r, pos, v, vv, p);
+                }
             }
         }
         run += btot;
@@ -312,9 +343,12 @@ cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *l
         e = cudaMemsetAsync(a.scratch, 0, finalize_zero_bytes(), st);
         if (e != cudaSuccess) return e;
     }
+    const int smem = F_STAGE_ROWS * 9;
     int occ = 0;
-    e = per_device_setup((const void *)finalize_compact_kernel, 0, &occ, [](int, int *v) {
-        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(v, finalize_compact_kernel, F_THREADS, 0);
+    e = per_device_setup((const void *)finalize_compact_kernel, 0, &occ, [&](int, int *v) {
+        cudaError_t e1 = cudaFuncSetAttribute(finalize_compact_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e1 != cudaSuccess) return e1;
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(v, finalize_compact_kernel, F_THREADS, smem);
     });
     if (e != cudaSuccess) return e;
     if (occ < 1) return cudaErrorInvalidConfiguration;
@@ -332,7 +366,7 @@ cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *l
     FinalizeArgs aa = a;
     void *args[] = {(void *)&aa, (void *)&chunk, (void *)&bits, (void *)&counts, (void *)&barrier};
     e = cudaLaunchCooperativeKernel((const void *)finalize_compact_kernel, dim3((unsigned)grid), dim3(F_THREADS),
-                                    args, 0, st);
+                                    args, (size_t)smem, st);
     ++*launches;
     return e;
 }
