@@ -705,6 +705,9 @@ def test_exec_graph_replay_matches(eng):
                 for rep in range(11):   # 8 direct runs, the capture, replays
                     g = eng.result_to_numpy(eng.exec(plan, R, S, index=idx, emit_all=True))
                     assert_parity(g, ref, plan, True, ctx=("graphs", graphs, plan["corr_op"], plan["agg"], rep))
+                    # survivors only: the cooperative compaction kernel inside the graph
+                    g = eng.result_to_numpy(eng.exec(plan, R, S, index=idx, emit_all=False))
+                    assert_parity(g, ref, plan, False, ctx=("graphs survivors", graphs, plan["corr_op"], rep))
         # in-place change of R.col2 (the compared column): replays read the new values
         eng.set_option(OPT_GRAPHS, 1)
         plan, mode = plans[1]

@@ -32,3 +32,21 @@ for name, k, v in (("16M u32+v32", rng.integers(0, 2 ** 31 - 1, 16_000_000).asty
     out.append("%s filter %.3f ms sort %.3f ms" % (name, best[0], best[1]))
     eng.release(m)
 print(os.path.basename(os.environ.get("NESTGPU_LIB", "default")), " | ".join(out))
+
+# library baseline on the same inputs: torch.sort (CUB radix sort pairs: key +
+# int64 index), CUDA events, best of 5
+import torch  # noqa: E402
+lib = []
+for name, k in (("16M u32 keys (+ int64 idx)", rng.integers(0, 2 ** 31 - 1, 16_000_000).astype(np.int32)),
+                ("38M u64-range keys (+ int64 idx)", (rng.integers(0, 15_000_000, 38_000_000) // 8 * 32).astype(np.int64))):
+    t = torch.from_numpy(k).cuda()
+    best = 1e9
+    for _ in range(6):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        torch.sort(t, stable=True)
+        b.record()
+        torch.cuda.synchronize()
+        best = min(best, a.elapsed_time(b))
+    lib.append("%s %.3f ms" % (name, best))
+print("torch.sort (CUB):", " | ".join(lib))
