@@ -470,8 +470,14 @@ nestgpu_status nestgpu_result_put(nestgpu_ctx *ctx, const nestgpu_result *res, v
  *     replayed afterwards (one graph launch instead of one launch per
  *     kernel; not with dedup, profiling or the malloc ablation).  Results
  *     are identical either way.
+ *   NESTGPU_OPT_SORT (value 0/1/2): the index build's sort -- 0 (default)
+ *     and 1 the LSD onesweep; 2 the two-round-trip MSD bucket sort
+ *     (partition by the top varying key bits, finish each bucket in shared
+ *     memory) wherever it fits, else the LSD onesweep.  An experiment kept
+ *     for measurement: 1.2-1.9x slower than the onesweep on every measured
+ *     shape.  Both are stable sorts of the same S'.
  * Errors: INVALID (unknown option). */
-enum { NESTGPU_OPT_MALLOC_SCRATCH = 1, NESTGPU_OPT_BNL_SHAPE = 2, NESTGPU_OPT_GRAPHS = 3 };
+enum { NESTGPU_OPT_MALLOC_SCRATCH = 1, NESTGPU_OPT_BNL_SHAPE = 2, NESTGPU_OPT_GRAPHS = 3, NESTGPU_OPT_SORT = 4 };
 nestgpu_status nestgpu_set_option(nestgpu_ctx *ctx, int32_t option, int64_t value);
 
 /* Per-stage device times (ms, CUDA events on the context stream) of the last

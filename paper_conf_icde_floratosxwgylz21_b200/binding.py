@@ -39,6 +39,7 @@ STRATEGIES = ("nested_loop", "index", "nested_loop_cached", "index_cached")
 OPT_MALLOC_SCRATCH = 1
 OPT_BNL_SHAPE = 2
 OPT_GRAPHS = 3
+OPT_SORT = 4   # 0 / 1 LSD onesweep (default), 2 MSD bucket sort experiment
 
 
 class NestGPUError(RuntimeError):

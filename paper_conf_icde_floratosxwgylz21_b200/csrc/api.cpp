@@ -109,6 +109,7 @@ struct nestgpu_ctx {
     bool malloc_scratch;
     std::vector<void *> mallocs;
     int bnl_shape;   // NESTGPU_OPT_BNL_SHAPE (test knob): 0 automatic, 1 full, 2 warp-split
+    int sort_mode;   // NESTGPU_OPT_SORT: 0 / 1 LSD onesweep, 2 MSD bucket sort (experiment)
     cudaEvent_t ev[NESTGPU_N_STAGES][2];
     // CUDA graphs of exec launch sequences (NESTGPU_OPT_GRAPHS, default on):
     // key = every argument that determines the sequence (plan, column /
@@ -449,6 +450,7 @@ nestgpu_status nestgpu_create(int device, void *d_arena, size_t arena_bytes, voi
     c->profiling = false;
     c->malloc_scratch = false;
     c->bnl_shape = 0;
+    c->sort_mode = 0;
     c->cap_stream = nullptr;
     {
         const char *gr = getenv("NESTGPU_GRAPHS");
@@ -741,26 +743,6 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     // pass: the first pass drops the high word, the last re-attaches it.
     const bool narrow = pre_narrow || (kb == 8 && np >= 2 && ((kand ^ kor) >> 32) == 0);
     const unsigned hi = pre_narrow ? pre_hi : (unsigned)(kand >> 32);
-    // one scratch region per pass, all zeroed with the digit histograms by
-    // one fill kernel
-    if (!small) {
-        ng::FillList fl;
-        fl.add(hist, ng::hist_bytes());
-        for (int p = 0; p < np; p++) {
-            const int kin = pre_narrow || (narrow && p > 0) ? 4 : kb;
-            const size_t zb = ng::sort_pass_zero_bytes(nsp, kin, vb, rb);
-            pscr[p] = salloc(c, zb);
-            if (!pscr[p]) return fail(c, NESTGPU_ERR_OOM, "arena exhausted (sort scratch)");
-            fl.add(pscr[p], zb);
-        }
-        CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
-    }
-    prof_begin(c, 2);
-    htrace(c, "fill2");
-    CUDA_TRY(c, ng::launch_digit_hist(fkb, tk, nsp, shifts, np, hist, dbase, c->num_sms, c->stream, &c->launches,
-                                      rb, true));
-    htrace(c, "hist");
-
     IndexRec ix{};
     ix.off = c->lo;
     ix.n = nsp;
@@ -776,7 +758,79 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     c->pinned[8 * 256 + 4] = (unsigned)(nsp & 0xffffffffu);
     c->pinned[8 * 256 + 5] = (unsigned)((unsigned long long)nsp >> 32);
     CUDA_TRY(c, cudaMemcpyAsync(ix.d_n, c->pinned + 8 * 256 + 4, 8, cudaMemcpyHostToDevice, c->stream));
-    if (np == 0) {
+    prof_begin(c, 2);
+    // Two-round-trip MSD bucket sort (k_bsort.cu, NESTGPU_OPT_SORT = 2 only:
+    // measured 1.2-1.9x slower than the LSD onesweep on every shape, DESIGN
+    // §18): partition by the top D varying bits, finish every bucket in
+    // shared memory.  Its histograms report the largest bucket; one more sync
+    // reads it, and skewed keys (a bucket past the finish capacity) fall
+    // through to the LSD onesweep below.
+    bool sorted = false;
+    if (c->sort_mode == 2 && np >= 1 && (kand ^ kor) != 0) {
+        const int kmid = narrow ? 4 : kb;
+        const unsigned long long var = kand ^ kor;
+        const int top = 63 - __builtin_clzll(var), low = __builtin_ctzll(var);
+        const long long cap = ng::bsort_capacity(kmid, vb);
+        int D = 1;
+        while (D < 12 && (double)nsp / (double)(1ll << D) > 0.6 * (double)cap) D++;
+        const int s1 = top - D + 1;
+        // finish passes: <= 6-bit windows over the varying bits below s1
+        int sh2[12], bt2[12], np2 = 0;
+        for (int b = low; b < s1 && np2 < 12;) {
+            if (!((var >> b) & 1ull)) {
+                b++;
+                continue;
+            }
+            const int w = s1 - b < 6 ? s1 - b : 6;
+            sh2[np2] = b;
+            bt2[np2++] = w;
+            b += w;
+        }
+        bool fits = (double)nsp / (double)(1ll << D) <= 0.9 * (double)cap && s1 > low && np2 > 0 && np2 <= 12;
+        if (fits) {
+            const int nb = 1 << D;
+            void *hs = salloc(c, ng::bsort_hist_bytes(nsp, nb));
+            unsigned *zs = (unsigned *)salloc(c, ng::bsort_zero_bytes(nb));
+            unsigned *bbase = (unsigned *)salloc(c, (size_t)(nb + 1) * 4);
+            unsigned *maxb = (unsigned *)(dsmall + 4);
+            if (!hs || !zs || !bbase) return fail(c, NESTGPU_ERR_OOM, "arena exhausted (bucket sort scratch)");
+            ng::FillList fl;
+            fl.add(zs, ng::bsort_zero_bytes(nb));
+            CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
+            CUDA_TRY(c, ng::launch_bsort_hist(fkb, tk, nsp, s1, nb, hs, zs, bbase, maxb, c->stream, &c->launches));
+            CUDA_TRY(c, cudaMemcpyAsync(c->pinned + 16, maxb, 4, cudaMemcpyDeviceToHost, c->stream));
+            CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+            htrace(c, "bsort hist + sync");
+            if ((long long)c->pinned[16] <= cap) {
+                CUDA_TRY(c, ng::launch_bsort_sort(fkb, kmid, kb, vb, tk, tv, uk, uv, ix.keys, ix.payload, nsp, s1, D,
+                                                  sh2, bt2, np2, hs, bbase, hi, c->stream, &c->launches));
+                sorted = true;
+                htrace(c, "bsort");
+            }
+        }
+    }
+    // one scratch region per pass, all zeroed with the digit histograms by
+    // one fill kernel
+    if (!sorted && !small) {
+        ng::FillList fl;
+        fl.add(hist, ng::hist_bytes());
+        for (int p = 0; p < np; p++) {
+            const int kin = pre_narrow || (narrow && p > 0) ? 4 : kb;
+            const size_t zb = ng::sort_pass_zero_bytes(nsp, kin, vb, rb);
+            pscr[p] = salloc(c, zb);
+            if (!pscr[p]) return fail(c, NESTGPU_ERR_OOM, "arena exhausted (sort scratch)");
+            fl.add(pscr[p], zb);
+        }
+        CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
+    }
+    htrace(c, "fill2");
+    if (!sorted) {
+        CUDA_TRY(c, ng::launch_digit_hist(fkb, tk, nsp, shifts, np, hist, dbase, c->num_sms, c->stream, &c->launches,
+                                          rb, true));
+        htrace(c, "hist");
+    }
+    if (sorted) {
+    } else if (np == 0) {
         if (nsp > 0) {
             CUDA_TRY(c, cudaMemcpyAsync(ix.keys, tk, (size_t)nsp * kb, cudaMemcpyDeviceToDevice, c->stream));
             if (vb) CUDA_TRY(c, cudaMemcpyAsync(ix.payload, tv, (size_t)nsp * vb, cudaMemcpyDeviceToDevice, c->stream));
@@ -1702,6 +1756,10 @@ nestgpu_status nestgpu_set_option(nestgpu_ctx *c, int32_t option, int64_t value)
         return NESTGPU_OK;
     case NESTGPU_OPT_GRAPHS:
         c->graphs_on = value != 0;
+        return NESTGPU_OK;
+    case NESTGPU_OPT_SORT:
+        if (value < 0 || value > 2) return fail(c, NESTGPU_ERR_INVALID, "set_option: sort 0, 1 or 2");
+        c->sort_mode = (int)value;
         return NESTGPU_OK;
     }
     return fail(c, NESTGPU_ERR_INVALID, "set_option: unknown option %d", option);

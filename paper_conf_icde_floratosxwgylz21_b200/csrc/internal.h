@@ -140,6 +140,26 @@ cudaError_t launch_radix_pass_x(int kb_in, int kb_out, int vb, const void *kin, 
 // scratch bytes of one radix pass that must be zero (per-tile digit counts + counter)
 size_t sort_pass_zero_bytes(long long n, int kb, int vb, int rb);
 
+// a4 (large S'): two-round-trip MSD bucket sort (k_bsort.cu).
+//   bsort_capacity: largest bucket the finish kernel sorts in shared memory
+//   launch_bsort_hist: group histograms of the D-bit digit at s1 (nb = 2^D
+//     <= 4096 buckets), scanned into per-group starts (hscratch,
+//     bsort_hist_bytes), bucket bases base[0..nb] and the largest bucket
+//     *maxb (device); zscratch (bsort_zero_bytes) must be zero
+//   launch_bsort_sort: partition kin -> kmid (kb_in -> kb_mid key bytes) by
+//     the D-bit digit, then finish each bucket kmid -> kout (kb_mid ->
+//     kb_out; 4 -> 8 re-attaches hi) over the np2 <= 6-bit digit windows
+//     (pshift, pbits); valid only when *maxb <= bsort_capacity(kb_mid, vb)
+int bsort_capacity(int kb_mid, int vb);
+size_t bsort_hist_bytes(long long n, int nb);
+size_t bsort_zero_bytes(int nb);
+cudaError_t launch_bsort_hist(int kb_in, const void *keys, long long n, int s1, int nb, void *hscratch,
+                              unsigned *zscratch, unsigned *base, unsigned *maxb, cudaStream_t st, long long *launches);
+cudaError_t launch_bsort_sort(int kb_in, int kb_mid, int kb_out, int vb, const void *kin, const void *vin,
+                              void *kmid, void *vmid, void *kout, void *vout, long long n, int s1, int D,
+                              const int *pshift, const int *pbits, int np2, const void *hscratch,
+                              const unsigned *base, unsigned hi, cudaStream_t st, long long *launches);
+
 // Partial aggregates per R' tuple: acc (int64) + cnt (int64); identity init.
 // n: host upper bound (grid size); d_n: the actual count (device)
 cudaError_t launch_init_partials(long long n, const long long *d_n, int agg, long long *acc, long long *cnt,

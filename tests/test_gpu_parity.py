@@ -545,6 +545,98 @@ def test_index_sort_large(eng, pattern, pay):
     test_index_sort_digit_windows(eng, pattern, 3_000_017, pay)
 
 
+def _check_index_sorted(eng, ix, k, kdt, pay):
+    """The index is the encoded keys ascending, every payload exactly once and
+    carried by its own key (payload = row id, scaled for int64)."""
+    import torch
+    n = len(k)
+    info = eng.index_info(ix)
+    kb = 4 if kdt == "int32" else 8
+    assert info["n"] == n and info["key_bytes"] == kb
+    if kb == 4:
+        enc = k.astype(np.int32).view(np.uint32) ^ np.uint32(0x80000000)
+        keys = eng.arena_view(info["d_keys"], n * 4).view(torch.int32).cpu().numpy().view(np.uint32)
+    else:
+        enc = k.view(np.uint64) ^ np.uint64(1 << 63)
+        keys = eng.arena_view(info["d_keys"], n * 8).view(torch.int64).cpu().numpy().view(np.uint64)
+    assert np.array_equal(keys, np.sort(enc))
+    if pay is not None:
+        vb = 4 if pay == "int32" else 8
+        tdt = torch.int32 if vb == 4 else torch.int64
+        p = eng.arena_view(info["d_payload"], n * vb).view(tdt).cpu().numpy().astype(np.int64)
+        row = p if vb == 4 else p // ((1 << 33) + 1)
+        assert np.array_equal(np.sort(row), np.arange(n))
+        assert np.array_equal(keys, enc[row])
+        return keys, row
+    return keys, None
+
+
+def _skewed_keys(n, rng):
+    """27 varying bits, but 3/4 of the keys in one 2^12-wide range: one
+    partition bucket far past the finish capacity (falls back to the LSD
+    sort)."""
+    k = rng.integers(0, 1 << 27, n)
+    k[: 3 * n // 4] = (5 << 20) + rng.integers(0, 1 << 12, 3 * n // 4)
+    return rng.permutation(k), "int32"
+
+
+@pytest.mark.parametrize("pattern", ["mult32_lt2^26", "bits1_to_27", "i64_low_word", "i64_straddle",
+                                     "i64_full", "i64_all_equal", "i32_negative_dups", "skewed"])
+@pytest.mark.parametrize("n", [2, 4097, 100_003, 1_000_003])
+@pytest.mark.parametrize("pay", ["int32", "int64", None])
+def test_index_bucket_sort(eng, pattern, n, pay):
+    """The two-round-trip MSD bucket sort (k_bsort.cu; NESTGPU_OPT_SORT = 2
+    forces it wherever the keys vary in more bits than its partition digit):
+    every key pattern, 0/4/8-byte payloads (4- to 16-byte items: every tile /
+    bucket register shape), sizes inside one tile, across tiles and groups
+    with ragged tails.  Same checks as the LSD sort (which runs beside it on
+    the same S)."""
+    from paper_conf_icde_floratosxwgylz21_b200.binding import OPT_SORT
+    import torch
+    rng = np.random.default_rng([zlib.crc32(pattern.encode()), n, 3])
+    k, kdt = _skewed_keys(n, rng) if pattern == "skewed" else _key_pattern(pattern, n, rng)
+    k = np.asarray(k, dtype=np.int64)
+    cols, dts = {"k": k}, {"k": kdt}
+    if pay is not None:
+        cols["v"] = np.arange(n, dtype=np.int64) * (1 if pay == "int32" else (1 << 33) + 1)
+        dts["v"] = pay
+    m = eng.mark()
+    try:
+        S = eng.load_table(cols, dtypes=dts)
+        for mode in (2, 1):
+            eng.set_option(OPT_SORT, mode)
+            ix = eng.build_index(S, ["k"], "v" if pay else None)
+            _check_index_sorted(eng, ix, k, kdt, pay)
+    finally:
+        eng.set_option(OPT_SORT, 0)
+        eng.release(m)
+
+
+@pytest.mark.parametrize("pattern,pay", [("bits1_to_27", "int32"), ("i64_low_word", None),
+                                         ("i64_straddle", "int64"), ("skewed", "int32")])
+def test_index_bucket_sort_large(eng, pattern, pay):
+    """The bucket sort at 3M keys: ~90-370 partition groups, 4096 buckets (the
+    skewed keys fall back to the LSD sort after the bucket histogram)."""
+    from paper_conf_icde_floratosxwgylz21_b200.binding import OPT_SORT
+    eng.set_option(OPT_SORT, 2)
+    rng = np.random.default_rng([zlib.crc32(pattern.encode()), 7])
+    n = 3_000_017
+    k, kdt = _skewed_keys(n, rng) if pattern == "skewed" else _key_pattern(pattern, n, rng)
+    k = np.asarray(k, dtype=np.int64)
+    cols, dts = {"k": k}, {"k": kdt}
+    if pay is not None:
+        cols["v"] = np.arange(n, dtype=np.int64) * (1 if pay == "int32" else (1 << 33) + 1)
+        dts["v"] = pay
+    m = eng.mark()
+    try:
+        S = eng.load_table(cols, dtypes=dts)
+        ix = eng.build_index(S, ["k"], "v" if pay else None)
+        _check_index_sorted(eng, ix, k, kdt, pay)
+    finally:
+        eng.set_option(OPT_SORT, 0)
+        eng.release(m)
+
+
 @pytest.mark.parametrize("pattern", ["mult32_lt2^26", "bits1_to_27", "i64_low_word", "i64_straddle"])
 def test_dedup_sort_digit_windows(eng, pattern):
     """The R' key sort of caching on the same key patterns: results
