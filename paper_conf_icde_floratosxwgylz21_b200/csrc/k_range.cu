@@ -441,10 +441,19 @@ __global__ void __launch_bounds__(P_THREADS) block_prefix_kernel(const V *__rest
     const long long b0 = blockIdx.x * (long long)P_BLOCK;
     if (threadIdx.x == 0) s_carry = bpre[blockIdx.x];
     if (blockIdx.x == 0 && threadIdx.x == 0) out[BACK ? N : 0] = ident<AGG>();
+    // every row of the block loaded up front (one DRAM round trip, not one
+    // per 256-row step of the barrier-separated scan below)
+    long long xs[P_ITEMS];
+#pragma unroll
+    for (int j = 0; j < P_ITEMS; j++) {
+        const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
+        xs[j] = e < N ? elem<V, BACK, PART>(v, N, e) : ident<AGG>();
+    }
     __syncthreads();
+#pragma unroll
     for (int j = 0; j < P_ITEMS; j++) {   // rows of the block in order, 256 at a time
         const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
-        long long incl = e < N ? elem<V, BACK, PART>(v, N, e) : ident<AGG>();
+        long long incl = xs[j];
         for (int o = 1; o < 32; o <<= 1) {
             const long long y = __shfl_up_sync(FULL, incl, o);
             if (lane >= o) incl = comb<AGG>(incl, y);
@@ -514,11 +523,19 @@ __global__ void __launch_bounds__(P_THREADS) seg_block_kernel(const K *__restric
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const long long b0 = blockIdx.x * (long long)G_BLOCK;
     if (threadIdx.x == 0) s_carry = WRITE ? SegPair<AGG>{bv[blockIdx.x], 0} : SegPair<AGG>{ident<AGG>(), 0};
-    __syncthreads();
+    // the block's rows loaded up front (one DRAM round trip per CTA)
+    SegPair<AGG> xs[G_ITEMS];
+#pragma unroll
     for (int j = 0; j < G_ITEMS; j++) {
         const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
-        SegPair<AGG> x{ident<AGG>(), 0};
-        if (e < N) x = SegPair<AGG>{(long long)v[e], (e == 0 || keys[e] != keys[e - 1]) ? 1 : 0};
+        xs[j] = SegPair<AGG>{ident<AGG>(), 0};
+        if (e < N) xs[j] = SegPair<AGG>{(long long)v[e], (e == 0 || keys[e] != keys[e - 1]) ? 1 : 0};
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < G_ITEMS; j++) {
+        const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
+        const SegPair<AGG> x = xs[j];
         const SegPair<AGG> incl = warp_seg_scan<AGG>(x, lane);
         if (lane == 31) {
             s_wv[warp] = incl.v;

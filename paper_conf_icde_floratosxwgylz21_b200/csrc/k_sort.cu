@@ -385,12 +385,22 @@ __global__ void __launch_bounds__(256) digit_hist_kernel(const K *__restrict__ k
     __shared__ unsigned s_w[8];
     for (int i = threadIdx.x; i < dl.n * NB; i += 256) s_hist[i] = 0;
     __syncthreads();
+    // HB keys per thread per round are loaded before any is counted: the
+    // shared-memory atomics would otherwise serialise one DRAM round trip per
+    // key (a small S' has only a few CTAs, each with a long chain)
+    constexpr int HB = 8;
     const long long stride = (long long)gridDim.x * 256;
-    for (long long i = blockIdx.x * 256LL + threadIdx.x; i < n; i += stride) {
-        const K k = keys[i];
+    for (long long i0 = blockIdx.x * 256LL + threadIdx.x; i0 < n; i0 += stride * HB) {
+        K k[HB];
 #pragma unroll
-        for (int p = 0; p < 8; p++)
-            if (p < dl.n) atomicAdd(&s_hist[p * NB + (unsigned)((k >> dl.shift[p]) & (NB - 1))], 1u);
+        for (int u = 0; u < HB; u++) k[u] = i0 + u * stride < n ? __ldg(keys + i0 + u * stride) : (K)0;
+#pragma unroll
+        for (int u = 0; u < HB; u++) {
+            if (i0 + u * stride >= n) break;
+#pragma unroll
+            for (int p = 0; p < 8; p++)
+                if (p < dl.n) atomicAdd(&s_hist[p * NB + (unsigned)((k[u] >> dl.shift[p]) & (NB - 1))], 1u);
+        }
     }
     __syncthreads();
     for (int i = threadIdx.x; i < dl.n * NB; i += 256)
