@@ -43,6 +43,7 @@ struct Column {
     bool alive;
     bool stats;         // host-side min/max known
     long long mn, mx;
+    bool sorted;        // (with stats) NOT NULL and stored in ascending key order
     bool caller_filled; // nestgpu_alloc_column: contents may change behind our back (stats not cached)
 };
 
@@ -389,13 +390,16 @@ namespace {
 nestgpu_status column_stats(nestgpu_ctx *c, Column &col)
 {
     if (col.stats) return NESTGPU_OK;
-    long long *d = (long long *)salloc(c, 16);
+    long long *d = (long long *)salloc(c, 24);
     if (!d) return fail(c, NESTGPU_ERR_OOM, "arena exhausted (stats)");
     CUDA_TRY(c, ng::launch_minmax(col.d, dtype_width(col.dtype), col.valid, col.n, d, c->stream, &c->launches));
-    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, d, 16, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, d, 24, cudaMemcpyDeviceToHost, c->stream));
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    long long desc;
     memcpy(&col.mn, c->pinned, 8);
     memcpy(&col.mx, (char *)c->pinned + 8, 8);
+    memcpy(&desc, (char *)c->pinned + 16, 8);
+    col.sorted = !col.valid && desc == 0;
     col.stats = true;
     return NESTGPU_OK;
 }
@@ -642,6 +646,68 @@ nestgpu_status nestgpu_gather_column(nestgpu_ctx *c, int32_t src_col, const int6
     return NESTGPU_OK;
 }
 
+// Sort-free index build for a key-ordered column (column statistics: NOT
+// NULL, every row >= its predecessor -- e.g. TPC-H lineitem stored by
+// l_orderkey, partsupp by ps_partkey): the stable sort of S' is then the
+// identity, so the index is S' itself, compacted IN ROW ORDER by the ordered
+// two-pass filter straight into the index arrays.  The count pass + scan run
+// first; one sync reads |S'|; the index is allocated at its exact size and
+// the write pass fills it.  Same bytes as the sorting build.
+static nestgpu_status build_index_ordered(nestgpu_ctx *c, const int32_t *key_cols, int32_t n_key_cols,
+                                          int32_t payload_col, const nestgpu_pred *inner_preds,
+                                          int32_t n_inner_preds, const ng::KeySrc &ks, const ng::PredSet &ps,
+                                          const ng::ValSrc &vs, int kb, int vb, int64_t n, const Column *pc,
+                                          int32_t *out_index)
+{
+    scratch_reset(c);
+    for (int st = 0; st < NESTGPU_N_STAGES; st++) c->ran[st] = false;
+    void *fscr = salloc(c, ng::filter_scratch_bytes(n));
+    long long *dsmall = (long long *)salloc(c, 64);
+    if (!fscr || !dsmall) return fail(c, NESTGPU_ERR_OOM, "arena exhausted building an index over %lld rows", (long long)n);
+    {
+        ng::FillList fl;
+        fl.add(dsmall, 16);
+        fl.add(fscr, ng::filter_zero_bytes(n, false));
+        CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
+    }
+    prof_begin(c, 1);
+    CUDA_TRY(c, ng::launch_filter(n, ps, ks, kb, vs, vb, 0, 0, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr,
+                                  fscr, dsmall, c->stream, &c->launches, true, 1));
+    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, dsmall, 8, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    htrace(c, "ordered count + sync");
+    long long nsp;
+    memcpy(&nsp, c->pinned, 8);
+    IndexRec ix{};
+    ix.off = c->lo;
+    ix.n = nsp;
+    ix.kb = kb;
+    ix.vb = vb;
+    ix.d_n = (long long *)palloc(c, 8);
+    ix.keys = palloc(c, (size_t)(nsp > 0 ? nsp : 1) * kb);
+    ix.payload = vb ? palloc(c, (size_t)(nsp > 0 ? nsp : 1) * vb) : nullptr;
+    if (!ix.d_n || !ix.keys || (vb && !ix.payload)) {
+        c->lo = ix.off;
+        return fail(c, NESTGPU_ERR_OOM, "arena exhausted storing an index of %lld rows", nsp);
+    }
+    CUDA_TRY(c, cudaMemcpyAsync(ix.d_n, dsmall, 8, cudaMemcpyDeviceToDevice, c->stream));
+    if (nsp > 0)
+        CUDA_TRY(c, ng::launch_filter(n, ps, ks, kb, vs, vb, 0, 0, nullptr, ix.keys, nullptr, ix.payload, nullptr,
+                                      nullptr, fscr, dsmall, c->stream, &c->launches, true, 2));
+    prof_end(c, 1);
+    ix.key_cols[0] = key_cols[0];
+    ix.key_cols[1] = n_key_cols == 2 ? key_cols[1] : -1;
+    ix.n_key = n_key_cols;
+    ix.payload_col = payload_col;
+    ix.inner.assign(inner_preds, inner_preds + n_inner_preds);
+    ix.payload_nullable = pc && pc->valid;
+    ix.alive = true;
+    *out_index = put_slot(c->idx, ix);
+    CUDA_TRY(c, cudaGetLastError());
+    htrace_end(c, "build_index (key-ordered column, no sort)");
+    return NESTGPU_OK;
+}
+
 nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int32_t n_key_cols, int32_t payload_col,
                                    const nestgpu_pred *inner_preds, int32_t n_inner_preds, int32_t *out_index)
 {
@@ -666,6 +732,18 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     }
     const int kb = key_bytes(c, key_cols, n_key_cols);
     const int vb = pc ? vs.w : 0;
+    bool stats_fresh = false;
+    if (n_key_cols == 1 && c->sort_mode != 1) {
+        Column &kc = c->cols[key_cols[0]];
+        if (!kc.valid && !(pc && pc->valid)) {
+            if (kc.caller_filled) kc.stats = false;   // recomputed: the caller may have rewritten it
+            stats_fresh = true;
+            if ((s = column_stats(c, kc))) return s;
+            if (kc.sorted)
+                return build_index_ordered(c, key_cols, n_key_cols, payload_col, inner_preds, n_inner_preds, ks, ps,
+                                           vs, kb, vb, n, pc, out_index);
+        }
+    }
     // 64-bit keys of one column whose encoded min and max share the high word
     // (column statistics, computed once per column): every key does, so the
     // S' filter already writes 32-bit keys and the whole sort runs on them;
@@ -675,7 +753,7 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     unsigned pre_hi = 0;
     if (kb == 8 && n_key_cols == 1) {
         Column &kc = c->cols[key_cols[0]];
-        if (kc.caller_filled) kc.stats = false;   // recomputed: the caller may have rewritten it
+        if (kc.caller_filled && !stats_fresh) kc.stats = false;   // recomputed: the caller may have rewritten it
         if ((s = column_stats(c, kc))) return s;
         const unsigned long long emn = (unsigned long long)kc.mn ^ 0x8000000000000000ull;
         const unsigned long long emx = (unsigned long long)kc.mx ^ 0x8000000000000000ull;

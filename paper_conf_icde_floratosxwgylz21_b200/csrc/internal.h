@@ -107,12 +107,17 @@ size_t finalize_zero_bytes();   // the part of the finalize scratch that must be
 //                (u64)[2..3] = max |payload| (atomicMax; 32-bit partial sums)
 //   scratch    : tile status + counter, from filter_scratch_bytes(n)
 //   out_count  : int64 survivor count (device)
+//   ordered_phase: 0 = one call (ordered iff out_ids); 1 / 2 = the two
+//     halves of an ordered filter without row ids: 1 counts + scans (the
+//     caller reads *out_count and sizes the outputs), 2 writes the outputs
+//     (same arguments and scratch; drop_null_* must be 0)
 size_t filter_scratch_bytes(long long n);
 cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, int kb,
                           const ValSrc &val, int vb, int drop_null_key, int drop_null_val,
                           int *out_ids, void *out_keys, uint8_t *out_kvalid, void *out_vals,
                           unsigned long long *keymask, unsigned *extreme, void *scratch,
-                          long long *out_count, cudaStream_t st, long long *launches, bool prezeroed = false);
+                          long long *out_count, cudaStream_t st, long long *launches, bool prezeroed = false,
+                          int ordered_phase = 0);
 
 // a4: histograms of the digits at `shifts` (np of them) over n encoded keys,
 // and their exclusive scans into digit_base[np][256].

@@ -1004,9 +1004,10 @@ static void resolve(const SrcCols &sc, const SrcPlan &sp, TPlan &tp)
 cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, int kb, const ValSrc &val, int vb,
                           int drop_null_key, int drop_null_val, int *out_ids, void *out_keys, uint8_t *out_kvalid,
                           void *out_vals, unsigned long long *keymask, unsigned *extreme, void *scratch,
-                          long long *out_count, cudaStream_t st, long long *launches, bool prezeroed)
+                          long long *out_count, cudaStream_t st, long long *launches, bool prezeroed,
+                          int ordered_phase)
 {
-    cudaError_t e = prezeroed ? cudaSuccess : cudaMemsetAsync(out_count, 0, sizeof(long long), st);
+    cudaError_t e = prezeroed || ordered_phase == 2 ? cudaSuccess : cudaMemsetAsync(out_count, 0, sizeof(long long), st);
     if (e != cudaSuccess || n <= 0) return e;
     // the column segments a tile needs, deduplicated
     SrcCols sc;
@@ -1046,9 +1047,10 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
     const int items = layout(sc, 16);
     if (!items) return cudaErrorInvalidValue;
     resolve(sc, sp, tp);
-    const bool one_pass = out_ids && !out_vals && !extreme && !drop_null_key && !drop_null_val && k &&
+    const bool ordered = out_ids || ordered_phase;
+    const bool one_pass = out_ids && !ordered_phase && !out_vals && !extreme && !drop_null_key && !drop_null_val && k &&
                           !getenv_two_pass();
-    if (!prezeroed || (out_ids && !one_pass)) {
+    if (ordered_phase != 2 && (!prezeroed || (out_ids && !one_pass))) {
         e = cudaMemsetAsync(scratch, 0, 1024, st);
         if (e != cudaSuccess) return e;
     }
@@ -1073,13 +1075,22 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
         ++*launches;
         return e;
     }
-    if (out_ids) {
-        // Ordered (R'): pass 1 counts survivors per tile reading only the
-        // predicate columns (same tile size as pass 2), then an exclusive scan.
+    if (ordered) {
+        // Ordered (R', or S' of a key-ordered column): pass 1 counts
+        // survivors per tile reading only the predicate columns (same tile
+        // size as pass 2), then an exclusive scan.  ordered_phase 1 stops
+        // after the scan (*out_count is final: the caller sizes the output),
+        // 2 runs only pass 2 with the same scratch.
         if (drop_null_key || drop_null_val) return cudaErrorInvalidValue;
         const long long tiles = (n + T_THREADS * items - 1) / (T_THREADS * items);
         unsigned *tcount = (unsigned *)((char *)scratch + 1024);
         unsigned long long *tbase = (unsigned long long *)((char *)scratch + 1024 + ((tiles * 4 + 255) & ~255ll));
+        if (ordered_phase == 2) {
+            o.tile_base = tbase;
+            e = dispatch(k, v, items, n, sc, tp, o, num_sms, st);
+            ++*launches;
+            return e;
+        }
         SrcCols sc1 = sc;
         sc1.n = n_pred_src;   // predicate columns come first in the source list
         int off = 0;
@@ -1099,6 +1110,7 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
         tile_scan_kernel<<<1, 1024, 0, st>>>(tcount, tiles, tbase, out_count);
         o.tile_base = tbase;
         *launches += 2;
+        if (ordered_phase == 1) return cudaGetLastError();
     }
     e = dispatch(k, v, items, n, sc, tp, o, num_sms, st);
     ++*launches;

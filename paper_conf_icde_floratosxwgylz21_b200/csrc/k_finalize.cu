@@ -396,29 +396,36 @@ cudaError_t launch_init_partials(long long n, const long long *d_n, int agg, lon
 
 // ------------------------------------------------------------------ column min / max
 // (for the SUM/AVG overflow pre-check, reading R5)
+// (and out[2] != 0 iff some row is smaller than its predecessor: the
+// column is not stored in key order -- the index build's sort-free path)
 __global__ void minmax_init_kernel(long long *out)
 {
     out[0] = LLONG_MAX;
     out[1] = LLONG_MIN;
+    out[2] = 0;
 }
 
 __global__ void minmax_kernel(const void *__restrict__ col, int w, const uint8_t *__restrict__ valid, long long n,
                               long long *__restrict__ out)
 {
     long long mn = LLONG_MAX, mx = LLONG_MIN;
+    bool desc = false;
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
         if (valid && !valid[i]) continue;
         const long long v = load_w(col, w, i);
         mn = min(mn, v);
         mx = max(mx, v);
+        if (i > 0 && !valid) desc |= load_w(col, w, i - 1) > v;
     }
     for (int o = 16; o > 0; o >>= 1) {
         mn = min(mn, __shfl_xor_sync(FULL, mn, o));
         mx = max(mx, __shfl_xor_sync(FULL, mx, o));
     }
+    desc = __any_sync(FULL, desc);
     if ((threadIdx.x & 31) == 0) {
         atomicMin(&out[0], mn);
         atomicMax(&out[1], mx);
+        if (desc) atomicOr((unsigned long long *)&out[2], 1ull);
     }
 }
 

@@ -571,6 +571,122 @@ def _check_index_sorted(eng, ix, k, kdt, pay):
     return keys, None
 
 
+@pytest.mark.parametrize("kdt", ["int32", "int64"])
+@pytest.mark.parametrize("pay", ["int32", "int64", None])
+@pytest.mark.parametrize("n,pred", [(1, False), (5000, False), (300_007, True), (2_000_003, True),
+                                    (2_000_003, False)])
+def test_index_key_ordered_column(eng, kdt, pay, n, pred):
+    """Sort-free index build: a NOT NULL key column stored in ascending order
+    (column statistics; TPC-H lineitem by l_orderkey, partsupp by ps_partkey)
+    is compacted in row order by the ordered filter straight into the index.
+    The stable sort of S' is the identity, so the index must be S' exactly:
+    keys ascending and, within equal keys, payloads in row order -- and the
+    LSD sort of the same S (NESTGPU_OPT_SORT = 1) must hold the same keys and
+    the same (key, payload) pairs.  Then '=' / '<' plans through both indexes
+    vs the oracle."""
+    from paper_conf_icde_floratosxwgylz21_b200.binding import OPT_SORT
+    import torch
+    rng = np.random.default_rng([n, len(kdt), 0 if pay is None else len(pay)])
+    k = np.sort(rng.integers(-(1 << 33) if kdt == "int64" else -(1 << 20), 1 << 20, n))
+    k[n // 3: n // 3 + min(n, 50)] = k[n // 3] if n > 1 else k[:1]   # a long run of one key
+    k = np.sort(k)
+    v = rng.integers(-1000, 1000, n) * (1 if pay != "int64" else (1 << 34))
+    c3 = rng.integers(0, 4, n)
+    cols, dts = {"col1": k, "col3": c3}, {"col1": kdt, "col3": "int32"}
+    if pay is not None:
+        cols["col2"], dts["col2"] = v, pay
+    preds = [{"col": "col3", "op": "!=", "lit": 1}] if pred else []
+    keep = c3 != 1 if pred else np.ones(n, bool)
+    m = eng.mark()
+    try:
+        S = eng.load_table(cols, dtypes=dts)
+        got = {}
+        for mode in (0, 1):
+            eng.set_option(OPT_SORT, mode)
+            eng.set_profiling(True)
+            ix = eng.build_index(S, ["col1"], "col2" if pay else None, preds)
+            prof = eng.last_profile()
+            eng.set_profiling(False)
+            info = eng.index_info(ix)
+            ns = int(keep.sum())
+            assert info["n"] == ns
+            kb = 4 if kdt == "int32" else 8
+            tdt = torch.int32 if kb == 4 else torch.int64
+            keys = np.zeros(0, np.int64)
+            if ns:
+                kr = eng.arena_view(info["d_keys"], ns * kb).view(tdt).cpu().numpy()
+                keys = kr.view(np.uint32).astype(np.int64) if kb == 4 else kr
+            enc = k[keep].astype(np.int64)
+            enc_u = (enc.astype(np.int32).view(np.uint32) ^ np.uint32(1 << 31)).astype(np.int64) if kb == 4 else \
+                (enc.view(np.uint64) ^ np.uint64(1 << 63)).view(np.int64)
+            assert np.array_equal(keys, enc_u)
+            p = None
+            if pay is not None and ns:
+                vbt = torch.int32 if pay == "int32" else torch.int64
+                vbb = 4 if pay == "int32" else 8
+                p = eng.arena_view(info["d_payload"], ns * vbb).view(vbt).cpu().numpy().astype(np.int64)
+            got[mode] = (keys, p, prof)
+            if mode == 0:
+                if pay is not None and ns:
+                    assert np.array_equal(p, v[keep])          # row order inside every key run
+                assert np.isnan(prof["sort"])                   # no sort ran
+        if pay is not None and info["n"]:
+            a = np.lexsort((got[0][1], got[0][0]))
+            b = np.lexsort((got[1][1], got[1][0]))
+            assert np.array_equal(got[0][0][a], got[1][0][b]) and np.array_equal(got[0][1][a], got[1][1][b])
+        eng.set_option(OPT_SORT, 0)
+        R = {"col1": rng.integers(int(k.min()) - 2, int(k.max()) + 3, 2001), "col2": rng.integers(-1000, 1000, 2001)}
+        t = {"R": R, "S": cols}
+        dt = {"R": {"col1": kdt, "col2": pay or "int32"}, "S": dts}
+        for corr_op, agg in (("=", "min" if pay else "count"), ("=", "exists"), ("<", "count"), ("=", "sum" if pay else "count")):
+            plan = make_plan(corr_op, agg, "<=", inner_preds=preds)
+            if pay is None and agg in ("min", "sum"):
+                continue
+            assert_parity(run(eng, t, plan, "index", emit_all=True, dtypes=dt), oracle.evaluate(t, plan), plan, True,
+                          ctx=(kdt, pay, n, pred, corr_op, agg))
+    finally:
+        eng.set_option(OPT_SORT, 0)
+        eng.set_profiling(False)
+        eng.release(m)
+
+
+def test_index_almost_ordered_column_sorts(eng):
+    """One descent in an otherwise ascending column: not key-ordered, the
+    index is sorted (LSD) and still exact; and a caller-filled column whose
+    contents change between builds has its order re-checked."""
+    import torch
+    n = 100_003
+    k = np.arange(n, dtype=np.int32) * 3
+    k[n // 2], k[n // 2 + 1] = k[n // 2 + 1], k[n // 2]
+    m = eng.mark()
+    try:
+        S = eng.load_table({"col1": k, "col2": np.arange(n, dtype=np.int32)})
+        assert eng.index_info(eng.build_index(S, ["col1"], "col2"))["key_bytes"] == 4
+        ix = eng.build_index(S, ["col1"], "col2")
+        info = eng.index_info(ix)
+        keys = eng.arena_view(info["d_keys"], n * 4).view(torch.int32).cpu().numpy().view(np.uint32)
+        assert np.array_equal(keys, np.sort(k.astype(np.int32).view(np.uint32) ^ np.uint32(1 << 31)))
+        # caller-filled column: first ordered, then rewritten unordered
+        cid = eng.alloc_column(n, "int32")
+        view = eng.arena_view(eng.column_info(cid)["d_values"], n * 4).view(torch.int32)
+        view.copy_(torch.from_numpy(np.arange(n, dtype=np.int32)))
+        S2 = dict(S)
+        S2["col1"] = cid
+        ix2 = eng.build_index(S2, ["col1"], "col2")
+        i2 = eng.index_info(ix2)
+        got = eng.arena_view(i2["d_keys"], n * 4).view(torch.int32).cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), np.arange(n, dtype=np.uint32) ^ np.uint32(1 << 31))
+        view.copy_(torch.from_numpy(np.arange(n, dtype=np.int32)[::-1].copy()))
+        ix3 = eng.build_index(S2, ["col1"], "col2")
+        i3 = eng.index_info(ix3)
+        got = eng.arena_view(i3["d_keys"], n * 4).view(torch.int32).cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), np.arange(n, dtype=np.uint32) ^ np.uint32(1 << 31))
+        pay = eng.arena_view(i3["d_payload"], n * 4).view(torch.int32).cpu().numpy()
+        assert np.array_equal(pay, np.arange(n)[::-1])
+    finally:
+        eng.release(m)
+
+
 def _skewed_keys(n, rng):
     """27 varying bits, but 3/4 of the keys in one 2^12-wide range: one
     partition bucket far past the finish capacity (falls back to the LSD

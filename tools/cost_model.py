@@ -106,9 +106,18 @@ def stats(tables, plan, survivors):
     k = {"=": ub - lb, "!=": N - (ub - lb), "<": N - ub, "<=": N - lb, ">": lb, ">=": ub}[op]
     value = plan["agg"] in ("min", "max", "sum", "avg")
     vb = S[plan["agg_col"]].dtype.itemsize if value else 0
+    sp = _passes(sk, kb)
+    # a NOT NULL key column stored in ascending order needs no sort (the
+    # engine's key-ordered index build, api.cpp build_index_ordered)
+    sv = tables.get("S_valid") or {}
+    if (len(plan["inner_key"]) == 1 and sv.get(plan["inner_key"][0]) is None
+            and (not value or sv.get(plan["agg_col"]) is None)):
+        col = np.asarray(S[plan["inner_key"][0]])
+        if len(col) < 2 or bool(np.all(col[1:] >= col[:-1])):
+            sp = 0
     return dict(n_r=len(rm), n_s=len(sm), n_rp=int(rm.sum()), n_sp=int(sm.sum()),
                 n_distinct=int(len(np.unique(rk))), sum_k=int(k.sum()), survivors=int(survivors),
-                key_bytes=kb, payload_bytes=vb, sort_passes=_passes(sk, kb), dedup_passes=_passes(rk, kb),
+                key_bytes=kb, payload_bytes=vb, sort_passes=sp, dedup_passes=_passes(rk, kb),
                 narrow_keys=_narrow(sk, kb), corr_op=op, agg=plan["agg"])
 
 

@@ -32,7 +32,8 @@ def ideal_stages(tabs, plan, st, use_index, survivors, hbm_gbps, alu_ms):
     nested loop runs at its integer-pipe bound.  Bytes per stage:
       S' filter  n_S x (inner predicate + key + payload column widths) read
                  + |S'| x (key + payload) written
-      sort       one read + one write of |S'| x (key + payload) (lower bound)
+      sort       one read + one write of |S'| x (key + payload) (lower bound;
+                 none for a key-ordered column, which the engine does not sort)
       R' filter  n_R x (outer predicate + key column widths) read
                  + |R'| x (4-byte id + key) written
       probe      |R'| x key read + sum_k x payload read + |R'| x 16 B partials
@@ -54,8 +55,9 @@ def ideal_stages(tabs, plan, st, use_index, survivors, hbm_gbps, alu_ms):
     b = {"inner_filter": n_s * in_w + st["n_sp"] * (kb + vb),
          "outer_filter": n_r * out_w + st["n_rp"] * (4 + kb),
          "finalize": st["n_rp"] * (16 + 4 + xw) + survivors * 18}
-    if use_index:
+    if use_index and st["sort_passes"] > 0:   # key-ordered columns need no sort (cost_model.stats)
         b["sort"] = 2 * st["n_sp"] * (kb + vb)
+    if use_index:
         b["probe"] = st["n_rp"] * (kb + 16) + st["sum_k"] * vb
     out = {k: v / (hbm_gbps * 1e9) * 1e3 for k, v in b.items()}
     if not use_index:
@@ -194,7 +196,8 @@ def main():
         if use_index or alu_ms is not None:
             ideal, nbytes = ideal_stages(tabs, plan, st, use_index, res_n, hbm, alu_ms)
             ideal_total = sum(ideal.values())
-            dev = stages["total"] + (sum(ix_prof[k] for k in ("inner_filter", "sort")) if ix_prof else 0.0)
+            dev = stages["total"] + (sum(ix_prof[k] for k in ("inner_filter", "sort") if ix_prof[k] == ix_prof[k])
+                                     if ix_prof else 0.0)
             rec["roofline"] = {"ideal_ms": {k: round(v, 5) for k, v in ideal.items()},
                                "algorithmic_bytes": nbytes, "hbm_gbps": hbm,
                                "query_frac": ideal_total / p50, "device_frac": ideal_total / dev if dev > 0 else None}
