@@ -174,7 +174,13 @@ nestgpu_status nestgpu_gather_column(nestgpu_ctx *ctx, int32_t src_col, const in
  * satisfy no correlated predicate); rows with a NULL payload are dropped too
  * (MIN/MAX/SUM/AVG skip them), so an index with a nullable payload column
  * cannot serve COUNT/EXISTS plans.  All columns must have S's row count.
- * Synchronises the stream once (to size the sort).
+ * A NOT NULL single key column stored in ascending order (checked once per
+ * column with its min / max statistics; every build for a column created by
+ * nestgpu_alloc_column) with a NOT NULL payload needs no sort: S' is
+ * compacted in row order straight into the index (the stable sort of a
+ * sorted S' is the identity; same bytes).
+ * Synchronises the stream once (to size the sort or the index), plus once
+ * when a key column's statistics are computed.
  * Errors: INVALID, TYPE, UNSUPPORTED, OOM, CUDA. */
 nestgpu_status nestgpu_build_index(nestgpu_ctx *ctx, const int32_t *key_cols, int32_t n_key_cols,
                                    int32_t payload_col,
@@ -471,7 +477,8 @@ nestgpu_status nestgpu_result_put(nestgpu_ctx *ctx, const nestgpu_result *res, v
  *     kernel; not with dedup, profiling or the malloc ablation).  Results
  *     are identical either way.
  *   NESTGPU_OPT_SORT (value 0/1/2): the index build's sort -- 0 (default)
- *     and 1 the LSD onesweep; 2 the two-round-trip MSD bucket sort
+ *     the LSD onesweep, none for a key-ordered column; 1 always the LSD
+ *     onesweep (the key-ordered shortcut off); 2 the two-round-trip MSD bucket sort
  *     (partition by the top varying key bits, finish each bucket in shared
  *     memory) wherever it fits, else the LSD onesweep.  An experiment kept
  *     for measurement: 1.2-1.9x slower than the onesweep on every measured
