@@ -687,6 +687,30 @@ def test_index_almost_ordered_column_sorts(eng):
         eng.release(m)
 
 
+@pytest.mark.parametrize("agg", ["exists", "not_exists", "min", "count"])
+def test_result_to_host_survivor_fields(eng, agg):
+    """result_to_host writes a survivors-only result's valid / passed (and an
+    EXISTS / NOT EXISTS value) on the host instead of copying them: they
+    must equal the device fields, on a result too large for the exec's
+    pinned staging (C2 '=' plans: 60k-980k survivors)."""
+    t = query1.config("C2")
+    plan = make_plan("=", agg, "=")
+    m = eng.mark()
+    try:
+        from tests.gpu_helpers import load
+        R, S = load(eng, t)
+        idx = eng.index_for_plan(plan, S)
+        res = eng.exec(plan, R, S, index=idx)
+        host = eng.result_to_numpy(res)
+        dev = eng.result_tensors(res)
+        assert res.n_rows > 20000
+        for k in ("row", "value", "valid", "passed"):
+            assert np.array_equal(host[k].astype(np.int64), dev[k].cpu().numpy().astype(np.int64)), (agg, k)
+        assert host["valid"].all() and host["passed"].all()
+    finally:
+        eng.release(m)
+
+
 def _skewed_keys(n, rng):
     """27 varying bits, but 3/4 of the keys in one 2^12-wide range: one
     partition bucket far past the finish capacity (falls back to the LSD
