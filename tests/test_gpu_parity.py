@@ -954,3 +954,38 @@ def test_exec_graph_replay_matches(eng):
     finally:
         eng.set_option(OPT_GRAPHS, 1)
         eng.release(m)
+
+
+def test_two_contexts_two_host_threads():
+    """Two contexts in one process driven by two host threads at once (the
+    ADVICE r1 case: the per-kernel launch setup -- shared-memory opt-ins of
+    the nested loop, filter and sort kernels, occupancy -- is cached per
+    (kernel, device) under a mutex, not in a process-global static): every
+    plan of each thread matches the oracle.  One GPU on this box, so both
+    contexts share device 0; each has its own arena and stream."""
+    import threading
+    from tests.gpu_helpers import make_engine
+    t = query1.config("C1")
+    plans = [make_plan(op, agg, "=") for op in ("=", ">", "!=") for agg in ("min", "count", "exists")]
+    refs = [oracle.evaluate(t, p) for p in plans]
+    errors = []
+
+    def work(k):
+        try:
+            e = make_engine(1)
+            try:
+                for rep in range(3):
+                    for i, p in enumerate(plans):
+                        mode = "index" if (i + k + rep) % 2 == 0 else "bnl"
+                        assert_parity(run(e, t, p, mode, emit_all=True), refs[i], p, True, ctx=(k, rep, i, mode))
+            finally:
+                e.close()
+        except Exception as ex:   # surfaced below
+            errors.append(repr(ex))
+
+    th = [threading.Thread(target=work, args=(k,)) for k in range(2)]
+    for x in th:
+        x.start()
+    for x in th:
+        x.join()
+    assert not errors, errors
