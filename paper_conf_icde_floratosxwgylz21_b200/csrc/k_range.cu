@@ -42,7 +42,10 @@ struct LongItem {
 // by each CTA, narrow a binary search to one stride-wide window of the keys
 // before it touches global memory (the top ~12 levels of the search come from
 // shared memory instead of ~12 dependent L2 round trips).
-constexpr int SAMP_BYTES = 16384;
+#ifndef NG_SAMP_BYTES
+#define NG_SAMP_BYTES 16384
+#endif
+constexpr int SAMP_BYTES = NG_SAMP_BYTES;
 
 size_t range_scratch_bytes(long long n_rp_max)
 {

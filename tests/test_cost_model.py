@@ -161,3 +161,24 @@ def test_sort_pass_plan_mirror(bits, lo, kb, want):
         top = (1 << bits) - 1
         keys = np.array([0, top << lo], dtype=np.uint64).astype(dt)
     assert _passes(keys, kb) == want
+
+
+def test_stats_key_ordered_column_needs_no_sort():
+    """tools/cost_model.stats mirrors the engine's key-ordered index build:
+    a NOT NULL inner key column stored in ascending order (TPC-H lineitem by
+    l_orderkey) has no sort passes; the same column shuffled, or with NULLs,
+    keeps its radix passes."""
+    import numpy as np
+    from datagen import make_plan
+    from tools.cost_model import stats
+    rng = np.random.default_rng(1)
+    k = np.sort(rng.integers(0, 1 << 24, 5000)).astype(np.int32)
+    t = {"R": {"col1": k[:100].copy(), "col2": np.zeros(100, np.int32)},
+         "S": {"col1": k, "col2": rng.integers(0, 9, 5000).astype(np.int32)}}
+    plan = make_plan("=", "min", "=")
+    assert stats(t, plan, 0)["sort_passes"] == 0
+    t["S"]["col1"] = rng.permutation(k)
+    assert stats(t, plan, 0)["sort_passes"] == 3
+    t["S"]["col1"] = k
+    t["S_valid"] = {"col1": np.ones(5000, bool)}
+    assert stats(t, plan, 0)["sort_passes"] == 3
