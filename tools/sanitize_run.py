@@ -5,7 +5,8 @@ group), finalize, gather, minmax, type-J collections + IN + materialise,
 cost-model calibration (fills), the radix-sort variants (pre-narrowed
 64-bit keys, 9-bit digit passes, keys without payload), and (round 2) the
 exact split SUM/AVG, the one-launch ordered R' filter with and without
-predicates, group aggregates, staged small results and a window put."""
+predicates, group aggregates, staged small results and a window put; the
+key-ordered index build and the MSD bucket sort experiment (session 2)."""
 import os
 import sys
 
@@ -96,6 +97,34 @@ er, ev = oracle.survivors(oracle.evaluate(tn, plan))
 wi, wv = eng.window_tensors(win, res.n_rows + 5, res.n_rows)
 bad += not (np.array_equal(wi.cpu().numpy(), er) and np.array_equal(wv.cpu().numpy(), ev))
 eng.window_free(win)
+# round 2, session 2: the key-ordered (sort-free) index build with and
+# without inner predicates, and the MSD bucket sort experiment
+# (NESTGPU_OPT_SORT = 2: group histograms, column scan, partition, finish)
+from paper_conf_icde_floratosxwgylz21_b200.binding import OPT_SORT  # noqa: E402
+ko = np.sort(rng.integers(-5000, 5000, 50011)).astype(np.int64)
+to = {"R": {"col1": rng.integers(-5010, 5010, 7001).astype(np.int64), "col2": rng.integers(-50, 50, 7001)},
+      "S": {"col1": ko, "col2": rng.integers(-50, 50, 50011), "col3": rng.integers(0, 3, 50011)}}
+Ro, So = eng.load_table(to["R"], dtypes={"col1": "int64"}), eng.load_table(to["S"], dtypes={"col1": "int64"})
+for preds in ([], [{"col": "col3", "op": "!=", "lit": 1}]):
+    for agg in ("min", "exists"):
+        plan = make_plan("=", agg, "<=", inner_preds=preds)
+        g = eng.result_to_numpy(eng.exec(plan, Ro, So, index=eng.index_for_plan(plan, So), emit_all=True))
+        ref = oracle.evaluate(to, plan)
+        bad += not np.array_equal(g["value"], ref["value"][ref["in_rp"].astype(bool)])
+eng.set_option(OPT_SORT, 2)
+for keys, dt, pay in ((rng.integers(0, 1 << 27, 100003), "int32", True),
+                      (rng.integers(0, 1 << 29, 100003) + (7 << 40), "int64", False),
+                      (rng.integers(-2 ** 40, 2 ** 40, 60007), "int64", True)):
+    cols = {"k": keys, "v": np.arange(len(keys))} if pay else {"k": keys}
+    T = eng.load_table(cols, dtypes={"k": dt, "v": "int32"} if pay else {"k": dt})
+    ix = eng.build_index(T, ["k"], "v" if pay else None)
+    info = eng.index_info(ix)
+    kb = info["key_bytes"]
+    got = eng.arena_view(info["d_keys"], len(keys) * kb).view(torch.int64 if kb == 8 else torch.int32).cpu().numpy()
+    enc = (keys.astype(np.int64).view(np.uint64) ^ np.uint64(1 << 63)) if kb == 8 else \
+        (keys.astype(np.int32).view(np.uint32) ^ np.uint32(1 << 31))
+    bad += not np.array_equal(got.view(enc.dtype), np.sort(enc))
+eng.set_option(OPT_SORT, 0)
 eng.cost_calibrate(1 << 16)
 print("sanitize workload done, mismatches:", bad)
 sys.exit(1 if bad else 0)
