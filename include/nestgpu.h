@@ -483,8 +483,15 @@ nestgpu_status nestgpu_result_put(nestgpu_ctx *ctx, const nestgpu_result *res, v
  *     memory) wherever it fits, else the LSD onesweep.  An experiment kept
  *     for measurement: 1.2-1.9x slower than the onesweep on every measured
  *     shape.  Both are stable sorts of the same S'.
+ *   NESTGPU_OPT_TINY (value 0/1, default 1): a nested-loop exec (index -1,
+ *     no dedup) over |S| <= 4096, |R| <= 4096 rows and |R| x |S| <= 2^21 pairs
+ *     runs as ONE kernel launch of one CTA (S' in shared memory, a warp per
+ *     outer tuple, finalize and ordered compaction in the same kernel)
+ *     instead of the fill / filter / nested-loop / finalize sequence; 0
+ *     forces the sequence.  Results are identical either way.
  * Errors: INVALID (unknown option). */
-enum { NESTGPU_OPT_MALLOC_SCRATCH = 1, NESTGPU_OPT_BNL_SHAPE = 2, NESTGPU_OPT_GRAPHS = 3, NESTGPU_OPT_SORT = 4 };
+enum { NESTGPU_OPT_MALLOC_SCRATCH = 1, NESTGPU_OPT_BNL_SHAPE = 2, NESTGPU_OPT_GRAPHS = 3, NESTGPU_OPT_SORT = 4,
+       NESTGPU_OPT_TINY = 5 };
 nestgpu_status nestgpu_set_option(nestgpu_ctx *ctx, int32_t option, int64_t value);
 
 /* Per-stage device times (ms, CUDA events on the context stream) of the last

@@ -40,6 +40,7 @@ OPT_MALLOC_SCRATCH = 1
 OPT_BNL_SHAPE = 2
 OPT_GRAPHS = 3
 OPT_SORT = 4   # 0 / 1 LSD onesweep (default), 2 MSD bucket sort experiment
+OPT_TINY = 5   # 1 (default): one-launch path for tiny nested-loop queries; 0: the regular sequence
 
 
 class NestGPUError(RuntimeError):

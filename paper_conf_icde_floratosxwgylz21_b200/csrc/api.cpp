@@ -111,6 +111,7 @@ struct nestgpu_ctx {
     std::vector<void *> mallocs;
     int bnl_shape;   // NESTGPU_OPT_BNL_SHAPE (test knob): 0 automatic, 1 full, 2 warp-split
     int sort_mode;   // NESTGPU_OPT_SORT: 0 / 1 LSD onesweep, 2 MSD bucket sort (experiment)
+    bool tiny_on;    // NESTGPU_OPT_TINY: one-launch path for tiny nested-loop queries (default on)
     cudaEvent_t ev[NESTGPU_N_STAGES][2];
     // CUDA graphs of exec launch sequences (NESTGPU_OPT_GRAPHS, default on):
     // key = every argument that determines the sequence (plan, column /
@@ -455,6 +456,7 @@ nestgpu_status nestgpu_create(int device, void *d_arena, size_t arena_bytes, voi
     c->malloc_scratch = false;
     c->bnl_shape = 0;
     c->sort_mode = 0;
+    c->tiny_on = true;
     c->cap_stream = nullptr;
     {
         const char *gr = getenv("NESTGPU_GRAPHS");
@@ -1257,7 +1259,8 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
     uint8_t *rkvalid = ravalid ? (uint8_t *)salloc(c, (size_t)nR) : nullptr;
     long long *acc = (long long *)salloc(c, (size_t)nR * 8);
     long long *cnt = (long long *)salloc(c, (size_t)nR * 8);
-    long long *counts = (long long *)salloc(c, 128);  // [0] |R'| [1] |S'| [2] survivors; [4..5] extreme; [8] overflow
+    long long *counts = (long long *)salloc(c, 128 + 8 * ng::TINY_G_MAX);  // [0] |R'| [1] |S'| [2] survivors;
+                                                                          // [4..5] extreme; [8] overflow; tiny: CTA counts
     long long *acc_hi = wide ? (long long *)salloc(c, (size_t)nR * 8) : nullptr;
     // one scratch per filter / finalize (all zeroed up front by one fill kernel)
     void *fscr = salloc(c, ng::filter_scratch_bytes(nR));
@@ -1358,10 +1361,51 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
 
     const long long krows = std::min<long long>(nR, (long long)(STAGE_BYTES / (8 * w8 + 2)));
     long long n_distinct = -1;
+    // Tiny inputs: the nested-loop strategy's whole sequence as one launch of
+    // one CTA (k_finalize.cu tiny_exec_kernel; NESTGPU_OPT_TINY, off when a
+    // test forces a nested-loop R-block shape)
+    const bool tiny = c->tiny_on && !ix && !P->dedup && c->bnl_shape == 0 && nS <= ng::TINY_S_MAX &&
+                      nR <= ng::TINY_R_MAX && nR * nS <= ng::TINY_PAIRS_MAX;
     // Everything enqueued from here to the result copies: run directly, or
     // captured once into a CUDA graph and replayed (§17) -- a repeated small
     // query then costs one graph launch instead of one launch per kernel.
     auto enqueue = [&]() -> nestgpu_status {
+      if (tiny) {
+        prof_begin(c, 5);
+        prof_begin(c, 3);
+        ng::TinyArgs ta{};
+        ta.nR = nR;
+        ta.nS = nS;
+        ta.rp = ops;
+        ta.sp = ips;
+        ta.rk = rks;
+        ta.sk = sks;
+        if (value_agg) ta.v = ng::ValSrc{ac->d, ac->valid, vb};
+        ta.corr_op = P->corr_op;
+        ng::FinalizeArgs &fa = ta.f;
+        fa.x_col = xc ? xc->d : nullptr;
+        fa.x_valid = xc ? xc->valid : nullptr;
+        fa.x_w = xc ? dtype_width(xc->dtype) : 4;
+        fa.agg = P->agg;
+        fa.outer_op = P->outer_op;
+        fa.a = P->lhs_mult;
+        fa.b = P->rhs_mult;
+        fa.row_id_base = P->row_id_base;
+        fa.emit_all = P->emit_all;
+        fa.out_ids = o_ids;
+        fa.out_vals = o_vals;
+        fa.out_sum = o_sum;
+        fa.out_cnt = o_cnt;
+        fa.out_valid = o_valid;
+        fa.out_passed = o_pass;
+        fa.out_count = d_out;
+        ta.counts = counts;
+        ta.status = (unsigned long long *)(counts + 16);
+        CUDA_TRY(c, ng::launch_tiny_exec(ta, c->num_sms, c->stream, &c->launches));
+        htrace(c, "tiny");
+        prof_end(c, 3);
+        prof_end(c, 5);
+      } else {
         // ------------------------------------------------------------ a2: R'
         prof_begin(c, 5);
         prof_begin(c, 0);
@@ -1498,6 +1542,7 @@ nestgpu_status nestgpu_exec_correlated(nestgpu_ctx *c, const nestgpu_plan *P, ne
         htrace(c, "finalize");
         prof_end(c, 4);
         prof_end(c, 5);
+      }
         CUDA_TRY(c, cudaMemcpyAsync(c->pinned, counts, 72, cudaMemcpyDeviceToHost, c->stream));
         // the first rows of every result field, staged on the host before the
         // one synchronisation (8-byte fields, then the two byte fields)
@@ -1834,6 +1879,9 @@ nestgpu_status nestgpu_set_option(nestgpu_ctx *c, int32_t option, int64_t value)
         return NESTGPU_OK;
     case NESTGPU_OPT_GRAPHS:
         c->graphs_on = value != 0;
+        return NESTGPU_OK;
+    case NESTGPU_OPT_TINY:
+        c->tiny_on = value != 0;
         return NESTGPU_OK;
     case NESTGPU_OPT_SORT:
         if (value < 0 || value > 2) return fail(c, NESTGPU_ERR_INVALID, "set_option: sort 0, 1 or 2");

@@ -244,6 +244,28 @@ struct FinalizeArgs {
 };
 cudaError_t launch_finalize(const FinalizeArgs &a, cudaStream_t st, long long *launches, bool prezeroed = false);
 
+// Tiny queries (k_finalize.cu): the nested-loop strategy's whole sequence in
+// one launch of one CTA when |S| <= TINY_S_MAX, |R| <= TINY_R_MAX and
+// |R| x |S| <= TINY_PAIRS_MAX.  f: the finalize arguments (outputs,
+// out_count = counts + 2, overflow unused); counts[0] |R'|, [1] |S'|, [8]
+// overflow flag are written by the kernel.
+// counts must have 128 + 8 * TINY_G_MAX bytes (the launcher zeroes them;
+// the tail holds the per-CTA emit counts).
+constexpr long long TINY_S_MAX = 4096, TINY_R_MAX = 4096, TINY_PAIRS_MAX = 1ll << 21;
+constexpr int TINY_G_MAX = 256;
+struct TinyArgs {
+    long long nR, nS;
+    PredSet rp, sp;
+    KeySrc rk, sk;
+    ValSrc v;
+    int corr_op;
+    int chunk;                      // outer tuples per CTA (set by the launcher)
+    FinalizeArgs f;
+    long long *counts;
+    unsigned long long *status;     // counts + 16: per-CTA emit counts
+};
+cudaError_t launch_tiny_exec(const TinyArgs &t, int num_sms, cudaStream_t st, long long *launches);
+
 // Survivor rows into a (peer) window: win_ids[off + i] = ids[i],
 // win_vals[off + i] = vals[i], i < n; ends with __threadfence_system.
 cudaError_t launch_put_rows(const long long *ids, const long long *vals, long long n, long long *win_ids,

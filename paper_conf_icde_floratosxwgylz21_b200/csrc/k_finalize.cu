@@ -394,6 +394,275 @@ cudaError_t launch_init_partials(long long n, const long long *d_n, int agg, lon
     return cudaGetLastError();
 }
 
+// ------------------------------------------------------------------ tiny queries
+// The whole nested-method query in ONE launch for tiny inputs (|S| <= 4096,
+// |R| <= 4096, |R| x |S| <= 2^21 pairs; the plan template's nested-loop
+// strategy without caching).  Every stage of the regular sequence (fill, R'
+// filter, S' filter, partial init, tiled nested loop, finalize + ordered
+// compaction) costs a launch and a few microseconds of latency on inputs
+// this small, so one kernel does them all.  CTA c of G owns a contiguous
+// slice of R:
+//   1. S' = rows of S whose inner predicates hold, key NOT NULL (and payload
+//      NOT NULL for MIN/MAX/SUM/AVG), compacted into the CTA's shared memory
+//      (any order: the aggregates are order-free; every CTA holds all of S');
+//   2. warp w evaluates outer tuple r of the slice: outer predicates, then
+//      the Fig. 2 loop over S' with the lanes striding S' (the correlated
+//      predicate as one unsigned range test), a warp reduction (SUM / AVG
+//      exact in int128, OVERFLOW when a sum leaves int64, as the oracle),
+//      then fin_eval -- the finalize kernel's reading R1/R2/R6/R7 code;
+//   3. a block scan of the slice's emit flags (row order inside the slice),
+//      the slice's emit count published at once; the CTA's offset is the
+//      sum of its predecessors' counts (no chain: each waits only for their
+//      counts), then fin_write.
+// Results are the regular path's, field for field (tests run the C1 plans
+// and NULL / predicate / 64-bit / composite cases through both).
+constexpr int TINY_T = 1024;   // one S row per thread for |S| <= 1024, one outer tuple per warp
+constexpr int TINY_W = TINY_T / 32;
+
+__device__ __forceinline__ bool tiny_pred_row(const DevPred &p, long long i)
+{
+    if (p.valid && !p.valid[i]) return false;
+    const long long x = load_w(p.col, p.w, i);
+    long long y = p.lit;
+    if (p.rhs) {
+        if (p.rhs_valid && !p.rhs_valid[i]) return false;
+        y = load_w(p.rhs, p.rhs_w, i);
+    }
+    return cmp_rt<long long>(x, p.op, y);
+}
+
+__device__ __forceinline__ bool tiny_preds(const PredSet &ps, long long i)
+{
+    for (int k = 0; k < ps.n; k++)
+        if (!tiny_pred_row(ps.p[k], i)) return false;
+    return true;
+}
+
+// key of row i as a comparable int64 (single column: the signed value, the
+// order of the encoded keys; composite: the packed pair, '=' only); false if NULL
+__device__ __forceinline__ bool tiny_key(const KeySrc &k, long long i, long long &out)
+{
+    if (k.v0 && !k.v0[i]) return false;
+    if (k.n_key == 2) {
+        if (k.v1 && !k.v1[i]) return false;
+        out = (long long)(((unsigned long long)(unsigned)__ldg((const int *)k.c0 + i) << 32) |
+                          (unsigned)__ldg((const int *)k.c1 + i));
+    } else {
+        out = load_w(k.c0, k.w0, i);
+    }
+    return true;
+}
+
+// lanes fold S' entries j = lane, lane + 32, ... with s.key in [lo, hi]
+// (unsigned offset test) XOR neg -- the correlated predicate r.key OP s.key
+template <int AGG>
+__device__ __forceinline__ void tiny_fold(const long long *s_key, const long long *s_val, int ns, int lane,
+                                          long long lo, unsigned long long span, bool neg, long long &c,
+                                          long long &m, __int128 &sm)
+{
+    for (int j = lane; j < ns; j += 32) {
+        const bool q = ((unsigned long long)(s_key[j] - lo) <= span) != neg;
+        if (q) {
+            c++;
+            if constexpr (AGG == MIN) m = min(m, s_val[j]);
+            else if constexpr (AGG == MAX) m = max(m, s_val[j]);
+            else if constexpr (AGG == SUM) sm += s_val[j];
+        }
+    }
+}
+
+__global__ void __launch_bounds__(TINY_T) tiny_exec_kernel(TinyArgs T)
+{
+    const FinalizeArgs &A = T.f;
+    extern __shared__ __align__(16) unsigned char smem[];
+    long long *s_key = (long long *)smem;                       // [TINY_S_MAX]
+    long long *s_val = s_key + TINY_S_MAX;                      // [TINY_S_MAX]
+    long long *r_val = s_val + TINY_S_MAX;                      // [chunk] Res value (0 when NULL)
+    long long *r_sum = r_val + T.chunk;                         // [chunk] AVG: exact sum
+    long long *r_cnt = r_sum + T.chunk;                         // [chunk] AVG: nn
+    uint8_t *r_flag = (uint8_t *)(r_cnt + T.chunk);             // [chunk] bit0 valid, bit1 passed, bit2 in R'
+    __shared__ int s_ns, s_ovf;
+    __shared__ unsigned s_wsum[TINY_W];
+    __shared__ unsigned long long s_pre;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const bool value_agg = A.agg == MIN || A.agg == MAX || A.agg == SUM || A.agg == AVG;
+    const long long rb = (long long)blockIdx.x * T.chunk;
+    const int m_rows = (int)max(0ll, min((long long)T.chunk, T.nR - rb));
+    if (tid == 0) {
+        s_ns = 0;
+        s_ovf = 0;
+    }
+    __syncthreads();
+    // 1. S' into shared memory
+    for (long long i = tid; i < T.nS; i += TINY_T) {
+        long long k;
+        if (!tiny_key(T.sk, i, k) || !tiny_preds(T.sp, i)) continue;
+        if (value_agg && T.v.v && !T.v.v[i]) continue;
+        const int slot = atomicAdd(&s_ns, 1);
+        s_key[slot] = k;
+        if (value_agg) s_val[slot] = load_w(T.v.c, T.v.w, i);
+    }
+    __syncthreads();
+    const int ns = s_ns;
+    // 2. warp per outer tuple of the slice
+    for (int q = warp; q < m_rows; q += TINY_W) {
+        const long long r = rb + q;
+        const bool in_rp = tiny_preds(T.rp, r);
+        long long rk = 0;
+        const bool kval = tiny_key(T.rk, r, rk);
+        long long lo = rk, hi = rk;
+        bool neg = false, empty = !(in_rp && kval);
+        switch (T.corr_op) {   // r.key OP s.key  <=>  s.key in [lo, hi] (XOR neg)
+        case NE: neg = true; break;
+        case LT: if (rk == LLONG_MAX) empty = true; else { lo = rk + 1; hi = LLONG_MAX; } break;
+        case LE: hi = LLONG_MAX; break;
+        case GT: if (rk == LLONG_MIN) empty = true; else { lo = LLONG_MIN; hi = rk - 1; } break;
+        case GE: lo = LLONG_MIN; break;
+        default: break;
+        }
+        const unsigned long long span = (unsigned long long)hi - (unsigned long long)lo;
+        long long c = 0, m = A.agg == MAX ? LLONG_MIN : LLONG_MAX;
+        __int128 sm = 0;
+        if (!empty) {
+            switch (A.agg) {
+            case MIN: tiny_fold<MIN>(s_key, s_val, ns, lane, lo, span, neg, c, m, sm); break;
+            case MAX: tiny_fold<MAX>(s_key, s_val, ns, lane, lo, span, neg, c, m, sm); break;
+            case SUM: case AVG: tiny_fold<SUM>(s_key, s_val, ns, lane, lo, span, neg, c, m, sm); break;
+            default: tiny_fold<COUNT>(s_key, s_val, ns, lane, lo, span, neg, c, m, sm); break;
+            }
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            c += __shfl_xor_sync(FULL, c, o);
+            const long long m2 = __shfl_xor_sync(FULL, m, o);
+            m = A.agg == MAX ? max(m, m2) : min(m, m2);
+            const long long lo2 = __shfl_xor_sync(FULL, (long long)(unsigned long long)sm, o);
+            const long long hi2 = __shfl_xor_sync(FULL, (long long)(sm >> 64), o);
+            sm += ((__int128)hi2 << 64) | (__int128)(unsigned long long)lo2;
+        }
+        if (lane == 0) {
+            uint8_t f = 0;
+            if (in_rp) {
+                long long acc = m;
+                if (A.agg == SUM || A.agg == AVG) {
+                    acc = 0;
+                    if (sm > (__int128)LLONG_MAX || sm < (__int128)LLONG_MIN) s_ovf = 1;
+                    else acc = (long long)sm;
+                }
+                FinIn in;
+                in.acc = acc;
+                in.cnt = c;
+                in.g = 0;
+                in.row = (int)r;
+                in.kval = kval;
+                fin_load_x(A, in);
+                long long value;
+                bool valid, passed;
+                fin_eval(A, in, value, valid, passed);
+                r_val[q] = value;
+                r_sum[q] = kval ? acc : 0;
+                r_cnt[q] = kval ? c : 0;
+                f = (valid ? 1 : 0) | (passed ? 2 : 0) | 4;
+            }
+            r_flag[q] = f;
+        }
+    }
+    __syncthreads();
+    // 3. positions in row order: consecutive rows per thread, a block scan
+    const int per = (m_rows + TINY_T - 1) / TINY_T;
+    const int q0 = tid * per;
+    unsigned cnt_e = 0, cnt_rp = 0;
+    for (int k = 0; k < per; k++) {
+        const int q = q0 + k;
+        if (q < m_rows) {
+            const uint8_t f = r_flag[q];
+            cnt_rp += (f >> 2) & 1;
+            cnt_e += (f & 4) && (A.emit_all || (f & 2)) ? 1 : 0;
+        }
+    }
+    unsigned inc = cnt_e;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned t = __shfl_up_sync(FULL, inc, o);
+        if (lane >= o) inc += t;
+    }
+    if (lane == 31) s_wsum[warp] = inc;
+    unsigned rp_w = cnt_rp;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) rp_w += __shfl_xor_sync(FULL, rp_w, o);
+    if (lane == 0 && rp_w) atomicAdd((unsigned long long *)&T.counts[0], (unsigned long long)rp_w);
+    __syncthreads();
+    unsigned pos = inc - cnt_e, total = 0;
+    for (int w = 0; w < TINY_W; w++) {
+        const unsigned t = s_wsum[w];
+        if (w < warp) pos += t;
+        total += t;
+    }
+    // this CTA's count for its successors, then the sum of its predecessors'
+    if (tid == 0) {
+        st_relaxed_u64(T.status + blockIdx.x, (1ull << 63) | total);
+        if (s_ovf) atomicOr((unsigned long long *)&T.counts[8], 1ull);
+    }
+    if (warp == 0) {
+        unsigned long long pre = 0;
+        for (int j = lane; j < (int)blockIdx.x; j += 32) {
+            unsigned long long v;
+            while (((v = ld_relaxed_u64(T.status + j)) >> 63) == 0) {
+            }
+            pre += v & ~(1ull << 63);
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) pre += __shfl_xor_sync(FULL, pre, o);
+        if (lane == 0) s_pre = pre;
+    }
+    __syncthreads();
+    const unsigned long long base = s_pre;
+    for (int k = 0; k < per; k++) {
+        const int q = q0 + k;
+        if (q >= m_rows) break;
+        const uint8_t f = r_flag[q];
+        if (!((f & 4) && (A.emit_all || (f & 2)))) continue;
+        FinIn in;
+        in.acc = r_sum[q];
+        in.cnt = r_cnt[q];
+        in.g = 0;
+        in.row = (int)(rb + q);
+        in.kval = true;   // r_sum / r_cnt already hold 0 for a NULL key
+        fin_write(A, in, (long long)(base + pos), r_val[q], (f & 1) != 0, (f & 2) != 0);
+        pos++;
+    }
+    if (tid == 0) {
+        if (blockIdx.x == 0) T.counts[1] = ns;
+        if (blockIdx.x == gridDim.x - 1) *A.out_count = (long long)(base + total);
+    }
+}
+
+cudaError_t launch_tiny_exec(const TinyArgs &t0, int num_sms, cudaStream_t st, long long *launches)
+{
+    TinyArgs t = t0;
+    // a slice of >= 32 outer tuples per CTA (one per warp), at most one CTA per SM
+    long long g = (t.nR + 31) / 32;
+    if (g > num_sms) g = num_sms;
+    if (g > TINY_G_MAX) g = TINY_G_MAX;
+    if (g < 1) g = 1;
+    t.chunk = (int)((t.nR + g - 1) / g);
+    if (t.chunk < 1) t.chunk = 1;
+    g = t.nR > 0 ? (t.nR + t.chunk - 1) / t.chunk : 1;
+    const size_t smem = (size_t)TINY_S_MAX * 16 + (size_t)t.chunk * 25;
+    int dummy = 0;
+    cudaError_t e = per_device_setup((const void *)tiny_exec_kernel, 0, &dummy, [](int, int *v) {
+        *v = 1;
+        return cudaFuncSetAttribute(tiny_exec_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)((size_t)TINY_S_MAX * 16 + (size_t)TINY_R_MAX * 25));
+    });
+    if (e != cudaSuccess) return e;
+    e = cudaMemsetAsync(t.counts, 0, 128 + (size_t)TINY_G_MAX * 8, st);   // counts + the per-CTA emit counts
+    if (e != cudaSuccess) return e;
+    tiny_exec_kernel<<<(unsigned)g, TINY_T, smem, st>>>(t);
+    ++*launches;
+    return cudaGetLastError();
+}
+
 // ------------------------------------------------------------------ column min / max
 // (for the SUM/AVG overflow pre-check, reading R5)
 // (and out[2] != 0 iff some row is smaller than its predecessor: the

@@ -321,14 +321,22 @@ def test_launch_count_and_profile(eng):
     m = eng.mark()
     try:
         R, S = eng.load_table(t["R"]), eng.load_table(t["S"])
+        from paper_conf_icde_floratosxwgylz21_b200.binding import OPT_TINY
         eng.set_profiling(True)
         before = eng.launch_count()
         eng.exec(make_plan(">", "min", "="), R, S)
-        assert eng.launch_count() - before >= 4  # R' filter, S' filter, init, BNL, finalize
+        assert eng.launch_count() - before == 1   # the one-launch tiny path
         prof = eng.last_profile()
         assert prof["subquery"] > 0 and prof["total"] >= prof["subquery"]
-        eng.set_profiling(False)
+        eng.set_option(OPT_TINY, 0)
+        before = eng.launch_count()
+        eng.exec(make_plan(">", "min", "="), R, S)
+        assert eng.launch_count() - before >= 4  # fill, R' filter, S' filter, BNL, finalize
+        prof = eng.last_profile()
+        assert prof["subquery"] > 0 and prof["total"] >= prof["subquery"]
     finally:
+        eng.set_option(OPT_TINY, 1)
+        eng.set_profiling(False)
         eng.release(m)
 
 
@@ -989,3 +997,51 @@ def test_two_contexts_two_host_threads():
     for x in th:
         x.join()
     assert not errors, errors
+
+
+@pytest.mark.parametrize("tiny", [1, 0])
+def test_tiny_one_launch_path(eng, tiny):
+    """The one-launch path for tiny nested-loop queries (NESTGPU_OPT_TINY,
+    k_finalize.cu tiny_exec_kernel) against the oracle and with it switched
+    off (the regular fill / filter / nested loop / finalize sequence):
+    NULL-bearing random tables with outer and inner predicates (literal and
+    column-vs-column), every operator x aggregate x emit mode, a row-id base,
+    64-bit keys and decimal payloads, composite keys, and the SUM overflow
+    error; sizes at the path's limits (4096 rows, 2^21 pairs)."""
+    from paper_conf_icde_floratosxwgylz21_b200.binding import OPT_TINY, NestGPUError
+    eng.set_option(OPT_TINY, tiny)
+    try:
+        t = query1.random_small(23, n_r=511, n_s=4096, key_hi=60, val_lo=-40, val_hi=40, null_frac=0.15)
+        for corr_op in PLAN_OPS:
+            for agg in AGGS:
+                for emit_all in (True, False):
+                    plan = make_plan(corr_op, agg, "<=", outer_preds=[{"col": "col3", "op": "<=", "lit": 1}],
+                                     inner_preds=[{"col": "col3", "op": "!=", "rhs": "col2"}])
+                    ref = oracle.evaluate(t, plan)
+                    g = run(eng, t, plan, "bnl", emit_all=emit_all, row_id_base=1000)
+                    g["row"] = g["row"] - 1000
+                    assert_parity(g, ref, plan, emit_all, ctx=(tiny, corr_op, agg, emit_all))
+        rng = np.random.default_rng(5)
+        t64 = {"R": {"col1": rng.integers(-3, 40, 4096) * (1 << 35), "col2": rng.integers(-9, 9, 4096) * 10 ** 9},
+               "S": {"col1": rng.integers(-3, 40, 512) * (1 << 35), "col2": rng.integers(-9, 9, 512) * 10 ** 12}}
+        dt = {"R": {"col1": "int64", "col2": "int64"}, "S": {"col1": "int64", "col2": "decimal"}}
+        for corr_op in ("=", "<", "!="):
+            for agg in ("min", "sum", "avg", "count"):
+                plan = make_plan(corr_op, agg, ">", lhs_mult=1000, rhs_mult=1)
+                assert_parity(run(eng, t64, plan, "bnl", emit_all=True, dtypes=dt), oracle.evaluate(t64, plan), plan,
+                              True, ctx=(tiny, "i64", corr_op, agg))
+        i32 = lambda lo, hi, n: rng.integers(lo, hi, n).astype(np.int32)   # noqa: E731
+        tc = {"R": {"a": i32(0, 5, 1500), "b": i32(0, 5, 1500), "x": i32(-5, 5, 1500)},
+              "S": {"a": i32(0, 5, 1300), "b": i32(0, 5, 1300), "v": i32(-5, 5, 1300)}}
+        for agg in ("max", "count", "not_exists"):
+            plan = make_plan("=", agg, "<", outer_key=["a", "b"], inner_key=["a", "b"], agg_col="v", outer_cmp_col="x")
+            assert_parity(run(eng, tc, plan, "bnl", emit_all=False), oracle.evaluate(tc, plan), plan, False,
+                          ctx=(tiny, "composite", agg))
+        big = (1 << 62) + (1 << 61)
+        tov = {"R": {"col1": np.zeros(3, np.int64), "col2": np.zeros(3, np.int64)},
+               "S": {"col1": np.zeros(4, np.int64), "col2": np.full(4, big, np.int64)}}
+        with pytest.raises(NestGPUError):
+            run(eng, tov, make_plan("=", "sum", "<"), "bnl", dtypes={"R": {"col1": "int64", "col2": "int64"},
+                                                                  "S": {"col1": "int64", "col2": "int64"}})
+    finally:
+        eng.set_option(OPT_TINY, 1)
