@@ -43,6 +43,9 @@ namespace ng {
 #ifndef NG_S_PREAGG
 #define NG_S_PREAGG 0   // 1: a tile-histogram kernel publishes every tile's digit counts before the pass
 #endif
+#ifndef NG_H_KEYS
+#define NG_H_KEYS 4096   // digit histogram: keys per CTA (fewer CTAs = fewer same-bin global atomics)
+#endif
 #ifndef NG_S_PMINB
 #define NG_S_PMINB 3  // persistent pass: CTAs per SM the register budget must allow
 #endif
@@ -458,7 +461,7 @@ cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *
     for (int p = 0; p < np; p++) dl.shift[p] = shifts[p];
     // >= 4096 keys per CTA: the shared bins' init / merge and the last CTA's
     // scan stay small next to the counting
-    long long blocks = (n + 4095) / 4096;
+    long long blocks = (n + NG_H_KEYS - 1) / NG_H_KEYS;
     if (blocks > (long long)num_sms * 8) blocks = (long long)num_sms * 8;
     if (blocks < 1) blocks = 1;
     if (rb == 8) {

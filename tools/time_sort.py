@@ -14,10 +14,12 @@ from paper_conf_icde_floratosxwgylz21_b200.binding import OPT_SORT  # noqa: E402
 
 eng = Engine(0, arena_bytes=8 << 30)
 eng.set_profiling(True)
-MODES = {"auto": 0, "lsd": 1, "bucket": 2}
+MODES = {"auto": 0}
 rng = np.random.default_rng(0)
 out = []
-for name, k, v in (("16M u32+v32", rng.integers(0, 2 ** 31 - 1, 16_000_000).astype(np.int32),
+for name, k, v in (("1M u32 (18 bits, C2-like)+v32", rng.integers(0, 1 << 18, 1_000_000).astype(np.int32),
+                    rng.integers(0, 1 << 20, 1_000_000).astype(np.int32)),
+                   ("16M u32+v32", rng.integers(0, 2 ** 31 - 1, 16_000_000).astype(np.int32),
                     rng.integers(0, 2 ** 20, 16_000_000).astype(np.int32)),
                    ("38M u64", (rng.integers(0, 15_000_000, 38_000_000) // 8 * 32).astype(np.int64), None),
                    ("60M u32+v32", rng.integers(0, 2 ** 26, 60_000_000).astype(np.int32),
