@@ -812,6 +812,8 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     memcpy(&nsp, c->pinned, 8);
     memcpy(&kand, c->pinned + 4, 8);
     memcpy(&kor, c->pinned + 6, 8);
+    if (nsp >= (1ll << 30))   // radix-pass look-back words carry 30-bit counts
+        return fail(c, NESTGPU_ERR_UNSUPPORTED, "build_index: |S'| = %lld >= 2^30 rows to sort", nsp);
     int shifts[8], rb = 8;
     int np = plan_sort_passes(fkb, kand, kor, nsp, shifts, &rb);
     if (pre_narrow && np == 0 && nsp > 0) {   // equal keys: one pass still widens them to 64 bits

@@ -594,10 +594,123 @@ __global__ void __launch_bounds__(1024) seg_block_scan_kernel(long long *__restr
     }
 }
 
+// Single pass (round 2, session 2): one launch instead of block totals +
+// one-CTA scan + rewrite.  CTA b (dynamic id, so its predecessors run)
+// scans its 4096 rows (16 consecutive per thread, a sequential segmented
+// scan, then a block scan of the thread totals), publishes its block pair
+// (f, v) at once, and thread 0 walks back over the predecessors' published
+// pairs until one is an inclusive prefix or holds a run start (f = 1:
+// nothing before it reaches this block) -- for short runs the walk is one
+// step.  status[b]: 0 = not yet, 1 = block pair, 2 = inclusive; bit 2 = f.
+constexpr int SG_ITEMS = 16;
+constexpr int SG_BLOCK = P_THREADS * SG_ITEMS;
+template <typename K, typename V, int AGG>
+__global__ void __launch_bounds__(P_THREADS) seg_onepass_kernel(const K *__restrict__ keys, const V *__restrict__ v,
+                                                                long long N, long long *__restrict__ grp,
+                                                                unsigned *__restrict__ status,
+                                                                long long *__restrict__ sagg,
+                                                                long long *__restrict__ sinc,
+                                                                unsigned *__restrict__ counter)
+{
+    __shared__ long long s_wv[P_THREADS / 32];
+    __shared__ int s_wf[P_THREADS / 32];
+    __shared__ SegPair<AGG> s_carry;
+    __shared__ long long s_b;
+    __shared__ int s_head0;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) s_b = atomicAdd(counter, 1u);
+    __syncthreads();
+    const long long b = s_b;
+    const long long e0 = b * SG_BLOCK + (long long)tid * SG_ITEMS;
+    // this thread's 16 rows: sequential segmented inclusive scan
+    SegPair<AGG> x[SG_ITEMS];
+    K prev = e0 > 0 && e0 - 1 < N ? keys[e0 - 1] : (K)0;
+#pragma unroll
+    for (int i = 0; i < SG_ITEMS; i++) {
+        const long long e = e0 + i;
+        if (e < N) {
+            const K k = keys[e];
+            x[i] = SegPair<AGG>{(long long)v[e], (e == 0 || k != prev) ? 1 : 0};
+            prev = k;
+        } else {
+            x[i] = SegPair<AGG>{ident<AGG>(), 0};
+        }
+    }
+    if (tid == 0) s_head0 = x[0].f;
+#pragma unroll
+    for (int i = 1; i < SG_ITEMS; i++) x[i] = seg_comb<AGG>(x[i - 1], x[i]);
+    // block exclusive scan of the thread totals
+    const SegPair<AGG> tot = x[SG_ITEMS - 1];
+    const SegPair<AGG> incl = warp_seg_scan<AGG>(tot, lane);
+    if (lane == 31) {
+        s_wv[warp] = incl.v;
+        s_wf[warp] = incl.f;
+    }
+    __syncthreads();
+    SegPair<AGG> wpre{ident<AGG>(), 0};
+    for (int w = 0; w < warp; w++) wpre = seg_comb<AGG>(wpre, SegPair<AGG>{s_wv[w], s_wf[w]});
+    SegPair<AGG> up{__shfl_up_sync(FULL, incl.v, 1), __shfl_up_sync(FULL, incl.f, 1)};
+    if (lane == 0) up = SegPair<AGG>{ident<AGG>(), 0};
+    const SegPair<AGG> tex = seg_comb<AGG>(wpre, up);   // the block's rows before this thread's
+    if (tid == P_THREADS - 1) {
+        const SegPair<AGG> blk = seg_comb<AGG>(tex, tot);   // the whole block
+        SegPair<AGG> carry{ident<AGG>(), 0};
+        if (b == 0 || blk.f) {   // the block's inclusive pair does not depend on its predecessors
+            sinc[b] = blk.v;
+            __threadfence();
+            st_relaxed_u32(status + b, 2u | ((unsigned)blk.f << 2));
+        } else {
+            sagg[b] = blk.v;
+            __threadfence();
+            st_relaxed_u32(status + b, 1u);
+        }
+        if (b > 0 && !s_head0) {   // rows before the block's first run start take the carry
+            for (long long p = b - 1; p >= 0; p--) {
+                unsigned st;
+                while (((st = ld_relaxed_u32(status + p)) & 3u) == 0) {
+                }
+                __threadfence();
+                const long long pv = (st & 3u) == 2u ? ld_relaxed_u64((const unsigned long long *)(sinc + p))
+                                                     : ld_relaxed_u64((const unsigned long long *)(sagg + p));
+                carry = seg_comb<AGG>(SegPair<AGG>{pv, (int)((st >> 2) & 1u)}, carry);
+                if ((st & 3u) == 2u || ((st >> 2) & 1u)) break;
+            }
+            if (!blk.f) {
+                sinc[b] = seg_comb<AGG>(carry, blk).v;
+                __threadfence();
+                st_relaxed_u32(status + b, 2u);
+            }
+        }
+        s_carry = carry;
+    }
+    __syncthreads();
+    const SegPair<AGG> pre = seg_comb<AGG>(s_carry, tex);
+#pragma unroll
+    for (int i = 0; i < SG_ITEMS; i++) {
+        const long long e = e0 + i;
+        if (e < N) grp[e] = seg_comb<AGG>(pre, x[i]).v;
+    }
+}
+
 template <typename K, typename V, int AGG>
 static void seg_scan(const void *keys, const void *v, long long N, long long *grp, void *scratch, cudaStream_t st,
                      long long *launches)
 {
+#ifndef NG_SEG_THREE_PASS
+    {
+        const long long nb = (N + SG_BLOCK - 1) / SG_BLOCK;
+        unsigned *counter = (unsigned *)scratch;
+        unsigned *status = counter + 1;
+        const size_t zb = ((size_t)(nb + 1) * 4 + 15) & ~(size_t)15;
+        long long *sagg = (long long *)((char *)scratch + zb);
+        long long *sinc = sagg + nb;
+        cudaMemsetAsync(scratch, 0, zb, st);
+        seg_onepass_kernel<K, V, AGG><<<(unsigned)nb, P_THREADS, 0, st>>>((const K *)keys, (const V *)v, N, grp,
+                                                                           status, sagg, sinc, counter);
+        *launches += 1;
+        return;
+    }
+#endif
     const long long nb = (N + G_BLOCK - 1) / G_BLOCK;
     long long *bv = (long long *)scratch;
     int *bf = (int *)(bv + nb + 1);
