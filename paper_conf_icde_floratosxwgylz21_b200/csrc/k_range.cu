@@ -510,90 +510,6 @@ __device__ __forceinline__ SegPair<AGG> warp_seg_scan(SegPair<AGG> x, int lane)
     return x;
 }
 
-// One block of G_BLOCK sorted (key, payload) rows scanned in order, 256 at a
-// time; WRITE: write grp[e], else only the block's total pair (bv, bf).
-// Small blocks (4 rows of 256): the scan is latency-bound, so many CTAs.
-constexpr int G_ITEMS = 4;
-constexpr int G_BLOCK = P_THREADS * G_ITEMS;
-template <typename K, typename V, int AGG, bool WRITE>
-__global__ void __launch_bounds__(P_THREADS) seg_block_kernel(const K *__restrict__ keys, const V *__restrict__ v,
-                                                              long long N, long long *__restrict__ bv,
-                                                              int *__restrict__ bf, long long *__restrict__ grp)
-{
-    __shared__ long long s_wv[P_THREADS / 32];
-    __shared__ int s_wf[P_THREADS / 32];
-    __shared__ SegPair<AGG> s_carry;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const long long b0 = blockIdx.x * (long long)G_BLOCK;
-    if (threadIdx.x == 0) s_carry = WRITE ? SegPair<AGG>{bv[blockIdx.x], 0} : SegPair<AGG>{ident<AGG>(), 0};
-    // the block's rows loaded up front (one DRAM round trip per CTA)
-    SegPair<AGG> xs[G_ITEMS];
-#pragma unroll
-    for (int j = 0; j < G_ITEMS; j++) {
-        const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
-        xs[j] = SegPair<AGG>{ident<AGG>(), 0};
-        if (e < N) xs[j] = SegPair<AGG>{(long long)v[e], (e == 0 || keys[e] != keys[e - 1]) ? 1 : 0};
-    }
-    __syncthreads();
-#pragma unroll
-    for (int j = 0; j < G_ITEMS; j++) {
-        const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
-        const SegPair<AGG> x = xs[j];
-        const SegPair<AGG> incl = warp_seg_scan<AGG>(x, lane);
-        if (lane == 31) {
-            s_wv[warp] = incl.v;
-            s_wf[warp] = incl.f;
-        }
-        __syncthreads();
-        SegPair<AGG> wpre{ident<AGG>(), 0};
-        for (int w = 0; w < warp; w++) wpre = seg_comb<AGG>(wpre, SegPair<AGG>{s_wv[w], s_wf[w]});
-        const SegPair<AGG> val = seg_comb<AGG>(s_carry, seg_comb<AGG>(wpre, incl));
-        if (WRITE && e < N) grp[e] = val.v;
-        __syncthreads();
-        if (threadIdx.x == P_THREADS - 1) s_carry = val;
-        __syncthreads();
-    }
-    if (!WRITE && threadIdx.x == 0) {
-        bv[blockIdx.x] = s_carry.v;
-        bf[blockIdx.x] = s_carry.f;
-    }
-}
-
-// exclusive scan of the block pairs: one CTA of 1024 threads, chunks of
-// 1024 pairs in order (segmented warp scans + a scan of the warp totals)
-template <int AGG>
-__global__ void __launch_bounds__(1024) seg_block_scan_kernel(long long *__restrict__ bv, const int *__restrict__ bf,
-                                                              long long nb)
-{
-    __shared__ long long s_wv[32];
-    __shared__ int s_wf[32];
-    __shared__ SegPair<AGG> s_carry;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    if (threadIdx.x == 0) s_carry = SegPair<AGG>{ident<AGG>(), 0};
-    __syncthreads();
-    for (long long b0 = 0; b0 < nb; b0 += 1024) {
-        const long long b = b0 + threadIdx.x;
-        const SegPair<AGG> x = b < nb ? SegPair<AGG>{bv[b], bf[b]} : SegPair<AGG>{ident<AGG>(), 0};
-        const SegPair<AGG> incl = warp_seg_scan<AGG>(x, lane);
-        if (lane == 31) {
-            s_wv[warp] = incl.v;
-            s_wf[warp] = incl.f;
-        }
-        __syncthreads();
-        SegPair<AGG> wpre{ident<AGG>(), 0};
-        for (int w = 0; w < warp; w++) wpre = seg_comb<AGG>(wpre, SegPair<AGG>{s_wv[w], s_wf[w]});
-        const SegPair<AGG> carry = s_carry;
-        // exclusive: everything before b = carry (+) warps before (+) lanes before
-        SegPair<AGG> up{__shfl_up_sync(FULL, incl.v, 1), __shfl_up_sync(FULL, incl.f, 1)};
-        if (lane == 0) up = SegPair<AGG>{ident<AGG>(), 0};
-        const SegPair<AGG> ex = seg_comb<AGG>(carry, seg_comb<AGG>(wpre, up));
-        __syncthreads();
-        if (b < nb) bv[b] = ex.v;
-        if (threadIdx.x == 1023) s_carry = seg_comb<AGG>(carry, seg_comb<AGG>(wpre, incl));
-        __syncthreads();
-    }
-}
-
 // Single pass (round 2, session 2): one launch instead of block totals +
 // one-CTA scan + rewrite.  CTA b (dynamic id, so its predecessors run)
 // scans its 4096 rows (16 consecutive per thread, a sequential segmented
@@ -696,30 +612,16 @@ template <typename K, typename V, int AGG>
 static void seg_scan(const void *keys, const void *v, long long N, long long *grp, void *scratch, cudaStream_t st,
                      long long *launches)
 {
-#ifndef NG_SEG_THREE_PASS
-    {
-        const long long nb = (N + SG_BLOCK - 1) / SG_BLOCK;
-        unsigned *counter = (unsigned *)scratch;
-        unsigned *status = counter + 1;
-        const size_t zb = ((size_t)(nb + 1) * 4 + 15) & ~(size_t)15;
-        long long *sagg = (long long *)((char *)scratch + zb);
-        long long *sinc = sagg + nb;
-        cudaMemsetAsync(scratch, 0, zb, st);
-        seg_onepass_kernel<K, V, AGG><<<(unsigned)nb, P_THREADS, 0, st>>>((const K *)keys, (const V *)v, N, grp,
-                                                                           status, sagg, sinc, counter);
-        *launches += 1;
-        return;
-    }
-#endif
-    const long long nb = (N + G_BLOCK - 1) / G_BLOCK;
-    long long *bv = (long long *)scratch;
-    int *bf = (int *)(bv + nb + 1);
-    seg_block_kernel<K, V, AGG, false><<<(unsigned)nb, P_THREADS, 0, st>>>((const K *)keys, (const V *)v, N, bv, bf,
-                                                                           nullptr);
-    seg_block_scan_kernel<AGG><<<1, 1024, 0, st>>>(bv, bf, nb);
-    seg_block_kernel<K, V, AGG, true><<<(unsigned)nb, P_THREADS, 0, st>>>((const K *)keys, (const V *)v, N, bv, bf,
-                                                                          grp);
-    *launches += 3;
+    const long long nb = (N + SG_BLOCK - 1) / SG_BLOCK;
+    unsigned *counter = (unsigned *)scratch;
+    unsigned *status = counter + 1;
+    const size_t zb = ((size_t)(nb + 1) * 4 + 15) & ~(size_t)15;
+    long long *sagg = (long long *)((char *)scratch + zb);
+    long long *sinc = sagg + nb;
+    cudaMemsetAsync(scratch, 0, zb, st);
+    seg_onepass_kernel<K, V, AGG><<<(unsigned)nb, P_THREADS, 0, st>>>((const K *)keys, (const V *)v, N, grp, status,
+                                                                       sagg, sinc, counter);
+    *launches += 1;
 }
 
 cudaError_t launch_index_group_agg(int agg, int kb, int vb, const void *keys, const void *payload, long long n,
