@@ -533,6 +533,7 @@ __global__ void __launch_bounds__(P_THREADS) seg_onepass_kernel(const K *__restr
     __shared__ SegPair<AGG> s_carry;
     __shared__ long long s_b;
     __shared__ int s_head0;
+    __shared__ SegPair<AGG> s_blk;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) s_b = atomicAdd(counter, 1u);
     __syncthreads();
@@ -568,36 +569,55 @@ __global__ void __launch_bounds__(P_THREADS) seg_onepass_kernel(const K *__restr
     SegPair<AGG> up{__shfl_up_sync(FULL, incl.v, 1), __shfl_up_sync(FULL, incl.f, 1)};
     if (lane == 0) up = SegPair<AGG>{ident<AGG>(), 0};
     const SegPair<AGG> tex = seg_comb<AGG>(wpre, up);   // the block's rows before this thread's
-    if (tid == P_THREADS - 1) {
-        const SegPair<AGG> blk = seg_comb<AGG>(tex, tot);   // the whole block
-        SegPair<AGG> carry{ident<AGG>(), 0};
-        if (b == 0 || blk.f) {   // the block's inclusive pair does not depend on its predecessors
-            sinc[b] = blk.v;
-            __threadfence();
-            st_relaxed_u32(status + b, 2u | ((unsigned)blk.f << 2));
-        } else {
-            sagg[b] = blk.v;
-            __threadfence();
-            st_relaxed_u32(status + b, 1u);
-        }
-        if (b > 0 && !s_head0) {   // rows before the block's first run start take the carry
-            for (long long p = b - 1; p >= 0; p--) {
-                unsigned st;
-                while (((st = ld_relaxed_u32(status + p)) & 3u) == 0) {
-                }
+    if (tid == P_THREADS - 1) s_blk = seg_comb<AGG>(tex, tot);   // the whole block
+    __syncthreads();
+    if (warp == 0) {
+        const SegPair<AGG> blk = s_blk;
+        if (lane == 0) {
+            if (b == 0 || blk.f) {   // the block's inclusive pair does not depend on its predecessors
+                sinc[b] = blk.v;
                 __threadfence();
-                const long long pv = (st & 3u) == 2u ? ld_relaxed_u64((const unsigned long long *)(sinc + p))
-                                                     : ld_relaxed_u64((const unsigned long long *)(sagg + p));
-                carry = seg_comb<AGG>(SegPair<AGG>{pv, (int)((st >> 2) & 1u)}, carry);
-                if ((st & 3u) == 2u || ((st >> 2) & 1u)) break;
+                st_relaxed_u32(status + b, 2u | ((unsigned)blk.f << 2));
+            } else {
+                sagg[b] = blk.v;
+                __threadfence();
+                st_relaxed_u32(status + b, 1u);
             }
-            if (!blk.f) {
+        }
+        SegPair<AGG> carry{ident<AGG>(), 0};
+        if (b > 0 && !s_head0) {   // rows before the block's first run start take the carry
+            // 32 predecessors per round (lane l: block top - l); the walk stops
+            // at the nearest one that is inclusive or holds a run start
+            for (long long top = b - 1; top >= 0; top -= 32) {
+                const long long p = top - lane;
+                unsigned st = 2u;
+                long long pv = ident<AGG>();
+                if (p >= 0) {
+                    while (((st = ld_relaxed_u32(status + p)) & 3u) == 0) {
+                    }
+                    __threadfence();
+                    pv = (st & 3u) == 2u ? ld_relaxed_u64((const unsigned long long *)(sinc + p))
+                                         : ld_relaxed_u64((const unsigned long long *)(sagg + p));
+                }
+                const int pf = (int)((st >> 2) & 1u);
+                const unsigned stopm = __ballot_sync(FULL, (st & 3u) == 2u || pf);
+                const int stop = stopm ? __ffs(stopm) - 1 : 31;
+                // in order: pair[stop] (farthest) ... pair[0] (nearest), then carry
+                SegPair<AGG> w{ident<AGG>(), 0};
+                for (int l = stop; l >= 0; l--) {
+                    const SegPair<AGG> q{__shfl_sync(FULL, pv, l), __shfl_sync(FULL, pf, l)};
+                    w = seg_comb<AGG>(w, q);
+                }
+                carry = seg_comb<AGG>(w, carry);
+                if (stopm) break;
+            }
+            if (lane == 0 && !blk.f) {
                 sinc[b] = seg_comb<AGG>(carry, blk).v;
                 __threadfence();
                 st_relaxed_u32(status + b, 2u);
             }
         }
-        s_carry = carry;
+        if (lane == 0) s_carry = carry;
     }
     __syncthreads();
     const SegPair<AGG> pre = seg_comb<AGG>(s_carry, tex);
