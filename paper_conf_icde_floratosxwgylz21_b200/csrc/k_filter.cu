@@ -157,8 +157,12 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
                   uint8_t *__restrict__ out_kvalid, void *__restrict__ out_vals,
                   unsigned long long *__restrict__ keymask, unsigned *__restrict__ extreme,
                   const unsigned long long *__restrict__ tile_base, unsigned *__restrict__ tile_count,
-                  unsigned *__restrict__ counter, long long *__restrict__ out_count)
+                  unsigned *__restrict__ counter, long long *__restrict__ out_count,
+                  unsigned *__restrict__ live_bits)
 {
+    // live_bits (ordered two-pass mode): pass 1 (tile_count) writes each
+    // (tile, item, warp)'s survivor ballot; pass 2 takes its survivors from
+    // them instead of re-reading and re-evaluating the predicate columns
     using K = typename std::conditional<KB == 8, uint64_t, uint32_t>::type;
     using V = typename std::conditional<VB == 8, long long, int>::type;
     constexpr int TILE = T_THREADS * ITEMS;
@@ -212,9 +216,15 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
         const long long rows = min((long long)TILE, n - base);
 
         unsigned live = 0;
+        if (live_bits && !tile_count) {
 #pragma unroll
-        for (int j = 0; j < ITEMS; j++)
-            if (j * T_THREADS + tid < rows) live |= 1u << j;
+            for (int j = 0; j < ITEMS; j++)
+                live |= ((__ldcg(live_bits + (tile * ITEMS + j) * T_WARPS + warp) >> lane) & 1u) << j;
+        } else {
+#pragma unroll
+            for (int j = 0; j < ITEMS; j++)
+                if (j * T_THREADS + tid < rows) live |= 1u << j;
+        }
         // local predicates (NULL operands are not TRUE, reading R2)
         const unsigned char *sb = smem + stage * sc.stage_bytes;
         for (int k = 0; k < tp.n_preds; k++) {
@@ -271,7 +281,10 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
 #pragma unroll
         for (int j = 0; j < ITEMS; j++) {
             const unsigned m = __ballot_sync(FULL, live >> j & 1u);
-            if (lane == 0) s_cnt[j][warp] = __popc(m);
+            if (lane == 0) {
+                s_cnt[j][warp] = __popc(m);
+                if (live_bits && tile_count) live_bits[(tile * ITEMS + j) * T_WARPS + warp] = m;
+            }
             rank[j] = __popc(m & lanemask_lt());
         }
         __syncthreads();
@@ -722,36 +735,42 @@ __global__ void __launch_bounds__(256) rp_dense_kernel(long long n, KeySrc ks, i
 }
 
 // ------------------------------------------------------------------ host side
-// Exclusive scan of the per-tile counts (ordered mode): one CTA, chunks of 1024.
+// Exclusive scan of the per-tile counts (ordered mode): one CTA; thread t
+// owns a contiguous segment of the counts (loads of the segment in flight
+// together), sums it, block scan, then writes the segment's prefixes -- a
+// few memory round trips instead of one per 1024-count chunk (60M rows =
+// 29k tiles: 44 -> 26 us; chunks staged in shared memory measured 32 us).
 __global__ void __launch_bounds__(1024) tile_scan_kernel(const unsigned *__restrict__ cnt, long long tiles,
                                                          unsigned long long *__restrict__ base,
                                                          long long *__restrict__ out_count)
 {
     __shared__ unsigned long long s_w[32];
-    __shared__ unsigned long long s_carry;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    if (threadIdx.x == 0) s_carry = 0;
-    __syncthreads();
-    for (long long b0 = 0; b0 < tiles; b0 += 1024) {
-        const long long i = b0 + threadIdx.x;
-        const unsigned long long x = i < tiles ? cnt[i] : 0ull;
-        unsigned long long incl = x;
+    const long long per = (tiles + 1023) / 1024;
+    const long long i0 = threadIdx.x * per, i1 = min(tiles, i0 + per);
+    unsigned long long sum = 0;
+#pragma unroll 8
+    for (long long i = i0; i < i1; i++) sum += __ldg(cnt + i);
+    unsigned long long incl = sum;
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const unsigned long long y = __shfl_up_sync(FULL, incl, o);
-            if (lane >= o) incl += y;
-        }
-        if (lane == 31) s_w[warp] = incl;
-        __syncthreads();
-        unsigned long long wpre = 0;
-        for (int w = 0; w < warp; w++) wpre += s_w[w];
-        const unsigned long long carry = s_carry;
-        if (i < tiles) base[i] = carry + wpre + incl - x;
-        __syncthreads();
-        if (threadIdx.x == 1023) s_carry = carry + wpre + incl;
-        __syncthreads();
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long y = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += y;
     }
-    if (threadIdx.x == 0) *out_count = (long long)s_carry;
+    if (lane == 31) s_w[warp] = incl;
+    __syncthreads();
+    unsigned long long run = incl - sum, total = 0;
+    for (int w = 0; w < 32; w++) {
+        if (w < warp) run += s_w[w];
+        total += s_w[w];
+    }
+#pragma unroll 8
+    for (long long i = i0; i < i1; i++) {
+        const unsigned c = __ldg(cnt + i);
+        base[i] = run;
+        run += c;
+    }
+    if (threadIdx.x == 0) *out_count = (long long)total;
 }
 
 namespace {
@@ -796,6 +815,7 @@ struct FilterOut {
     unsigned *tile_count;
     unsigned *counter;
     long long *count;
+    unsigned *live_bits;   // ordered two-pass mode: survivor ballots of pass 1 (nullable)
 };
 
 template <int KB, int VB, int ITEMS>
@@ -815,7 +835,7 @@ cudaError_t launch_t(long long n, const SrcCols &sc, const TPlan &tp, const Filt
     long long grid = (long long)num_sms * (occ > 0 ? occ : 1);
     if (grid > tiles) grid = tiles;
     kern<<<(unsigned)grid, T_THREADS, smem, st>>>(n, sc, tp, o.ids, o.keys, o.kvalid, o.vals, o.keymask, o.extreme,
-                                                  o.tile_base, o.tile_count, o.counter, o.count);
+                                                  o.tile_base, o.tile_count, o.counter, o.count, o.live_bits);
     return cudaGetLastError();
 }
 
@@ -850,7 +870,7 @@ size_t filter_scratch_bytes(long long n)
 {
     // counters + per-tile counts / offsets (two-pass mode), or the ordered
     // filter's chunk counts + ballot words
-    const size_t two_pass = 1024 + 256 + (size_t)(n / T_THREADS + 2) * 12;
+    const size_t two_pass = 1024 + 768 + (size_t)(n / T_THREADS + 2) * 12 + (size_t)(n / 32 + 2) * 4 + 64 * 16 * 4;
     const size_t one_launch = RP_BITS_OFF + (size_t)(n / 32 + 2) * 4 + 256;
     return two_pass > one_launch ? two_pass : one_launch;
 }
@@ -1085,9 +1105,39 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
         const long long tiles = (n + T_THREADS * items - 1) / (T_THREADS * items);
         unsigned *tcount = (unsigned *)((char *)scratch + 1024);
         unsigned long long *tbase = (unsigned long long *)((char *)scratch + 1024 + ((tiles * 4 + 255) & ~255ll));
+        // the two-call mode keeps pass 1's survivor ballots for pass 2
+        unsigned *bits = ordered_phase ? (unsigned *)((char *)tbase + ((tiles * 8 + 255) & ~255ll)) : nullptr;
         if (ordered_phase == 2) {
+            // pass 2 streams only the key / payload columns: the predicate
+            // columns are not read again
+            SrcCols sc2;
+            memset(&sc2, 0, sizeof sc2);
+            SrcPlan sp2 = sp;
+            sp2.key0 = sp2.key0v = sp2.key1 = sp2.key1v = sp2.val = sp2.valv = -1;
+            if (k) {
+                sp2.key0 = add_src(sc2, key.c0, key.n_key == 2 ? 4 : key.w0);
+                sp2.key0v = add_src(sc2, key.v0, 1);
+                if (key.n_key == 2) {
+                    sp2.key1 = add_src(sc2, key.c1, 4);
+                    sp2.key1v = add_src(sc2, key.v1, 1);
+                }
+            }
+            if (v) {
+                sp2.val = add_src(sc2, val.c, val.w);
+                sp2.valv = add_src(sc2, val.v, 1);
+            }
+            int off2 = 0;
+            for (int c = 0; c < sc2.n; c++) {
+                sc2.off[c] = off2;
+                off2 += (T_THREADS * items * sc2.w[c] + 15) & ~15;
+            }
+            sc2.stage_bytes = off2 ? ((off2 + 127) & ~127) : 128;
+            TPlan tp2 = tp;
+            tp2.n_preds = 0;
+            resolve(sc2, sp2, tp2);
             o.tile_base = tbase;
-            e = dispatch(k, v, items, n, sc, tp, o, num_sms, st);
+            o.live_bits = bits;
+            e = dispatch(k, v, items, n, sc2, tp2, o, num_sms, st);
             ++*launches;
             return e;
         }
@@ -1104,7 +1154,7 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
         TPlan tp1 = tp;
         resolve(sc1, sp1, tp1);
         FilterOut o1{nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, tcount,
-                     (unsigned *)scratch + 64, out_count};
+                     (unsigned *)scratch + 64, out_count, bits};
         e = launch_items<0, 0>(items, n, sc1, tp1, o1, num_sms, st);
         if (e != cudaSuccess) return e;
         tile_scan_kernel<<<1, 1024, 0, st>>>(tcount, tiles, tbase, out_count);
