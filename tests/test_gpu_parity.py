@@ -1045,3 +1045,22 @@ def test_tiny_one_launch_path(eng, tiny):
                                                                   "S": {"col1": "int64", "col2": "int64"}})
     finally:
         eng.set_option(OPT_TINY, 1)
+
+
+@pytest.mark.parametrize("spread", ["dense", "sparse"])
+def test_key_ordered_outer_index_path(eng, spread):
+    """Ascending outer keys (TPC-H orders by o_orderkey) through the index
+    path: every operator x aggregate vs the oracle, ragged warps, duplicate
+    outer keys, keys below / above S's range, dense and sparse key spreads."""
+    rng = np.random.default_rng(31 if spread == "dense" else 32)
+    n_s = 200_003
+    s_keys = rng.integers(0, 50_000 if spread == "dense" else 5_000_000, n_s)
+    n_r = 40_013
+    r_keys = np.sort(rng.integers(-100, (50_000 if spread == "dense" else 5_000_000) + 100, n_r))
+    t = {"R": {"col1": r_keys.astype(np.int32), "col2": rng.integers(-60, 60, n_r).astype(np.int32)},
+         "S": {"col1": s_keys.astype(np.int32), "col2": rng.integers(-60, 60, n_s).astype(np.int32)}}
+    for corr_op in PLAN_OPS:
+        for agg in ("min", "count", "sum", "exists"):
+            plan = make_plan(corr_op, agg, "<=")
+            assert_parity(run(eng, t, plan, "index", emit_all=True), oracle.evaluate(t, plan), plan, True,
+                          ctx=(spread, corr_op, agg))
