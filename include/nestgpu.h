@@ -179,8 +179,10 @@ nestgpu_status nestgpu_gather_column(nestgpu_ctx *ctx, int32_t src_col, const in
  * nestgpu_alloc_column) with a NOT NULL payload needs no sort: S' is
  * compacted in row order straight into the index (the stable sort of a
  * sorted S' is the identity; same bytes).
- * Synchronises the stream once (to size the sort or the index), plus once
- * when a key column's statistics are computed.  UNSUPPORTED when a sort
+ * Synchronises the stream once (to size the sort or the index) -- not at
+ * all for an index over all of S (no inner predicates, NOT NULL key and
+ * payload: the radix plan comes from the key column's statistics) -- plus
+ * once when a key column's statistics are computed.  UNSUPPORTED when a sort
  * would see |S'| >= 2^30 rows (columns hold < 2^31).
  * Errors: INVALID, TYPE, UNSUPPORTED, OOM, CUDA. */
 nestgpu_status nestgpu_build_index(nestgpu_ctx *ctx, const int32_t *key_cols, int32_t n_key_cols,

@@ -44,6 +44,7 @@ struct Column {
     bool stats;         // host-side min/max known
     long long mn, mx;
     bool sorted;        // (with stats) NOT NULL and stored in ascending key order
+    long long band, bor;   // (with stats) AND / OR of the non-NULL (sign-extended) values
     bool caller_filled; // nestgpu_alloc_column: contents may change behind our back (stats not cached)
 };
 
@@ -391,15 +392,17 @@ namespace {
 nestgpu_status column_stats(nestgpu_ctx *c, Column &col)
 {
     if (col.stats) return NESTGPU_OK;
-    long long *d = (long long *)salloc(c, 24);
+    long long *d = (long long *)salloc(c, 40);
     if (!d) return fail(c, NESTGPU_ERR_OOM, "arena exhausted (stats)");
     CUDA_TRY(c, ng::launch_minmax(col.d, dtype_width(col.dtype), col.valid, col.n, d, c->stream, &c->launches));
-    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, d, 24, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, d, 40, cudaMemcpyDeviceToHost, c->stream));
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
     long long desc;
     memcpy(&col.mn, c->pinned, 8);
     memcpy(&col.mx, (char *)c->pinned + 8, 8);
     memcpy(&desc, (char *)c->pinned + 16, 8);
+    memcpy(&col.band, (char *)c->pinned + 24, 8);
+    memcpy(&col.bor, (char *)c->pinned + 32, 8);
     col.sorted = !col.valid && desc == 0;
     col.stats = true;
     return NESTGPU_OK;
@@ -765,6 +768,18 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
         }
     }
     const int fkb = pre_narrow ? 4 : kb;   // key width the S' filter writes
+    // an index over all of S (no predicates, NOT NULL key / payload) needs no
+    // sync: |S'| = |S| and the radix plan comes from the key column's stats
+    bool nosync = false;
+    if (n_key_cols == 1 && n_inner_preds == 0 && c->sort_mode != 2) {
+        Column &kc = c->cols[key_cols[0]];
+        if (!kc.valid && !(pc && pc->valid)) {
+            if (kc.caller_filled && !stats_fresh) kc.stats = false;
+            if ((s = column_stats(c, kc))) return s;
+            stats_fresh = true;
+            nosync = true;
+        }
+    }
     scratch_reset(c);
     for (int st = 0; st < NESTGPU_N_STAGES; st++) c->ran[st] = false;
     void *tk = salloc(c, (size_t)n * kb), *tv = vb ? salloc(c, (size_t)n * vb) : nullptr;
@@ -804,14 +819,35 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
                                   fscr, d_count, c->stream, &c->launches, true));
     prof_end(c, 1);
     htrace(c, "filter");
-    CUDA_TRY(c, cudaMemcpyAsync(c->pinned, dsmall, 32, cudaMemcpyDeviceToHost, c->stream));
-    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
-    htrace(c, "sync");
     long long nsp;
     unsigned long long kand, kor;
-    memcpy(&nsp, c->pinned, 8);
-    memcpy(&kand, c->pinned + 4, 8);
-    memcpy(&kor, c->pinned + 6, 8);
+    if (nosync) {
+        // no predicates, NOT NULL key and payload: S' = S, and the key bits
+        // that vary come from the column statistics (AND / OR of the values,
+        // encoded as the filter encodes them) -- no host round trip
+        const Column &kc = c->cols[key_cols[0]];
+        const unsigned long long sb = fkb == 8 ? (1ull << 63) : (kb == 4 ? 0x80000000ull : 0ull);
+        unsigned long long ka = (unsigned long long)kc.band, ko = (unsigned long long)kc.bor;
+        if (fkb == 4) {
+            ka &= 0xffffffffull;
+            ko &= 0xffffffffull;
+        }
+        kand = (ka & ~sb) | (~ko & sb);
+        kor = (ko & ~sb) | (~ka & sb);
+        if (fkb == 4) {   // 4-byte keys: the filter's AND / OR of zero-extended keys
+            kand &= 0xffffffffull;
+            kor &= 0xffffffffull;
+        }
+        nsp = n;
+        htrace(c, "plan from stats");
+    } else {
+        CUDA_TRY(c, cudaMemcpyAsync(c->pinned, dsmall, 32, cudaMemcpyDeviceToHost, c->stream));
+        CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+        htrace(c, "sync");
+        memcpy(&nsp, c->pinned, 8);
+        memcpy(&kand, c->pinned + 4, 8);
+        memcpy(&kor, c->pinned + 6, 8);
+    }
     if (nsp >= (1ll << 30))   // radix-pass look-back words carry 30-bit counts
         return fail(c, NESTGPU_ERR_UNSUPPORTED, "build_index: |S'| = %lld >= 2^30 rows to sort", nsp);
     int shifts[8], rb = 8;

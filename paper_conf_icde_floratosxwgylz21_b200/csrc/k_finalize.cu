@@ -666,24 +666,31 @@ cudaError_t launch_tiny_exec(const TinyArgs &t0, int num_sms, cudaStream_t st, l
 // ------------------------------------------------------------------ column min / max
 // (for the SUM/AVG overflow pre-check, reading R5)
 // (and out[2] != 0 iff some row is smaller than its predecessor: the
-// column is not stored in key order -- the index build's sort-free path)
+// column is not stored in key order -- the index build's sort-free path;
+// out[3] / out[4] the AND / OR of the values: the key bits that vary, so an
+// index build without predicates plans its radix passes with no sync)
 __global__ void minmax_init_kernel(long long *out)
 {
     out[0] = LLONG_MAX;
     out[1] = LLONG_MIN;
     out[2] = 0;
+    out[3] = -1;   // AND of the (sign-extended) values
+    out[4] = 0;    // OR
 }
 
 __global__ void minmax_kernel(const void *__restrict__ col, int w, const uint8_t *__restrict__ valid, long long n,
                               long long *__restrict__ out)
 {
     long long mn = LLONG_MAX, mx = LLONG_MIN;
+    unsigned long long ka = ~0ull, ko = 0ull;
     bool desc = false;
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
         if (valid && !valid[i]) continue;
         const long long v = load_w(col, w, i);
         mn = min(mn, v);
         mx = max(mx, v);
+        ka &= (unsigned long long)v;
+        ko |= (unsigned long long)v;
         if (i > 0 && !valid) desc |= load_w(col, w, i - 1) > v;
     }
     for (int o = 16; o > 0; o >>= 1) {
@@ -691,10 +698,16 @@ __global__ void minmax_kernel(const void *__restrict__ col, int w, const uint8_t
         mx = max(mx, __shfl_xor_sync(FULL, mx, o));
     }
     desc = __any_sync(FULL, desc);
+    for (int o = 16; o > 0; o >>= 1) {
+        ka &= __shfl_xor_sync(FULL, ka, o);
+        ko |= __shfl_xor_sync(FULL, ko, o);
+    }
     if ((threadIdx.x & 31) == 0) {
         atomicMin(&out[0], mn);
         atomicMax(&out[1], mx);
         if (desc) atomicOr((unsigned long long *)&out[2], 1ull);
+        atomicAnd((unsigned long long *)&out[3], ka);
+        atomicOr((unsigned long long *)&out[4], ko);
     }
 }
 
