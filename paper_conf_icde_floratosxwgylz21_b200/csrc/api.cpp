@@ -814,9 +814,37 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
         CUDA_TRY(c, ng::launch_fill(fl, c->stream, &c->launches));
         htrace(c, "fill");
     }
+    // the encoded key AND / OR the S' filter would report, from the key
+    // column's statistics (nosync: S' = S)
+    auto stats_mask = [&](unsigned long long &ka_out, unsigned long long &ko_out) {
+        const Column &kc = c->cols[key_cols[0]];
+        const unsigned long long sb = fkb == 8 ? (1ull << 63) : (kb == 4 ? 0x80000000ull : 0ull);
+        unsigned long long ka = (unsigned long long)kc.band, ko = (unsigned long long)kc.bor;
+        if (fkb == 4) {   // 4-byte keys: the filter's AND / OR of zero-extended keys
+            ka &= 0xffffffffull;
+            ko &= 0xffffffffull;
+        }
+        ka_out = (ka & ~sb) | (~ko & sb);
+        ko_out = (ko & ~sb) | (~ka & sb);
+        if (fkb == 4) {
+            ka_out &= 0xffffffffull;
+            ko_out &= 0xffffffffull;
+        }
+    };
+    // with S' = S and at least one radix pass, the first pass and the
+    // histogram read the raw key / payload columns and encode keys as they
+    // load them: no filter pass at all
+    bool raw_input = false;
+    if (nosync && n > 1 && n < (1ll << 30)) {
+        unsigned long long ka, ko;
+        stats_mask(ka, ko);
+        int sh0[8], rb0 = 8;
+        raw_input = plan_sort_passes(fkb, ka, ko, n, sh0, &rb0) >= 1;
+    }
     prof_begin(c, 1);
-    CUDA_TRY(c, ng::launch_filter(n, ps, ks, fkb, vs, vb, 1, pc ? 1 : 0, nullptr, tk, nullptr, tv, keymask, nullptr,
-                                  fscr, d_count, c->stream, &c->launches, true));
+    if (!raw_input)
+        CUDA_TRY(c, ng::launch_filter(n, ps, ks, fkb, vs, vb, 1, pc ? 1 : 0, nullptr, tk, nullptr, tv, keymask, nullptr,
+                                      fscr, d_count, c->stream, &c->launches, true));
     prof_end(c, 1);
     htrace(c, "filter");
     long long nsp;
@@ -825,19 +853,7 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
         // no predicates, NOT NULL key and payload: S' = S, and the key bits
         // that vary come from the column statistics (AND / OR of the values,
         // encoded as the filter encodes them) -- no host round trip
-        const Column &kc = c->cols[key_cols[0]];
-        const unsigned long long sb = fkb == 8 ? (1ull << 63) : (kb == 4 ? 0x80000000ull : 0ull);
-        unsigned long long ka = (unsigned long long)kc.band, ko = (unsigned long long)kc.bor;
-        if (fkb == 4) {
-            ka &= 0xffffffffull;
-            ko &= 0xffffffffull;
-        }
-        kand = (ka & ~sb) | (~ko & sb);
-        kor = (ko & ~sb) | (~ka & sb);
-        if (fkb == 4) {   // 4-byte keys: the filter's AND / OR of zero-extended keys
-            kand &= 0xffffffffull;
-            kor &= 0xffffffffull;
-        }
+        stats_mask(kand, kor);
         nsp = n;
         htrace(c, "plan from stats");
     } else {
@@ -933,7 +949,7 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
         ng::FillList fl;
         fl.add(hist, ng::hist_bytes());
         for (int p = 0; p < np; p++) {
-            const int kin = pre_narrow || (narrow && p > 0) ? 4 : kb;
+            const int kin = raw_input && p == 0 ? kb : (pre_narrow || (narrow && p > 0) ? 4 : kb);
             const size_t zb = ng::sort_pass_zero_bytes(nsp, kin, vb, rb);
             pscr[p] = salloc(c, zb);
             if (!pscr[p]) return fail(c, NESTGPU_ERR_OOM, "arena exhausted (sort scratch)");
@@ -943,8 +959,14 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
     }
     htrace(c, "fill2");
     if (!sorted) {
-        CUDA_TRY(c, ng::launch_digit_hist(fkb, tk, nsp, shifts, np, hist, dbase, c->num_sms, c->stream, &c->launches,
-                                          rb, true));
+        const Column &kcol = c->cols[key_cols[0]];
+        const unsigned long long rencx = kb == 8 ? (1ull << 63) : 0x80000000ull;   // raw column -> encoded key
+        if (raw_input)
+            CUDA_TRY(c, ng::launch_digit_hist(kb, kcol.d, nsp, shifts, np, hist, dbase, c->num_sms, c->stream,
+                                              &c->launches, rb, true, rencx));
+        else
+            CUDA_TRY(c, ng::launch_digit_hist(fkb, tk, nsp, shifts, np, hist, dbase, c->num_sms, c->stream,
+                                              &c->launches, rb, true));
         htrace(c, "hist");
     }
     if (sorted) {
@@ -954,16 +976,20 @@ nestgpu_status nestgpu_build_index(nestgpu_ctx *c, const int32_t *key_cols, int3
             if (vb) CUDA_TRY(c, cudaMemcpyAsync(ix.payload, tv, (size_t)nsp * vb, cudaMemcpyDeviceToDevice, c->stream));
         }
     } else {
-        // T -> ... -> P with ping-pong so that the last pass writes P.
-        const void *ik = tk, *iv = tv;
+        // T -> ... -> P with ping-pong so that the last pass writes P (the
+        // first pass reads the raw columns when the filter was skipped)
+        const Column &kcol = c->cols[key_cols[0]];
+        const void *ik = raw_input ? kcol.d : tk, *iv = raw_input ? (pc ? pc->d : nullptr) : tv;
         for (int p = 0; p < np; p++) {
             const bool to_final = ((np - 1 - p) % 2) == 0;
             void *ok = to_final ? ix.keys : uk;
             void *ov = to_final ? ix.payload : uv;
             if (ok == ik) { ok = tk; ov = tv; }
-            const int kin = pre_narrow || (narrow && p > 0) ? 4 : kb, kout = narrow && p < np - 1 ? 4 : kb;
+            const bool rawp = raw_input && p == 0;
+            const int kin = rawp ? kb : (pre_narrow || (narrow && p > 0) ? 4 : kb), kout = narrow && p < np - 1 ? 4 : kb;
+            const unsigned long long encx = rawp ? (kb == 8 ? (1ull << 63) : 0x80000000ull) : 0ull;
             CUDA_TRY(c, ng::launch_radix_pass_x(kin, kout, vb, ik, ok, iv, ov, nsp, shifts[p], dbase + p * (1 << rb),
-                                                pscr[p], hi, c->stream, &c->launches, rb, true));
+                                                pscr[p], hi, c->stream, &c->launches, rb, true, encx));
             ik = ok;
             iv = ov;
         }

@@ -125,9 +125,10 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
 // hist: hist_bytes() of scratch (8 x 512 bins + a CTA-done counter); the
 // kernel's last CTA scans the bins into digit_base (one launch).
 size_t hist_bytes();
+//   encx: XOR applied to every key read (encodes a raw signed key column)
 cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *shifts, int np, unsigned *hist,
                               unsigned *digit_base, int num_sms, cudaStream_t st, long long *launches, int rb = 8,
-                              bool prezeroed = false);
+                              bool prezeroed = false, unsigned long long encx = 0);
 
 // a4: one stable LSD radix pass on the rb-bit digit (rb = 8 or 9) at bit
 // `shift` of the encoded keys.
@@ -141,7 +142,7 @@ cudaError_t launch_radix_pass(int kb, int vb, const void *kin, void *kout, const
 cudaError_t launch_radix_pass_x(int kb_in, int kb_out, int vb, const void *kin, void *kout, const void *vin,
                                 void *vout, long long n, int shift, const unsigned *digit_base, void *scratch,
                                 unsigned hi, cudaStream_t st, long long *launches, int rb = 8,
-                                bool prezeroed = false);
+                                bool prezeroed = false, unsigned long long encx = 0);
 // scratch bytes of one radix pass that must be zero (per-tile digit counts + counter)
 size_t sort_pass_zero_bytes(long long n, int kb, int vb, int rb);
 

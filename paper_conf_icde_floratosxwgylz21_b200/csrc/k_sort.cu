@@ -150,8 +150,10 @@ template <typename K, int VB, typename KO, int RB>
 __global__ void __launch_bounds__(S_THREADS, NG_S_PMINB)
 onesweep_p_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *__restrict__ vin_,
                   void *__restrict__ vout_, long long n, int shift, const unsigned *__restrict__ digit_base,
-                  unsigned *__restrict__ status, unsigned *__restrict__ counter, unsigned hi)
+                  unsigned *__restrict__ status, unsigned *__restrict__ counter, unsigned hi, K encx)
 {
+    // encx: XOR applied to every key read (the sign-bit flip that encodes a
+    // raw signed key column; 0 when the input is already encoded)
     using C = PassCfg<K, VB, RB>;
     using V = typename C::V;
     constexpr int ITEMS = C::ITEMS, TILE = C::TILE;
@@ -217,7 +219,7 @@ onesweep_p_kernel(const K *__restrict__ kin, KO *__restrict__ kout, const void *
         for (int j = 0; j < ITEMS; j++) {
             const int p = warp * 32 * ITEMS + j * 32 + lane;
             const bool ok = p < tile_n;
-            key[j] = ok ? s_k[p] : (K)0;
+            key[j] = ok ? (K)(s_k[p] ^ encx) : (K)0;
             if constexpr (VB > 0) val[j] = ok ? s_v[p] : (V)0;
             if (ok) atomicAdd(&s_cnt[warp][(unsigned)(key[j] >> shift) & DM], 1u);
         }
@@ -381,7 +383,7 @@ template <typename K, int NB>
 __global__ void __launch_bounds__(256) digit_hist_kernel(const K *__restrict__ keys, long long n, DigitList dl,
                                                          unsigned *__restrict__ hist,
                                                          unsigned *__restrict__ done,
-                                                         unsigned *__restrict__ digit_base)
+                                                         unsigned *__restrict__ digit_base, K encx)
 {
     __shared__ unsigned s_hist[8 * NB];
     __shared__ bool s_last;
@@ -396,7 +398,7 @@ __global__ void __launch_bounds__(256) digit_hist_kernel(const K *__restrict__ k
     for (long long i0 = blockIdx.x * 256LL + threadIdx.x; i0 < n; i0 += stride * HB) {
         K k[HB];
 #pragma unroll
-        for (int u = 0; u < HB; u++) k[u] = i0 + u * stride < n ? __ldg(keys + i0 + u * stride) : (K)0;
+        for (int u = 0; u < HB; u++) k[u] = i0 + u * stride < n ? (K)(__ldg(keys + i0 + u * stride) ^ encx) : (K)0;
 #pragma unroll
         for (int u = 0; u < HB; u++) {
             if (i0 + u * stride >= n) break;
@@ -448,7 +450,7 @@ size_t hist_bytes() { return 8 * 512 * 4 + 256; }
 
 cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *shifts, int np, unsigned *hist,
                               unsigned *digit_base, int num_sms, cudaStream_t st, long long *launches, int rb,
-                              bool prezeroed)
+                              bool prezeroed, unsigned long long encx)
 {
     if (np <= 0) return cudaSuccess;
     const int nb = 1 << rb;
@@ -465,11 +467,11 @@ cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *
     if (blocks > (long long)num_sms * 8) blocks = (long long)num_sms * 8;
     if (blocks < 1) blocks = 1;
     if (rb == 8) {
-        if (kb == 4) digit_hist_kernel<uint32_t, 256><<<(unsigned)blocks, 256, 0, st>>>((const uint32_t *)keys, n, dl, hist, done, digit_base);
-        else digit_hist_kernel<uint64_t, 256><<<(unsigned)blocks, 256, 0, st>>>((const uint64_t *)keys, n, dl, hist, done, digit_base);
+        if (kb == 4) digit_hist_kernel<uint32_t, 256><<<(unsigned)blocks, 256, 0, st>>>((const uint32_t *)keys, n, dl, hist, done, digit_base, (uint32_t)encx);
+        else digit_hist_kernel<uint64_t, 256><<<(unsigned)blocks, 256, 0, st>>>((const uint64_t *)keys, n, dl, hist, done, digit_base, (uint64_t)encx);
     } else {
-        if (kb == 4) digit_hist_kernel<uint32_t, 512><<<(unsigned)blocks, 256, 0, st>>>((const uint32_t *)keys, n, dl, hist, done, digit_base);
-        else digit_hist_kernel<uint64_t, 512><<<(unsigned)blocks, 256, 0, st>>>((const uint64_t *)keys, n, dl, hist, done, digit_base);
+        if (kb == 4) digit_hist_kernel<uint32_t, 512><<<(unsigned)blocks, 256, 0, st>>>((const uint32_t *)keys, n, dl, hist, done, digit_base, (uint32_t)encx);
+        else digit_hist_kernel<uint64_t, 512><<<(unsigned)blocks, 256, 0, st>>>((const uint64_t *)keys, n, dl, hist, done, digit_base, (uint64_t)encx);
     }
     *launches += 1;
     return cudaGetLastError();
@@ -482,7 +484,8 @@ cudaError_t launch_digit_hist(int kb, const void *keys, long long n, const int *
 // inclusive prefix.  Also zeroes the tile counter.
 template <typename K, int NB, int TILE>
 __global__ void __launch_bounds__(256) tile_agg_kernel(const K *__restrict__ keys, long long n, int shift,
-                                                       unsigned *__restrict__ status, unsigned *__restrict__ counter)
+                                                       unsigned *__restrict__ status, unsigned *__restrict__ counter,
+                                                       K encx)
 {
     __shared__ unsigned h[NB];
     for (int d = threadIdx.x; d < NB; d += 256) h[d] = 0;
@@ -491,7 +494,7 @@ __global__ void __launch_bounds__(256) tile_agg_kernel(const K *__restrict__ key
     const long long b0 = t * TILE;
     const long long b1 = min(n, b0 + TILE);
     for (long long i = b0 + threadIdx.x; i < b1; i += 256)
-        atomicAdd(&h[(unsigned)(__ldg(keys + i) >> shift) & (NB - 1)], 1u);
+        atomicAdd(&h[(unsigned)((__ldg(keys + i) ^ encx) >> shift) & (NB - 1)], 1u);
     __syncthreads();
     for (int d = threadIdx.x; d < NB; d += 256) status[t * NB + d] = (t == 0 ? D_INC : D_AGG) | h[d];
     if (t == 0 && threadIdx.x == 0) *counter = 0;
@@ -499,7 +502,8 @@ __global__ void __launch_bounds__(256) tile_agg_kernel(const K *__restrict__ key
 
 template <typename K, int VB, typename KO, int RB>
 static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *vout, long long n, int shift,
-                            const unsigned *digit_base, void *scratch, unsigned hi, cudaStream_t st, bool prezeroed)
+                            const unsigned *digit_base, void *scratch, unsigned hi, cudaStream_t st, bool prezeroed,
+                            unsigned long long encx)
 {
     using Cfg = PassCfg<K, VB, RB>;
     const long long tiles = (n + Cfg::TILE - 1) / Cfg::TILE;
@@ -521,7 +525,7 @@ static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *
     if (e != cudaSuccess) return e;
     if (NG_S_PREAGG) {
         tile_agg_kernel<K, (1 << RB), Cfg::TILE><<<(unsigned)tiles, 256, 0, st>>>(
-            (const K *)kin, n, shift, (unsigned *)((char *)scratch + 256), (unsigned *)scratch);
+            (const K *)kin, n, shift, (unsigned *)((char *)scratch + 256), (unsigned *)scratch, (K)encx);
     } else if (!prezeroed) {
         e = cudaMemsetAsync(scratch, 0, (size_t)tiles * (1 << RB) * 4 + 256, st);
         if (e != cudaSuccess) return e;
@@ -529,44 +533,45 @@ static cudaError_t run_pass(const void *kin, void *kout, const void *vin, void *
     const unsigned grid = (unsigned)(tiles < grid_max ? tiles : grid_max);
     onesweep_p_kernel<K, VB, KO, RB><<<grid, S_THREADS, Cfg::SMEM, st>>>(
         (const K *)kin, (KO *)kout, vin, vout, n, shift, digit_base, (unsigned *)((char *)scratch + 256),
-        (unsigned *)scratch, hi);
+        (unsigned *)scratch, hi, (K)encx);
     return cudaGetLastError();
 }
 
 template <typename K, typename KO, int RB>
 static cudaError_t run_pass_v(int vb, const void *kin, void *kout, const void *vin, void *vout, long long n, int shift,
-                              const unsigned *digit_base, void *scratch, unsigned hi, cudaStream_t st, bool pz)
+                              const unsigned *digit_base, void *scratch, unsigned hi, cudaStream_t st, bool pz,
+                              unsigned long long encx)
 {
-    if (vb == 0) return run_pass<K, 0, KO, RB>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
-    if (vb == 4) return run_pass<K, 4, KO, RB>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
-    return run_pass<K, 8, KO, RB>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
+    if (vb == 0) return run_pass<K, 0, KO, RB>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz, encx);
+    if (vb == 4) return run_pass<K, 4, KO, RB>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz, encx);
+    return run_pass<K, 8, KO, RB>(kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz, encx);
 }
 
 template <int RB>
 static cudaError_t run_pass_kk(int kb_in, int kb_out, int vb, const void *kin, void *kout, const void *vin,
                                void *vout, long long n, int shift, const unsigned *digit_base, void *scratch,
-                               unsigned hi, cudaStream_t st, bool pz)
+                               unsigned hi, cudaStream_t st, bool pz, unsigned long long encx)
 {
-    if (kb_in == 4 && kb_out == 4)
-        return run_pass_v<uint32_t, uint32_t, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
-    if (kb_in == 8 && kb_out == 8)
-        return run_pass_v<uint64_t, uint64_t, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
-    if (kb_in == 8)
-        return run_pass_v<uint64_t, uint32_t, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
-    return run_pass_v<uint32_t, uint64_t, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz);
+#define NG_RPV(KI, KO_) run_pass_v<KI, KO_, RB>(vb, kin, kout, vin, vout, n, shift, digit_base, scratch, hi, st, pz, encx)
+    if (kb_in == 4 && kb_out == 4) return NG_RPV(uint32_t, uint32_t);
+    if (kb_in == 8 && kb_out == 8) return NG_RPV(uint64_t, uint64_t);
+    if (kb_in == 8) return NG_RPV(uint64_t, uint32_t);
+    return NG_RPV(uint32_t, uint64_t);
+#undef NG_RPV
 }
 
 cudaError_t launch_radix_pass_x(int kb_in, int kb_out, int vb, const void *kin, void *kout, const void *vin,
                                 void *vout, long long n, int shift, const unsigned *digit_base, void *scratch,
-                                unsigned hi, cudaStream_t st, long long *launches, int rb, bool prezeroed)
+                                unsigned hi, cudaStream_t st, long long *launches, int rb, bool prezeroed,
+                                unsigned long long encx)
 {
     if (n <= 0) return cudaSuccess;
     if (n >= (1ll << 30)) return cudaErrorInvalidValue;
     if (rb != 8 && rb != 9) return cudaErrorInvalidValue;
     const cudaError_t e = rb == 8 ? run_pass_kk<8>(kb_in, kb_out, vb, kin, kout, vin, vout, n, shift, digit_base,
-                                                   scratch, hi, st, prezeroed)
+                                                   scratch, hi, st, prezeroed, encx)
                                   : run_pass_kk<9>(kb_in, kb_out, vb, kin, kout, vin, vout, n, shift, digit_base,
-                                                   scratch, hi, st, prezeroed);
+                                                   scratch, hi, st, prezeroed, encx);
     ++*launches;
     return e;
 }
