@@ -438,39 +438,49 @@ __global__ void __launch_bounds__(P_THREADS) block_prefix_kernel(const V *__rest
 {
     // out has N+1 entries: forward out[e+1] = AGG(v[0..e]); backward
     // out[N-1-e] = AGG(v[N-1-e..N)); the identity entry is written by block 0.
+    // The block's rows come in by coalesced loads into shared memory (one
+    // padding word per P_ITEMS), each thread scans P_ITEMS consecutive rows in
+    // registers, one block scan of the thread totals, and the results leave
+    // through shared memory by coalesced stores (round 2, session 2: was 16
+    // barrier-separated steps of 256 rows)
+    constexpr int PAD = P_ITEMS + 1;
+    __shared__ long long s_x[P_THREADS * PAD];
     __shared__ long long s_w[P_THREADS / 32];
-    __shared__ long long s_carry;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const long long b0 = blockIdx.x * (long long)P_BLOCK;
-    if (threadIdx.x == 0) s_carry = bpre[blockIdx.x];
-    if (blockIdx.x == 0 && threadIdx.x == 0) out[BACK ? N : 0] = ident<AGG>();
-    // every row of the block loaded up front (one DRAM round trip, not one
-    // per 256-row step of the barrier-separated scan below)
-    long long xs[P_ITEMS];
+    if (blockIdx.x == 0 && tid == 0) out[BACK ? N : 0] = ident<AGG>();
 #pragma unroll
     for (int j = 0; j < P_ITEMS; j++) {
-        const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
-        xs[j] = e < N ? elem<V, BACK, PART>(v, N, e) : ident<AGG>();
+        const int q = j * P_THREADS + tid;   // block-local row, coalesced
+        const long long e = b0 + q;
+        s_x[(q / P_ITEMS) * PAD + q % P_ITEMS] = e < N ? elem<V, BACK, PART>(v, N, e) : ident<AGG>();
     }
     __syncthreads();
+    long long xs[P_ITEMS];
 #pragma unroll
-    for (int j = 0; j < P_ITEMS; j++) {   // rows of the block in order, 256 at a time
-        const long long e = b0 + (long long)j * P_THREADS + threadIdx.x;
-        long long incl = xs[j];
-        for (int o = 1; o < 32; o <<= 1) {
-            const long long y = __shfl_up_sync(FULL, incl, o);
-            if (lane >= o) incl = comb<AGG>(incl, y);
-        }
-        if (lane == 31) s_w[warp] = incl;
-        __syncthreads();
-        long long wpre = ident<AGG>();
-        for (int w = 0; w < warp; w++) wpre = comb<AGG>(wpre, s_w[w]);
-        const long long carry = s_carry;
-        const long long val = comb<AGG>(carry, comb<AGG>(wpre, incl));
-        if (e < N) out[BACK ? N - 1 - e : e + 1] = val;
-        __syncthreads();
-        if (threadIdx.x == P_THREADS - 1) s_carry = val;
-        __syncthreads();
+    for (int j = 0; j < P_ITEMS; j++) xs[j] = s_x[tid * PAD + j];
+#pragma unroll
+    for (int j = 1; j < P_ITEMS; j++) xs[j] = comb<AGG>(xs[j - 1], xs[j]);
+    long long incl = xs[P_ITEMS - 1];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const long long y = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl = comb<AGG>(y, incl);
+    }
+    if (lane == 31) s_w[warp] = incl;
+    __syncthreads();
+    long long pre = bpre[blockIdx.x];
+    for (int w = 0; w < warp; w++) pre = comb<AGG>(pre, s_w[w]);
+    const long long up = __shfl_up_sync(FULL, incl, 1);
+    if (lane) pre = comb<AGG>(pre, up);
+#pragma unroll
+    for (int j = 0; j < P_ITEMS; j++) s_x[tid * PAD + j] = comb<AGG>(pre, xs[j]);
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < P_ITEMS; j++) {
+        const int q = j * P_THREADS + tid;
+        const long long e = b0 + q;
+        if (e < N) out[BACK ? N - 1 - e : e + 1] = s_x[(q / P_ITEMS) * PAD + q % P_ITEMS];
     }
 }
 
