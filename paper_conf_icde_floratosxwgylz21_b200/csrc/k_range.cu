@@ -549,20 +549,29 @@ __global__ void __launch_bounds__(P_THREADS) seg_onepass_kernel(const K *__restr
     __syncthreads();
     const long long b = s_b;
     const long long e0 = b * SG_BLOCK + (long long)tid * SG_ITEMS;
-    // this thread's 16 rows: sequential segmented inclusive scan
-    SegPair<AGG> x[SG_ITEMS];
-    K prev = e0 > 0 && e0 - 1 < N ? keys[e0 - 1] : (K)0;
+    // the block's rows enter through shared memory (coalesced loads, one
+    // padding slot per SG_ITEMS) as (payload, run-start flag) pairs
+    constexpr int SPAD = SG_ITEMS + 1;
+    __shared__ long long s_xv[P_THREADS * SPAD];
+    __shared__ unsigned char s_xf[P_THREADS * SPAD];
 #pragma unroll
-    for (int i = 0; i < SG_ITEMS; i++) {
-        const long long e = e0 + i;
+    for (int j = 0; j < SG_ITEMS; j++) {
+        const int q = j * P_THREADS + tid;
+        const long long e = b * SG_BLOCK + q;
+        const int slot = (q / SG_ITEMS) * SPAD + q % SG_ITEMS;
         if (e < N) {
-            const K k = keys[e];
-            x[i] = SegPair<AGG>{(long long)v[e], (e == 0 || k != prev) ? 1 : 0};
-            prev = k;
+            s_xv[slot] = (long long)v[e];
+            s_xf[slot] = (e == 0 || keys[e] != keys[e - 1]) ? 1 : 0;
         } else {
-            x[i] = SegPair<AGG>{ident<AGG>(), 0};
+            s_xv[slot] = ident<AGG>();
+            s_xf[slot] = 0;
         }
     }
+    __syncthreads();
+    // this thread's 16 consecutive rows: sequential segmented inclusive scan
+    SegPair<AGG> x[SG_ITEMS];
+#pragma unroll
+    for (int i = 0; i < SG_ITEMS; i++) x[i] = SegPair<AGG>{s_xv[tid * SPAD + i], (int)s_xf[tid * SPAD + i]};
     if (tid == 0) s_head0 = x[0].f;
 #pragma unroll
     for (int i = 1; i < SG_ITEMS; i++) x[i] = seg_comb<AGG>(x[i - 1], x[i]);
@@ -632,10 +641,15 @@ __global__ void __launch_bounds__(P_THREADS) seg_onepass_kernel(const K *__restr
     __syncthreads();
     const SegPair<AGG> pre = seg_comb<AGG>(s_carry, tex);
 #pragma unroll
-    for (int i = 0; i < SG_ITEMS; i++) {
-        const long long e = e0 + i;
-        if (e < N) grp[e] = seg_comb<AGG>(pre, x[i]).v;
+    for (int i = 0; i < SG_ITEMS; i++) s_xv[tid * SPAD + i] = seg_comb<AGG>(pre, x[i]).v;
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < SG_ITEMS; j++) {   // and leave the same way (coalesced stores)
+        const int q = j * P_THREADS + tid;
+        const long long e = b * SG_BLOCK + q;
+        if (e < N) grp[e] = s_xv[(q / SG_ITEMS) * SPAD + q % SG_ITEMS];
     }
+    (void)e0;
 }
 
 template <typename K, typename V, int AGG>
