@@ -15,7 +15,9 @@ eng = Engine(0, arena_bytes=16 << 30)
 eng.set_profiling(True)
 out = []
 t4, p4 = tpch.flattened("q4", 10.0, 5)
-for name, t, plan in (("Q4 SF10", t4, p4), ("C5", query1.config("C5"), make_plan("=", "count", "="))):
+t2, p2 = tpch.flattened("q2", 1.0, 3)
+for name, t, plan in (("Q4 SF10", t4, p4), ("C5", query1.config("C5"), make_plan("=", "count", "=")),
+                      ("Q2 SF1", t2, p2)):
     m0 = eng.mark()
     R, S = load(eng, t)
     idx = eng.index_for_plan(plan, S)
