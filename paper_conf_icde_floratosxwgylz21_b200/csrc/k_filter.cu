@@ -158,7 +158,7 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
                   unsigned long long *__restrict__ keymask, unsigned *__restrict__ extreme,
                   const unsigned long long *__restrict__ tile_base, unsigned *__restrict__ tile_count,
                   unsigned *__restrict__ counter, long long *__restrict__ out_count,
-                  unsigned *__restrict__ live_bits)
+                  unsigned *__restrict__ live_bits, const unsigned long long *__restrict__ chunk_off)
 {
     // live_bits (ordered two-pass mode): pass 1 (tile_count) writes each
     // (tile, item, warp)'s survivor ballot; pass 2 takes its survivors from
@@ -311,7 +311,7 @@ filter_tma_kernel(long long n, SrcCols sc, TPlan tp, int *__restrict__ out_ids, 
             }
             if (lane == 31) {
                 if (tile_count) tile_count[tile] = incl;
-                else if (tile_base) s_claim = tile_base[tile];
+                else if (tile_base) s_claim = tile_base[tile] + (chunk_off ? __ldcg(chunk_off + (tile >> 10)) : 0ull);
                 else s_claim = incl ? atomicAdd((unsigned long long *)out_count, (unsigned long long)incl) : 0ull;
             }
         }
@@ -735,23 +735,25 @@ __global__ void __launch_bounds__(256) rp_dense_kernel(long long n, KeySrc ks, i
 }
 
 // ------------------------------------------------------------------ host side
-// Exclusive scan of the per-tile counts (ordered mode): one CTA; thread t
-// owns a contiguous segment of the counts (loads of the segment in flight
-// together), sums it, block scan, then writes the segment's prefixes -- a
-// few memory round trips instead of one per 1024-count chunk (60M rows =
-// 29k tiles: 44 -> 26 us; chunks staged in shared memory measured 32 us).
-__global__ void __launch_bounds__(1024) tile_scan_kernel(const unsigned *__restrict__ cnt, long long tiles,
-                                                         unsigned long long *__restrict__ base,
-                                                         long long *__restrict__ out_count)
+// Exclusive scan of the per-tile counts (ordered mode) over many CTAs:
+// CTA c scans tiles [1024c, 1024c + 1024)
+// (one coalesced load each, a block scan) into base[] as chunk-local
+// exclusive prefixes and its total into ctot[c]; the last CTA to finish
+// scans the chunk totals into coff[] (and *out_count).  A tile's offset is
+// base[t] + coff[t >> 10] (29k tiles: one round trip instead of ~29).
+__global__ void __launch_bounds__(1024) tile_scan_chunks_kernel(const unsigned *__restrict__ cnt, long long tiles,
+                                                                unsigned long long *__restrict__ base,
+                                                                unsigned long long *__restrict__ ctot,
+                                                                unsigned long long *__restrict__ coff,
+                                                                long long *__restrict__ out_count,
+                                                                unsigned *__restrict__ done)
 {
     __shared__ unsigned long long s_w[32];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const long long per = (tiles + 1023) / 1024;
-    const long long i0 = threadIdx.x * per, i1 = min(tiles, i0 + per);
-    unsigned long long sum = 0;
-#pragma unroll 8
-    for (long long i = i0; i < i1; i++) sum += __ldg(cnt + i);
-    unsigned long long incl = sum;
+    __shared__ bool s_last;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const long long i = blockIdx.x * 1024ll + tid;
+    const unsigned long long x = i < tiles ? __ldg(cnt + i) : 0ull;
+    unsigned long long incl = x;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
         const unsigned long long y = __shfl_up_sync(FULL, incl, o);
@@ -759,18 +761,37 @@ __global__ void __launch_bounds__(1024) tile_scan_kernel(const unsigned *__restr
     }
     if (lane == 31) s_w[warp] = incl;
     __syncthreads();
-    unsigned long long run = incl - sum, total = 0;
+    unsigned long long pre = incl - x, total = 0;
     for (int w = 0; w < 32; w++) {
-        if (w < warp) run += s_w[w];
+        if (w < warp) pre += s_w[w];
         total += s_w[w];
     }
-#pragma unroll 8
-    for (long long i = i0; i < i1; i++) {
-        const unsigned c = __ldg(cnt + i);
-        base[i] = run;
-        run += c;
+    if (i < tiles) base[i] = pre;
+    if (tid == 0) ctot[blockIdx.x] = total;
+    __threadfence();
+    __syncthreads();
+    if (tid == 0) s_last = atomicAdd(done, 1u) == gridDim.x - 1;
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    // the last CTA: exclusive scan of the chunk totals (<= 1024 chunks)
+    const unsigned long long c = tid < (int)gridDim.x ? __ldcg(ctot + tid) : 0ull;
+    unsigned long long ci = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long y = __shfl_up_sync(FULL, ci, o);
+        if (lane >= o) ci += y;
     }
-    if (threadIdx.x == 0) *out_count = (long long)total;
+    __syncthreads();
+    if (lane == 31) s_w[warp] = ci;
+    __syncthreads();
+    unsigned long long cp = ci - c, ct = 0;
+    for (int w = 0; w < 32; w++) {
+        if (w < warp) cp += s_w[w];
+        ct += s_w[w];
+    }
+    if (tid < (int)gridDim.x) coff[tid] = cp;
+    if (tid == 0) *out_count = (long long)ct;
 }
 
 namespace {
@@ -816,6 +837,7 @@ struct FilterOut {
     unsigned *counter;
     long long *count;
     unsigned *live_bits;   // ordered two-pass mode: survivor ballots of pass 1 (nullable)
+    const unsigned long long *chunk_off = nullptr;   // + offset of the tile's 1024-tile chunk (nullable)
 };
 
 template <int KB, int VB, int ITEMS>
@@ -835,7 +857,7 @@ cudaError_t launch_t(long long n, const SrcCols &sc, const TPlan &tp, const Filt
     long long grid = (long long)num_sms * (occ > 0 ? occ : 1);
     if (grid > tiles) grid = tiles;
     kern<<<(unsigned)grid, T_THREADS, smem, st>>>(n, sc, tp, o.ids, o.keys, o.kvalid, o.vals, o.keymask, o.extreme,
-                                                  o.tile_base, o.tile_count, o.counter, o.count, o.live_bits);
+                                                  o.tile_base, o.tile_count, o.counter, o.count, o.live_bits, o.chunk_off);
     return cudaGetLastError();
 }
 
@@ -870,7 +892,8 @@ size_t filter_scratch_bytes(long long n)
 {
     // counters + per-tile counts / offsets (two-pass mode), or the ordered
     // filter's chunk counts + ballot words
-    const size_t two_pass = 1024 + 768 + (size_t)(n / T_THREADS + 2) * 12 + (size_t)(n / 32 + 2) * 4 + 64 * 16 * 4;
+    const size_t two_pass = 1024 + 1024 + (size_t)(n / T_THREADS + 2) * 12 + (size_t)(n / 32 + 2) * 4 + 64 * 16 * 4 +
+                            (size_t)(n / T_THREADS / 1024 + 2) * 16;
     const size_t one_launch = RP_BITS_OFF + (size_t)(n / 32 + 2) * 4 + 256;
     return two_pass > one_launch ? two_pass : one_launch;
 }
@@ -1105,8 +1128,12 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
         const long long tiles = (n + T_THREADS * items - 1) / (T_THREADS * items);
         unsigned *tcount = (unsigned *)((char *)scratch + 1024);
         unsigned long long *tbase = (unsigned long long *)((char *)scratch + 1024 + ((tiles * 4 + 255) & ~255ll));
+        const long long nchunks = (tiles + 1023) / 1024;
+        unsigned long long *ctot = (unsigned long long *)((char *)tbase + ((tiles * 8 + 255) & ~255ll));
+        unsigned long long *coff = ctot + nchunks;
+        unsigned *cdone = (unsigned *)scratch + 128;   // a zeroed counter word (scratch bytes 512..515)
         // the two-call mode keeps pass 1's survivor ballots for pass 2
-        unsigned *bits = ordered_phase ? (unsigned *)((char *)tbase + ((tiles * 8 + 255) & ~255ll)) : nullptr;
+        unsigned *bits = ordered_phase ? (unsigned *)((char *)ctot + ((nchunks * 16 + 255) & ~255ll)) : nullptr;
         if (ordered_phase == 2) {
             // pass 2 streams only the key / payload columns: the predicate
             // columns are not read again
@@ -1136,6 +1163,7 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
             tp2.n_preds = 0;
             resolve(sc2, sp2, tp2);
             o.tile_base = tbase;
+            o.chunk_off = coff;
             o.live_bits = bits;
             e = dispatch(k, v, items, n, sc2, tp2, o, num_sms, st);
             ++*launches;
@@ -1157,8 +1185,10 @@ cudaError_t launch_filter(long long n, const PredSet &preds, const KeySrc &key, 
                      (unsigned *)scratch + 64, out_count, bits};
         e = launch_items<0, 0>(items, n, sc1, tp1, o1, num_sms, st);
         if (e != cudaSuccess) return e;
-        tile_scan_kernel<<<1, 1024, 0, st>>>(tcount, tiles, tbase, out_count);
+        tile_scan_chunks_kernel<<<(unsigned)nchunks, 1024, 0, st>>>(tcount, tiles, tbase, ctot, coff, out_count,
+                                                                    cdone);
         o.tile_base = tbase;
+        o.chunk_off = coff;
         *launches += 2;
         if (ordered_phase == 1) return cudaGetLastError();
     }
